@@ -1,0 +1,100 @@
+"""CPU oracle for exact triangle counting — TEST INFRASTRUCTURE.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
+``cpu_baseline`` / ``--impl reference`` leg may import this module.  The
+product path (``paper_conf_ipps_li0ptz24_b200``) never imports it, and it
+never imports the product path; both take their inputs from ``tcgen``.
+
+The arithmetic lives in ``oracle/tc_oracle.cpp`` (plain C++17 + std::thread,
+node-iterator with ``std::set_intersection``; each step cites PAPER.md).
+This wrapper only marshals arguments.  Pins: ``tests/test_oracle_pins.py``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "libtcoracle.so")
+_lib = None
+
+ORDER_DEGREE, ORDER_ID, ORDER_HASH = 0, 1, 2
+
+
+class _Result(ctypes.Structure):
+    _fields_ = [
+        ("triangles", ctypes.c_uint64),
+        ("m", ctypes.c_int64),
+        ("n_active", ctypes.c_int64),
+        ("max_out_degree", ctypes.c_int64),
+        ("merge_steps_total", ctypes.c_uint64),
+        ("merge_steps_counted", ctypes.c_uint64),
+        ("build_ms", ctypes.c_double),
+        ("count_ms", ctypes.c_double),
+        ("threads", ctypes.c_int32),
+        ("sampled", ctypes.c_int32),
+    ]
+
+
+@dataclass
+class OracleResult:
+    triangles: int
+    m: int
+    n_active: int
+    max_out_degree: int
+    merge_steps_total: int
+    merge_steps_counted: int
+    build_ms: float
+    count_ms: float
+    threads: int
+    sampled: bool
+
+
+def build_lib() -> str:
+    """Compile the oracle with g++ (building the checker is not using it)."""
+    src = os.path.join(_HERE, "tc_oracle.cpp")
+    if not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(src):
+        subprocess.check_call(["g++", "-O3", "-std=c++17", "-fPIC", "-shared", "-pthread",
+                               src, "-o", _LIB_PATH])
+    return _LIB_PATH
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build_lib()
+        L = ctypes.CDLL(_LIB_PATH)
+        L.tco_count.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64,
+                                ctypes.c_int, ctypes.c_int, ctypes.c_int64, ctypes.POINTER(_Result)]
+        L.tco_count.restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def count(src, dst, n: int = -1, order: int = ORDER_DEGREE, threads: int = 0,
+          sample_stride: int = 1) -> OracleResult:
+    """Exact T of the cleaned simple graph given by raw pairs (src[i], dst[i]).
+
+    Raises ValueError on an id outside [0, n).
+    """
+    src = np.ascontiguousarray(src, dtype=np.int32)
+    dst = np.ascontiguousarray(dst, dtype=np.int32)
+    if src.shape != dst.shape:
+        raise ValueError("src and dst differ in length")
+    r = _Result()
+    rc = lib().tco_count(src.ctypes.data_as(ctypes.c_void_p), dst.ctypes.data_as(ctypes.c_void_p),
+                         len(src), int(n), int(order), int(threads), int(sample_stride),
+                         ctypes.byref(r))
+    if rc != 0:
+        raise ValueError("oracle: invalid input (vertex id out of range)")
+    return OracleResult(int(r.triangles), int(r.m), int(r.n_active), int(r.max_out_degree),
+                        int(r.merge_steps_total), int(r.merge_steps_counted), float(r.build_ms),
+                        float(r.count_ms), int(r.threads), bool(r.sampled))
+
+
+def triangles(src, dst, n: int = -1, **kw) -> int:
+    return count(src, dst, n, **kw).triangles
