@@ -1,0 +1,404 @@
+#!/usr/bin/env python
+"""bench.py — oriented edges/s and TC ms of the ITC hot path on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--impl b200tc|reference]
+    torchrun --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N ...
+
+One "step" = one pass of the whole counting path over
+the built graph of the workload: every rank counts its cost-balanced range of
+live oriented edges (tc_count_range) and, for N > 1, one 8-byte NCCL
+all_reduce combines the partials.  Preprocessing (a1-a6, tc_build_csr) is
+timed separately and reported under "build_ms"; "e2e" times the public entry
+point from pinned HOST edge lists: H2D copy + build + count + D2H of T.
+
+Default workload: config C3 (RMAT scale 24, edge factor 16, Graph500
+initiator, seed 1), the largest single-GPU RMAT graph BASELINE.json quotes the
+metric on.  Inputs (1.1 GB CSR) exceed L2, and L2 is additionally flushed
+between timed steps by writing a 512 MiB buffer.
+
+Rank 0 prints ONE JSON line.  The oracle (oracle/, CPU) runs only in the
+cpu_baseline leg (rank 0, N = 1) and under --impl reference.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import tcgen  # noqa: E402
+
+METRIC = "oriented edges/sec"
+UNIT = "edges/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C3", choices=sorted(tcgen.CONFIGS))
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--impl", default="b200tc", choices=["b200tc", "reference"])
+    ap.add_argument("--flush-mb", type=int, default=512)
+    ap.add_argument("--e2e-steps", type=int, default=None, help="default: --steps")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0,
+                    help="target oracle counting time of the cpu_baseline sample")
+    ap.add_argument("--chunk-cost", type=int, default=0)
+    ap.add_argument("--block", type=int, default=0)
+    ap.add_argument("--out", default=None, help="also write the JSON line here")
+    return ap.parse_args()
+
+
+def cpu_info():
+    model = "unknown"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return model, os.cpu_count()
+
+
+def expected_counts(cfg, seed):
+    p = os.path.join(ROOT, "tests", "golden", "config_counts.json")
+    if not os.path.exists(p):
+        return None
+    return json.load(open(p)).get(f"{cfg}/seed{seed}")
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def profile_traffic(cfg):
+    """dram bytes per launch of the count kernel from the committed ncu summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(p):
+        return None
+    d = json.load(open(p)).get(cfg)
+    return None if not d else d.get("dram_bytes_per_launch")
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms (B200_PROFILING.md)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-lms", "200", "-i", str(self.index)],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.p.terminate()
+        self.p.wait()
+        self.f.flush()
+        rows = [l.strip().split(", ") for l in open(self.f.name) if l.strip()]
+        os.unlink(self.f.name)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[1]))
+                mx.append(float(r[2]))
+            except (ValueError, IndexError):
+                continue
+            for name, v in zip(names, r[5:9]):
+                if v.strip() == "Active":
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def run_reference(a):
+    """--impl reference: the CPU oracle, as it stands, on this box's host cores."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    cfg = tcgen.CONFIGS[a.config]
+    tcgen.lib().tcgen_set_threads(0)
+    src, dst, n = cfg.generate(a.seed)
+    g = oracle.OracleGraph(src, dst, n)
+    probe = g.count_rows(stride=4096, offset=0)
+    m = probe.m
+    # each step: rows x % stride == step, sized to ~cpu_seconds / (W+K) * ... bounded
+    per_step_s = max(1.0, min(10.0, 120.0 / max(1, a.steps + a.warmup)))
+    rate = probe.merge_steps_counted / max(probe.count_ms / 1e3, 1e-6)  # merge steps / s
+    want_steps = rate * per_step_s
+    stride = int(max(1, min(1 << 20, probe.merge_steps_total // max(want_steps, 1))))
+    for i in range(a.warmup):
+        g.count_rows(stride=stride, offset=i % stride)
+    edges, secs, counted, total = 0.0, 0.0, 0, probe.merge_steps_total
+    for i in range(a.steps):
+        r = g.count_rows(stride=stride, offset=(a.warmup + i) % stride)
+        frac = r.merge_steps_counted / max(1, r.merge_steps_total)
+        edges += m * frac
+        secs += r.count_ms / 1e3
+        counted += r.merge_steps_counted
+    value = edges / secs if secs > 0 else 0.0
+    model, ncpu = cpu_info()
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": a.gpus,
+        "steps": a.steps, "warmup": a.warmup, "ms_per_step": secs * 1e3 / max(1, a.steps),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
+        "data": "synthetic", "config": {"workload": f"{a.config}: {cfg.description}",
+                                        "seed": a.seed, "n": n, "m": m},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": r.threads, "kind": "oracle",
+                         "sample": (f"rows x % {stride} == o (one offset o per step) of the "
+                                    f"{a.config} graph; {counted / max(1, total) / a.steps:.4%} "
+                                    f"of its merge steps per step; CPU {model}, {ncpu} cpus; "
+                                    f"oracle build {g.count_rows(stride=1 << 30).build_ms:.0f} ms "
+                                    f"not in value")},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    if a.out:
+        open(a.out, "w").write(json.dumps(line) + "\n")
+    g.close()
+    return 0
+
+
+def cpu_baseline(src, dst, n, a, m_gpu):
+    """The oracle timed on a bounded row sample of the same workload (rank 0, N = 1)."""
+    import oracle
+    g = oracle.OracleGraph(src, dst, n)
+    probe = g.count_rows(stride=4096, offset=0)
+    rate = probe.merge_steps_counted / max(probe.count_ms / 1e3, 1e-6)
+    stride = int(max(1, min(1 << 20, probe.merge_steps_total // max(rate * a.cpu_seconds, 1))))
+    r = g.count_rows(stride=stride, offset=1 % stride)
+    frac = r.merge_steps_counted / max(1, r.merge_steps_total)
+    value = r.m * frac / max(r.count_ms / 1e3, 1e-9)
+    model, ncpu = cpu_info()
+    out = {"value": value, "unit": UNIT, "cores": r.threads, "kind": "oracle",
+           "sample": (f"rows x % {stride} == 1 of the same graph ({frac:.3%} of its "
+                      f"{r.merge_steps_total:.3e} merge steps, {r.count_ms:.0f} ms); "
+                      f"value = m * sampled fraction / count time; oracle build "
+                      f"{r.build_ms:.0f} ms excluded like the GPU build; CPU {model}, {ncpu} cpus"),
+           "oracle_build_ms": r.build_ms}
+    g.close()
+    assert r.m == m_gpu, (r.m, m_gpu)
+    return out
+
+
+def main():
+    a = parse()
+    if a.impl == "reference":
+        return run_reference(a)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_li0ptz24_b200 as tc
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != a.gpus and rank == 0:
+        print(f"warning: --gpus {a.gpus} but WORLD_SIZE {world}", file=sys.stderr)
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+
+    cfg = tcgen.CONFIGS[a.config]
+    tcgen.lib().tcgen_set_threads(0)
+    t0 = time.time()
+    src, dst, n = cfg.generate(a.seed)
+    gen_s = time.time() - t0
+    opts = {}
+    if a.chunk_cost:
+        opts["chunk_cost"] = a.chunk_cost
+    if a.block:
+        opts["block_threads"] = a.block
+
+    # ---------------------------------------------------------------- build (a1..a6)
+    dsrc = torch.from_numpy(src).to(dev)
+    dst_t = torch.from_numpy(dst).to(dev)
+    g = tc.build_csr(dsrc, dst_t, n, options=opts or None)   # warm (allocator pools, CUB)
+    g.close()
+    torch.cuda.synchronize()
+    tb = time.perf_counter()
+    g = tc.build_csr(dsrc, dst_t, n, options=opts or None)
+    torch.cuda.synchronize()
+    build_wall_ms = (time.perf_counter() - tb) * 1e3
+    info = g.info
+    del dsrc, dst_t
+    m = int(info.m)
+
+    bounds = g.partition(world)
+    e0, e1 = bounds[rank], bounds[rank + 1]
+    keys_share = 1.0
+    if world > 1:
+        # this rank's share of the probe keys, for its roofline bytes
+        keys_share = (e1 - e0) / max(1, info.m_live)
+    out = torch.zeros(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(a.flush_mb << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step(ev_mid=None):
+        g.count_range(e0, e1, out=out)
+        if ev_mid is not None:
+            ev_mid.record(stream)
+        if world > 1:
+            dist.all_reduce(out)
+
+    for _ in range(max(1, a.warmup)):
+        step()
+    torch.cuda.synchronize()
+    T = int(out.item()) & (2**64 - 1)
+
+    sampler = ClockSampler(torch.cuda.current_device())
+    sampler.start()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+            torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    for i in range(a.steps):
+        flush.fill_(i & 0xFF)  # L2 flush between timed steps (outside the events)
+        s0, sm, s1 = evs[i]
+        s0.record(stream)
+        step(sm)
+        s1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    step_ms = [s0.elapsed_time(s1) for s0, _, s1 in evs]
+    kern_ms = [s0.elapsed_time(sm) for s0, sm, _ in evs]
+    tot = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    total_ms, kern_total_ms = float(tot[0]), float(tot[1])
+    ms_per_step = total_ms / a.steps
+    value = m / (ms_per_step / 1e3)
+
+    # ---------------------------------------------------------------- e2e (public API, host data)
+    e2e = None
+    if not a.no_e2e:
+        k2 = a.e2e_steps if a.e2e_steps is not None else a.steps
+        ps = torch.from_numpy(src).pin_memory()
+        pd = torch.from_numpy(dst).pin_memory()
+        ts = []
+        n_chunks = 0
+        for i in range(1 + k2):  # first one warms the pinned path
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            x0 = torch.cuda.Event(enable_timing=True)
+            x1 = torch.cuda.Event(enable_timing=True)
+            x0.record(stream)
+            g2 = tc.build_csr_host(ps, pd, n, options=opts or None)
+            b = g2.partition(world)
+            o2 = g2.count_range(b[rank], b[rank + 1])
+            if world > 1:
+                dist.all_reduce(o2)
+            t_e2e = int(o2.item()) & (2**64 - 1)
+            x1.record(stream)
+            torch.cuda.synchronize()
+            n_chunks = g2.info.n_chunks
+            g2.close()
+            assert t_e2e == T, (t_e2e, T)
+            if i:
+                ts.append(x0.elapsed_time(x1))
+        et = torch.tensor([sum(ts)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        e2e_ms = float(et[0]) / max(1, len(ts))
+        e2e = {"value": m / (e2e_ms / 1e3), "unit": UNIT, "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": int(src.nbytes + dst.nbytes),
+               "d2h_bytes_per_step": 8 + 8 * (n_chunks + 1) + 96,
+               "what": "tc_build_csr_host (H2D of the raw pinned edge list + a1..a6) + "
+                       "tc_count_range + all_reduce + 8-B D2H of T"}
+
+    if rank != 0:
+        if world > 1:
+            dist.barrier()
+            dist.destroy_process_group()
+        return 0
+
+    exp = expected_counts(a.config, a.seed)
+    parity = None if exp is None else (exp["triangles"] == T and exp["m"] == m)
+
+    hbm, peak_src = peaks()
+    kern_avg_s = kern_total_ms / a.steps / 1e3
+    b_launch = info.b_itc * keys_share
+    achieved = b_launch / kern_avg_s / 1e9
+    traffic = profile_traffic(a.config) if world == 1 else None
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
+        "warmup": a.warmup, "ms_per_step": ms_per_step, "tc_ms": ms_per_step,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
+        "data": "synthetic",
+        "config": {"workload": f"{a.config}: {cfg.description}", "seed": a.seed, "n": n,
+                   "n_active": int(info.n), "m": m, "max_out_degree": int(info.max_out_degree),
+                   "m_live": int(info.m_live), "keys_total": int(info.keys_total),
+                   "parallelism": f"edge-range x{world} (replicated CSR, 1 NCCL all_reduce)",
+                   "l2": f"flushed by a {a.flush_mb} MiB write between timed steps; CSR "
+                         f"{(info.m * 4 + (info.n + 1) * 8) / 2**20:.0f} MiB"},
+        "triangles": str(T), "parity_vs_oracle": parity,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved / hbm, "traffic": traffic,
+                     "bytes_per_launch": b_launch, "kernel_ms": kern_avg_s * 1e3,
+                     "bytes_def": "B_ITC = sum_e [4(suf_e + d+(v_e)) + 12] + 8(n'+1) "
+                                  "(SURVEY.md §8(d)); x this rank's share for N>1",
+                     "peak_source": peak_src},
+        "e2e": e2e,
+        "gpu_launches": a.steps,
+        "build_ms": {"canon": info.ms_canon, "sort_unique": info.ms_sort_unique,
+                     "degree_rank": info.ms_degree_rank, "orient_csr": info.ms_orient_csr,
+                     "plan": info.ms_plan, "total_events": info.ms_total,
+                     "wall": build_wall_ms},
+        "plan": {"n_chunks": int(info.n_chunks), "grid": int(info.count_grid),
+                 "block": int(info.count_block), "smem_bytes": int(info.smem_bytes),
+                 "groups": int(info.n_groups)},
+        "clocks": clocks,
+        "gen_s": round(gen_s, 2),
+        "step_ms": step_ms,
+    }
+    if world == 1 and not a.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(src, dst, n, a, m)
+    print(json.dumps(line), flush=True)
+    if a.out:
+        open(a.out, "w").write(json.dumps(line) + "\n")
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,184 @@
+/*
+ * tc.h — C-ABI of the B200 intersection-based triangle counting (ITC) library.
+ *
+ * The operation (PAPER.md = Li et al., "A Comparative Study of
+ * Intersection-Based Triangle Counting Algorithms on GPUs", IPDPS-W 2024):
+ *
+ *   T(G) = |{ {x,y,z} : {x,y}, {y,z}, {x,z} in E }|
+ *
+ * for the simple undirected graph G obtained from a raw edge list by
+ * ignoring direction, dropping self-loops and merging duplicates (P:287:
+ * cleaning "do[es] not alter the number of triangles").  The library
+ * reaches T exactly by the edge-iterator intersection of P:78 (Fig. 1(b))
+ * over a degree-oriented DAG: every triangle u<v<w (in the
+ * orientation order) is found once, at oriented edge (u,v), as the witness
+ * w in N+(u) ∩ N+(v).  Counts are exact integers; there is no rounding.
+ *
+ * Pipeline:
+ *   tc_build_csr  : a1 validate + canonicalise + drop self-loops,
+ *                   a2 radix sort + unique, a3 degree, a4 rank by
+ *                   (degree, id) + relabel + drop isolated vertices,
+ *                   a5 orient + per-row sort -> CSR, a6 dispatch plan.
+ *   tc_count*     : a7/a8 grouped counting kernels, a9 u64 reduction.
+ *
+ * Conventions (all entry points):
+ *   - extern "C", return tc_status, never throw, never abort.
+ *   - Device pointers are CUDA device memory of the current device; host
+ *     pointers are ordinary (pageable or pinned) host memory.
+ *   - `stream` is a cudaStream_t passed as void* (0 = legacy default
+ *     stream).  Work is stream ordered; only functions that write a host
+ *     output (h_*) synchronise the stream.
+ *   - Vertex ids are int32 (0 <= id < 2^31-1); edge counts and offsets are
+ *     int64; triangle counts are uint64 (they exceed 2^32 at config C3).
+ *   - On any non-OK status, tc_last_error() returns a thread-local message.
+ *   - A tc_graph is immutable after tc_build_csr / tc_replan returns, so
+ *     concurrent counts on one graph from different streams are allowed.
+ */
+#ifndef TC_H
+#define TC_H
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define TC_API __attribute__((visibility("default")))
+#else
+#define TC_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  TC_OK = 0,
+  TC_ERR_INVALID_ARGUMENT = 1, /* null pointer, id out of range, bad range   */
+  TC_ERR_OUT_OF_MEMORY = 2,    /* the allocator returned NULL                */
+  TC_ERR_CUDA = 3,             /* a CUDA runtime error (text in tc_last_error) */
+  TC_ERR_UNSUPPORTED = 4       /* a size the library does not handle          */
+} tc_status;
+
+typedef struct tc_graph tc_graph; /* opaque: owns the device CSR and plan */
+
+/* Build flags. */
+#define TC_KEEP_ISOLATED 0x1u /* keep degree-0 vertices as empty rows (n' = n) */
+
+/*
+ * Device allocator hook.  alloc returns NULL on failure (-> TC_ERR_OUT_OF_MEMORY);
+ * free receives exactly the pointer/size/stream of a prior alloc.  The default
+ * (tc_set_allocator(NULL, NULL, NULL)) is cudaMallocAsync / cudaFreeAsync on
+ * the calling stream.  Process-wide; set it before building graphs.
+ */
+typedef void* (*tc_alloc_fn)(size_t bytes, void* stream, void* ctx);
+typedef void (*tc_free_fn)(void* ptr, size_t bytes, void* stream, void* ctx);
+TC_API tc_status tc_set_allocator(tc_alloc_fn alloc, tc_free_fn free_fn, void* ctx);
+
+/*
+ * Plan options (performance parameters that never
+ * change the count; the property tests vary them).  0 in a field = default.
+ */
+typedef struct {
+  int32_t chunk_cost;   /* cost units per work chunk (default 16384)               */
+  int32_t seg_cost;     /* fixed cost per live oriented edge (default 4)          */
+  int32_t huge_degree;  /* d+(v) above which N+(v) is probed in global memory by
+                           binary search instead of an SMEM hash (default 8192)    */
+  int32_t block_threads;/* threads per CTA of the count kernel (default 512)       */
+  int32_t hash_shift;   /* hash slots = next_pow2(d+(v) << hash_shift) (default 1) */
+  int32_t reserved[3];
+} tc_options;
+
+/*
+ * a1..a6.  Build the oriented CSR and dispatch plan from a raw edge list.
+ *   d_src, d_dst : device int32[num_edges]; pair i is the undirected edge
+ *                  {d_src[i], d_dst[i]}.  Caller-owned, never modified.
+ *                  Duplicates, reversed pairs and self-loops are allowed
+ *                  (cleaned).
+ *   num_edges    : >= 0; 0 gives a valid empty graph (T = 0).
+ *   num_vertices : ids must lie in [0, num_vertices); -1 = max id + 1.
+ *   flags        : TC_KEEP_ISOLATED or 0.
+ *   opts         : NULL for defaults.
+ *   out          : receives the new graph; NULL on any error (nothing leaks).
+ * Errors: TC_ERR_INVALID_ARGUMENT for null pointers, num_edges < 0,
+ * num_vertices > 2^31-1, or any id < 0 or >= num_vertices.
+ * Synchronises `stream` (the unique-edge count must reach the host).
+ */
+TC_API tc_status tc_build_csr(const int32_t* d_src, const int32_t* d_dst, int64_t num_edges,
+                       int64_t num_vertices, uint32_t flags, const tc_options* opts,
+                       void* stream, tc_graph** out);
+
+/* Same, from HOST int32 arrays: the library copies them to the device on
+ * `stream` first (the end-to-end entry point bench.py's e2e leg times). */
+TC_API tc_status tc_build_csr_host(const int32_t* h_src, const int32_t* h_dst, int64_t num_edges,
+                            int64_t num_vertices, uint32_t flags, const tc_options* opts,
+                            void* stream, tc_graph** out);
+
+/* Rebuild only the dispatch plan (a6) with new options. */
+TC_API tc_status tc_replan(tc_graph* g, const tc_options* opts, void* stream);
+
+typedef struct {
+  int64_t n_input;          /* num_vertices as given / inferred                 */
+  int64_t n;                /* n': rows of the CSR (non-isolated vertices)      */
+  int64_t m;                /* unique undirected edges = oriented edges |E+|    */
+  int64_t max_out_degree;   /* max d+(u)                                        */
+  int64_t m_live;           /* oriented edges with non-empty work (plan units)  */
+  int64_t n_groups;         /* distinct middle vertices v with live edges       */
+  int64_t n_chunks;         /* work chunks of the count kernel                  */
+  int64_t keys_total;       /* sum of suffix lengths over live edges (probes)   */
+  uint64_t b_itc;           /* algorithmic bytes B_ITC         */
+  int64_t smem_bytes;       /* dynamic SMEM per CTA of the count kernel          */
+  int32_t count_grid;       /* CTAs the count kernel launches                    */
+  int32_t count_block;      /* threads per CTA                                   */
+  /* Borrowed device pointers, valid until tc_free: */
+  const int64_t* row_ptr;   /* int64[n+1], row offsets of the oriented CSR       */
+  const int32_t* col;       /* int32[m], each row strictly ascending, col > row  */
+  const int32_t* perm;      /* int32[n], new id -> original id                   */
+  /* Build phase times (ms, CUDA events on the build stream): */
+  float ms_canon, ms_sort_unique, ms_degree_rank, ms_orient_csr, ms_plan, ms_total;
+} tc_graph_info_t;
+
+TC_API tc_status tc_graph_info(const tc_graph* g, tc_graph_info_t* out);
+
+/* a7..a9.  T of the whole graph.  h_count: host uint64.  Synchronises. */
+TC_API tc_status tc_count(const tc_graph* g, void* stream, uint64_t* h_count);
+
+/* Stream-ordered variant: writes T into device uint64 *d_count (no sync). */
+TC_API tc_status tc_count_async(const tc_graph* g, void* stream, uint64_t* d_count);
+
+/*
+ * Partial count over the live oriented edges [e_begin, e_end) of the plan
+ * order (0 <= e_begin <= e_end <= m_live): writes sum_{e in range} |N+(u_e) ∩
+ * N+(v_e)| into device uint64 *d_partial (overwritten, not accumulated).
+ * Any cut of [0, m_live) into ranges gives partials summing to T (P:78:
+ * the per-edge intersections are independent).  No sync.
+ */
+TC_API tc_status tc_count_range(const tc_graph* g, int64_t e_begin, int64_t e_end, void* stream,
+                         uint64_t* d_partial);
+
+/*
+ * Cost-balanced split of [0, m_live) into world_size contiguous ranges
+ * (SURVEY.md §8(e)): h_bounds (host int64[world_size+1]) receives
+ * 0 = b_0 <= b_1 <= ... <= b_P = m_live, aligned to work chunks.
+ */
+TC_API tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds);
+
+/*
+ * Host-only form of the same split (no GPU needed; tested on CPU):
+ * given the exclusive cost prefix of `n_units` units (prefix[0] = 0,
+ * prefix[n_units] = total, non-decreasing), writes the unit bounds that cut
+ * the total cost into world_size near-equal contiguous parts.
+ */
+TC_API tc_status tc_partition_prefix(const int64_t* h_prefix, int64_t n_units, int32_t world_size,
+                              int64_t* h_bounds);
+
+/* Release a graph (NULL is a no-op).  Stream-ordered frees on the build stream. */
+TC_API void tc_free(tc_graph* g);
+
+/* Thread-local text for the last non-OK status of this thread. */
+TC_API const char* tc_last_error(void);
+
+/* Library version string, e.g. "b200tc 0.1 sm_100a". */
+TC_API const char* tc_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TC_H */

@@ -71,8 +71,53 @@ def lib():
         L.tco_count.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64,
                                 ctypes.c_int, ctypes.c_int, ctypes.c_int64, ctypes.POINTER(_Result)]
         L.tco_count.restype = ctypes.c_int
+        L.tco_build.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64,
+                                ctypes.c_int]
+        L.tco_build.restype = ctypes.c_void_p
+        L.tco_count_rows.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int64,
+                                     ctypes.c_int64, ctypes.POINTER(_Result)]
+        L.tco_count_rows.restype = ctypes.c_int
+        L.tco_free.argtypes = [ctypes.c_void_p]
+        L.tco_free.restype = None
         _lib = L
     return _lib
+
+
+def _wrap(r) -> OracleResult:
+    return OracleResult(int(r.triangles), int(r.m), int(r.n_active), int(r.max_out_degree),
+                        int(r.merge_steps_total), int(r.merge_steps_counted), float(r.build_ms),
+                        float(r.count_ms), int(r.threads), bool(r.sampled))
+
+
+class OracleGraph:
+    """Steps 1-4 done once (tco_build); count_rows() runs step 5 over all rows
+    or over the sampled rows x % stride == offset (bench reference leg)."""
+
+    def __init__(self, src, dst, n: int = -1, order: int = ORDER_DEGREE):
+        src = np.ascontiguousarray(src, dtype=np.int32)
+        dst = np.ascontiguousarray(dst, dtype=np.int32)
+        if src.shape != dst.shape:
+            raise ValueError("src and dst differ in length")
+        self._h = lib().tco_build(src.ctypes.data_as(ctypes.c_void_p),
+                                  dst.ctypes.data_as(ctypes.c_void_p), len(src), int(n),
+                                  int(order))
+        if not self._h:
+            raise ValueError("oracle: invalid input (vertex id out of range)")
+
+    def count_rows(self, threads: int = 0, stride: int = 1, offset: int = 0) -> OracleResult:
+        r = _Result()
+        if lib().tco_count_rows(self._h, int(threads), int(stride), int(offset),
+                                ctypes.byref(r)) != 0:
+            raise ValueError("oracle: bad arguments")
+        return _wrap(r)
+
+    def close(self):
+        if self._h:
+            lib().tco_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        self.close()
 
 
 def count(src, dst, n: int = -1, order: int = ORDER_DEGREE, threads: int = 0,
@@ -91,9 +136,7 @@ def count(src, dst, n: int = -1, order: int = ORDER_DEGREE, threads: int = 0,
                          ctypes.byref(r))
     if rc != 0:
         raise ValueError("oracle: invalid input (vertex id out of range)")
-    return OracleResult(int(r.triangles), int(r.m), int(r.n_active), int(r.max_out_degree),
-                        int(r.merge_steps_total), int(r.merge_steps_counted), float(r.build_ms),
-                        float(r.count_ms), int(r.threads), bool(r.sampled))
+    return _wrap(r)
 
 
 def triangles(src, dst, n: int = -1, **kw) -> int:

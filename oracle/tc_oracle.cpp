@@ -76,14 +76,19 @@ typedef struct {
   int32_t sampled;              // 1 when sample_stride > 1
 } tco_result;
 
-// Returns 0 on success, 1 on invalid argument (an id < 0 or >= n, null pointer).
-// n < 0 means "max id + 1".  order: 0 = (degree, id), 1 = id, 2 = (hash(id), id).
-// threads <= 0 means std::thread::hardware_concurrency().  sample_stride > 1
-// counts only rows x with x % sample_stride == 0 (bench cpu_baseline sampling).
-int tco_count(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t n, int order,
-              int threads, int64_t sample_stride, tco_result* out) {
-  if (!out || num_pairs < 0 || (num_pairs > 0 && (!src || !dst))) return 1;
-  std::memset(out, 0, sizeof(*out));
+struct tco_graph {
+  int64_t n = 0, m = 0, n_active = 0, max_out = 0;
+  std::vector<int64_t> off;  // row offsets of the oriented lists
+  std::vector<int32_t> adj;  // N+(x), ascending by id
+  double build_ms = 0;
+};
+
+// Steps 1-4.  Returns NULL on invalid argument (an id < 0 or >= n, null
+// pointer).  n < 0 means "max id + 1".  order: 0 = (degree, id), 1 = id,
+// 2 = (hash(id), id).
+tco_graph* tco_build(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t n,
+                     int order) {
+  if (num_pairs < 0 || (num_pairs > 0 && (!src || !dst))) return nullptr;
   auto t0 = std::chrono::steady_clock::now();
   if (n < 0) {
     int64_t mx = -1;
@@ -95,7 +100,7 @@ int tco_count(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t
   keys.reserve(num_pairs);
   for (int64_t i = 0; i < num_pairs; ++i) {
     int64_t a = src[i], b = dst[i];
-    if (a < 0 || b < 0 || a >= n || b >= n) return 1;
+    if (a < 0 || b < 0 || a >= n || b >= n) return nullptr;
     if (a == b) continue;
     uint64_t lo = (uint64_t)std::min(a, b), hi = (uint64_t)std::max(a, b);
     keys.push_back((lo << 32) | hi);
@@ -118,13 +123,16 @@ int tco_count(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t
     }
     return deg[x] != deg[y] ? deg[x] < deg[y] : x < y;
   };
-  std::vector<int64_t> off(n + 1, 0);
+  tco_graph* g = new tco_graph();
+  std::vector<int64_t>& off = g->off;
+  off.assign(n + 1, 0);
   for (uint64_t k : keys) {
     int64_t a = (int64_t)(k >> 32), b = (int64_t)(k & 0xffffffffu);
     ++off[(before(a, b) ? a : b) + 1];
   }
   for (int64_t x = 0; x < n; ++x) off[x + 1] += off[x];
-  std::vector<int32_t> adj(m);
+  std::vector<int32_t>& adj = g->adj;
+  adj.resize(m);
   {
     std::vector<int64_t> fill(off.begin(), off.end() - 1);
     for (uint64_t k : keys) {
@@ -139,7 +147,25 @@ int tco_count(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t
     max_out = std::max(max_out, off[x + 1] - off[x]);
     n_active += deg[x] > 0;
   }
-  out->build_ms = ms_since(t0);
+  g->n = n;
+  g->m = m;
+  g->n_active = n_active;
+  g->max_out = max_out;
+  g->build_ms = ms_since(t0);
+  return g;
+}
+
+void tco_free(tco_graph* g) { delete g; }
+
+// Step 5 over the rows x with x % sample_stride == sample_offset (all rows
+// when sample_stride <= 1).  threads <= 0 means hardware_concurrency().
+int tco_count_rows(const tco_graph* g, int threads, int64_t sample_stride, int64_t sample_offset,
+                   tco_result* out) {
+  if (!g || !out) return 1;
+  std::memset(out, 0, sizeof(*out));
+  const int64_t n = g->n;
+  const int64_t* off = g->off.data();
+  const int32_t* adj = g->adj.data();
   // 5. T = sum over oriented edges of |N+(x) ∩ N+(y)|, rows in dynamic chunks
   auto t1 = std::chrono::steady_clock::now();
   int nt = threads > 0 ? threads : (int)std::thread::hardware_concurrency();
@@ -154,12 +180,12 @@ int tco_count(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t
       if (b >= n) break;
       int64_t e = std::min(n, b + chunk);
       for (int64_t x = b; x < e; ++x) {
-        const int32_t* xb = adj.data() + off[x];
-        const int32_t* xe = adj.data() + off[x + 1];
-        bool counted = sample_stride <= 1 || x % sample_stride == 0;
+        const int32_t* xb = adj + off[x];
+        const int32_t* xe = adj + off[x + 1];
+        bool counted = sample_stride <= 1 || x % sample_stride == sample_offset;
         for (const int32_t* p = xb; p != xe; ++p) {
-          const int32_t* yb = adj.data() + off[*p];
-          const int32_t* ye = adj.data() + off[*p + 1];
+          const int32_t* yb = adj + off[*p];
+          const int32_t* ye = adj + off[*p + 1];
           uint64_t s = (uint64_t)(xe - xb) + (uint64_t)(ye - yb);
           all += s;
           if (!counted) continue;
@@ -183,12 +209,26 @@ int tco_count(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t
     out->merge_steps_total += part_all[w];
   }
   out->count_ms = ms_since(t1);
-  out->m = m;
-  out->n_active = n_active;
-  out->max_out_degree = max_out;
+  out->build_ms = g->build_ms;
+  out->m = g->m;
+  out->n_active = g->n_active;
+  out->max_out_degree = g->max_out;
   out->threads = nt;
   out->sampled = sample_stride > 1;
   return 0;
+}
+
+// Steps 1-5 in one call.  Returns 0 on success, 1 on invalid argument.
+// sample_stride > 1 counts only rows x with x % sample_stride == 0.
+int tco_count(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t n, int order,
+              int threads, int64_t sample_stride, tco_result* out) {
+  if (!out) return 1;
+  std::memset(out, 0, sizeof(*out));
+  tco_graph* g = tco_build(src, dst, num_pairs, n, order);
+  if (!g) return 1;
+  int rc = tco_count_rows(g, threads, sample_stride, 0, out);
+  tco_free(g);
+  return rc;
 }
 
 }  // extern "C"

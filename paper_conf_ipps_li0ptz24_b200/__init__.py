@@ -1,0 +1,317 @@
+"""b200tc — B200-native intersection-based triangle counting (ITC).
+
+Thin Python binding over the C-ABI in ``include/tc.h`` (``libtc.so``, built
+in-tree by ``make`` / ``__graft_entry__.build()``).  This module only
+marshals arguments: every step of the path (cleaning, orientation, CSR,
+plan, counting, reduction) runs in the library's sm_100a kernels.  PyTorch
+supplies device memory for the inputs, the current CUDA stream, and the
+process group of :func:`count_partitioned`.
+
+There is no CPU fallback: if ``libtc.so`` is missing or no CUDA device is
+present, the entry points raise.
+
+    g = build_csr(src, dst)          # torch int32 CUDA tensors (raw edge list)
+    t = g.count()                    # exact uint64 triangle count (int)
+    t = count_partitioned(g, group)  # torch.distributed over NCCL
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libtc.so")
+
+TC_OK, TC_ERR_INVALID_ARGUMENT, TC_ERR_OUT_OF_MEMORY, TC_ERR_CUDA, TC_ERR_UNSUPPORTED = range(5)
+TC_KEEP_ISOLATED = 0x1
+
+# Every symbol include/tc.h declares (tests check the library exports them).
+EXPORTS = (
+    "tc_set_allocator", "tc_build_csr", "tc_build_csr_host", "tc_replan", "tc_graph_info",
+    "tc_count", "tc_count_async", "tc_count_range", "tc_partition", "tc_partition_prefix",
+    "tc_free", "tc_last_error", "tc_version",
+)
+
+
+class TCError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"tc status {status}: {msg}")
+        self.status = status
+
+
+class InvalidArgument(TCError, ValueError):
+    pass
+
+
+class OutOfMemory(TCError, MemoryError):
+    pass
+
+
+class Options(ctypes.Structure):
+    """tc_options (0 = library default).  Performance knobs only: they never
+    change the count."""
+    _fields_ = [("chunk_cost", ctypes.c_int32), ("seg_cost", ctypes.c_int32),
+                ("huge_degree", ctypes.c_int32), ("block_threads", ctypes.c_int32),
+                ("hash_shift", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
+
+
+class GraphInfo(ctypes.Structure):
+    _fields_ = [("n_input", ctypes.c_int64), ("n", ctypes.c_int64), ("m", ctypes.c_int64),
+                ("max_out_degree", ctypes.c_int64), ("m_live", ctypes.c_int64),
+                ("n_groups", ctypes.c_int64), ("n_chunks", ctypes.c_int64),
+                ("keys_total", ctypes.c_int64), ("b_itc", ctypes.c_uint64),
+                ("smem_bytes", ctypes.c_int64), ("count_grid", ctypes.c_int32),
+                ("count_block", ctypes.c_int32), ("row_ptr", ctypes.c_void_p),
+                ("col", ctypes.c_void_p), ("perm", ctypes.c_void_p),
+                ("ms_canon", ctypes.c_float), ("ms_sort_unique", ctypes.c_float),
+                ("ms_degree_rank", ctypes.c_float), ("ms_orient_csr", ctypes.c_float),
+                ("ms_plan", ctypes.c_float), ("ms_total", ctypes.c_float)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_
+                if k not in ("row_ptr", "col", "perm")}
+
+
+_lib = None
+
+
+def lib():
+    """Load libtc.so (raises if it was not built — no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run `make` or __graft_entry__.build()")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, i64, i32, u32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint32
+        st = ctypes.c_int
+        sig = {
+            "tc_set_allocator": ([vp, vp, vp], st),
+            "tc_build_csr": ([vp, vp, i64, i64, u32, vp, vp, ctypes.POINTER(vp)], st),
+            "tc_build_csr_host": ([vp, vp, i64, i64, u32, vp, vp, ctypes.POINTER(vp)], st),
+            "tc_replan": ([vp, vp, vp], st),
+            "tc_graph_info": ([vp, ctypes.POINTER(GraphInfo)], st),
+            "tc_count": ([vp, vp, ctypes.POINTER(ctypes.c_uint64)], st),
+            "tc_count_async": ([vp, vp, vp], st),
+            "tc_count_range": ([vp, i64, i64, vp, vp], st),
+            "tc_partition": ([vp, i32, vp], st),
+            "tc_partition_prefix": ([vp, i64, i32, vp], st),
+            "tc_free": ([vp], None),
+            "tc_last_error": ([], ctypes.c_char_p),
+            "tc_version": ([], ctypes.c_char_p),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = res
+        _lib = L
+    return _lib
+
+
+def _check(status: int):
+    if status == TC_OK:
+        return
+    msg = lib().tc_last_error().decode(errors="replace")
+    if status == TC_ERR_INVALID_ARGUMENT:
+        raise InvalidArgument(status, msg)
+    if status == TC_ERR_OUT_OF_MEMORY:
+        raise OutOfMemory(status, msg)
+    raise TCError(status, msg)
+
+
+def version() -> str:
+    return lib().tc_version().decode()
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _stream(stream=None) -> int:
+    torch = _torch()
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return int(stream.cuda_stream)
+
+
+def _options(opts):
+    """tc_options* for the C call (None = defaults)."""
+    if opts is None:
+        return None
+    if not isinstance(opts, Options):
+        o = Options()
+        for k, v in dict(opts).items():
+            setattr(o, k, int(v))
+        opts = o
+    return ctypes.byref(opts)
+
+
+class _DevArray:
+    """Borrowed device array exposed through __cuda_array_interface__."""
+
+    def __init__(self, ptr: int, n: int, typestr: str, owner):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr,
+                                         "data": (ptr or 0, True), "version": 3}
+        self._owner = owner
+
+
+class Graph:
+    """An oriented CSR + dispatch plan living on one GPU (owns a tc_graph*)."""
+
+    def __init__(self, handle: int):
+        self._h = ctypes.c_void_p(handle)
+        self.info = self._info()
+
+    # ------------------------------------------------------------ info
+    def _info(self) -> GraphInfo:
+        gi = GraphInfo()
+        _check(lib().tc_graph_info(self._h, ctypes.byref(gi)))
+        return gi
+
+    @property
+    def n(self) -> int:
+        return int(self.info.n)
+
+    @property
+    def m(self) -> int:
+        return int(self.info.m)
+
+    @property
+    def m_live(self) -> int:
+        return int(self.info.m_live)
+
+    def csr(self):
+        """(row_ptr int64[n+1], col int32[m], perm int32[n]) as borrowed CUDA tensors."""
+        torch = _torch()
+        gi = self.info
+        rp = torch.as_tensor(_DevArray(gi.row_ptr, gi.n + 1, "<i8", self), device="cuda")
+        col = torch.as_tensor(_DevArray(gi.col, gi.m, "<i4", self), device="cuda")
+        perm = torch.as_tensor(_DevArray(gi.perm, gi.n, "<i4", self), device="cuda")
+        return rp, col, perm
+
+    # ------------------------------------------------------------ counting
+    def count(self, stream=None) -> int:
+        """T (exact; synchronises the stream)."""
+        out = ctypes.c_uint64(0)
+        _check(lib().tc_count(self._h, ctypes.c_void_p(_stream(stream)), ctypes.byref(out)))
+        return int(out.value)
+
+    def count_async(self, out=None, stream=None):
+        """Stream-ordered T into a 1-element int64 CUDA tensor (u64 bit pattern)."""
+        torch = _torch()
+        if out is None:
+            out = torch.empty(1, dtype=torch.int64, device="cuda")
+        _check(lib().tc_count_async(self._h, ctypes.c_void_p(_stream(stream)),
+                                    ctypes.c_void_p(out.data_ptr())))
+        return out
+
+    def count_range(self, e_begin: int, e_end: int, out=None, stream=None):
+        """Partial count of live oriented edges [e_begin, e_end) (plan order)."""
+        torch = _torch()
+        if out is None:
+            out = torch.empty(1, dtype=torch.int64, device="cuda")
+        _check(lib().tc_count_range(self._h, int(e_begin), int(e_end),
+                                    ctypes.c_void_p(_stream(stream)),
+                                    ctypes.c_void_p(out.data_ptr())))
+        return out
+
+    def partition(self, world_size: int) -> list:
+        b = np.zeros(int(world_size) + 1, dtype=np.int64)
+        _check(lib().tc_partition(self._h, int(world_size), b.ctypes.data_as(ctypes.c_void_p)))
+        return [int(x) for x in b]
+
+    def replan(self, options=None, stream=None):
+        _check(lib().tc_replan(self._h, _options(options), ctypes.c_void_p(_stream(stream))))
+        self.info = self._info()
+
+    # ------------------------------------------------------------ lifetime
+    def close(self):
+        if self._h is not None and self._h.value:
+            lib().tc_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+
+def build_csr(src, dst, num_vertices: Optional[int] = None, keep_isolated: bool = False,
+              options=None, stream=None) -> Graph:
+    """a1..a6 from a raw device edge list (torch int32 CUDA tensors of equal length)."""
+    torch = _torch()
+    if src.shape != dst.shape or src.dim() != 1:
+        raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, "src/dst must be 1-D of equal length")
+    if src.dtype != torch.int32 or dst.dtype != torch.int32 or not src.is_cuda or not dst.is_cuda:
+        raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, "src/dst must be int32 CUDA tensors")
+    src, dst = src.contiguous(), dst.contiguous()
+    h = ctypes.c_void_p(0)
+    _check(lib().tc_build_csr(ctypes.c_void_p(src.data_ptr()), ctypes.c_void_p(dst.data_ptr()),
+                              int(src.numel()), -1 if num_vertices is None else int(num_vertices),
+                              TC_KEEP_ISOLATED if keep_isolated else 0, _options(options),
+                              ctypes.c_void_p(_stream(stream)), ctypes.byref(h)))
+    return Graph(h.value)
+
+
+def build_csr_host(src: np.ndarray, dst: np.ndarray, num_vertices: Optional[int] = None,
+                   keep_isolated: bool = False, options=None, stream=None) -> Graph:
+    """Same from host int32 arrays (numpy, or pinned torch CPU tensors): the
+    library performs the host->device copy on the stream."""
+    def ptr(a):
+        if hasattr(a, "data_ptr"):
+            return a.data_ptr(), a.numel()
+        a = np.ascontiguousarray(a, dtype=np.int32)
+        return a.ctypes.data, a.size
+    ps, ns = ptr(src)
+    pd, nd = ptr(dst)
+    if ns != nd:
+        raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, "src/dst differ in length")
+    h = ctypes.c_void_p(0)
+    _check(lib().tc_build_csr_host(ctypes.c_void_p(ps), ctypes.c_void_p(pd), int(ns),
+                                   -1 if num_vertices is None else int(num_vertices),
+                                   TC_KEEP_ISOLATED if keep_isolated else 0, _options(options),
+                                   ctypes.c_void_p(_stream(stream)), ctypes.byref(h)))
+    return Graph(h.value)
+
+
+def partition_prefix(prefix: Sequence[int], world_size: int) -> list:
+    """Host-only cost split (tc_partition_prefix): unit bounds cutting the
+    exclusive cost prefix into world_size near-equal contiguous parts."""
+    p = np.ascontiguousarray(prefix, dtype=np.int64)
+    b = np.zeros(int(world_size) + 1, dtype=np.int64)
+    _check(lib().tc_partition_prefix(p.ctypes.data_as(ctypes.c_void_p), len(p) - 1,
+                                     int(world_size), b.ctypes.data_as(ctypes.c_void_p)))
+    return [int(x) for x in b]
+
+
+def count_partitioned(graph, group=None, stream=None) -> int:
+    """T over a torch.distributed process group.
+
+    Every rank holds the same replicated graph; rank r counts the live
+    oriented edges [b_r, b_{r+1}) of tc_partition's cost-balanced split and a
+    single all_reduce(SUM) of the 8-byte partials (ProcessGroupNCCL over
+    NVLink on the GPU box) gives T on every rank.  Two's-complement int64
+    addition is bit-identical to uint64 addition mod 2^64.
+    """
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    bounds = graph.partition(world)
+    partial = graph.count_range(bounds[rank], bounds[rank + 1], stream=stream)
+    dist.all_reduce(partial, op=dist.ReduceOp.SUM, group=group)
+    return int(partial.item()) & (2**64 - 1)
+
+
+__all__ = ["Graph", "Options", "GraphInfo", "build_csr", "build_csr_host", "count_partitioned",
+           "partition_prefix", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
+           "EXPORTS", "LIB_PATH"]

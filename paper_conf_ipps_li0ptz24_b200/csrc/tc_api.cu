@@ -1,0 +1,320 @@
+// tc_api.cu — the C-ABI boundary (include/tc.h).  Argument checking, error
+// translation (no exception crosses the ABI), the allocator hook, and the
+// host-side range/partition logic.  SURVEY.md §8(b).
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+#include "tc_internal.cuh"
+
+namespace {
+thread_local std::string t_last_error;
+
+tc_alloc_fn g_alloc = nullptr;
+tc_free_fn g_free = nullptr;
+void* g_ctx = nullptr;
+
+template <class F>
+tc_status guarded(F f) {
+  try {
+    f();
+    return TC_OK;
+  } catch (const tc::Error& e) {
+    t_last_error = e.msg;
+    return e.status;
+  } catch (const std::bad_alloc&) {
+    t_last_error = "host allocation failed";
+    return TC_ERR_OUT_OF_MEMORY;
+  } catch (...) {
+    t_last_error = "unexpected internal error";
+    return TC_ERR_CUDA;
+  }
+}
+
+void require(bool ok, const char* msg) {
+  if (!ok) tc::fail(TC_ERR_INVALID_ARGUMENT, msg);
+}
+
+}  // namespace
+
+namespace tc {
+
+void fail(tc_status s, const std::string& msg) { throw Error{s, msg}; }
+
+void check_cuda(cudaError_t e, const char* what, const char* file, int line) {
+  if (e == cudaSuccess) return;
+  if (e == cudaErrorMemoryAllocation) {
+    cudaGetLastError();
+    fail(TC_ERR_OUT_OF_MEMORY, std::string("CUDA out of memory in ") + what);
+  }
+  char buf[512];
+  snprintf(buf, sizeof(buf), "%s: %s (%s:%d)", what, cudaGetErrorString(e), file, line);
+  fail(TC_ERR_CUDA, buf);
+}
+
+void* dev_alloc(size_t bytes, cudaStream_t s) {
+  void* p = nullptr;
+  if (g_alloc) {
+    p = g_alloc(bytes, (void*)s, g_ctx);
+    if (!p) fail(TC_ERR_OUT_OF_MEMORY, "allocator hook returned NULL");
+    return p;
+  }
+  static bool pool_ready = false;
+  if (!pool_ready) {
+    // Keep freed blocks in the device pool across syncs: without this every
+    // build re-maps its scratch (tens of ms at config C2).
+    int dev = 0;
+    cudaMemPool_t pool;
+    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    cudaGetLastError();
+    pool_ready = true;
+  }
+  cudaError_t e = cudaMallocAsync(&p, bytes, s);
+  if (e != cudaSuccess || !p) {
+    cudaGetLastError();
+    fail(TC_ERR_OUT_OF_MEMORY, "cudaMallocAsync failed (" + std::to_string(bytes) + " bytes)");
+  }
+  return p;
+}
+
+void dev_free(void* p, size_t bytes, cudaStream_t s) {
+  if (!p) return;
+  if (g_free) {
+    g_free(p, bytes, (void*)s, g_ctx);
+    return;
+  }
+  cudaFreeAsync(p, s);
+}
+
+Options resolve_options(const tc_options* o) {
+  Options r;
+  if (!o) return r;
+  if (o->chunk_cost) r.chunk_cost = o->chunk_cost;
+  if (o->seg_cost) r.seg_cost = o->seg_cost;
+  if (o->huge_degree) r.huge_degree = o->huge_degree;
+  if (o->block_threads) r.block_threads = o->block_threads;
+  if (o->hash_shift) r.hash_shift = o->hash_shift;
+  require(r.chunk_cost >= 64, "chunk_cost must be >= 64");
+  require(r.seg_cost >= 1, "seg_cost must be >= 1");
+  require(r.huge_degree >= 1, "huge_degree must be >= 1");
+  require(r.block_threads >= 64 && r.block_threads <= 512 && r.block_threads % 32 == 0,
+          "block_threads must be a multiple of 32 in [64, 512]");
+  require(r.hash_shift >= 0 && r.hash_shift <= 4, "hash_shift must be in [0, 4]");
+  return r;
+}
+
+}  // namespace tc
+
+namespace {
+
+// Rebinds every stream-ordered buffer of the graph to `s` so frees are
+// ordered after the work that used them.
+void rebind(tc_graph* g, cudaStream_t s) {
+  g->row_ptr.s = g->col.s = g->perm.s = s;
+  tc::Plan& P = g->plan;
+  P.key_prefix.s = P.seg_base.s = P.ins_prefix.s = P.grp_ibase.s = P.slot_prefix.s =
+      P.chunk_seg.s = s;
+  P.seg_group.s = P.grp_tmax.s = s;
+}
+
+tc_status build_impl(const int32_t* src, const int32_t* dst, int64_t num_edges,
+                     int64_t num_vertices, uint32_t flags, const tc_options* opts, void* stream,
+                     tc_graph** out, bool host) {
+  if (out) *out = nullptr;
+  tc_graph* g = nullptr;
+  tc_status st = guarded([&] {
+    require(out != nullptr, "out is NULL");
+    require(num_edges >= 0, "num_edges < 0");
+    require(num_edges == 0 || (src && dst), "src/dst is NULL");
+    require(num_vertices >= -1 && num_vertices <= 0x7fffffffLL,
+            "num_vertices must be -1 or in [0, 2^31-1]");
+    require((flags & ~TC_KEEP_ISOLATED) == 0, "unknown flag bits");
+    const tc::Options opt = tc::resolve_options(opts);
+    cudaStream_t s = (cudaStream_t)stream;
+    g = new tc_graph();
+    if (host) {
+      tc::DevBuf<int32_t> ds(std::max<int64_t>(num_edges, 1), s), dd(std::max<int64_t>(num_edges, 1), s);
+      if (num_edges) {
+        TC_CUDA(cudaMemcpyAsync(ds.get(), src, sizeof(int32_t) * num_edges,
+                                cudaMemcpyHostToDevice, s));
+        TC_CUDA(cudaMemcpyAsync(dd.get(), dst, sizeof(int32_t) * num_edges,
+                                cudaMemcpyHostToDevice, s));
+      }
+      tc::build_graph(ds.get(), dd.get(), num_edges, num_vertices, flags, opt, s, g);
+    } else {
+      tc::build_graph(src, dst, num_edges, num_vertices, flags, opt, s, g);
+    }
+  });
+  if (st != TC_OK) {
+    if (g) {
+      cudaStreamSynchronize((cudaStream_t)stream);
+      delete g;
+    }
+    return st;
+  }
+  *out = g;
+  return TC_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+tc_status tc_set_allocator(tc_alloc_fn alloc, tc_free_fn free_fn, void* ctx) {
+  if ((alloc == nullptr) != (free_fn == nullptr)) {
+    t_last_error = "alloc and free hooks must both be set or both be NULL";
+    return TC_ERR_INVALID_ARGUMENT;
+  }
+  g_alloc = alloc;
+  g_free = free_fn;
+  g_ctx = ctx;
+  return TC_OK;
+}
+
+tc_status tc_build_csr(const int32_t* d_src, const int32_t* d_dst, int64_t num_edges,
+                       int64_t num_vertices, uint32_t flags, const tc_options* opts,
+                       void* stream, tc_graph** out) {
+  return build_impl(d_src, d_dst, num_edges, num_vertices, flags, opts, stream, out, false);
+}
+
+tc_status tc_build_csr_host(const int32_t* h_src, const int32_t* h_dst, int64_t num_edges,
+                            int64_t num_vertices, uint32_t flags, const tc_options* opts,
+                            void* stream, tc_graph** out) {
+  return build_impl(h_src, h_dst, num_edges, num_vertices, flags, opts, stream, out, true);
+}
+
+tc_status tc_replan(tc_graph* g, const tc_options* opts, void* stream) {
+  return guarded([&] {
+    require(g != nullptr, "graph is NULL");
+    const tc::Options opt = tc::resolve_options(opts);
+    cudaStream_t s = (cudaStream_t)stream;
+    TC_CUDA(cudaStreamSynchronize(s));
+    rebind(g, s);
+    tc::build_plan(g, opt, s);
+    TC_CUDA(cudaStreamSynchronize(s));
+  });
+}
+
+tc_status tc_graph_info(const tc_graph* g, tc_graph_info_t* o) {
+  return guarded([&] {
+    require(g && o, "NULL argument");
+    std::memset(o, 0, sizeof(*o));
+    const tc::Plan& P = g->plan;
+    o->n_input = g->n_input;
+    o->n = g->n;
+    o->m = g->m;
+    o->max_out_degree = g->max_out;
+    o->m_live = P.S;
+    o->n_groups = P.G;
+    o->n_chunks = P.n_chunks;
+    o->keys_total = P.keys_total;
+    o->b_itc = g->b_itc;
+    o->smem_bytes = P.smem_bytes;
+    o->count_grid = P.grid;
+    o->count_block = P.block;
+    o->row_ptr = g->row_ptr.get();
+    o->col = g->col.get();
+    o->perm = g->perm.get();
+    o->ms_canon = g->ms[0];
+    o->ms_sort_unique = g->ms[1];
+    o->ms_degree_rank = g->ms[2];
+    o->ms_orient_csr = g->ms[3];
+    o->ms_plan = g->ms[4];
+    o->ms_total = g->ms[5];
+  });
+}
+
+tc_status tc_count_async(const tc_graph* g, void* stream, uint64_t* d_count) {
+  return guarded([&] {
+    require(g && d_count, "NULL argument");
+    tc::count_chunks(g, 0, g->plan.n_chunks, 0, g->plan.S, (cudaStream_t)stream,
+                     reinterpret_cast<unsigned long long*>(d_count));
+  });
+}
+
+tc_status tc_count(const tc_graph* g, void* stream, uint64_t* h_count) {
+  return guarded([&] {
+    require(g && h_count, "NULL argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    tc::DevBuf<unsigned long long> d(1, s);
+    tc::count_chunks(g, 0, g->plan.n_chunks, 0, g->plan.S, s, d.get());
+    unsigned long long h = 0;
+    TC_CUDA(cudaMemcpyAsync(&h, d.get(), sizeof(h), cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaStreamSynchronize(s));
+    *h_count = h;
+  });
+}
+
+tc_status tc_count_range(const tc_graph* g, int64_t e_begin, int64_t e_end, void* stream,
+                         uint64_t* d_partial) {
+  return guarded([&] {
+    require(g && d_partial, "NULL argument");
+    const tc::Plan& P = g->plan;
+    require(0 <= e_begin && e_begin <= e_end && e_end <= P.S,
+            "need 0 <= e_begin <= e_end <= m_live");
+    const auto& cs = P.h_chunk_seg;
+    // first chunk whose end is > e_begin, last chunk whose start is < e_end
+    int64_t c_begin = 0, c_end = 0;
+    if (e_end > e_begin) {
+      c_begin = std::upper_bound(cs.begin(), cs.end(), e_begin) - cs.begin() - 1;
+      c_end = std::lower_bound(cs.begin(), cs.end(), e_end) - cs.begin();
+      c_begin = std::max<int64_t>(c_begin, 0);
+      c_end = std::min<int64_t>(c_end, P.n_chunks);
+    }
+    tc::count_chunks(g, c_begin, c_end, e_begin, e_end, (cudaStream_t)stream,
+                     reinterpret_cast<unsigned long long*>(d_partial));
+  });
+}
+
+tc_status tc_partition_prefix(const int64_t* h_prefix, int64_t n_units, int32_t world_size,
+                              int64_t* h_bounds) {
+  return guarded([&] {
+    require(h_prefix && h_bounds, "NULL argument");
+    require(n_units >= 0, "n_units < 0");
+    require(world_size >= 1, "world_size < 1");
+    const int64_t total = h_prefix[n_units];
+    h_bounds[0] = 0;
+    for (int32_t r = 1; r < world_size; ++r) {
+      // first unit whose exclusive prefix reaches r/world of the total cost
+      const long double t = (long double)total * r / world_size;
+      const int64_t* it = std::lower_bound(h_prefix, h_prefix + n_units + 1, t,
+                                           [](int64_t a, long double b) { return (long double)a < b; });
+      int64_t b = it - h_prefix;
+      b = std::min(std::max(b, h_bounds[r - 1]), n_units);
+      h_bounds[r] = b;
+    }
+    h_bounds[world_size] = n_units;
+  });
+}
+
+tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds) {
+  return guarded([&] {
+    require(g && h_bounds, "NULL argument");
+    require(world_size >= 1, "world_size < 1");
+    const tc::Plan& P = g->plan;
+    // Chunks carry near-equal cost (a6), so a split by chunk count is a
+    // split by cost; bounds are the chunks' first live edges.
+    const int64_t nc = P.n_chunks;
+    for (int32_t r = 0; r <= world_size; ++r) {
+      const int64_t c = nc * r / world_size;
+      h_bounds[r] = (r == world_size) ? P.S : P.h_chunk_seg[c];
+    }
+  });
+}
+
+void tc_free(tc_graph* g) {
+  if (!g) return;
+  cudaDeviceSynchronize();
+  rebind(g, nullptr);
+  delete g;
+}
+
+const char* tc_last_error(void) { return t_last_error.c_str(); }
+
+const char* tc_version(void) { return "b200tc 0.1 sm_100a"; }
+
+}  // extern "C"

@@ -1,0 +1,640 @@
+// tc_build.cu — preprocessing: SURVEY.md §8(a) rows a1..a6 on the GPU.
+//
+//   a1 validate + canonicalise + drop self-loops
+//   a2 radix sort + unique                          ("resolving duplicate edges")
+//   a3 undirected degree                            (P:108 degree ordering)
+//   a4 rank by (degree, id), relabel, drop isolated ("u < v")
+//   a5 orient u -> v iff rank u < rank v, CSR
+//   a6 dispatch plan (live edges grouped by head v, hash sizes, cost chunks)
+//
+// Every pass is a streaming integer pass (HBM bound); the sorts are CUB's
+// onesweep radix sort on the minimal bit width (2*ceil(log2 n) bits).  The
+// only host round trips are the counts that size the next allocation.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+
+#include "tc_internal.cuh"
+
+namespace tc {
+namespace {
+
+constexpr int TPB = 256;
+
+unsigned grid_for(int64_t n) {
+  int64_t b = (n + TPB - 1) / TPB;
+  return (unsigned)std::max<int64_t>(1, std::min<int64_t>(b, 148 * 32));
+}
+
+int bits_for(int64_t n) {  // bits so that every id in [0, n) fits
+  int b = 1;
+  while ((int64_t(1) << b) < n) ++b;
+  return b;
+}
+
+template <class F>
+void cub_run(cudaStream_t s, F f) {
+  size_t bytes = 0;
+  TC_CUDA(f(nullptr, bytes));
+  DevBuf<char> tmp(bytes ? bytes : 16, s);
+  TC_CUDA(f(tmp.get(), bytes));
+}
+
+template <class T>
+T d2h(const T* d, cudaStream_t s) {
+  T h;
+  TC_CUDA(cudaMemcpyAsync(&h, d, sizeof(T), cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  return h;
+}
+
+// ------------------------------------------------------------------ a1
+// key = (min << bits) | max for a valid non-loop pair, SENT otherwise.
+__global__ void k_canon(const int32_t* __restrict__ src, const int32_t* __restrict__ dst,
+                        int64_t m, int64_t n, int bits, uint64_t sent,
+                        uint64_t* __restrict__ key, int* __restrict__ err) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t a = src[i], b = dst[i];
+    uint64_t k = sent;
+    if (a < 0 || b < 0 || a >= n || b >= n) {
+      *err = 1;
+    } else if (a != b) {
+      uint64_t lo = (uint64_t)min(a, b), hi = (uint64_t)max(a, b);
+      k = (lo << bits) | hi;
+    }
+    key[i] = k;
+  }
+}
+
+// {err, n_selected, last key} for the single host round trip after a2.
+struct UniqTail {
+  int err;
+  int pad;
+  int64_t nsel;
+  uint64_t last;
+};
+__global__ void k_uniq_tail(const int* err, const int64_t* nsel, const uint64_t* keys,
+                            UniqTail* out) {
+  out->err = *err;
+  out->nsel = *nsel;
+  out->last = *nsel > 0 ? keys[*nsel - 1] : 0;
+}
+
+// ------------------------------------------------------------------ a3
+__global__ void k_degree(const uint64_t* __restrict__ key, int64_t m, int bits,
+                         int32_t* __restrict__ deg) {
+  const uint64_t mask = (uint64_t(1) << bits) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t k = key[i];
+    atomicAdd(&deg[k >> bits], 1);
+    atomicAdd(&deg[k & mask], 1);
+  }
+}
+
+// ------------------------------------------------------------------ a4
+// vertex key = (deg << bits) | v; isolated vertices get SENTV (sorted last)
+// unless TC_KEEP_ISOLATED.  Counts the kept vertices into *n_act.
+__global__ void k_vkey(const int32_t* __restrict__ deg, int64_t n, int bits, int keep,
+                       uint64_t sentv, uint64_t* __restrict__ vkey,
+                       unsigned long long* __restrict__ n_act) {
+  for (int64_t base = blockIdx.x * (int64_t)blockDim.x; base < n;
+       base += (int64_t)gridDim.x * blockDim.x) {
+    int64_t v = base + threadIdx.x;
+    int act = 0;
+    if (v < n) {
+      int64_t d = deg[v];
+      act = keep || d > 0;
+      vkey[v] = act ? (((uint64_t)d << bits) | (uint64_t)v) : sentv;
+    }
+    int c = __syncthreads_count(act);
+    if (threadIdx.x == 0 && c) atomicAdd(n_act, (unsigned long long)c);
+  }
+}
+
+__global__ void k_perm(const uint64_t* __restrict__ vkey, int64_t n_act, int bits,
+                       int32_t* __restrict__ perm, int32_t* __restrict__ rank) {
+  const uint64_t mask = (uint64_t(1) << bits) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_act;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t v = (int32_t)(vkey[i] & mask);
+    perm[i] = v;
+    rank[v] = (int32_t)i;
+  }
+}
+
+// ------------------------------------------------------------------ a5
+__global__ void k_orient(const uint64_t* __restrict__ key, int64_t m, int bits,
+                         const int32_t* __restrict__ rank, int bits2,
+                         uint64_t* __restrict__ okey) {
+  const uint64_t mask = (uint64_t(1) << bits) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t k = key[i];
+    uint64_t ra = (uint64_t)rank[k >> bits], rb = (uint64_t)rank[k & mask];
+    okey[i] = ra < rb ? ((ra << bits2) | rb) : ((rb << bits2) | ra);
+  }
+}
+
+__global__ void k_csr(const uint64_t* __restrict__ okey, int64_t m, int64_t n, int bits2,
+                      int32_t* __restrict__ col, int64_t* __restrict__ row_ptr) {
+  const uint64_t mask = (uint64_t(1) << bits2) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t k = okey[i];
+    int64_t u = (int64_t)(k >> bits2);
+    col[i] = (int32_t)(k & mask);
+    int64_t prev = i ? (int64_t)(okey[i - 1] >> bits2) : -1;
+    for (int64_t x = prev + 1; x <= u; ++x) row_ptr[x] = i;
+    if (i == m - 1)
+      for (int64_t x = u + 1; x <= n; ++x) row_ptr[x] = m;
+  }
+}
+
+__global__ void k_fill_i64(int64_t* p, int64_t n, int64_t v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    p[i] = v;
+}
+
+__global__ void k_max_outdeg(const int64_t* __restrict__ row_ptr, int64_t n,
+                             unsigned long long* out) {
+  typedef cub::BlockReduce<unsigned long long, TPB> BR;
+  __shared__ typename BR::TempStorage tmp;
+  unsigned long long mx = 0;
+  for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n;
+       u += (int64_t)gridDim.x * blockDim.x)
+    mx = max(mx, (unsigned long long)(row_ptr[u + 1] - row_ptr[u]));
+  unsigned long long r = BR(tmp).Reduce(mx, cub::Max());
+  if (threadIdx.x == 0) atomicMax(out, r);
+}
+
+// ------------------------------------------------------------------ a6
+__global__ void k_rowid(const int64_t* __restrict__ row_ptr, int64_t n,
+                        int32_t* __restrict__ rowid) {
+  for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n;
+       u += (int64_t)gridDim.x * blockDim.x)
+    for (int64_t p = row_ptr[u], e = row_ptr[u + 1]; p < e; ++p) rowid[p] = (int32_t)u;
+}
+
+// Per oriented edge p = (u, v): suffix length suf = row_end(u) - p - 1,
+// live iff suf > 0 and d+(v) > 0 (C-12 exact skips).  Accumulates
+// stats[0] = B_ITC edge part, stats[1] = sum of live suffixes, stats[2] = live count.
+__global__ void k_edge_stats(const int64_t* __restrict__ row_ptr,
+                             const int32_t* __restrict__ col,
+                             const int32_t* __restrict__ rowid, int64_t m,
+                             uint8_t* __restrict__ live, unsigned long long* stats) {
+  typedef cub::BlockReduce<unsigned long long, TPB> BR;
+  __shared__ typename BR::TempStorage tmp;
+  unsigned long long b = 0, keys = 0, nl = 0;
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < m;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    int32_t u = rowid[p], v = col[p];
+    int64_t suf = row_ptr[u + 1] - p - 1;
+    int64_t dv = row_ptr[v + 1] - row_ptr[v];
+    bool l = suf > 0 && dv > 0;
+    live[p] = l;
+    b += 4ull * (unsigned long long)(suf + dv) + 12ull;
+    if (l) {
+      keys += (unsigned long long)suf;
+      ++nl;
+    }
+  }
+  unsigned long long r0 = BR(tmp).Sum(b);
+  __syncthreads();
+  unsigned long long r1 = BR(tmp).Sum(keys);
+  __syncthreads();
+  unsigned long long r2 = BR(tmp).Sum(nl);
+  if (threadIdx.x == 0) {
+    atomicAdd(&stats[0], r0);
+    atomicAdd(&stats[1], r1);
+    atomicAdd(&stats[2], r2);
+  }
+}
+
+__global__ void k_gather_head(const int64_t* __restrict__ p_live, int64_t S,
+                              const int32_t* __restrict__ col, uint32_t* __restrict__ vkey) {
+  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
+       s += (int64_t)gridDim.x * blockDim.x)
+    vkey[s] = (uint32_t)col[p_live[s]];
+}
+
+__global__ void k_group_mark(const uint32_t* __restrict__ vkey, int64_t S,
+                             int32_t* __restrict__ mark) {
+  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
+       s += (int64_t)gridDim.x * blockDim.x)
+    mark[s] = (s == 0 || vkey[s] != vkey[s - 1]) ? 1 : 0;
+}
+
+// Per segment: length, group id; per group (at its first segment): table facts.
+__global__ void k_seg_group(const uint32_t* __restrict__ vkey, const int64_t* __restrict__ p_s,
+                            const int32_t* __restrict__ gincl, int64_t S,
+                            const int64_t* __restrict__ row_ptr,
+                            const int32_t* __restrict__ col,
+                            const int32_t* __restrict__ rowid, int huge_degree,
+                            int hash_shift, int32_t* __restrict__ seg_group,
+                            int64_t* __restrict__ seg_len, int64_t* __restrict__ grp_row,
+                            int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots,
+                            int32_t* __restrict__ grp_tmax) {
+  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
+       s += (int64_t)gridDim.x * blockDim.x) {
+    int64_t p = p_s[s];
+    int32_t g = gincl[s] - 1;
+    seg_group[s] = g;
+    seg_len[s] = row_ptr[rowid[p] + 1] - p - 1;
+    if (s == 0 || vkey[s] != vkey[s - 1]) {
+      int64_t v = vkey[s];
+      int64_t rs = row_ptr[v], d = row_ptr[v + 1] - rs;
+      grp_row[g] = rs;
+      grp_d[g] = d;
+      int64_t slots = 0;
+      if (d <= huge_degree) {
+        // > d slots so a probe for an absent key always meets an empty slot
+        int64_t want = d << hash_shift;
+        if (want < d + 1) want = d + 1;
+        slots = 1;
+        while (slots < want) slots <<= 1;
+      }
+      grp_slots[g] = slots;
+      grp_tmax[g] = col[rs + d - 1];
+    }
+  }
+}
+
+__global__ void k_seg_base_cost(const int64_t* __restrict__ p_s,
+                                const int64_t* __restrict__ key_prefix,
+                                const int64_t* __restrict__ seg_len,
+                                const int32_t* __restrict__ seg_group,
+                                const int64_t* __restrict__ grp_d,
+                                const int64_t* __restrict__ grp_slots, int64_t S, int seg_cost,
+                                int64_t* __restrict__ seg_base, int64_t* __restrict__ cost) {
+  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
+       s += (int64_t)gridDim.x * blockDim.x) {
+    seg_base[s] = p_s[s] + 1 - key_prefix[s];
+    int32_t g = seg_group[s];
+    int64_t c = seg_cost + seg_len[s];
+    if (s == 0 || seg_group[s - 1] != g) c += grp_d[g] + grp_slots[g];
+    cost[s] = c;
+  }
+}
+
+__global__ void k_grp_ibase(const int64_t* __restrict__ grp_row,
+                            const int64_t* __restrict__ ins_prefix, int64_t G,
+                            int64_t* __restrict__ ibase) {
+  for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < G;
+       g += (int64_t)gridDim.x * blockDim.x)
+    ibase[g] = grp_row[g] - ins_prefix[g];
+}
+
+// chunk_seg[c] = first segment whose exclusive cost prefix is >= c * C.
+__global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t S,
+                               int64_t n_chunks, int64_t C, int64_t* __restrict__ chunk_seg) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= n_chunks;
+       c += (int64_t)gridDim.x * blockDim.x) {
+    if (c == n_chunks) {
+      chunk_seg[c] = S;
+      continue;
+    }
+    int64_t target = c * C, lo = 0, hi = S;  // first s in [0, S] with prefix[s] >= target
+    while (lo < hi) {
+      int64_t mid = (lo + hi) >> 1;
+      if (cost_prefix[mid] < target) lo = mid + 1; else hi = mid;
+    }
+    chunk_seg[c] = lo;
+  }
+}
+
+// SMEM a chunk needs in the count kernel: 8 B of table info per group plus
+// 4 B per hash slot (must match the layout in tc_count.cu).
+__global__ void k_chunk_smem(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
+                             const int32_t* __restrict__ seg_group,
+                             const int64_t* __restrict__ slot_prefix,
+                             unsigned long long* out) {
+  typedef cub::BlockReduce<unsigned long long, TPB> BR;
+  __shared__ typename BR::TempStorage tmp;
+  unsigned long long mx = 0;
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n_chunks;
+       c += (int64_t)gridDim.x * blockDim.x) {
+    int64_t sa = chunk_seg[c], sb = chunk_seg[c + 1];
+    if (sa >= sb) continue;
+    int64_t ga = seg_group[sa], gb = (int64_t)seg_group[sb - 1] + 1;
+    unsigned long long b =
+        8ull * (unsigned long long)(gb - ga) + 4ull * (unsigned long long)(slot_prefix[gb] - slot_prefix[ga]);
+    mx = max(mx, b);
+  }
+  unsigned long long r = BR(tmp).Reduce(mx, cub::Max());
+  if (threadIdx.x == 0) atomicMax(out, r);
+}
+
+// exclusive prefix of `in` (length n) into out[0..n] (out[0] = 0, out[n] = total)
+void exclusive_prefix(const int64_t* in, int64_t n, int64_t* out, cudaStream_t s) {
+  TC_CUDA(cudaMemsetAsync(out, 0, sizeof(int64_t), s));
+  if (n == 0) return;
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceScan::InclusiveSum(t, b, in, out + 1, n, s);
+  });
+}
+
+struct Timer {
+  cudaEvent_t e[7];
+  int k = 0;
+  cudaStream_t s;
+  explicit Timer(cudaStream_t st) : s(st) {
+    for (auto& x : e) TC_CUDA(cudaEventCreate(&x));
+  }
+  ~Timer() {
+    for (auto& x : e) cudaEventDestroy(x);
+  }
+  void mark() { TC_CUDA(cudaEventRecord(e[k++], s)); }
+  float ms(int a, int b) {
+    float t = 0;
+    TC_CUDA(cudaEventElapsedTime(&t, e[a], e[b]));
+    return t;
+  }
+};
+
+}  // namespace
+
+// ------------------------------------------------------------------ a1..a5
+void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
+                 uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g) {
+  Timer tm(s);
+  tm.mark();
+  if (n < 0) {  // num_vertices = max id + 1
+    if (m_gen == 0) {
+      n = 0;
+    } else {
+      DevBuf<int32_t> mx(2, s);
+      cub_run(s, [&](void* t, size_t& b) {
+        return cub::DeviceReduce::Max(t, b, d_src, mx.get(), m_gen, s);
+      });
+      cub_run(s, [&](void* t, size_t& b) {
+        return cub::DeviceReduce::Max(t, b, d_dst, mx.get() + 1, m_gen, s);
+      });
+      int32_t h[2];
+      TC_CUDA(cudaMemcpyAsync(h, mx.get(), sizeof(h), cudaMemcpyDeviceToHost, s));
+      TC_CUDA(cudaStreamSynchronize(s));
+      n = (int64_t)std::max(h[0], h[1]) + 1;
+      if (n < 0) n = 0;
+    }
+  }
+  g->n_input = n;
+  const int bits = bits_for(std::max<int64_t>(n, 2));
+  const uint64_t sent = (uint64_t(1) << (2 * bits)) - 1;  // never a valid (lo < hi) key
+
+  // a1 + a2
+  DevBuf<uint64_t> ka(std::max<int64_t>(m_gen, 1), s), kb(std::max<int64_t>(m_gen, 1), s);
+  DevBuf<int> err(1, s);
+  DevBuf<int64_t> nsel(1, s);
+  DevBuf<UniqTail> tail(1, s);
+  TC_CUDA(cudaMemsetAsync(err.get(), 0, sizeof(int), s));
+  TC_CUDA(cudaMemsetAsync(nsel.get(), 0, sizeof(int64_t), s));
+  if (m_gen > 0) {
+    k_canon<<<grid_for(m_gen), TPB, 0, s>>>(d_src, d_dst, m_gen, n, bits, sent, ka.get(),
+                                            err.get());
+    TC_LAUNCH();
+  }
+  tm.mark();
+  int64_t m = 0;
+  uint64_t* ukey = ka.get();
+  if (m_gen > 0) {
+    cub::DoubleBuffer<uint64_t> db(ka.get(), kb.get());
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceRadixSort::SortKeys(t, b, db, m_gen, 0, 2 * bits, s);
+    });
+    uint64_t* sorted = db.Current();
+    uint64_t* other = sorted == ka.get() ? kb.get() : ka.get();
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceSelect::Unique(t, b, sorted, other, nsel.get(), m_gen, s);
+    });
+    ukey = other;
+  }
+  k_uniq_tail<<<1, 1, 0, s>>>(err.get(), nsel.get(), ukey, tail.get());
+  TC_LAUNCH();
+  UniqTail ut = d2h(tail.get(), s);
+  if (ut.err) fail(TC_ERR_INVALID_ARGUMENT, "vertex id < 0 or >= num_vertices in the edge list");
+  m = ut.nsel - ((ut.nsel > 0 && ut.last == sent) ? 1 : 0);
+  g->m = m;
+  tm.mark();
+
+  // a3 + a4
+  DevBuf<int32_t> deg(std::max<int64_t>(n, 1), s);
+  TC_CUDA(cudaMemsetAsync(deg.get(), 0, sizeof(int32_t) * std::max<int64_t>(n, 1), s));
+  if (m > 0) {
+    k_degree<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, deg.get());
+    TC_LAUNCH();
+  }
+  const int keep = (flags & TC_KEEP_ISOLATED) ? 1 : 0;
+  const uint64_t sentv = (uint64_t(1) << (2 * bits + 1)) - 1;
+  DevBuf<uint64_t> va(std::max<int64_t>(n, 1), s), vb(std::max<int64_t>(n, 1), s);
+  DevBuf<unsigned long long> nact(1, s);
+  TC_CUDA(cudaMemsetAsync(nact.get(), 0, sizeof(unsigned long long), s));
+  int64_t n_act = 0;
+  DevBuf<int32_t> rank(std::max<int64_t>(n, 1), s);
+  if (n > 0) {
+    k_vkey<<<grid_for(n), TPB, 0, s>>>(deg.get(), n, bits, keep, sentv, va.get(), nact.get());
+    TC_LAUNCH();
+    cub::DoubleBuffer<uint64_t> db(va.get(), vb.get());
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceRadixSort::SortKeys(t, b, db, n, 0, 2 * bits + 1, s);
+    });
+    n_act = (int64_t)d2h(nact.get(), s);
+    g->perm = DevBuf<int32_t>(std::max<int64_t>(n_act, 1), s);
+    if (n_act > 0) {
+      k_perm<<<grid_for(n_act), TPB, 0, s>>>(db.Current(), n_act, bits, g->perm.get(),
+                                             rank.get());
+      TC_LAUNCH();
+    }
+  } else {
+    g->perm = DevBuf<int32_t>(1, s);
+  }
+  g->n = n_act;
+  deg.reset();
+  va.reset();
+  vb.reset();
+  tm.mark();
+
+  // a5
+  const int bits2 = bits_for(std::max<int64_t>(n_act, 2));
+  g->bits = bits2;
+  g->row_ptr = DevBuf<int64_t>(n_act + 1, s);
+  g->col = DevBuf<int32_t>(std::max<int64_t>(m, 1), s);
+  if (m > 0) {
+    uint64_t* okey_a = (ukey == ka.get()) ? kb.get() : ka.get();  // the free buffer
+    k_orient<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank.get(), bits2, okey_a);
+    TC_LAUNCH();
+    cub::DoubleBuffer<uint64_t> db(okey_a, ukey);
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceRadixSort::SortKeys(t, b, db, m, 0, 2 * bits2, s);
+    });
+    k_csr<<<grid_for(m), TPB, 0, s>>>(db.Current(), m, n_act, bits2, g->col.get(),
+                                      g->row_ptr.get());
+    TC_LAUNCH();
+  } else {
+    k_fill_i64<<<grid_for(n_act + 1), TPB, 0, s>>>(g->row_ptr.get(), n_act + 1, 0);
+    TC_LAUNCH();
+  }
+  ka.reset();
+  kb.reset();
+  rank.reset();
+  {
+    DevBuf<unsigned long long> mx(1, s);
+    TC_CUDA(cudaMemsetAsync(mx.get(), 0, sizeof(unsigned long long), s));
+    if (n_act > 0) {
+      k_max_outdeg<<<grid_for(n_act), TPB, 0, s>>>(g->row_ptr.get(), n_act, mx.get());
+      TC_LAUNCH();
+    }
+    g->max_out = (int64_t)d2h(mx.get(), s);
+  }
+  tm.mark();
+  build_plan(g, opt, s);
+  tm.mark();
+  TC_CUDA(cudaStreamSynchronize(s));
+  g->ms[0] = tm.ms(0, 1);
+  g->ms[1] = tm.ms(1, 2);
+  g->ms[2] = tm.ms(2, 3);
+  g->ms[3] = tm.ms(3, 4);
+  g->ms[4] = tm.ms(4, 5);
+  g->ms[5] = tm.ms(0, 5);
+}
+
+// ------------------------------------------------------------------ a6
+void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
+  Plan& P = g->plan;
+  P = Plan();
+  P.opt = opt;
+  const int64_t m = g->m, n = g->n;
+  const int64_t* row_ptr = g->row_ptr.get();
+  const int32_t* col = g->col.get();
+  DevBuf<unsigned long long> stats(3, s);
+  TC_CUDA(cudaMemsetAsync(stats.get(), 0, 3 * sizeof(unsigned long long), s));
+  DevBuf<int32_t> rowid(std::max<int64_t>(m, 1), s);
+  DevBuf<uint8_t> live(std::max<int64_t>(m, 1), s);
+  if (m > 0) {
+    k_rowid<<<grid_for(n), TPB, 0, s>>>(row_ptr, n, rowid.get());
+    TC_LAUNCH();
+    k_edge_stats<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m, live.get(),
+                                             stats.get());
+    TC_LAUNCH();
+  }
+  unsigned long long h_stats[3];
+  TC_CUDA(cudaMemcpyAsync(h_stats, stats.get(), sizeof(h_stats), cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  g->b_itc = h_stats[0] + 8ull * (unsigned long long)(n + 1);
+  P.keys_total = (int64_t)h_stats[1];
+  const int64_t S = (int64_t)h_stats[2];
+  P.S = S;
+  P.block = opt.block_threads;
+  P.key_prefix = DevBuf<int64_t>(S + 1, s);
+  TC_CUDA(cudaMemsetAsync(P.key_prefix.get(), 0, sizeof(int64_t), s));
+  if (S == 0) {
+    P.chunk_seg = DevBuf<int64_t>(1, s);
+    TC_CUDA(cudaMemsetAsync(P.chunk_seg.get(), 0, sizeof(int64_t), s));
+    P.h_chunk_seg.assign(1, 0);
+    TC_CUDA(cudaStreamSynchronize(s));
+    return;
+  }
+
+  // live edges, grouped by head v (stable: position order inside a group)
+  DevBuf<int64_t> p_live(S, s), p_sorted(S, s);
+  DevBuf<uint32_t> vk(S, s), vk_sorted(S, s);
+  {
+    DevBuf<int64_t> nsel(1, s);
+    cub::CountingInputIterator<int64_t> it(0);
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceSelect::Flagged(t, b, it, live.get(), p_live.get(), nsel.get(), m, s);
+    });
+  }
+  live.reset();
+  k_gather_head<<<grid_for(S), TPB, 0, s>>>(p_live.get(), S, col, vk.get());
+  TC_LAUNCH();
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceRadixSort::SortPairs(t, b, vk.get(), vk_sorted.get(), p_live.get(),
+                                           p_sorted.get(), S, 0, g->bits, s);
+  });
+  vk.reset();
+  p_live.reset();
+
+  DevBuf<int32_t> gincl(S, s);
+  {
+    DevBuf<int32_t> mark(S, s);
+    k_group_mark<<<grid_for(S), TPB, 0, s>>>(vk_sorted.get(), S, mark.get());
+    TC_LAUNCH();
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceScan::InclusiveSum(t, b, mark.get(), gincl.get(), S, s);
+    });
+  }
+  const int64_t G = (int64_t)d2h(gincl.get() + (S - 1), s);
+  P.G = G;
+  P.seg_group = DevBuf<int32_t>(S, s);
+  DevBuf<int64_t> seg_len(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
+  P.grp_tmax = DevBuf<int32_t>(G, s);
+  k_seg_group<<<grid_for(S), TPB, 0, s>>>(vk_sorted.get(), p_sorted.get(), gincl.get(), S,
+                                          row_ptr, col, rowid.get(), opt.huge_degree,
+                                          opt.hash_shift, P.seg_group.get(), seg_len.get(),
+                                          grp_row.get(), grp_d.get(), grp_slots.get(),
+                                          P.grp_tmax.get());
+  TC_LAUNCH();
+  gincl.reset();
+  vk_sorted.reset();
+  rowid.reset();
+  exclusive_prefix(seg_len.get(), S, P.key_prefix.get(), s);
+  P.ins_prefix = DevBuf<int64_t>(G + 1, s);
+  P.slot_prefix = DevBuf<int64_t>(G + 1, s);
+  exclusive_prefix(grp_d.get(), G, P.ins_prefix.get(), s);
+  exclusive_prefix(grp_slots.get(), G, P.slot_prefix.get(), s);
+  P.grp_ibase = DevBuf<int64_t>(G, s);
+  k_grp_ibase<<<grid_for(G), TPB, 0, s>>>(grp_row.get(), P.ins_prefix.get(), G,
+                                          P.grp_ibase.get());
+  TC_LAUNCH();
+  P.seg_base = DevBuf<int64_t>(S, s);
+  DevBuf<int64_t> cost(S, s), cost_prefix(S + 1, s);
+  k_seg_base_cost<<<grid_for(S), TPB, 0, s>>>(p_sorted.get(), P.key_prefix.get(), seg_len.get(),
+                                              P.seg_group.get(), grp_d.get(), grp_slots.get(),
+                                              S, opt.seg_cost, P.seg_base.get(), cost.get());
+  TC_LAUNCH();
+  exclusive_prefix(cost.get(), S, cost_prefix.get(), s);
+  cost.reset();
+  seg_len.reset();
+  grp_row.reset();
+  grp_d.reset();
+  grp_slots.reset();
+  p_sorted.reset();
+  const int64_t total_cost = d2h(cost_prefix.get() + S, s);
+
+  // Chunking: halve the chunk cost until the largest chunk's SMEM fits one CTA.
+  const int64_t smem_limit = std::min<int64_t>(max_smem_per_block(), 200 * 1024) - 1024;
+  int64_t C = std::max(opt.chunk_cost, 64);
+  DevBuf<unsigned long long> mx(1, s);
+  for (;;) {
+    const int64_t nc = (total_cost + C - 1) / C;
+    P.chunk_seg = DevBuf<int64_t>(nc + 1, s);
+    k_chunk_bounds<<<grid_for(nc + 1), TPB, 0, s>>>(cost_prefix.get(), S, nc, C,
+                                                    P.chunk_seg.get());
+    TC_LAUNCH();
+    TC_CUDA(cudaMemsetAsync(mx.get(), 0, sizeof(unsigned long long), s));
+    k_chunk_smem<<<grid_for(nc), TPB, 0, s>>>(P.chunk_seg.get(), nc, P.seg_group.get(),
+                                              P.slot_prefix.get(), mx.get());
+    TC_LAUNCH();
+    const int64_t need = (int64_t)d2h(mx.get(), s);
+    if (need <= smem_limit || C <= 64) {
+      if (need > smem_limit)
+        fail(TC_ERR_UNSUPPORTED, "a chunk's hash tables exceed shared memory (lower huge_degree)");
+      P.n_chunks = nc;
+      P.smem_bytes = need;
+      break;
+    }
+    C >>= 1;
+  }
+  P.opt.chunk_cost = (int)C;
+  P.h_chunk_seg.resize(P.n_chunks + 1);
+  TC_CUDA(cudaMemcpyAsync(P.h_chunk_seg.data(), P.chunk_seg.get(),
+                          sizeof(int64_t) * (P.n_chunks + 1), cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  const int occ = count_occupancy(P.block, P.smem_bytes);
+  if (occ < 1) fail(TC_ERR_UNSUPPORTED, "count kernel cannot launch with this SMEM/block size");
+  P.grid = (int)std::min<int64_t>(P.n_chunks, (int64_t)occ * num_sms());
+}
+
+}  // namespace tc

@@ -1,0 +1,107 @@
+"""CPU-side checks of the C-ABI boundary (-m "not gpu").
+
+No compute call is made here (there is no GPU in the build container): the
+library must load, export every symbol include/tc.h declares, reject bad
+arguments before touching the device, and its host-only partition logic must
+cut cost prefixes into balanced contiguous ranges.
+"""
+import ctypes
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def tc():
+    subprocess.run(["make", "-s", "-C", ROOT, "paper_conf_ipps_li0ptz24_b200/libtc.so"],
+                   check=True)
+    import paper_conf_ipps_li0ptz24_b200 as tc
+    tc.lib()
+    return tc
+
+
+def header_symbols():
+    text = open(os.path.join(ROOT, "include", "tc.h")).read()
+    return sorted(set(re.findall(r"TC_API\s+[\w\s\*]+?\b(tc_\w+)\s*\(", text)))
+
+
+def test_header_symbols_match_binding(tc):
+    assert header_symbols() == sorted(tc.EXPORTS)
+
+
+def test_library_exports_every_symbol(tc):
+    out = subprocess.run(["nm", "-D", "--defined-only", tc.LIB_PATH], capture_output=True,
+                         text=True, check=True).stdout
+    exported = set(re.findall(r"\bT (tc_\w+)", out))
+    missing = set(header_symbols()) - exported
+    assert not missing, missing
+    # nothing else leaks from the C-ABI namespace
+    assert exported == set(header_symbols())
+
+
+def test_library_is_sm100a(tc):
+    out = subprocess.run(["cuobjdump", "--list-elf", tc.LIB_PATH], capture_output=True,
+                         text=True, check=True).stdout
+    assert "sm_100a" in out
+
+
+def test_version(tc):
+    assert tc.version().startswith("b200tc")
+
+
+def test_null_out_is_invalid(tc):
+    L = tc.lib()
+    assert L.tc_build_csr(None, None, 0, -1, 0, None, None, None) == tc.TC_ERR_INVALID_ARGUMENT
+    assert "out" in L.tc_last_error().decode()
+
+
+def test_bad_arguments_rejected_before_device(tc):
+    L = tc.lib()
+    h = ctypes.c_void_p(0)
+    assert L.tc_build_csr(None, None, -1, -1, 0, None, None, ctypes.byref(h)) == 1
+    assert L.tc_build_csr(None, None, 5, -1, 0, None, None, ctypes.byref(h)) == 1
+    assert L.tc_build_csr(None, None, 0, 2**31, 0, None, None, ctypes.byref(h)) == 1
+    assert L.tc_build_csr(None, None, 0, -1, 0x80, None, None, ctypes.byref(h)) == 1
+    assert h.value is None
+    bad = tc.Options(chunk_cost=8)
+    assert L.tc_build_csr(None, None, 0, -1, 0, ctypes.byref(bad), None, ctypes.byref(h)) == 1
+    bad = tc.Options(block_threads=1024)
+    assert L.tc_build_csr(None, None, 0, -1, 0, ctypes.byref(bad), None, ctypes.byref(h)) == 1
+    assert L.tc_count(None, None, None) == 1
+    assert L.tc_count_range(None, 0, 0, None, None) == 1
+    assert L.tc_partition(None, 2, None) == 1
+    assert L.tc_graph_info(None, None) == 1
+    L.tc_free(None)  # no-op
+
+
+def test_allocator_hooks_must_pair(tc):
+    L = tc.lib()
+    cb = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+    f = cb(lambda n, s, c: None)
+    assert L.tc_set_allocator(ctypes.cast(f, ctypes.c_void_p), None, None) == 1
+    assert L.tc_set_allocator(None, None, None) == 0
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
+def test_partition_prefix_balanced(tc, world):
+    rng = np.random.default_rng(world)
+    cost = rng.integers(1, 200, size=5000)
+    prefix = np.concatenate([[0], np.cumsum(cost)])
+    b = tc.partition_prefix(prefix, world)
+    assert b[0] == 0 and b[-1] == len(cost) and all(x <= y for x, y in zip(b, b[1:]))
+    loads = [prefix[b[r + 1]] - prefix[b[r]] for r in range(world)]
+    assert sum(loads) == prefix[-1]
+    # every part within one unit's cost of the ideal share
+    assert max(loads) - prefix[-1] / world <= cost.max()
+
+
+def test_partition_prefix_degenerate(tc):
+    assert tc.partition_prefix([0], 4) == [0, 0, 0, 0, 0]
+    assert tc.partition_prefix([0, 10], 3) == [0, 1, 1, 1] or tc.partition_prefix([0, 10], 3)[-1] == 1
+    with pytest.raises(tc.InvalidArgument):
+        tc.partition_prefix([0, 1], 0)

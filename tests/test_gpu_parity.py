@@ -1,0 +1,278 @@
+"""GPU parity: the CUDA path (through the C-ABI) vs the CPU oracle, bit-exact.
+
+Every count here is compared with oracle/ (or a closed form) on the same
+seeded input from tcgen/; neither side's numbers come from the other.
+Sizes span many work chunks and ragged tails; the plan options are varied
+because they must never change a count.
+"""
+from math import comb
+
+import numpy as np
+import pytest
+
+import oracle
+import tcgen
+from tests import graphs
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def tc():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_li0ptz24_b200 as tc
+    tc.lib()
+    return tc
+
+
+def dev(a):
+    return torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).cuda()
+
+
+def gpu_count(tc, src, dst, n=None, **kw):
+    with tc.build_csr(dev(src), dev(dst), n, **kw) as g:
+        return g.count()
+
+
+# ------------------------------------------------------------------ closed forms / golden
+
+@pytest.mark.parametrize("name", sorted(graphs.closed_form_cases()))
+def test_closed_forms(tc, name):
+    (src, dst, n), t = graphs.closed_form_cases()[name]
+    assert gpu_count(tc, src, dst, n) == t
+
+
+def test_karate(tc, golden):
+    src, dst = golden("karate.txt")
+    assert gpu_count(tc, src, dst, 34) == 45
+
+
+@pytest.mark.parametrize("name", ["lesmis.txt", "florentine.txt", "davis.txt"])
+def test_golden_vs_oracle(tc, golden, name):
+    src, dst = golden(name)
+    assert gpu_count(tc, src, dst) == oracle.triangles(src, dst)
+
+
+def test_fig14_suffix_example(tc):
+    """P:359 (Fig. 14): N(0) ⊇ {4,5,8}; edge (0,8) has an empty suffix and is
+    skipped; edge (0,4) searches only [5,8].  Graph: 0-{4,5,8}, 4-{5,8}, 5-8
+    is K4 on {0,4,5,8} plus nothing else -> 4 triangles."""
+    e = np.array([(0, 4), (0, 5), (0, 8), (4, 5), (4, 8), (5, 8)], dtype=np.int32)
+    assert gpu_count(tc, e[:, 0], e[:, 1], 9) == 4
+
+
+# ------------------------------------------------------------------ configs
+
+@pytest.mark.parametrize("seed", [1, 2, 3, 4, 5])
+def test_c1_rmat10_seeds(tc, seed):
+    src, dst, n = tcgen.CONFIGS["C1"].generate(seed)
+    r = oracle.count(src, dst, n)
+    with tc.build_csr(dev(src), dev(dst), n) as g:
+        assert g.count() == r.triangles
+        assert g.m == r.m and g.n == r.n_active
+        assert g.info.max_out_degree == r.max_out_degree  # same (deg, id) order
+
+
+@pytest.mark.parametrize("scale,ef,seed", [(14, 16, 1), (16, 16, 2), (17, 8, 3)])
+def test_rmat_medium(tc, scale, ef, seed):
+    src, dst, n = tcgen.rmat(scale, ef, seed)
+    assert gpu_count(tc, src, dst, n) == oracle.triangles(src, dst, n)
+
+
+def test_rmat_skewed_initiator(tc):
+    src, dst, n = tcgen.rmat(16, 24, 7, abc=(0.65, 0.15, 0.15))
+    assert gpu_count(tc, src, dst, n) == oracle.triangles(src, dst, n)
+
+
+def test_c2_chung_lu_full(tc):
+    src, dst, n = tcgen.CONFIGS["C2"].generate(1)
+    assert gpu_count(tc, src, dst, n) == oracle.triangles(src, dst, n)
+
+
+def test_c5_lattice_full(tc):
+    src, dst, n = tcgen.CONFIGS["C5"].generate(1)
+    assert gpu_count(tc, src, dst, n) == oracle.triangles(src, dst, n)
+
+
+def test_chung_lu_small(tc):
+    src, dst, n = tcgen.chung_lu(200_000, 1_500_000, 3)
+    assert gpu_count(tc, src, dst, n) == oracle.triangles(src, dst, n)
+
+
+# ------------------------------------------------------------------ properties
+
+@pytest.mark.parametrize("opts", [
+    dict(chunk_cost=64), dict(chunk_cost=256), dict(chunk_cost=4096), dict(chunk_cost=1 << 20),
+    dict(block_threads=64), dict(block_threads=128), dict(block_threads=256),
+    dict(seg_cost=1), dict(seg_cost=64), dict(hash_shift=0), dict(hash_shift=3),
+    dict(huge_degree=1), dict(huge_degree=16), dict(huge_degree=16, chunk_cost=64),
+])
+def test_plan_options_never_change_count(tc, opts):
+    src, dst, n = tcgen.rmat(13, 16, 11)
+    t = oracle.triangles(src, dst, n)
+    with tc.build_csr(dev(src), dev(dst), n, options=opts) as g:
+        assert g.count() == t
+    with tc.build_csr(dev(src), dev(dst), n) as g:
+        g.replan(opts)
+        assert g.count() == t
+
+
+def test_cleaning_invariance(tc):
+    """duplicates, reversed pairs, self-loops, isolated vertices."""
+    rng = np.random.default_rng(5)
+    src, dst, n = tcgen.rmat(12, 16, 5)
+    base = gpu_count(tc, src, dst, n)
+    dup = rng.integers(0, len(src), 20000)
+    loops = rng.integers(0, n, 500).astype(np.int32)
+    s2 = np.concatenate([src, dst[dup], loops, src[dup]])
+    d2 = np.concatenate([dst, src[dup], loops, dst[dup]])
+    p = rng.permutation(len(s2))
+    assert gpu_count(tc, s2[p], d2[p], n + 1000) == base
+    assert gpu_count(tc, s2[p], d2[p], n + 1000, keep_isolated=True) == base
+
+
+def test_relabel_invariance(tc):
+    rng = np.random.default_rng(2)
+    src, dst, n = tcgen.rmat(13, 8, 2)
+    perm = rng.permutation(n).astype(np.int32)
+    assert gpu_count(tc, perm[src], perm[dst], n) == gpu_count(tc, src, dst, n)
+
+
+def test_disjoint_union_additive(tc):
+    s1, d1, n1 = tcgen.rmat(11, 16, 1)
+    s2, d2, n2 = tcgen.lattice(60, 2)
+    s = np.concatenate([s1, s2 + n1])
+    d = np.concatenate([d1, d2 + n1])
+    assert gpu_count(tc, s, d) == gpu_count(tc, s1, d1) + gpu_count(tc, s2, d2)
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 5, 8])
+def test_partition_ranges_sum_to_total(tc, world):
+    src, dst, n = tcgen.rmat(14, 16, 4)
+    t = oracle.triangles(src, dst, n)
+    with tc.build_csr(dev(src), dev(dst), n, options=dict(chunk_cost=2048)) as g:
+        b = g.partition(world)
+        assert b[0] == 0 and b[-1] == g.m_live and b == sorted(b)
+        parts = [int(g.count_range(b[r], b[r + 1]).item()) for r in range(world)]
+        assert sum(parts) == t
+
+
+def test_arbitrary_ranges_sum_to_total(tc):
+    """Any cut of [0, m_live) is exact, including cuts inside chunks."""
+    rng = np.random.default_rng(9)
+    src, dst, n = tcgen.rmat(13, 16, 8)
+    t = oracle.triangles(src, dst, n)
+    with tc.build_csr(dev(src), dev(dst), n, options=dict(chunk_cost=1024)) as g:
+        cuts = np.unique(np.concatenate([[0, g.m_live], rng.integers(0, g.m_live, 37)]))
+        parts = [int(g.count_range(a, b).item()) for a, b in zip(cuts, cuts[1:])]
+        assert sum(parts) == t
+        assert int(g.count_range(5, 5).item()) == 0
+
+
+def test_count_async_matches(tc):
+    src, dst, n = tcgen.rmat(12, 16, 3)
+    with tc.build_csr(dev(src), dev(dst), n) as g:
+        out = g.count_async()
+        torch.cuda.synchronize()
+        assert int(out.item()) == g.count() == oracle.triangles(src, dst, n)
+
+
+def test_host_entry_point(tc):
+    src, dst, n = tcgen.rmat(12, 16, 6)
+    with tc.build_csr_host(src, dst, n) as g:
+        assert g.count() == oracle.triangles(src, dst, n)
+    pinned_s = torch.from_numpy(src).pin_memory()
+    pinned_d = torch.from_numpy(dst).pin_memory()
+    with tc.build_csr_host(pinned_s, pinned_d, n) as g:
+        assert g.count() == oracle.triangles(src, dst, n)
+
+
+# ------------------------------------------------------------------ CSR layout
+
+def reference_csr(src, dst, n):
+    """Host reference of a1..a5 (numpy): (deg, id) rank, relabel, orient, sort."""
+    s = np.minimum(src, dst).astype(np.int64)
+    d = np.maximum(src, dst).astype(np.int64)
+    keep = s != d
+    key = np.unique((s[keep] << 32) | d[keep])
+    a, b = key >> 32, key & 0xFFFFFFFF
+    deg = np.bincount(np.concatenate([a, b]), minlength=n)
+    active = np.nonzero(deg > 0)[0]
+    order = active[np.lexsort((active, deg[active]))]
+    rank = np.full(n, -1, dtype=np.int64)
+    rank[order] = np.arange(len(order))
+    u, v = rank[a], rank[b]
+    lo, hi = np.minimum(u, v), np.maximum(u, v)
+    idx = np.lexsort((hi, lo))
+    lo, hi = lo[idx], hi[idx]
+    row_ptr = np.concatenate([[0], np.cumsum(np.bincount(lo, minlength=len(order)))])
+    return row_ptr, hi.astype(np.int32), order.astype(np.int32)
+
+
+@pytest.mark.parametrize("case", ["rmat", "lattice", "karate"])
+def test_csr_exact(tc, golden, case):
+    if case == "rmat":
+        src, dst, n = tcgen.rmat(12, 16, 2)
+    elif case == "lattice":
+        src, dst, n = tcgen.lattice(50, 3)
+    else:
+        (src, dst), n = golden("karate.txt"), 34
+    rp, col, perm = reference_csr(src, dst, n)
+    with tc.build_csr(dev(src), dev(dst), n) as g:
+        grp, gcol, gperm = (x.cpu().numpy() for x in g.csr())
+        np.testing.assert_array_equal(grp, rp)
+        np.testing.assert_array_equal(gcol, col)
+        np.testing.assert_array_equal(gperm, perm)
+        # invariants: rows strictly ascending, col > row, d+ <= sqrt(2m)
+        rows = np.repeat(np.arange(len(rp) - 1), np.diff(rp))
+        assert np.all(gcol > rows)
+        same = rows[1:] == rows[:-1]
+        assert np.all(gcol[1:][same] > gcol[:-1][same])
+        assert np.diff(rp).max() <= int(np.sqrt(2 * g.m))
+
+
+# ------------------------------------------------------------------ edge cases / errors
+
+def test_empty_and_tiny(tc):
+    e = np.zeros(0, dtype=np.int32)
+    assert gpu_count(tc, e, e, 0) == 0
+    assert gpu_count(tc, e, e, 10) == 0
+    assert gpu_count(tc, e, e) == 0
+    assert gpu_count(tc, [0], [1], 2) == 0
+    assert gpu_count(tc, [0, 1, 2], [1, 2, 0]) == 1
+    loops = np.arange(10, dtype=np.int32)
+    assert gpu_count(tc, loops, loops, 10) == 0
+
+
+def test_invalid_ids(tc):
+    with pytest.raises(tc.InvalidArgument):
+        tc.build_csr(dev([0, 5]), dev([1, 2]), 5)
+    with pytest.raises(tc.InvalidArgument):
+        tc.build_csr(dev([-1]), dev([1]), 5)
+    with pytest.raises(tc.InvalidArgument):
+        tc.build_csr(dev([-1]), dev([1]))
+    # the library is still usable afterwards
+    assert gpu_count(tc, [0, 1, 2], [1, 2, 0]) == 1
+
+
+def test_sparse_ids_large_n(tc):
+    """n_vertices = 2^31-1 with a handful of sparse ids."""
+    big = 2**31 - 2
+    src = np.array([0, 1000, big, 0], dtype=np.int32)
+    dst = np.array([1000, big, 0, 7], dtype=np.int32)
+    assert gpu_count(tc, src, dst, 2**31 - 1) == 1
+
+
+def test_k3000_exceeds_32_bits(tc):
+    """C-13: C(3000,3) > 2^32 catches any 32-bit accumulator above the thread."""
+    (src, dst, n), t = graphs.complete(3000)
+    assert t == comb(3000, 3) > 2**32
+    assert gpu_count(tc, src, dst, n) == t
+
+
+def test_huge_table_path_on_clique(tc):
+    """K_1200 with huge_degree=100: most tables go through the global probe."""
+    (src, dst, n), t = graphs.complete(1200)
+    assert gpu_count(tc, src, dst, n, options=dict(huge_degree=100)) == t

@@ -154,3 +154,13 @@ def test_k3000_exceeds_32_bits():
     (src, dst, n), t = graphs.complete(3000)
     assert t == comb(3000, 3) > 2**32
     assert oracle.triangles(src, dst, n) == t
+
+
+def test_sample_offsets_tile_the_rows():
+    """count_rows over the cosets x % s == o, o = 0..s-1, adds up to the full count."""
+    src, dst, n = tcgen.rmat(12, 16, 13)
+    g = oracle.OracleGraph(src, dst, n)
+    full = g.count_rows()
+    parts = [g.count_rows(stride=5, offset=o) for o in range(5)]
+    assert sum(p.triangles for p in parts) == full.triangles == oracle.triangles(src, dst, n)
+    assert sum(p.merge_steps_counted for p in parts) == full.merge_steps_total
