@@ -82,8 +82,14 @@ typedef struct {
   int32_t huge_degree;  /* d+(v) above which N+(v) is probed in global memory by
                            binary search instead of an SMEM hash (default 8192)    */
   int32_t block_threads;/* threads per CTA of the count kernel (default 512)       */
-  int32_t hash_shift;   /* hash slots = next_pow2(d+(v) << hash_shift) (default 1) */
-  int32_t reserved[3];
+  int32_t table_factor; /* hash slots = next_pow2(table_factor * d+(v)), 2..16
+                           (default 3, i.e. load <= 1/3)                            */
+  int32_t long_min;     /* trimmed suffixes with >= long_min keys go to the
+                           warp-per-edge class, shorter ones to the flattened
+                           class (default 32; 1 = all long, 2^30 = all short)     */
+  int32_t probe_mode;   /* 0 = two-choice (cuckoo) tables with linear-probing
+                           fallback per chunk, 1 = linear probing only (default 0) */
+  int32_t reserved;
 } tc_options;
 
 /*

@@ -55,7 +55,8 @@ class Options(ctypes.Structure):
     change the count."""
     _fields_ = [("chunk_cost", ctypes.c_int32), ("seg_cost", ctypes.c_int32),
                 ("huge_degree", ctypes.c_int32), ("block_threads", ctypes.c_int32),
-                ("hash_shift", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
+                ("table_factor", ctypes.c_int32), ("long_min", ctypes.c_int32),
+                ("probe_mode", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 class GraphInfo(ctypes.Structure):
@@ -154,7 +155,7 @@ class _DevArray:
 
     def __init__(self, ptr: int, n: int, typestr: str, owner):
         self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr,
-                                         "data": (ptr or 0, True), "version": 3}
+                                         "data": (ptr or 0, False), "version": 3}
         self._owner = owner
 
 

@@ -97,13 +97,17 @@ Options resolve_options(const tc_options* o) {
   if (o->seg_cost) r.seg_cost = o->seg_cost;
   if (o->huge_degree) r.huge_degree = o->huge_degree;
   if (o->block_threads) r.block_threads = o->block_threads;
-  if (o->hash_shift) r.hash_shift = o->hash_shift;
+  if (o->table_factor) r.table_factor = o->table_factor;
+  if (o->long_min) r.long_min = o->long_min;
+  if (o->probe_mode) r.probe_mode = o->probe_mode;
   require(r.chunk_cost >= 64, "chunk_cost must be >= 64");
   require(r.seg_cost >= 1, "seg_cost must be >= 1");
   require(r.huge_degree >= 1, "huge_degree must be >= 1");
   require(r.block_threads >= 64 && r.block_threads <= 512 && r.block_threads % 32 == 0,
           "block_threads must be a multiple of 32 in [64, 512]");
-  require(r.hash_shift >= 0 && r.hash_shift <= 4, "hash_shift must be in [0, 4]");
+  require(r.table_factor >= 2 && r.table_factor <= 16, "table_factor must be in [2, 16]");
+  require(r.long_min >= 1, "long_min must be >= 1");
+  require(r.probe_mode == 0 || r.probe_mode == 1, "probe_mode must be 0 or 1");
   return r;
 }
 
@@ -116,9 +120,9 @@ namespace {
 void rebind(tc_graph* g, cudaStream_t s) {
   g->row_ptr.s = g->col.s = g->perm.s = s;
   tc::Plan& P = g->plan;
-  P.key_prefix.s = P.seg_base.s = P.ins_prefix.s = P.grp_ibase.s = P.slot_prefix.s =
+  P.key_prefix.s = P.seg_start.s = P.ins_prefix.s = P.grp_ibase.s = P.slot_prefix.s =
       P.chunk_seg.s = s;
-  P.seg_group.s = P.grp_tmax.s = s;
+  P.seg_len.s = P.seg_group.s = s;
 }
 
 tc_status build_impl(const int32_t* src, const int32_t* dst, int64_t num_edges,

@@ -178,102 +178,133 @@ __global__ void k_rowid(const int64_t* __restrict__ row_ptr, int64_t n,
     for (int64_t p = row_ptr[u], e = row_ptr[u + 1]; p < e; ++p) rowid[p] = (int32_t)u;
 }
 
-// Per oriented edge p = (u, v): suffix length suf = row_end(u) - p - 1,
-// live iff suf > 0 and d+(v) > 0 (C-12 exact skips).  Accumulates
-// stats[0] = B_ITC edge part, stats[1] = sum of live suffixes, stats[2] = live count.
-__global__ void k_edge_stats(const int64_t* __restrict__ row_ptr,
-                             const int32_t* __restrict__ col,
-                             const int32_t* __restrict__ rowid, int64_t m,
-                             uint8_t* __restrict__ live, unsigned long long* stats) {
+__device__ __forceinline__ int64_t lower_bound_i32(const int32_t* __restrict__ a, int64_t lo,
+                                                   int64_t hi, int32_t x) {
+  while (lo < hi) {
+    int64_t mid = (lo + hi) >> 1;
+    if (a[mid] < x) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ int64_t upper_bound_i32(const int32_t* __restrict__ a, int64_t lo,
+                                                   int64_t hi, int32_t x) {
+  while (lo < hi) {
+    int64_t mid = (lo + hi) >> 1;
+    if (a[mid] <= x) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+// Per oriented edge p = (u, v): the keys are the suffix of N+(u) after v,
+// col[p+1, row_end(u)), trimmed to [min N+(v), max N+(v)] because a
+// key outside that range cannot be in N+(v) (both lists sorted; exact, C-12).
+// Live iff the trimmed suffix is non-empty.  stats: [0] B_ITC edge part
+// (untrimmed), [1] trimmed keys, [2] live, [3] live long.
+__global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
+                            const int32_t* __restrict__ rowid, int64_t m, int long_min,
+                            int64_t* __restrict__ e_lo, int32_t* __restrict__ e_len,
+                            uint8_t* __restrict__ live, unsigned long long* stats) {
   typedef cub::BlockReduce<unsigned long long, TPB> BR;
   __shared__ typename BR::TempStorage tmp;
-  unsigned long long b = 0, keys = 0, nl = 0;
+  unsigned long long b = 0, keys = 0, nl = 0, nlong = 0;
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < m;
        p += (int64_t)gridDim.x * blockDim.x) {
-    int32_t u = rowid[p], v = col[p];
-    int64_t suf = row_ptr[u + 1] - p - 1;
-    int64_t dv = row_ptr[v + 1] - row_ptr[v];
-    bool l = suf > 0 && dv > 0;
-    live[p] = l;
+    const int32_t u = rowid[p], v = col[p];
+    const int64_t rend = row_ptr[u + 1], suf = rend - p - 1;
+    const int64_t rv = row_ptr[v], dv = row_ptr[v + 1] - rv;
     b += 4ull * (unsigned long long)(suf + dv) + 12ull;
-    if (l) {
-      keys += (unsigned long long)suf;
-      ++nl;
+    int64_t lo = p + 1, len = 0;
+    if (suf > 0 && dv > 0) {
+      lo = lower_bound_i32(col, p + 1, rend, col[rv]);
+      len = upper_bound_i32(col, lo, rend, col[rv + dv - 1]) - lo;
     }
+    e_lo[p] = lo;
+    e_len[p] = (int32_t)len;
+    live[p] = len > 0;
+    keys += (unsigned long long)len;
+    nl += len > 0;
+    nlong += len >= long_min;
   }
   unsigned long long r0 = BR(tmp).Sum(b);
   __syncthreads();
   unsigned long long r1 = BR(tmp).Sum(keys);
   __syncthreads();
   unsigned long long r2 = BR(tmp).Sum(nl);
+  __syncthreads();
+  unsigned long long r3 = BR(tmp).Sum(nlong);
   if (threadIdx.x == 0) {
     atomicAdd(&stats[0], r0);
     atomicAdd(&stats[1], r1);
     atomicAdd(&stats[2], r2);
+    atomicAdd(&stats[3], r3);
   }
 }
 
-__global__ void k_gather_head(const int64_t* __restrict__ p_live, int64_t S,
-                              const int32_t* __restrict__ col, uint32_t* __restrict__ vkey) {
+// sort key of a live edge: class (0 = long, 1 = short) above the head v.
+__global__ void k_class_key(const int64_t* __restrict__ p_live, int64_t S,
+                            const int32_t* __restrict__ col, const int32_t* __restrict__ e_len,
+                            int long_min, int bits, uint32_t* __restrict__ key) {
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
-       s += (int64_t)gridDim.x * blockDim.x)
-    vkey[s] = (uint32_t)col[p_live[s]];
+       s += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p = p_live[s];
+    const uint32_t cls = e_len[p] < long_min ? 1u : 0u;
+    key[s] = (cls << bits) | (uint32_t)col[p];
+  }
 }
 
-__global__ void k_group_mark(const uint32_t* __restrict__ vkey, int64_t S,
+__global__ void k_group_mark(const uint32_t* __restrict__ key, int64_t S,
                              int32_t* __restrict__ mark) {
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
        s += (int64_t)gridDim.x * blockDim.x)
-    mark[s] = (s == 0 || vkey[s] != vkey[s - 1]) ? 1 : 0;
+    mark[s] = (s == 0 || key[s] != key[s - 1]) ? 1 : 0;
 }
 
-// Per segment: length, group id; per group (at its first segment): table facts.
-__global__ void k_seg_group(const uint32_t* __restrict__ vkey, const int64_t* __restrict__ p_s,
-                            const int32_t* __restrict__ gincl, int64_t S,
-                            const int64_t* __restrict__ row_ptr,
-                            const int32_t* __restrict__ col,
-                            const int32_t* __restrict__ rowid, int huge_degree,
-                            int hash_shift, int32_t* __restrict__ seg_group,
-                            int64_t* __restrict__ seg_len, int64_t* __restrict__ grp_row,
-                            int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots,
-                            int32_t* __restrict__ grp_tmax) {
+// Per segment: start, length, group, work units; per group (at its first
+// segment): row start, d+(v) and hash slots (> d+(v), or 0 for huge tables).
+__global__ void k_seg_fill(const uint32_t* __restrict__ key, const int64_t* __restrict__ p_s,
+                           const int32_t* __restrict__ gincl, int64_t S, int64_t S_long,
+                           int bits, const int64_t* __restrict__ row_ptr,
+                           const int64_t* __restrict__ e_lo, const int32_t* __restrict__ e_len,
+                           int huge_degree, int table_factor, int64_t* __restrict__ seg_start,
+                           int32_t* __restrict__ seg_len, int32_t* __restrict__ seg_group,
+                           int64_t* __restrict__ units, int64_t* __restrict__ grp_row,
+                           int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots) {
+  const uint32_t mask = (1u << bits) - 1u;
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
        s += (int64_t)gridDim.x * blockDim.x) {
-    int64_t p = p_s[s];
-    int32_t g = gincl[s] - 1;
+    const int64_t p = p_s[s];
+    const int32_t g = gincl[s] - 1;
+    const int32_t len = e_len[p];
     seg_group[s] = g;
-    seg_len[s] = row_ptr[rowid[p] + 1] - p - 1;
-    if (s == 0 || vkey[s] != vkey[s - 1]) {
-      int64_t v = vkey[s];
-      int64_t rs = row_ptr[v], d = row_ptr[v + 1] - rs;
+    seg_start[s] = e_lo[p];
+    seg_len[s] = len;
+    units[s] = s < S_long ? (int64_t)((len + 31) & ~31) : (int64_t)len;
+    if (s == 0 || key[s] != key[s - 1]) {
+      const int64_t v = key[s] & mask;
+      const int64_t rs = row_ptr[v], d = row_ptr[v + 1] - rs;
       grp_row[g] = rs;
       grp_d[g] = d;
       int64_t slots = 0;
       if (d <= huge_degree) {
-        // > d slots so a probe for an absent key always meets an empty slot
-        int64_t want = d << hash_shift;
-        if (want < d + 1) want = d + 1;
-        slots = 1;
+        int64_t want = d * table_factor;
+        if (want < d + 1) want = d + 1;  // an empty slot always exists
+        slots = 2;
         while (slots < want) slots <<= 1;
       }
       grp_slots[g] = slots;
-      grp_tmax[g] = col[rs + d - 1];
     }
   }
 }
 
-__global__ void k_seg_base_cost(const int64_t* __restrict__ p_s,
-                                const int64_t* __restrict__ key_prefix,
-                                const int64_t* __restrict__ seg_len,
-                                const int32_t* __restrict__ seg_group,
-                                const int64_t* __restrict__ grp_d,
-                                const int64_t* __restrict__ grp_slots, int64_t S, int seg_cost,
-                                int64_t* __restrict__ seg_base, int64_t* __restrict__ cost) {
+__global__ void k_seg_cost(const int64_t* __restrict__ units, const int32_t* __restrict__ seg_group,
+                           const int64_t* __restrict__ grp_d,
+                           const int64_t* __restrict__ grp_slots, int64_t S, int seg_cost,
+                           int64_t* __restrict__ cost) {
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
        s += (int64_t)gridDim.x * blockDim.x) {
-    seg_base[s] = p_s[s] + 1 - key_prefix[s];
-    int32_t g = seg_group[s];
-    int64_t c = seg_cost + seg_len[s];
+    const int32_t g = seg_group[s];
+    int64_t c = seg_cost + units[s];
     if (s == 0 || seg_group[s - 1] != g) c += grp_d[g] + grp_slots[g];
     cost[s] = c;
   }
@@ -287,17 +318,29 @@ __global__ void k_grp_ibase(const int64_t* __restrict__ grp_row,
     ibase[g] = grp_row[g] - ins_prefix[g];
 }
 
-// chunk_seg[c] = first segment whose exclusive cost prefix is >= c * C.
-__global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t S,
-                               int64_t n_chunks, int64_t C, int64_t* __restrict__ chunk_seg) {
-  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= n_chunks;
+// Chunks never straddle the class boundary S_long: long chunk c < nL starts
+// at the first segment whose cost prefix reaches c*C; short chunk nL + j at
+// the first segment of [S_long, S) whose prefix reaches prefix[S_long] + j*C.
+__global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t S_long,
+                               int64_t S, int64_t nL, int64_t nS, int64_t C,
+                               int64_t* __restrict__ chunk_seg) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= nL + nS;
        c += (int64_t)gridDim.x * blockDim.x) {
-    if (c == n_chunks) {
+    if (c == nL + nS) {
       chunk_seg[c] = S;
       continue;
     }
-    int64_t target = c * C, lo = 0, hi = S;  // first s in [0, S] with prefix[s] >= target
-    while (lo < hi) {
+    int64_t lo, hi, target;
+    if (c < nL) {
+      lo = 0;
+      hi = S_long;
+      target = c * C;
+    } else {
+      lo = S_long;
+      hi = S;
+      target = cost_prefix[S_long] + (c - nL) * C;
+    }
+    while (lo < hi) {  // first s with prefix[s] >= target
       int64_t mid = (lo + hi) >> 1;
       if (cost_prefix[mid] < target) lo = mid + 1; else hi = mid;
     }
@@ -305,8 +348,6 @@ __global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t 
   }
 }
 
-// SMEM a chunk needs in the count kernel: 8 B of table info per group plus
-// 4 B per hash slot (must match the layout in tc_count.cu).
 __global__ void k_chunk_smem(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
                              const int32_t* __restrict__ seg_group,
                              const int64_t* __restrict__ slot_prefix,
@@ -316,12 +357,11 @@ __global__ void k_chunk_smem(const int64_t* __restrict__ chunk_seg, int64_t n_ch
   unsigned long long mx = 0;
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n_chunks;
        c += (int64_t)gridDim.x * blockDim.x) {
-    int64_t sa = chunk_seg[c], sb = chunk_seg[c + 1];
+    const int64_t sa = chunk_seg[c], sb = chunk_seg[c + 1];
     if (sa >= sb) continue;
-    int64_t ga = seg_group[sa], gb = (int64_t)seg_group[sb - 1] + 1;
-    unsigned long long b =
-        8ull * (unsigned long long)(gb - ga) + 4ull * (unsigned long long)(slot_prefix[gb] - slot_prefix[ga]);
-    mx = max(mx, b);
+    const int64_t ga = seg_group[sa], gb = (int64_t)seg_group[sb - 1] + 1;
+    const int64_t b = chunk_smem_bytes(sb - sa, gb - ga, slot_prefix[gb] - slot_prefix[ga]);
+    mx = max(mx, (unsigned long long)b);
   }
   unsigned long long r = BR(tmp).Reduce(mx, cub::Max());
   if (threadIdx.x == 0) atomicMax(out, r);
@@ -504,28 +544,31 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   Plan& P = g->plan;
   P = Plan();
   P.opt = opt;
+  P.block = opt.block_threads;
   const int64_t m = g->m, n = g->n;
   const int64_t* row_ptr = g->row_ptr.get();
   const int32_t* col = g->col.get();
-  DevBuf<unsigned long long> stats(3, s);
-  TC_CUDA(cudaMemsetAsync(stats.get(), 0, 3 * sizeof(unsigned long long), s));
-  DevBuf<int32_t> rowid(std::max<int64_t>(m, 1), s);
+  DevBuf<unsigned long long> stats(4, s);
+  TC_CUDA(cudaMemsetAsync(stats.get(), 0, 4 * sizeof(unsigned long long), s));
+  DevBuf<int32_t> rowid(std::max<int64_t>(m, 1), s), e_len(std::max<int64_t>(m, 1), s);
+  DevBuf<int64_t> e_lo(std::max<int64_t>(m, 1), s);
   DevBuf<uint8_t> live(std::max<int64_t>(m, 1), s);
   if (m > 0) {
     k_rowid<<<grid_for(n), TPB, 0, s>>>(row_ptr, n, rowid.get());
     TC_LAUNCH();
-    k_edge_stats<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m, live.get(),
-                                             stats.get());
+    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m, opt.long_min, e_lo.get(),
+                                            e_len.get(), live.get(), stats.get());
     TC_LAUNCH();
   }
-  unsigned long long h_stats[3];
+  rowid.reset();
+  unsigned long long h_stats[4];
   TC_CUDA(cudaMemcpyAsync(h_stats, stats.get(), sizeof(h_stats), cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));
   g->b_itc = h_stats[0] + 8ull * (unsigned long long)(n + 1);
   P.keys_total = (int64_t)h_stats[1];
-  const int64_t S = (int64_t)h_stats[2];
+  const int64_t S = (int64_t)h_stats[2], S_long = (int64_t)h_stats[3];
   P.S = S;
-  P.block = opt.block_threads;
+  P.S_long = S_long;
   P.key_prefix = DevBuf<int64_t>(S + 1, s);
   TC_CUDA(cudaMemsetAsync(P.key_prefix.get(), 0, sizeof(int64_t), s));
   if (S == 0) {
@@ -536,9 +579,9 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     return;
   }
 
-  // live edges, grouped by head v (stable: position order inside a group)
+  // live edges ordered by (class, head v, position): radix sort is stable
   DevBuf<int64_t> p_live(S, s), p_sorted(S, s);
-  DevBuf<uint32_t> vk(S, s), vk_sorted(S, s);
+  DevBuf<uint32_t> key(S, s), key_sorted(S, s);
   {
     DevBuf<int64_t> nsel(1, s);
     cub::CountingInputIterator<int64_t> it(0);
@@ -547,19 +590,20 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     });
   }
   live.reset();
-  k_gather_head<<<grid_for(S), TPB, 0, s>>>(p_live.get(), S, col, vk.get());
+  k_class_key<<<grid_for(S), TPB, 0, s>>>(p_live.get(), S, col, e_len.get(), opt.long_min, g->bits,
+                                          key.get());
   TC_LAUNCH();
   cub_run(s, [&](void* t, size_t& b) {
-    return cub::DeviceRadixSort::SortPairs(t, b, vk.get(), vk_sorted.get(), p_live.get(),
-                                           p_sorted.get(), S, 0, g->bits, s);
+    return cub::DeviceRadixSort::SortPairs(t, b, key.get(), key_sorted.get(), p_live.get(),
+                                           p_sorted.get(), S, 0, g->bits + 1, s);
   });
-  vk.reset();
+  key.reset();
   p_live.reset();
 
   DevBuf<int32_t> gincl(S, s);
   {
     DevBuf<int32_t> mark(S, s);
-    k_group_mark<<<grid_for(S), TPB, 0, s>>>(vk_sorted.get(), S, mark.get());
+    k_group_mark<<<grid_for(S), TPB, 0, s>>>(key_sorted.get(), S, mark.get());
     TC_LAUNCH();
     cub_run(s, [&](void* t, size_t& b) {
       return cub::DeviceScan::InclusiveSum(t, b, mark.get(), gincl.get(), S, s);
@@ -567,50 +611,58 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   }
   const int64_t G = (int64_t)d2h(gincl.get() + (S - 1), s);
   P.G = G;
+  P.seg_start = DevBuf<int64_t>(S, s);
+  P.seg_len = DevBuf<int32_t>(S, s);
   P.seg_group = DevBuf<int32_t>(S, s);
-  DevBuf<int64_t> seg_len(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
-  P.grp_tmax = DevBuf<int32_t>(G, s);
-  k_seg_group<<<grid_for(S), TPB, 0, s>>>(vk_sorted.get(), p_sorted.get(), gincl.get(), S,
-                                          row_ptr, col, rowid.get(), opt.huge_degree,
-                                          opt.hash_shift, P.seg_group.get(), seg_len.get(),
-                                          grp_row.get(), grp_d.get(), grp_slots.get(),
-                                          P.grp_tmax.get());
+  DevBuf<int64_t> units(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
+  k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted.get(), p_sorted.get(), gincl.get(), S, S_long,
+                                         g->bits, row_ptr, e_lo.get(), e_len.get(),
+                                         opt.huge_degree, opt.table_factor, P.seg_start.get(),
+                                         P.seg_len.get(), P.seg_group.get(), units.get(),
+                                         grp_row.get(), grp_d.get(), grp_slots.get());
   TC_LAUNCH();
   gincl.reset();
-  vk_sorted.reset();
-  rowid.reset();
-  exclusive_prefix(seg_len.get(), S, P.key_prefix.get(), s);
+  key_sorted.reset();
+  p_sorted.reset();
+  e_lo.reset();
+  e_len.reset();
+  exclusive_prefix(units.get(), S, P.key_prefix.get(), s);
   P.ins_prefix = DevBuf<int64_t>(G + 1, s);
   P.slot_prefix = DevBuf<int64_t>(G + 1, s);
   exclusive_prefix(grp_d.get(), G, P.ins_prefix.get(), s);
   exclusive_prefix(grp_slots.get(), G, P.slot_prefix.get(), s);
   P.grp_ibase = DevBuf<int64_t>(G, s);
-  k_grp_ibase<<<grid_for(G), TPB, 0, s>>>(grp_row.get(), P.ins_prefix.get(), G,
-                                          P.grp_ibase.get());
+  k_grp_ibase<<<grid_for(G), TPB, 0, s>>>(grp_row.get(), P.ins_prefix.get(), G, P.grp_ibase.get());
   TC_LAUNCH();
-  P.seg_base = DevBuf<int64_t>(S, s);
   DevBuf<int64_t> cost(S, s), cost_prefix(S + 1, s);
-  k_seg_base_cost<<<grid_for(S), TPB, 0, s>>>(p_sorted.get(), P.key_prefix.get(), seg_len.get(),
-                                              P.seg_group.get(), grp_d.get(), grp_slots.get(),
-                                              S, opt.seg_cost, P.seg_base.get(), cost.get());
+  k_seg_cost<<<grid_for(S), TPB, 0, s>>>(units.get(), P.seg_group.get(), grp_d.get(),
+                                         grp_slots.get(), S, opt.seg_cost, cost.get());
   TC_LAUNCH();
   exclusive_prefix(cost.get(), S, cost_prefix.get(), s);
   cost.reset();
-  seg_len.reset();
+  units.reset();
   grp_row.reset();
   grp_d.reset();
   grp_slots.reset();
-  p_sorted.reset();
-  const int64_t total_cost = d2h(cost_prefix.get() + S, s);
+  int64_t h_cp[3];
+  TC_CUDA(cudaMemcpyAsync(&h_cp[0], cost_prefix.get() + S_long, sizeof(int64_t),
+                          cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaMemcpyAsync(&h_cp[1], cost_prefix.get() + S, sizeof(int64_t), cudaMemcpyDeviceToHost,
+                          s));
+  TC_CUDA(cudaMemcpyAsync(&h_cp[2], P.key_prefix.get() + S, sizeof(int64_t),
+                          cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  const int64_t cost_long = h_cp[0], cost_short = h_cp[1] - h_cp[0];
+  P.units_total = h_cp[2];
 
   // Chunking: halve the chunk cost until the largest chunk's SMEM fits one CTA.
-  const int64_t smem_limit = std::min<int64_t>(max_smem_per_block(), 200 * 1024) - 1024;
+  const int64_t smem_limit = std::min<int64_t>(max_smem_per_block(), 200 * 1024);
   int64_t C = std::max(opt.chunk_cost, 64);
   DevBuf<unsigned long long> mx(1, s);
   for (;;) {
-    const int64_t nc = (total_cost + C - 1) / C;
+    const int64_t nL = (cost_long + C - 1) / C, nS = (cost_short + C - 1) / C, nc = nL + nS;
     P.chunk_seg = DevBuf<int64_t>(nc + 1, s);
-    k_chunk_bounds<<<grid_for(nc + 1), TPB, 0, s>>>(cost_prefix.get(), S, nc, C,
+    k_chunk_bounds<<<grid_for(nc + 1), TPB, 0, s>>>(cost_prefix.get(), S_long, S, nL, nS, C,
                                                     P.chunk_seg.get());
     TC_LAUNCH();
     TC_CUDA(cudaMemsetAsync(mx.get(), 0, sizeof(unsigned long long), s));
@@ -622,6 +674,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
       if (need > smem_limit)
         fail(TC_ERR_UNSUPPORTED, "a chunk's hash tables exceed shared memory (lower huge_degree)");
       P.n_chunks = nc;
+      P.n_long_chunks = nL;
       P.smem_bytes = need;
       break;
     }

@@ -3,28 +3,30 @@
 // What is computed (Fig. 1(b), Fig. 14): for every
 // oriented edge (u,v) of the degree-ordered DAG, |N+(u) ∩ (v,∞) ∩ N+(v)|,
 // the size of the intersection of u's suffix after v with v's out-list;
-// their sum is T.  Edges with an empty suffix or d+(v) = 0 are skipped
-// (exact, C-12); they never reach this kernel (tc_build.cu a6).
+// their sum is T.  The plan (tc_build.cu a6) already trimmed every suffix to
+// [min N+(v), max N+(v)] and dropped the edges left empty (exact, C-12).
 //
-// How.  Live edges are grouped by their head v (the plan's
-// "groups").  A CTA takes one work chunk = a run of consecutive live edges
-// of near-equal cost, which covers a run of groups:
-//   1. it builds, in shared memory, one open-addressing hash table per
-//      group from N+(v) (the GroupTC idea of a table shared by a block of
-//      edges, with TRUST-style hashing, instead of binary
-//      search, which P:369/P:379 name as the cost on large graphs);
-//   2. it streams the suffix keys of all its edges, flattened so that every
-//      lane of every warp handles one key per step regardless of how short
-//      the suffixes are (the flattened walk of P:349 / Alg. 1, with the
-//      `>=` boundary test of DESIGN.md reading C-7), and probes each key in
-//      its group's table;
+// How.  Live edges are grouped by their head v.  A CTA takes
+// one work chunk = a run of consecutive live edges of one class and
+// near-equal cost, covering a run of groups:
+//   1. it builds one hash table per group from N+(v) in shared memory (the
+//      GroupTC idea of a table shared by a block of edges, with the
+//      hashing TRUST uses, instead of binary search, the cost
+//      P:369/P:379 name on large graphs).  Tables are two-choice (cuckoo):
+//      a probe reads exactly two slots, so no warp waits on the longest of
+//      32 probe chains; if an insert ever fails the chunk falls back to
+//      linear probing;
+//   2. it streams the edges' suffix keys and probes the head's table:
+//      LONG class (suffix >= long_min keys): one warp walks one edge in
+//        32-key tiles, coalesced, with warp-uniform bookkeeping;
+//      SHORT class: the keys of all the chunk's edges are flattened over the
+//        lanes (the flattened walk of P:349 / Alg. 1 with the `>=` boundary
+//        of DESIGN.md reading C-7), 32 consecutive keys mapped to their
+//        edges with one SMEM load, a warp OR-reduce and popc;
+//      (degree-bucketed dispatch, the TRUST/Fox idea of P:176/P:254);
 //   3. counts go thread u32 -> warp shuffle -> CTA -> one u64 atomic.
 // Tables whose N+(v) exceeds huge_degree are not staged; their keys are
 // binary-searched in global memory (the TriCore-style probe).
-//
-// The flattened walk maps 32 consecutive flat keys to their segments with
-// one coalesced load of the next 32 segment starts and a warp OR-reduce
-// (__reduce_or_sync) + popc: no per-key search and no per-thread scanning.
 #include <algorithm>
 
 #include "tc_internal.cuh"
@@ -33,89 +35,77 @@ namespace tc {
 namespace {
 
 constexpr int kMaxBlock = 512;
-constexpr int kUnroll = 4;  // 32-key tiles in flight per warp iteration
+constexpr int kUnroll = 4;     // tiles in flight per warp iteration
+constexpr int kMaxKicks = 96;  // cuckoo displacement bound before the linear fallback
 
-__device__ __forceinline__ uint32_t hash_slot(int32_t key, int lg) {
+__device__ __forceinline__ uint32_t hash1(int32_t key, int lg) {
   return ((uint32_t)key * 0x9E3779B1u) >> (32 - lg);
+}
+__device__ __forceinline__ uint32_t hash2(int32_t key, int lg) {
+  return ((uint32_t)key * 0x85EBCA77u + 0x7F4A7C15u) >> (32 - lg);
 }
 
 // Largest s in [s_lo, s_hi) with P[s] <= k (segments are non-empty).
-__device__ __forceinline__ int64_t seg_of(const int64_t* __restrict__ P, int64_t s_lo,
-                                          int64_t s_hi, int64_t k) {
-  int64_t lo = s_lo, hi = s_hi - 1;
+template <class T>
+__device__ __forceinline__ T seg_of(const T* __restrict__ P, T s_lo, T s_hi, T k) {
+  T lo = s_lo, hi = s_hi - 1;
   while (lo < hi) {
-    int64_t mid = (lo + hi + 1) >> 1;
+    T mid = (lo + hi + 1) >> 1;
     if (P[mid] <= k) lo = mid; else hi = mid - 1;
   }
   return lo;
 }
 
-// Warp-cooperative walk over the flat index range [kbeg, kend) of the
-// segments [s_lo, s_hi) whose exclusive prefix is P (P[s_hi] = their end).
-// Every segment must be non-empty.  load(seg, k) returns the element, then
-// proc(seg, elem) consumes it; kUnroll tiles of 32 are loaded before any is
-// processed so that kUnroll independent global loads are in flight per lane.
-template <class Load, class Proc>
-__device__ __forceinline__ void warp_walk(const int64_t* __restrict__ P, int64_t s_lo,
-                                          int64_t s_hi, int64_t kbeg, int64_t kend, Load load,
-                                          Proc proc) {
+// Warp walk over the flat range [kbeg, kend) of the segments [s_lo, s_hi)
+// with (global, int64) exclusive prefix P; used to insert N+(v) keys.
+template <class Proc>
+__device__ __forceinline__ void warp_walk_global(const int64_t* __restrict__ P, int64_t s_lo,
+                                                 int64_t s_hi, int64_t kbeg, int64_t kend,
+                                                 const int32_t* __restrict__ col,
+                                                 const int64_t* __restrict__ base, Proc proc) {
   if (kbeg >= kend) return;
   const int lane = threadIdx.x & 31;
   const unsigned below = (1u << lane) - 1u;
-  int64_t s = seg_of(P, s_lo, s_hi, kbeg);
-  for (int64_t k0 = kbeg; k0 < kend; k0 += 32 * kUnroll) {
-    int64_t seg[kUnroll];
-#pragma unroll
-    for (int u = 0; u < kUnroll; ++u) {
-      const int64_t t0 = k0 + 32 * u;
-      const int64_t j = s + 1 + lane;
-      const int64_t pos = (j <= s_hi) ? P[j] - t0 : 64;
-      const unsigned bit = (pos >= 1 && pos <= 32) ? (1u << (pos - 1)) : 0u;
-      const unsigned M = __reduce_or_sync(0xffffffffu, bit);
-      seg[u] = s + __popc(M & below);
-      s += __popc(M);
-    }
-    int32_t elem[kUnroll];
-#pragma unroll
-    for (int u = 0; u < kUnroll; ++u) {
-      const int64_t k = k0 + 32 * u + lane;
-      elem[u] = (k < kend) ? load(seg[u], k) : 0;
-    }
-#pragma unroll
-    for (int u = 0; u < kUnroll; ++u) {
-      const int64_t k = k0 + 32 * u + lane;
-      if (k < kend) proc(seg[u], elem[u]);
-    }
+  int64_t s = seg_of<int64_t>(P, s_lo, s_hi, kbeg);
+  for (int64_t k0 = kbeg; k0 < kend; k0 += 32) {
+    const int64_t j = s + 1 + lane;
+    const int64_t pos = (j <= s_hi) ? P[j] - k0 : 64;
+    const unsigned bit = (pos >= 1 && pos <= 32) ? (1u << (pos - 1)) : 0u;
+    const unsigned M = __reduce_or_sync(0xffffffffu, bit);
+    const int64_t seg = s + __popc(M & below);
+    s += __popc(M);
+    const int64_t k = k0 + lane;
+    if (k < kend) proc(seg, __ldg(col + __ldg(base + seg) + k));
   }
 }
 
-__device__ __forceinline__ void hash_insert(int* __restrict__ table, int tab, int32_t key) {
+__device__ __forceinline__ bool cuckoo_insert(int* __restrict__ T, int tab, int32_t key) {
+  const int off = tab >> 5, lg = tab & 31;
+  uint32_t pos = hash1(key, lg);
+  for (int i = 0; i < kMaxKicks; ++i) {
+    const int old = atomicExch(&T[off + pos], key);
+    if (old < 0) return true;
+    key = old;  // displaced: move it to its other slot
+    const uint32_t p1 = hash1(key, lg);
+    pos = (pos == p1) ? hash2(key, lg) : p1;
+  }
+  return false;  // `key` is homeless: the chunk rebuilds with linear probing
+}
+
+__device__ __forceinline__ void linear_insert(int* __restrict__ T, int tab, int32_t key) {
   const int off = tab >> 5, lg = tab & 31;
   const uint32_t mask = (1u << lg) - 1u;
-  uint32_t h = hash_slot(key, lg);
+  uint32_t h = hash1(key, lg);
   for (;;) {
-    int prev = atomicCAS(&table[off + h], -1, key);
+    const int prev = atomicCAS(&T[off + h], -1, key);
     if (prev == -1 || prev == key) return;
     h = (h + 1) & mask;
   }
 }
 
-__device__ __forceinline__ unsigned hash_probe(const int* __restrict__ table, int tab,
-                                               int32_t key) {
-  const int off = tab >> 5, lg = tab & 31;
-  const uint32_t mask = (1u << lg) - 1u;
-  uint32_t h = hash_slot(key, lg);
-  for (;;) {
-    const int x = table[off + h];
-    if (x == key) return 1u;
-    if (x < 0) return 0u;
-    h = (h + 1) & mask;
-  }
-}
-
 // Binary search of key in the sorted list col[b, b+d) (huge tables only).
-__device__ __forceinline__ unsigned global_probe(const int32_t* __restrict__ col, int64_t b,
-                                                 int64_t d, int32_t key) {
+__device__ __noinline__ unsigned global_probe(const int32_t* __restrict__ col, int64_t b, int64_t d,
+                                              int32_t key) {
   int64_t lo = b, hi = b + d;
   while (lo < hi) {
     int64_t mid = (lo + hi) >> 1;
@@ -124,68 +114,220 @@ __device__ __forceinline__ unsigned global_probe(const int32_t* __restrict__ col
   return (lo < b + d && __ldg(col + lo) == key) ? 1u : 0u;
 }
 
+// Membership of key in group gl's table (tab = off << 5 | log2 slots, or -1).
+template <bool kLinear>
+__device__ __forceinline__ unsigned probe(const int* __restrict__ T, int tab, int32_t key,
+                                          const PlanView& pv, int64_t g) {
+  if (tab < 0) {
+    const int64_t ib = pv.ins_prefix[g];
+    return global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, key);
+  }
+  const int off = tab >> 5, lg = tab & 31;
+  if (!kLinear) {
+    // a key lives at hash1 or hash2; both reads are issued unconditionally
+    const int x1 = T[off + hash1(key, lg)];
+    const int x2 = T[off + hash2(key, lg)];
+    return (x1 == key) | (x2 == key);
+  }
+  const uint32_t mask = (1u << lg) - 1u;
+  uint32_t h = hash1(key, lg);
+  for (;;) {
+    const int x = T[off + h];
+    if (x == key) return 1u;
+    if (x < 0) return 0u;
+    h = (h + 1) & mask;
+  }
+}
+
+struct ChunkSmem {
+  int64_t* sB;  // long: key start in col; short: start - (chunk-relative first key)
+  int* sA;      // [S+1] long: tile prefix; short: key prefix (chunk-relative)
+  int* sC;      // long: suffix length
+  int* sD;      // group index (chunk-local)
+  int* sInfo;   // [G] table descriptor
+  int* sHash;   // slots
+};
+
+// LONG class: the warp owns tiles [t0, t1) of the chunk; each tile is 32
+// consecutive keys of one edge.  The edge bookkeeping is warp-uniform.
+template <bool kLinear>
+__device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int S, int t0, int t1,
+                                              const PlanView& pv, int64_t ga) {
+  unsigned cnt = 0;
+  if (t0 >= t1) return cnt;
+  const int lane = threadIdx.x & 31;
+  int s = seg_of<int>(c.sA, 0, S, t0);
+  int t_cur = c.sA[s], t_next = c.sA[s + 1];
+  int64_t st = c.sB[s];
+  int len = c.sC[s], gl = c.sD[s];
+  int tab = c.sInfo[gl];
+  for (int t = t0; t < t1; t += kUnroll) {
+    int64_t addr[kUnroll];
+    bool ok[kUnroll];
+    int tabu[kUnroll], glu[kUnroll];
+#pragma unroll
+    for (int u = 0; u < kUnroll; ++u) {
+      const int tt = t + u;
+      ok[u] = false;
+      addr[u] = 0;
+      tabu[u] = tab;
+      glu[u] = gl;
+      if (tt < t1) {
+        while (tt >= t_next) {  // warp-uniform: next edge of the chunk
+          ++s;
+          t_cur = t_next;
+          t_next = c.sA[s + 1];
+          st = c.sB[s];
+          len = c.sC[s];
+          gl = c.sD[s];
+          tab = c.sInfo[gl];
+        }
+        const int kl = ((tt - t_cur) << 5) + lane;
+        ok[u] = kl < len;
+        addr[u] = st + kl;
+        tabu[u] = tab;
+        glu[u] = gl;
+      }
+    }
+    int32_t key[kUnroll];
+#pragma unroll
+    for (int u = 0; u < kUnroll; ++u) key[u] = ok[u] ? __ldg(pv.col + addr[u]) : 0;
+#pragma unroll
+    for (int u = 0; u < kUnroll; ++u)
+      if (ok[u]) cnt += probe<kLinear>(c.sHash, tabu[u], key[u], pv, ga + glu[u]);
+  }
+  return cnt;
+}
+
+// SHORT class: the warp owns the flat keys [k0w, k1w) of the chunk.
+template <bool kLinear>
+__device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0w, int k1w,
+                                               const PlanView& pv, int64_t ga) {
+  unsigned cnt = 0;
+  if (k0w >= k1w) return cnt;
+  const int lane = threadIdx.x & 31;
+  const unsigned below = (1u << lane) - 1u;
+  int s = seg_of<int>(c.sA, 0, S, k0w);
+  for (int k0 = k0w; k0 < k1w; k0 += 32 * kUnroll) {
+    int seg[kUnroll];
+#pragma unroll
+    for (int u = 0; u < kUnroll; ++u) {
+      const int t0 = k0 + 32 * u;
+      const int j = s + 1 + lane;
+      const int pos = (j <= S) ? c.sA[j] - t0 : 64;
+      const unsigned bit = (pos >= 1 && pos <= 32) ? (1u << (pos - 1)) : 0u;
+      const unsigned M = __reduce_or_sync(0xffffffffu, bit);
+      seg[u] = s + __popc(M & below);
+      s += __popc(M);
+    }
+    int32_t key[kUnroll];
+    int gl[kUnroll];
+#pragma unroll
+    for (int u = 0; u < kUnroll; ++u) {
+      const int k = k0 + 32 * u + lane;
+      key[u] = 0;
+      gl[u] = 0;
+      if (k < k1w) {
+        key[u] = __ldg(pv.col + c.sB[seg[u]] + k);
+        gl[u] = c.sD[seg[u]];
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kUnroll; ++u) {
+      const int k = k0 + 32 * u + lane;
+      if (k < k1w) cnt += probe<kLinear>(c.sHash, c.sInfo[gl[u]], key[u], pv, ga + gl[u]);
+    }
+  }
+  return cnt;
+}
+
 __global__ void __launch_bounds__(kMaxBlock)
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
             unsigned long long* __restrict__ out) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ unsigned long long red[kMaxBlock / 32];
+  __shared__ int sFail;
   const int warp = threadIdx.x >> 5, nw = blockDim.x >> 5, lane = threadIdx.x & 31;
   unsigned long long acc = 0;
 
-  for (int64_t c = c_begin + blockIdx.x; c < c_end; c += gridDim.x) {
-    const int64_t sa = max(pv.chunk_seg[c], e_begin), sb = min(pv.chunk_seg[c + 1], e_end);
+  for (int64_t cix = c_begin + blockIdx.x; cix < c_end; cix += gridDim.x) {
+    const int64_t sa = max(pv.chunk_seg[cix], e_begin), sb = min(pv.chunk_seg[cix + 1], e_end);
     if (sa >= sb) continue;  // uniform over the CTA
+    const bool is_long = cix < pv.n_long_chunks;
+    const int S = (int)(sb - sa);
     const int64_t ga = pv.seg_group[sa], gb = (int64_t)pv.seg_group[sb - 1] + 1;
     const int G = (int)(gb - ga);
     const int64_t slot0 = pv.slot_prefix[ga];
     const int nslots = (int)(pv.slot_prefix[gb] - slot0);
-    int2* sInfo = reinterpret_cast<int2*>(smem);  // {tab = off << 5 | log2(slots) or -1, tmax}
-    int* sHash = reinterpret_cast<int*>(sInfo + G);
+    ChunkSmem c;
+    c.sB = reinterpret_cast<int64_t*>(smem);
+    c.sA = reinterpret_cast<int*>(c.sB + S);
+    c.sC = c.sA + S + 1;
+    c.sD = c.sC + S;
+    c.sInfo = c.sD + S;
+    c.sHash = c.sInfo + G;
 
-    // 1. table descriptors + empty slots
-    for (int i = threadIdx.x; i < G; i += blockDim.x) {
-      const int64_t g = ga + i;
-      const int64_t sp = pv.slot_prefix[g], ns = pv.slot_prefix[g + 1] - sp;
-      const int tab = ns > 0 ? (((int)(sp - slot0)) << 5) | (31 - __clz((int)ns)) : -1;
-      sInfo[i] = make_int2(tab, pv.grp_tmax[g]);
+    // 1. stage the chunk's edges and table descriptors; empty slots
+    const int64_t kp0 = pv.key_prefix[sa];
+    for (int i = threadIdx.x; i <= S; i += blockDim.x) {
+      const int64_t sg = sa + i;
+      const int rel = (int)(pv.key_prefix[sg] - kp0);
+      c.sA[i] = is_long ? (rel >> 5) : rel;
+      if (i < S) {
+        c.sB[i] = is_long ? pv.seg_start[sg] : pv.seg_start[sg] - rel;
+        c.sC[i] = pv.seg_len[sg];
+        c.sD[i] = pv.seg_group[sg] - (int)ga;
+      }
     }
-    for (int i = threadIdx.x; i < nslots; i += blockDim.x) sHash[i] = -1;
+    for (int i = threadIdx.x; i < G; i += blockDim.x) {
+      const int64_t sp = pv.slot_prefix[ga + i], ns = pv.slot_prefix[ga + i + 1] - sp;
+      c.sInfo[i] = ns > 0 ? (((int)(sp - slot0)) << 5) | (31 - __clz((int)ns)) : -1;
+    }
+    for (int i = threadIdx.x; i < nslots; i += blockDim.x) c.sHash[i] = -1;
+    if (threadIdx.x == 0) sFail = 0;
     __syncthreads();
 
     // 2. hash N+(v) of every group touched by the chunk
-    {
-      const int64_t kb = pv.ins_prefix[ga], len = pv.ins_prefix[gb] - kb;
-      warp_walk(
-          pv.ins_prefix, ga, gb, kb + len * warp / nw, kb + len * (warp + 1) / nw,
-          [&](int64_t g, int64_t k) { return __ldg(pv.col + pv.grp_ibase[g] + k); },
-          [&](int64_t g, int32_t key) {
-            const int tab = sInfo[g - ga].x;
-            if (tab >= 0) hash_insert(sHash, tab, key);
-          });
+    bool linear = pv.probe_mode == 1;
+    const int64_t ib = pv.ins_prefix[ga], ilen = pv.ins_prefix[gb] - ib;
+    const int64_t iw0 = ib + ilen * warp / nw, iw1 = ib + ilen * (warp + 1) / nw;
+    if (linear) {
+      warp_walk_global(pv.ins_prefix, ga, gb, iw0, iw1, pv.col, pv.grp_ibase,
+                       [&](int64_t g, int32_t key) {
+                         const int tab = c.sInfo[g - ga];
+                         if (tab >= 0) linear_insert(c.sHash, tab, key);
+                       });
+    } else {
+      bool ok = true;
+      warp_walk_global(pv.ins_prefix, ga, gb, iw0, iw1, pv.col, pv.grp_ibase,
+                       [&](int64_t g, int32_t key) {
+                         const int tab = c.sInfo[g - ga];
+                         if (tab >= 0 && !cuckoo_insert(c.sHash, tab, key)) ok = false;
+                       });
+      if (!ok) sFail = 1;
     }
     __syncthreads();
-
-    // 3. stream the suffix keys of the chunk's edges, probe the head's table
-    {
-      unsigned cnt = 0;
-      const int64_t kb = pv.key_prefix[sa], len = pv.key_prefix[sb] - kb;
-      warp_walk(
-          pv.key_prefix, sa, sb, kb + len * warp / nw, kb + len * (warp + 1) / nw,
-          [&](int64_t s, int64_t k) { return __ldg(pv.col + __ldg(pv.seg_base + s) + k); },
-          [&](int64_t s, int32_t key) {
-            const int gl = __ldg(pv.seg_group + s) - (int)ga;
-            const int2 info = sInfo[gl];
-            if (key > info.y) return;  // beyond max N+(v): cannot match
-            if (info.x >= 0) {
-              cnt += hash_probe(sHash, info.x, key);
-            } else {
-              const int64_t g = ga + gl;
-              const int64_t ib = pv.ins_prefix[g];
-              cnt += global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, key);
-            }
-          });
-      acc += cnt;
+    if (!linear && sFail) {  // uniform: rebuild this chunk's tables with linear probing
+      linear = true;
+      for (int i = threadIdx.x; i < nslots; i += blockDim.x) c.sHash[i] = -1;
+      __syncthreads();
+      warp_walk_global(pv.ins_prefix, ga, gb, iw0, iw1, pv.col, pv.grp_ibase,
+                       [&](int64_t g, int32_t key) {
+                         const int tab = c.sInfo[g - ga];
+                         if (tab >= 0) linear_insert(c.sHash, tab, key);
+                       });
+      __syncthreads();
     }
+
+    // 3. stream the chunk's suffix keys and probe the heads' tables
+    const int NU = c.sA[S];
+    const int w0 = (int)((int64_t)NU * warp / nw), w1 = (int)((int64_t)NU * (warp + 1) / nw);
+    unsigned cnt;
+    if (is_long)
+      cnt = linear ? walk_long<true>(c, S, w0, w1, pv, ga) : walk_long<false>(c, S, w0, w1, pv, ga);
+    else
+      cnt = linear ? walk_short<true>(c, S, w0, w1, pv, ga) : walk_short<false>(c, S, w0, w1, pv, ga);
+    acc += cnt;
     __syncthreads();  // SMEM is rebuilt by the next chunk
   }
 
@@ -243,13 +385,15 @@ void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_b
   PlanView pv;
   pv.col = g->col.get();
   pv.key_prefix = P.key_prefix.get();
-  pv.seg_base = P.seg_base.get();
+  pv.seg_start = P.seg_start.get();
+  pv.seg_len = P.seg_len.get();
   pv.seg_group = P.seg_group.get();
   pv.ins_prefix = P.ins_prefix.get();
   pv.grp_ibase = P.grp_ibase.get();
   pv.slot_prefix = P.slot_prefix.get();
-  pv.grp_tmax = P.grp_tmax.get();
   pv.chunk_seg = P.chunk_seg.get();
+  pv.n_long_chunks = P.n_long_chunks;
+  pv.probe_mode = P.opt.probe_mode;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c_end - c_begin, P.grid));
   k_count<<<grid, P.block, (size_t)P.smem_bytes, s>>>(pv, c_begin, c_end, e_begin, e_end, d_out);
   TC_LAUNCH();

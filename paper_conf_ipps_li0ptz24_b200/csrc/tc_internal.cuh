@@ -66,38 +66,54 @@ struct Options {
   int seg_cost = 4;
   int huge_degree = 8192;
   int block_threads = 512;
-  int hash_shift = 1;
+  int table_factor = 3;
+  int long_min = 32;
+  int probe_mode = 0;
 };
 Options resolve_options(const tc_options* o);
 
 // ---------------------------------------------------------------- plan
 // The dispatch plan.  Units:
-//   segment s  = one LIVE oriented edge (u,v) (suffix of N+(u) after v is
-//                non-empty and d+(v) > 0), in (v, position) order; its keys
-//                are col[p+1 .. row_end(u)), the suffix of P:359.
-//   group g    = one distinct head vertex v over the segments; its table is
-//                N+(v) = col[row_ptr[v] .. row_ptr[v+1]).
-//   flat key k = global index over all segments' keys, k in
-//                [key_prefix[s], key_prefix[s+1]) belongs to s and lives at
-//                col[seg_base[s] + k].
-//   chunk c    = segments [chunk_seg[c], chunk_seg[c+1]) of near-equal cost.
+//   segment s  = one LIVE oriented edge (u,v): its keys are the suffix of
+//                N+(u) after v trimmed to [min N+(v), max N+(v)]
+//                (keys outside cannot match), non-empty, stored as
+//                col[seg_start[s] .. seg_start[s] + seg_len[s]).
+//   class      = LONG (seg_len >= long_min: one warp walks the segment in
+//                32-key tiles) or SHORT (keys of many segments flattened
+//                over the lanes).  Segments [0, S_long) are long, [S_long,
+//                S) short; inside a class they are ordered by (v, position).
+//   group g    = one run of segments of one class with the same head v;
+//                its table is N+(v) = col[row_ptr[v] .. row_ptr[v+1]).
+//   work unit  = a key lane: a long segment has 32*ceil(len/32) (its tiles),
+//                a short one len; key_prefix is their exclusive prefix.
+//   chunk c    = segments [chunk_seg[c], chunk_seg[c+1]) of one class and
+//                near-equal cost; chunks [0, n_long_chunks) are long.
 struct PlanView {
   const int32_t* col;
-  const int64_t* key_prefix;   // [S+1]
-  const int64_t* seg_base;     // [S]  = (p+1) - key_prefix[s]
+  const int64_t* key_prefix;   // [S+1] work-unit prefix
+  const int64_t* seg_start;    // [S]
+  const int32_t* seg_len;      // [S]
   const int32_t* seg_group;    // [S]
   const int64_t* ins_prefix;   // [G+1] prefix of d+(v)
   const int64_t* grp_ibase;    // [G]  = row_ptr[v] - ins_prefix[g]
   const int64_t* slot_prefix;  // [G+1] prefix of hash slots (0 for huge groups)
-  const int32_t* grp_tmax;     // [G]  max element of N+(v)
   const int64_t* chunk_seg;    // [C+1]
+  int64_t n_long_chunks;
+  int probe_mode;
 };
+
+// SMEM a chunk needs (bytes): per segment staging + per group descriptor +
+// hash slots.  Shared by the plan (sizing) and the kernel (layout).
+__host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_t slots) {
+  return 4 * (S + 1) + 8 * S + 4 * S + 4 * S + 4 * G + 4 * slots + 64;
+}
 
 struct Plan {
   Options opt;
-  int64_t S = 0, G = 0, n_chunks = 0, keys_total = 0;
-  DevBuf<int64_t> key_prefix, seg_base, ins_prefix, grp_ibase, slot_prefix, chunk_seg;
-  DevBuf<int32_t> seg_group, grp_tmax;
+  int64_t S = 0, S_long = 0, G = 0, n_chunks = 0, n_long_chunks = 0, keys_total = 0;
+  int64_t units_total = 0;
+  DevBuf<int64_t> key_prefix, seg_start, ins_prefix, grp_ibase, slot_prefix, chunk_seg;
+  DevBuf<int32_t> seg_len, seg_group;
   std::vector<int64_t> h_chunk_seg;
   int64_t smem_bytes = 0;
   int grid = 0, block = 0;

@@ -106,8 +106,11 @@ def test_chung_lu_small(tc):
 @pytest.mark.parametrize("opts", [
     dict(chunk_cost=64), dict(chunk_cost=256), dict(chunk_cost=4096), dict(chunk_cost=1 << 20),
     dict(block_threads=64), dict(block_threads=128), dict(block_threads=256),
-    dict(seg_cost=1), dict(seg_cost=64), dict(hash_shift=0), dict(hash_shift=3),
+    dict(seg_cost=1), dict(seg_cost=64), dict(table_factor=2), dict(table_factor=16),
     dict(huge_degree=1), dict(huge_degree=16), dict(huge_degree=16, chunk_cost=64),
+    dict(long_min=1), dict(long_min=8), dict(long_min=1 << 30), dict(long_min=1 << 30, chunk_cost=64),
+    dict(probe_mode=1), dict(probe_mode=1, long_min=1), dict(probe_mode=1, long_min=1 << 30),
+    dict(table_factor=2, chunk_cost=1 << 20),
 ])
 def test_plan_options_never_change_count(tc, opts):
     src, dst, n = tcgen.rmat(13, 16, 11)
@@ -270,6 +273,24 @@ def test_k3000_exceeds_32_bits(tc):
     (src, dst, n), t = graphs.complete(3000)
     assert t == comb(3000, 3) > 2**32
     assert gpu_count(tc, src, dst, n) == t
+
+
+def test_classes_partition_the_edges(tc):
+    """long_min only moves edges between the two classes (C-10 analogue)."""
+    src, dst, n = tcgen.rmat(14, 16, 12)
+    t = oracle.triangles(src, dst, n)
+    for lm in (1, 4, 32, 200, 1 << 30):
+        with tc.build_csr(dev(src), dev(dst), n, options=dict(long_min=lm)) as g:
+            assert g.count() == t, lm
+
+
+def test_lattice_trim_drops_edges(tc):
+    """C5-like lattice: trimming the suffix to [min N+(v), max N+(v)] leaves
+    far fewer live edges than m, and the count is unchanged."""
+    src, dst, n = tcgen.lattice(300, 4)
+    with tc.build_csr(dev(src), dev(dst), n) as g:
+        assert g.count() == oracle.triangles(src, dst, n)
+        assert g.m_live < 0.5 * g.m
 
 
 def test_huge_table_path_on_clique(tc):
