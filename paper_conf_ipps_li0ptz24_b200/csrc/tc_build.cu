@@ -13,6 +13,9 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 
 #include "tc_internal.cuh"
 
@@ -39,6 +42,27 @@ void cub_run(cudaStream_t s, F f) {
   DevBuf<char> tmp(bytes ? bytes : 16, s);
   TC_CUDA(f(tmp.get(), bytes));
 }
+
+// TC_VERBOSE=1: plan sub-phase trace on stderr (host clock after a stream sync).
+struct Trace {
+  bool on;
+  cudaStream_t s;
+  std::chrono::steady_clock::time_point t0;
+  explicit Trace(cudaStream_t st) : on(std::getenv("TC_VERBOSE") != nullptr), s(st) {
+    if (on) {
+      cudaStreamSynchronize(s);
+      t0 = std::chrono::steady_clock::now();
+    }
+  }
+  void operator()(const char* what) {
+    if (!on) return;
+    cudaStreamSynchronize(s);
+    auto t = std::chrono::steady_clock::now();
+    fprintf(stderr, "[tc] %-28s %8.2f ms\n", what,
+            std::chrono::duration<double, std::milli>(t - t0).count());
+    t0 = t;
+  }
+};
 
 template <class T>
 T d2h(const T* d, cudaStream_t s) {
@@ -319,10 +343,10 @@ __global__ void k_grp_ibase(const int64_t* __restrict__ grp_row,
 }
 
 // Chunks never straddle the class boundary S_long: long chunk c < nL starts
-// at the first segment whose cost prefix reaches c*C; short chunk nL + j at
-// the first segment of [S_long, S) whose prefix reaches prefix[S_long] + j*C.
+// at the first segment whose cost prefix reaches c*CL; short chunk nL + j at
+// the first segment of [S_long, S) whose prefix reaches prefix[S_long] + j*CS.
 __global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t S_long,
-                               int64_t S, int64_t nL, int64_t nS, int64_t C,
+                               int64_t S, int64_t nL, int64_t nS, int64_t CL, int64_t CS,
                                int64_t* __restrict__ chunk_seg) {
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= nL + nS;
        c += (int64_t)gridDim.x * blockDim.x) {
@@ -334,11 +358,11 @@ __global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t 
     if (c < nL) {
       lo = 0;
       hi = S_long;
-      target = c * C;
+      target = c * CL;
     } else {
       lo = S_long;
       hi = S;
-      target = cost_prefix[S_long] + (c - nL) * C;
+      target = cost_prefix[S_long] + (c - nL) * CS;
     }
     while (lo < hi) {  // first s with prefix[s] >= target
       int64_t mid = (lo + hi) >> 1;
@@ -348,23 +372,28 @@ __global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t 
   }
 }
 
-__global__ void k_chunk_smem(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
+__global__ void k_chunk_smem(const int64_t* __restrict__ chunk_seg, int64_t n_chunks, int64_t nL,
                              const int32_t* __restrict__ seg_group,
                              const int64_t* __restrict__ slot_prefix,
-                             unsigned long long* out) {
+                             unsigned long long* out) {  // out[0] long max, out[1] short max
   typedef cub::BlockReduce<unsigned long long, TPB> BR;
   __shared__ typename BR::TempStorage tmp;
-  unsigned long long mx = 0;
+  unsigned long long mx[2] = {0, 0};
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n_chunks;
        c += (int64_t)gridDim.x * blockDim.x) {
     const int64_t sa = chunk_seg[c], sb = chunk_seg[c + 1];
     if (sa >= sb) continue;
     const int64_t ga = seg_group[sa], gb = (int64_t)seg_group[sb - 1] + 1;
     const int64_t b = chunk_smem_bytes(sb - sa, gb - ga, slot_prefix[gb] - slot_prefix[ga]);
-    mx = max(mx, (unsigned long long)b);
+    mx[c >= nL] = max(mx[c >= nL], (unsigned long long)b);
   }
-  unsigned long long r = BR(tmp).Reduce(mx, cub::Max());
-  if (threadIdx.x == 0) atomicMax(out, r);
+  unsigned long long r0 = BR(tmp).Reduce(mx[0], cub::Max());
+  __syncthreads();
+  unsigned long long r1 = BR(tmp).Reduce(mx[1], cub::Max());
+  if (threadIdx.x == 0) {
+    atomicMax(&out[0], r0);
+    atomicMax(&out[1], r1);
+  }
 }
 
 // exclusive prefix of `in` (length n) into out[0..n] (out[0] = 0, out[n] = total)
@@ -548,6 +577,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   const int64_t m = g->m, n = g->n;
   const int64_t* row_ptr = g->row_ptr.get();
   const int32_t* col = g->col.get();
+  Trace tr(s);
   DevBuf<unsigned long long> stats(4, s);
   TC_CUDA(cudaMemsetAsync(stats.get(), 0, 4 * sizeof(unsigned long long), s));
   DevBuf<int32_t> rowid(std::max<int64_t>(m, 1), s), e_len(std::max<int64_t>(m, 1), s);
@@ -561,6 +591,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     TC_LAUNCH();
   }
   rowid.reset();
+  tr("rowid + edge trim");
   unsigned long long h_stats[4];
   TC_CUDA(cudaMemcpyAsync(h_stats, stats.get(), sizeof(h_stats), cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));
@@ -599,6 +630,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   });
   key.reset();
   p_live.reset();
+  tr("select + class sort");
 
   DevBuf<int32_t> gincl(S, s);
   {
@@ -653,34 +685,54 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
                           cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));
   const int64_t cost_long = h_cp[0], cost_short = h_cp[1] - h_cp[0];
+  tr("groups + prefixes + costs");
   P.units_total = h_cp[2];
 
-  // Chunking: halve the chunk cost until the largest chunk's SMEM fits one CTA.
-  const int64_t smem_limit = std::min<int64_t>(max_smem_per_block(), 200 * 1024);
-  int64_t C = std::max(opt.chunk_cost, 64);
-  DevBuf<unsigned long long> mx(1, s);
+  // Chunking, per class: long chunks start 4x larger (their SMEM is one or
+  // two tables plus a few edges).  A class's chunk cost is halved while its
+  // largest chunk needs more SMEM than the 3-CTAs-per-SM target (down to 1024
+  // units), then while it exceeds what one CTA can have at all.
+  const int64_t hard = std::min<int64_t>(max_smem_per_block(), 200 * 1024);
+  const int64_t soft = std::min<int64_t>(hard, 72 * 1024);
+  int64_t CL = std::max<int64_t>(4ll * opt.chunk_cost, 64), CS = std::max<int64_t>(opt.chunk_cost, 64);
+  DevBuf<unsigned long long> mx(2, s);
   for (;;) {
-    const int64_t nL = (cost_long + C - 1) / C, nS = (cost_short + C - 1) / C, nc = nL + nS;
+    const int64_t nL = (cost_long + CL - 1) / CL, nS = (cost_short + CS - 1) / CS, nc = nL + nS;
     P.chunk_seg = DevBuf<int64_t>(nc + 1, s);
-    k_chunk_bounds<<<grid_for(nc + 1), TPB, 0, s>>>(cost_prefix.get(), S_long, S, nL, nS, C,
+    k_chunk_bounds<<<grid_for(nc + 1), TPB, 0, s>>>(cost_prefix.get(), S_long, S, nL, nS, CL, CS,
                                                     P.chunk_seg.get());
     TC_LAUNCH();
-    TC_CUDA(cudaMemsetAsync(mx.get(), 0, sizeof(unsigned long long), s));
-    k_chunk_smem<<<grid_for(nc), TPB, 0, s>>>(P.chunk_seg.get(), nc, P.seg_group.get(),
+    TC_CUDA(cudaMemsetAsync(mx.get(), 0, 2 * sizeof(unsigned long long), s));
+    k_chunk_smem<<<grid_for(nc), TPB, 0, s>>>(P.chunk_seg.get(), nc, nL, P.seg_group.get(),
                                               P.slot_prefix.get(), mx.get());
     TC_LAUNCH();
-    const int64_t need = (int64_t)d2h(mx.get(), s);
-    if (need <= smem_limit || C <= 64) {
-      if (need > smem_limit)
-        fail(TC_ERR_UNSUPPORTED, "a chunk's hash tables exceed shared memory (lower huge_degree)");
-      P.n_chunks = nc;
-      P.n_long_chunks = nL;
-      P.smem_bytes = need;
-      break;
-    }
-    C >>= 1;
+    unsigned long long need[2];
+    TC_CUDA(cudaMemcpyAsync(need, mx.get(), sizeof(need), cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaStreamSynchronize(s));
+    auto shrink = [&](int64_t& C, int64_t nd) {
+      if ((nd > (unsigned long long)soft && C > 1024) || (nd > (unsigned long long)hard && C > 64)) {
+        C >>= 1;
+        return true;
+      }
+      return false;
+    };
+    if (tr.on)
+      fprintf(stderr, "[tc]   chunks CL=%lld CS=%lld nL=%lld nS=%lld smem long %llu short %llu\n",
+              (long long)CL, (long long)CS, (long long)nL, (long long)nS, need[0], need[1]);
+    const bool again_l = shrink(CL, (int64_t)need[0]);
+    const bool again_s = shrink(CS, (int64_t)need[1]);
+    if (again_l || again_s) continue;
+    const int64_t nd = (int64_t)std::max(need[0], need[1]);
+    if (nd > hard)
+      fail(TC_ERR_UNSUPPORTED, "a chunk's hash tables exceed shared memory (lower huge_degree)");
+    P.n_chunks = nc;
+    P.n_long_chunks = nL;
+    P.smem_bytes = nd;
+    break;
   }
-  P.opt.chunk_cost = (int)C;
+  P.chunk_cost_long = CL;
+  P.chunk_cost_short = CS;
+  tr("chunking");
   P.h_chunk_seg.resize(P.n_chunks + 1);
   TC_CUDA(cudaMemcpyAsync(P.h_chunk_seg.data(), P.chunk_seg.get(),
                           sizeof(int64_t) * (P.n_chunks + 1), cudaMemcpyDeviceToHost, s));
@@ -688,6 +740,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   const int occ = count_occupancy(P.block, P.smem_bytes);
   if (occ < 1) fail(TC_ERR_UNSUPPORTED, "count kernel cannot launch with this SMEM/block size");
   P.grid = (int)std::min<int64_t>(P.n_chunks, (int64_t)occ * num_sms());
+  tr("chunk copy + occupancy");
 }
 
 }  // namespace tc

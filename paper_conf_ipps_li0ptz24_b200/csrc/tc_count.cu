@@ -38,11 +38,13 @@ constexpr int kMaxBlock = 512;
 constexpr int kUnroll = 4;     // tiles in flight per warp iteration
 constexpr int kMaxKicks = 96;  // cuckoo displacement bound before the linear fallback
 
-__device__ __forceinline__ uint32_t hash1(int32_t key, int lg) {
-  return ((uint32_t)key * 0x9E3779B1u) >> (32 - lg);
+// Table descriptor tab = (slot offset << 5) | sh with sh = 32 - log2(slots):
+// the slot of a key is the top log2(slots) bits of a multiplicative hash.
+__device__ __forceinline__ uint32_t hash1(int32_t key, int sh) {
+  return ((uint32_t)key * 0x9E3779B1u) >> sh;
 }
-__device__ __forceinline__ uint32_t hash2(int32_t key, int lg) {
-  return ((uint32_t)key * 0x85EBCA77u + 0x7F4A7C15u) >> (32 - lg);
+__device__ __forceinline__ uint32_t hash2(int32_t key, int sh) {
+  return ((uint32_t)key * 0x85EBCA77u + 0x7F4A7C15u) >> sh;
 }
 
 // Largest s in [s_lo, s_hi) with P[s] <= k (segments are non-empty).
@@ -80,22 +82,22 @@ __device__ __forceinline__ void warp_walk_global(const int64_t* __restrict__ P, 
 }
 
 __device__ __forceinline__ bool cuckoo_insert(int* __restrict__ T, int tab, int32_t key) {
-  const int off = tab >> 5, lg = tab & 31;
-  uint32_t pos = hash1(key, lg);
+  const int off = tab >> 5, sh = tab & 31;
+  uint32_t pos = hash1(key, sh);
   for (int i = 0; i < kMaxKicks; ++i) {
     const int old = atomicExch(&T[off + pos], key);
     if (old < 0) return true;
     key = old;  // displaced: move it to its other slot
-    const uint32_t p1 = hash1(key, lg);
-    pos = (pos == p1) ? hash2(key, lg) : p1;
+    const uint32_t p1 = hash1(key, sh);
+    pos = (pos == p1) ? hash2(key, sh) : p1;
   }
   return false;  // `key` is homeless: the chunk rebuilds with linear probing
 }
 
 __device__ __forceinline__ void linear_insert(int* __restrict__ T, int tab, int32_t key) {
-  const int off = tab >> 5, lg = tab & 31;
-  const uint32_t mask = (1u << lg) - 1u;
-  uint32_t h = hash1(key, lg);
+  const int off = tab >> 5, sh = tab & 31;
+  const uint32_t mask = 0xffffffffu >> sh;
+  uint32_t h = hash1(key, sh);
   for (;;) {
     const int prev = atomicCAS(&T[off + h], -1, key);
     if (prev == -1 || prev == key) return;
@@ -114,29 +116,37 @@ __device__ __noinline__ unsigned global_probe(const int32_t* __restrict__ col, i
   return (lo < b + d && __ldg(col + lo) == key) ? 1u : 0u;
 }
 
-// Membership of key in group gl's table (tab = off << 5 | log2 slots, or -1).
+// Membership of key in one SMEM table: T = first slot, sh = 32 - log2(slots).
+// Keys are >= 0, empty slots hold -1, and the sentinel -2 (padding lanes)
+// never matches and always terminates.
 template <bool kLinear>
-__device__ __forceinline__ unsigned probe(const int* __restrict__ T, int tab, int32_t key,
-                                          const PlanView& pv, int64_t g) {
-  if (tab < 0) {
-    const int64_t ib = pv.ins_prefix[g];
-    return global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, key);
-  }
-  const int off = tab >> 5, lg = tab & 31;
+__device__ __forceinline__ unsigned table_probe(const int* __restrict__ T, int sh, int32_t key) {
   if (!kLinear) {
-    // a key lives at hash1 or hash2; both reads are issued unconditionally
-    const int x1 = T[off + hash1(key, lg)];
-    const int x2 = T[off + hash2(key, lg)];
+    // two-choice table: a key lives at hash1 or hash2; both reads are issued
+    const int x1 = T[hash1(key, sh)];
+    const int x2 = T[hash2(key, sh)];
     return (x1 == key) | (x2 == key);
   }
-  const uint32_t mask = (1u << lg) - 1u;
-  uint32_t h = hash1(key, lg);
+  const uint32_t mask = 0xffffffffu >> sh;
+  uint32_t h = hash1(key, sh);
   for (;;) {
-    const int x = T[off + h];
+    const int x = T[h];
     if (x == key) return 1u;
     if (x < 0) return 0u;
     h = (h + 1) & mask;
   }
+}
+
+// Membership through a descriptor (tab = off << 5 | sh, or -1 = huge table
+// of group g, probed by binary search in global memory).
+template <bool kLinear, bool kHuge>
+__device__ __forceinline__ unsigned probe(const int* __restrict__ H, int tab, int32_t key,
+                                          const PlanView& pv, int64_t g) {
+  if (kHuge && tab < 0) {
+    const int64_t ib = pv.ins_prefix[g];
+    return global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, key);
+  }
+  return table_probe<kLinear>(H + (tab >> 5), tab & 31, key);
 }
 
 struct ChunkSmem {
@@ -149,58 +159,44 @@ struct ChunkSmem {
 };
 
 // LONG class: the warp owns tiles [t0, t1) of the chunk; each tile is 32
-// consecutive keys of one edge.  The edge bookkeeping is warp-uniform.
-template <bool kLinear>
+// consecutive keys of one edge.  The warp walks edge by edge (warp-uniform
+// bookkeeping); inside an edge, lane l reads keys l, l+32, ... through one
+// pointer with immediate offsets, kUnroll tiles in flight; lanes past the
+// end carry the never-matching sentinel so the probes run unpredicated.
+template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int S, int t0, int t1,
                                               const PlanView& pv, int64_t ga) {
   unsigned cnt = 0;
   if (t0 >= t1) return cnt;
   const int lane = threadIdx.x & 31;
   int s = seg_of<int>(c.sA, 0, S, t0);
-  int t_cur = c.sA[s], t_next = c.sA[s + 1];
-  int64_t st = c.sB[s];
-  int len = c.sC[s], gl = c.sD[s];
-  int tab = c.sInfo[gl];
-  for (int t = t0; t < t1; t += kUnroll) {
-    int64_t addr[kUnroll];
-    bool ok[kUnroll];
-    int tabu[kUnroll], glu[kUnroll];
-#pragma unroll
-    for (int u = 0; u < kUnroll; ++u) {
-      const int tt = t + u;
-      ok[u] = false;
-      addr[u] = 0;
-      tabu[u] = tab;
-      glu[u] = gl;
-      if (tt < t1) {
-        while (tt >= t_next) {  // warp-uniform: next edge of the chunk
-          ++s;
-          t_cur = t_next;
-          t_next = c.sA[s + 1];
-          st = c.sB[s];
-          len = c.sC[s];
-          gl = c.sD[s];
-          tab = c.sInfo[gl];
-        }
-        const int kl = ((tt - t_cur) << 5) + lane;
-        ok[u] = kl < len;
-        addr[u] = st + kl;
-        tabu[u] = tab;
-        glu[u] = gl;
-      }
+  for (int t = t0; t < t1; ++s) {
+    const int ts = c.sA[s], te = min(c.sA[s + 1], t1);
+    const int done = (t - ts) << 5;                             // keys of this edge before tile t
+    const int lim = min(c.sC[s] - done, (te - t) << 5) - lane;  // lane's keys: 32*i < lim
+    const int32_t* __restrict__ p = pv.col + c.sB[s] + done + lane;
+    const int gl = c.sD[s];
+    const int tab = c.sInfo[gl];
+    t = te;
+    if (kHuge && tab < 0) {
+      for (int i = 0; i < lim; i += 32) cnt += probe<kLinear, true>(c.sHash, tab, __ldg(p + i), pv, ga + gl);
+      continue;
     }
-    int32_t key[kUnroll];
+    const int* __restrict__ T = c.sHash + (tab >> 5);
+    const int sh = tab & 31;
+    for (int i = 0; i < lim; i += 32 * kUnroll) {
+      int32_t key[kUnroll];
 #pragma unroll
-    for (int u = 0; u < kUnroll; ++u) key[u] = ok[u] ? __ldg(pv.col + addr[u]) : 0;
+      for (int u = 0; u < kUnroll; ++u) key[u] = (i + 32 * u < lim) ? __ldg(p + i + 32 * u) : -2;
 #pragma unroll
-    for (int u = 0; u < kUnroll; ++u)
-      if (ok[u]) cnt += probe<kLinear>(c.sHash, tabu[u], key[u], pv, ga + glu[u]);
+      for (int u = 0; u < kUnroll; ++u) cnt += table_probe<kLinear>(T, sh, key[u]);
+    }
   }
   return cnt;
 }
 
 // SHORT class: the warp owns the flat keys [k0w, k1w) of the chunk.
-template <bool kLinear>
+template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0w, int k1w,
                                                const PlanView& pv, int64_t ga) {
   unsigned cnt = 0;
@@ -235,13 +231,13 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
 #pragma unroll
     for (int u = 0; u < kUnroll; ++u) {
       const int k = k0 + 32 * u + lane;
-      if (k < k1w) cnt += probe<kLinear>(c.sHash, c.sInfo[gl[u]], key[u], pv, ga + gl[u]);
+      if (k < k1w) cnt += probe<kLinear, kHuge>(c.sHash, c.sInfo[gl[u]], key[u], pv, ga + gl[u]);
     }
   }
   return cnt;
 }
 
-__global__ void __launch_bounds__(kMaxBlock)
+__global__ void __launch_bounds__(kMaxBlock, 3)  // 3 CTAs x 16 warps per SM
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
             unsigned long long* __restrict__ out) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -265,7 +261,9 @@ __global__ void __launch_bounds__(kMaxBlock)
     c.sC = c.sA + S + 1;
     c.sD = c.sC + S;
     c.sInfo = c.sD + S;
-    c.sHash = c.sInfo + G;
+    // 16-B aligned start of the slots, as an int offset from the (aligned) base
+    // so the compiler keeps every table access in the shared window (LDS/ATOMS)
+    c.sHash = reinterpret_cast<int*>(smem) + ((2 * S + (S + 1) + S + S + G + 3) & ~3);
 
     // 1. stage the chunk's edges and table descriptors; empty slots
     const int64_t kp0 = pv.key_prefix[sa];
@@ -279,13 +277,19 @@ __global__ void __launch_bounds__(kMaxBlock)
         c.sD[i] = pv.seg_group[sg] - (int)ga;
       }
     }
+    int huge = 0;
     for (int i = threadIdx.x; i < G; i += blockDim.x) {
       const int64_t sp = pv.slot_prefix[ga + i], ns = pv.slot_prefix[ga + i + 1] - sp;
-      c.sInfo[i] = ns > 0 ? (((int)(sp - slot0)) << 5) | (31 - __clz((int)ns)) : -1;
+      c.sInfo[i] = ns > 0 ? (((int)(sp - slot0)) << 5) | (32 - (31 - __clz((int)ns))) : -1;
+      huge |= ns == 0;
     }
-    for (int i = threadIdx.x; i < nslots; i += blockDim.x) c.sHash[i] = -1;
+    {
+      int4* h4 = reinterpret_cast<int4*>(c.sHash);
+      for (int i = threadIdx.x; i < (nslots >> 2); i += blockDim.x) h4[i] = make_int4(-1, -1, -1, -1);
+      for (int i = (nslots & ~3) + threadIdx.x; i < nslots; i += blockDim.x) c.sHash[i] = -1;
+    }
     if (threadIdx.x == 0) sFail = 0;
-    __syncthreads();
+    const bool any_huge = __syncthreads_or(huge);
 
     // 2. hash N+(v) of every group touched by the chunk
     bool linear = pv.probe_mode == 1;
@@ -310,7 +314,7 @@ __global__ void __launch_bounds__(kMaxBlock)
     if (!linear && sFail) {  // uniform: rebuild this chunk's tables with linear probing
       linear = true;
       for (int i = threadIdx.x; i < nslots; i += blockDim.x) c.sHash[i] = -1;
-      __syncthreads();
+      __syncthreads();  // (rare path: scalar init is fine)
       warp_walk_global(pv.ins_prefix, ga, gb, iw0, iw1, pv.col, pv.grp_ibase,
                        [&](int64_t g, int32_t key) {
                          const int tab = c.sInfo[g - ga];
@@ -323,10 +327,17 @@ __global__ void __launch_bounds__(kMaxBlock)
     const int NU = c.sA[S];
     const int w0 = (int)((int64_t)NU * warp / nw), w1 = (int)((int64_t)NU * (warp + 1) / nw);
     unsigned cnt;
-    if (is_long)
-      cnt = linear ? walk_long<true>(c, S, w0, w1, pv, ga) : walk_long<false>(c, S, w0, w1, pv, ga);
-    else
-      cnt = linear ? walk_short<true>(c, S, w0, w1, pv, ga) : walk_short<false>(c, S, w0, w1, pv, ga);
+    if (is_long) {
+      if (any_huge)
+        cnt = linear ? walk_long<true, true>(c, S, w0, w1, pv, ga) : walk_long<false, true>(c, S, w0, w1, pv, ga);
+      else
+        cnt = linear ? walk_long<true, false>(c, S, w0, w1, pv, ga) : walk_long<false, false>(c, S, w0, w1, pv, ga);
+    } else {
+      if (any_huge)
+        cnt = linear ? walk_short<true, true>(c, S, w0, w1, pv, ga) : walk_short<false, true>(c, S, w0, w1, pv, ga);
+      else
+        cnt = linear ? walk_short<true, false>(c, S, w0, w1, pv, ga) : walk_short<false, false>(c, S, w0, w1, pv, ga);
+    }
     acc += cnt;
     __syncthreads();  // SMEM is rebuilt by the next chunk
   }
@@ -366,7 +377,9 @@ int max_smem_per_block() {
   int dev = 0, v = 0;
   TC_CUDA(cudaGetDevice(&dev));
   TC_CUDA(cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
-  return v - (int)(sizeof(unsigned long long) * (kMaxBlock / 32));
+  cudaFuncAttributes fa;
+  TC_CUDA(cudaFuncGetAttributes(&fa, k_count));
+  return v - (int)fa.sharedSizeBytes;  // dynamic + static must fit the opt-in limit
 }
 
 int count_occupancy(int block, int64_t smem_bytes) {

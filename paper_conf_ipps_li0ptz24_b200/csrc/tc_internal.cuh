@@ -104,8 +104,10 @@ struct PlanView {
 
 // SMEM a chunk needs (bytes): per segment staging + per group descriptor +
 // hash slots.  Shared by the plan (sizing) and the kernel (layout).
+// Layout: sB int64[S] | sA int32[S+1] | sC int32[S] | sD int32[S] | sInfo
+// int32[G] | pad to 16 B | sHash int32[slots].
 __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_t slots) {
-  return 4 * (S + 1) + 8 * S + 4 * S + 4 * S + 4 * G + 4 * slots + 64;
+  return 8 * S + 4 * (S + 1) + 4 * S + 4 * S + 4 * G + 16 + 4 * slots;
 }
 
 struct Plan {
@@ -115,6 +117,7 @@ struct Plan {
   DevBuf<int64_t> key_prefix, seg_start, ins_prefix, grp_ibase, slot_prefix, chunk_seg;
   DevBuf<int32_t> seg_len, seg_group;
   std::vector<int64_t> h_chunk_seg;
+  int64_t chunk_cost_long = 0, chunk_cost_short = 0;  // after SMEM-driven halving
   int64_t smem_bytes = 0;
   int grid = 0, block = 0;
 };
