@@ -81,7 +81,8 @@ typedef struct {
   int32_t seg_cost;     /* fixed cost per live oriented edge (default 4)          */
   int32_t huge_degree;  /* d+(v) above which N+(v) is probed in global memory by
                            binary search instead of an SMEM hash (default 8192)    */
-  int32_t block_threads;/* threads per CTA of the count kernel (default 512)       */
+  int32_t block_threads;/* threads per CTA of the count kernel, 64..1024; 1/8 of
+                           the warps build tables, the rest probe (default 1024)   */
   int32_t table_factor; /* hash slots = next_pow2(table_factor * d+(v)), 2..16
                            (default 3, i.e. load <= 1/3)                            */
   int32_t long_min;     /* trimmed suffixes with >= long_min keys go to the

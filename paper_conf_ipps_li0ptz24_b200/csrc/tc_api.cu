@@ -103,8 +103,8 @@ Options resolve_options(const tc_options* o) {
   require(r.chunk_cost >= 64, "chunk_cost must be >= 64");
   require(r.seg_cost >= 1, "seg_cost must be >= 1");
   require(r.huge_degree >= 1, "huge_degree must be >= 1");
-  require(r.block_threads >= 64 && r.block_threads <= 512 && r.block_threads % 32 == 0,
-          "block_threads must be a multiple of 32 in [64, 512]");
+  require(r.block_threads >= 64 && r.block_threads <= 1024 && r.block_threads % 32 == 0,
+          "block_threads must be a multiple of 32 in [64, 1024]");
   require(r.table_factor >= 2 && r.table_factor <= 16, "table_factor must be in [2, 16]");
   require(r.long_min >= 1, "long_min must be >= 1");
   require(r.probe_mode == 0 || r.probe_mode == 1, "probe_mode must be 0 or 1");

@@ -690,10 +690,10 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
 
   // Chunking, per class: long chunks start 4x larger (their SMEM is one or
   // two tables plus a few edges).  A class's chunk cost is halved while its
-  // largest chunk needs more SMEM than the 3-CTAs-per-SM target (down to 1024
-  // units), then while it exceeds what one CTA can have at all.
-  const int64_t hard = std::min<int64_t>(max_smem_per_block(), 200 * 1024);
-  const int64_t soft = std::min<int64_t>(hard, 72 * 1024);
+  // largest chunk needs more SMEM than one of the count kernel's two chunk
+  // slots can hold.
+  const int64_t hard = max_chunk_smem();  // one of the kernel's two chunk slots
+  const int64_t soft = hard;
   int64_t CL = std::max<int64_t>(4ll * opt.chunk_cost, 64), CS = std::max<int64_t>(opt.chunk_cost, 64);
   DevBuf<unsigned long long> mx(2, s);
   for (;;) {

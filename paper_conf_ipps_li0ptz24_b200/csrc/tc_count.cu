@@ -4,27 +4,31 @@
 // oriented edge (u,v) of the degree-ordered DAG, |N+(u) ∩ (v,∞) ∩ N+(v)|,
 // the size of the intersection of u's suffix after v with v's out-list;
 // their sum is T.  The plan (tc_build.cu a6) already trimmed every suffix to
-// [min N+(v), max N+(v)] and dropped the edges left empty (exact, C-12).
+// [min N+(v), max N+(v)] and dropped the edges left empty (exact, C-12/C-21).
 //
-// How.  Live edges are grouped by their head v.  A CTA takes
-// one work chunk = a run of consecutive live edges of one class and
-// near-equal cost, covering a run of groups:
-//   1. it builds one hash table per group from N+(v) in shared memory (the
-//      GroupTC idea of a table shared by a block of edges, with the
-//      hashing TRUST uses, instead of binary search, the cost
-//      P:369/P:379 name on large graphs).  Tables are two-choice (cuckoo):
-//      a probe reads exactly two slots, so no warp waits on the longest of
-//      32 probe chains; if an insert ever fails the chunk falls back to
-//      linear probing;
-//   2. it streams the edges' suffix keys and probes the head's table:
-//      LONG class (suffix >= long_min keys): one warp walks one edge in
-//        32-key tiles, coalesced, with warp-uniform bookkeeping;
-//      SHORT class: the keys of all the chunk's edges are flattened over the
-//        lanes (the flattened walk of P:349 / Alg. 1 with the `>=` boundary
-//        of DESIGN.md reading C-7), 32 consecutive keys mapped to their
-//        edges with one SMEM load, a warp OR-reduce and popc;
-//      (degree-bucketed dispatch, the TRUST/Fox idea of P:176/P:254);
-//   3. counts go thread u32 -> warp shuffle -> CTA -> one u64 atomic.
+// How.  Live edges are grouped by their head v.  Work comes
+// in chunks = runs of consecutive live edges of one class and near-equal
+// cost, covering a run of groups.  One persistent CTA per SM, warp-specialised,
+// with two chunk slots in shared memory:
+//   PRODUCER warps (the first 1/4 of the CTA) take the CTA's chunk k+1 while
+//     the consumers work on chunk k: they stage the chunk's edges and table
+//     descriptors into the free slot and build one hash table per group from
+//     N+(v) (the GroupTC idea of a table shared by a block of edges, P:349,
+//     hashed as in TRUST, instead of binary search, the cost
+//     P:369/P:379 name on large graphs).  Tables are two-choice (cuckoo): a
+//     probe reads exactly two slots, so no warp waits on the longest of 32
+//     probe chains; if an insert ever fails the chunk falls back to linear
+//     probing.  They hand the slot over with an mbarrier.
+//   CONSUMER warps stream the chunk's suffix keys and probe the heads' tables:
+//     LONG class (suffix >= long_min keys): a warp walks one edge at a time
+//       in 32-key tiles, coalesced, with warp-uniform bookkeeping;
+//     SHORT class: the keys of all the chunk's edges are flattened over the
+//       lanes (the flattened walk of P:349 / Alg. 1 with the `>=` boundary
+//       of DESIGN.md reading C-7), 32 consecutive keys mapped to their edges
+//       with one SMEM load, a warp OR-reduce and popc
+//     (degree-bucketed dispatch, the TRUST/Fox idea of P:176/P:254), then
+//     release the slot with an mbarrier.
+//   Counts go thread u32 -> u64 -> warp shuffle -> CTA -> one atomic.
 // Tables whose N+(v) exceeds huge_degree are not staged; their keys are
 // binary-searched in global memory (the TriCore-style probe).
 #include <algorithm>
@@ -34,10 +38,48 @@
 namespace tc {
 namespace {
 
-constexpr int kMaxBlock = 512;
-constexpr int kUnroll = 4;     // tiles in flight per warp iteration
-constexpr int kMaxKicks = 96;  // cuckoo displacement bound before the linear fallback
+constexpr int kMaxBlock = 1024;
+constexpr int kUnrollLong = 8;   // tiles in flight per consumer warp (long class)
+constexpr int kUnrollShort = 4;  // tiles in flight per consumer warp (short class)
+constexpr int kMaxKicks = 96;    // cuckoo displacement bound before the linear fallback
+constexpr int kSlots = 2;        // chunk slots (double buffering)
+constexpr int kProdDiv = 4;      // 1/kProdDiv of the warps are producers
 
+// ------------------------------------------------------------------ mbarrier (PTX)
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n\t}" ::"r"(smem_u32(b))
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void named_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+// Named barrier that also ORs a predicate over its participants.
+__device__ __forceinline__ int named_sync_or(int id, int nthreads, int pred) {
+  int r;
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\tsetp.ne.s32 p, %1, 0;\n\t"
+      "bar.red.or.pred q, %2, %3, p;\n\tselp.s32 %0, 1, 0, q;\n\t}"
+      : "=r"(r)
+      : "r"(pred), "r"(id), "r"(nthreads)
+      : "memory");
+  return r;
+}
+
+// ------------------------------------------------------------------ hashing
 // Table descriptor tab = (slot offset << 5) | sh with sh = 32 - log2(slots):
 // the slot of a key is the top log2(slots) bits of a multiplicative hash.
 __device__ __forceinline__ uint32_t hash1(int32_t key, int sh) {
@@ -45,40 +87,6 @@ __device__ __forceinline__ uint32_t hash1(int32_t key, int sh) {
 }
 __device__ __forceinline__ uint32_t hash2(int32_t key, int sh) {
   return ((uint32_t)key * 0x85EBCA77u + 0x7F4A7C15u) >> sh;
-}
-
-// Largest s in [s_lo, s_hi) with P[s] <= k (segments are non-empty).
-template <class T>
-__device__ __forceinline__ T seg_of(const T* __restrict__ P, T s_lo, T s_hi, T k) {
-  T lo = s_lo, hi = s_hi - 1;
-  while (lo < hi) {
-    T mid = (lo + hi + 1) >> 1;
-    if (P[mid] <= k) lo = mid; else hi = mid - 1;
-  }
-  return lo;
-}
-
-// Warp walk over the flat range [kbeg, kend) of the segments [s_lo, s_hi)
-// with (global, int64) exclusive prefix P; used to insert N+(v) keys.
-template <class Proc>
-__device__ __forceinline__ void warp_walk_global(const int64_t* __restrict__ P, int64_t s_lo,
-                                                 int64_t s_hi, int64_t kbeg, int64_t kend,
-                                                 const int32_t* __restrict__ col,
-                                                 const int64_t* __restrict__ base, Proc proc) {
-  if (kbeg >= kend) return;
-  const int lane = threadIdx.x & 31;
-  const unsigned below = (1u << lane) - 1u;
-  int64_t s = seg_of<int64_t>(P, s_lo, s_hi, kbeg);
-  for (int64_t k0 = kbeg; k0 < kend; k0 += 32) {
-    const int64_t j = s + 1 + lane;
-    const int64_t pos = (j <= s_hi) ? P[j] - k0 : 64;
-    const unsigned bit = (pos >= 1 && pos <= 32) ? (1u << (pos - 1)) : 0u;
-    const unsigned M = __reduce_or_sync(0xffffffffu, bit);
-    const int64_t seg = s + __popc(M & below);
-    s += __popc(M);
-    const int64_t k = k0 + lane;
-    if (k < kend) proc(seg, __ldg(col + __ldg(base + seg) + k));
-  }
 }
 
 __device__ __forceinline__ bool cuckoo_insert(int* __restrict__ T, int tab, int32_t key) {
@@ -137,39 +145,103 @@ __device__ __forceinline__ unsigned table_probe(const int* __restrict__ T, int s
   }
 }
 
-// Membership through a descriptor (tab = off << 5 | sh, or -1 = huge table
-// of group g, probed by binary search in global memory).
-template <bool kLinear, bool kHuge>
-__device__ __forceinline__ unsigned probe(const int* __restrict__ H, int tab, int32_t key,
-                                          const PlanView& pv, int64_t g) {
-  if (kHuge && tab < 0) {
-    const int64_t ib = pv.ins_prefix[g];
-    return global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, key);
-  }
-  return table_probe<kLinear>(H + (tab >> 5), tab & 31, key);
-}
-
-struct ChunkSmem {
-  int64_t* sB;  // long: key start in col; short: start - (chunk-relative first key)
-  int* sA;      // [S+1] long: tile prefix; short: key prefix (chunk-relative)
-  int* sC;      // long: suffix length
-  int* sD;      // group index (chunk-local)
-  int* sInfo;   // [G] table descriptor
-  int* sHash;   // slots
+// ------------------------------------------------------------------ chunk slot
+// One slot = the staged edges, groups and tables of one chunk.  Layout (bytes,
+// region 16-B aligned): sB int64[S] | sGB int64[G] | sA int32[S+1] | sC
+// int32[S] | sD int32[S] | sInfo int32[G] | sGP int32[G+1] | pad | sHash.
+// chunk_smem_bytes (tc_internal.cuh) is the matching size.
+struct SlotHdr {
+  long long sa, ga;
+  int S, G, nslots, is_long, linear, done, huge, pad;
 };
 
+struct ChunkSmem {
+  int64_t* sB;   // long: key start in col; short: start - (chunk-relative first key)
+  int64_t* sGB;  // group: row start of N+(v) - sGP (so col[sGB[g] + k] is insert k)
+  int* sA;       // [S+1] long: tile prefix; short: key prefix (chunk-relative)
+  int* sC;       // long: suffix length
+  int* sD;       // group index (chunk-local)
+  int* sInfo;    // [G] table descriptor (-1: huge)
+  int* sGP;      // [G+1] insert prefix (chunk-relative)
+  int* sHash;    // slots
+};
+
+__device__ __forceinline__ ChunkSmem slot_view(unsigned char* region, int S, int G) {
+  ChunkSmem c;
+  c.sB = reinterpret_cast<int64_t*>(region);
+  c.sGB = c.sB + S;
+  c.sA = reinterpret_cast<int*>(c.sGB + G);
+  c.sC = c.sA + S + 1;
+  c.sD = c.sC + S;
+  c.sInfo = c.sD + S;
+  c.sGP = c.sInfo + G;
+  // 16-B aligned start of the slots as an int offset from the aligned region
+  // base, so every table access stays in the shared window (LDS/ATOMS)
+  c.sHash = reinterpret_cast<int*>(region) +
+            ((2 * S + 2 * G + (S + 1) + 2 * S + G + (G + 1) + 3) & ~3);
+  return c;
+}
+
+// Largest s in [0, S) with P[s] <= k (segments are non-empty).
+__device__ __forceinline__ int seg_of(const int* __restrict__ P, int S, int k) {
+  int lo = 0, hi = S - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (P[mid] <= k) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+// Warp walk over the flat range [kbeg, kend) of the segments [0, S) whose
+// exclusive prefix is the SMEM array P (P[S] = their end; segments non-empty).
+// 32 consecutive flat indices are mapped to their segments with one SMEM
+// load of the next 32 starts, a warp OR-reduce of a position mask and popc.
+// kU tiles are mapped, then load(seg, k) is issued for all of them (kU
+// independent global loads in flight per lane), then proc(seg, value).
+template <int kU, class Load, class Proc>
+__device__ __forceinline__ void warp_walk(const int* __restrict__ P, int S, int kbeg, int kend,
+                                          Load load, Proc proc) {
+  if (kbeg >= kend) return;
+  const int lane = threadIdx.x & 31;
+  const unsigned below = (1u << lane) - 1u;
+  int s = seg_of(P, S, kbeg);
+  for (int k0 = kbeg; k0 < kend; k0 += 32 * kU) {
+    int seg[kU];
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {
+      const int t0 = k0 + 32 * u;
+      const int j = s + 1 + lane;
+      const int pos = (j <= S) ? P[j] - t0 : 64;
+      const unsigned bit = (pos >= 1 && pos <= 32) ? (1u << (pos - 1)) : 0u;
+      const unsigned M = __reduce_or_sync(0xffffffffu, bit);
+      seg[u] = s + __popc(M & below);
+      s += __popc(M);
+    }
+    int32_t val[kU];
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {
+      const int k = k0 + 32 * u + lane;
+      val[u] = k < kend ? load(seg[u], k) : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < kU; ++u)
+      if (k0 + 32 * u + lane < kend) proc(seg[u], val[u]);
+  }
+}
+
+// ------------------------------------------------------------------ consumers
 // LONG class: the warp owns tiles [t0, t1) of the chunk; each tile is 32
 // consecutive keys of one edge.  The warp walks edge by edge (warp-uniform
 // bookkeeping); inside an edge, lane l reads keys l, l+32, ... through one
-// pointer with immediate offsets, kUnroll tiles in flight; lanes past the
-// end carry the never-matching sentinel so the probes run unpredicated.
+// pointer with immediate offsets, kUnrollLong tiles in flight; lanes past
+// the end carry the never-matching sentinel so the probes run unpredicated.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int S, int t0, int t1,
                                               const PlanView& pv, int64_t ga) {
   unsigned cnt = 0;
   if (t0 >= t1) return cnt;
   const int lane = threadIdx.x & 31;
-  int s = seg_of<int>(c.sA, 0, S, t0);
+  int s = seg_of(c.sA, S, t0);
   for (int t = t0; t < t1; ++s) {
     const int ts = c.sA[s], te = min(c.sA[s + 1], t1);
     const int done = (t - ts) << 5;                             // keys of this edge before tile t
@@ -179,17 +251,19 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int S, int t0,
     const int tab = c.sInfo[gl];
     t = te;
     if (kHuge && tab < 0) {
-      for (int i = 0; i < lim; i += 32) cnt += probe<kLinear, true>(c.sHash, tab, __ldg(p + i), pv, ga + gl);
+      const int64_t g = ga + gl, ib = pv.ins_prefix[g];
+      for (int i = 0; i < lim; i += 32)
+        cnt += global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, __ldg(p + i));
       continue;
     }
     const int* __restrict__ T = c.sHash + (tab >> 5);
     const int sh = tab & 31;
-    for (int i = 0; i < lim; i += 32 * kUnroll) {
-      int32_t key[kUnroll];
+    for (int i = 0; i < lim; i += 32 * kUnrollLong) {
+      int32_t key[kUnrollLong];
 #pragma unroll
-      for (int u = 0; u < kUnroll; ++u) key[u] = (i + 32 * u < lim) ? __ldg(p + i + 32 * u) : -2;
+      for (int u = 0; u < kUnrollLong; ++u) key[u] = (i + 32 * u < lim) ? __ldg(p + i + 32 * u) : -2;
 #pragma unroll
-      for (int u = 0; u < kUnroll; ++u) cnt += table_probe<kLinear>(T, sh, key[u]);
+      for (int u = 0; u < kUnrollLong; ++u) cnt += table_probe<kLinear>(T, sh, key[u]);
     }
   }
   return cnt;
@@ -203,11 +277,11 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
   if (k0w >= k1w) return cnt;
   const int lane = threadIdx.x & 31;
   const unsigned below = (1u << lane) - 1u;
-  int s = seg_of<int>(c.sA, 0, S, k0w);
-  for (int k0 = k0w; k0 < k1w; k0 += 32 * kUnroll) {
-    int seg[kUnroll];
+  int s = seg_of(c.sA, S, k0w);
+  for (int k0 = k0w; k0 < k1w; k0 += 32 * kUnrollShort) {
+    int seg[kUnrollShort];
 #pragma unroll
-    for (int u = 0; u < kUnroll; ++u) {
+    for (int u = 0; u < kUnrollShort; ++u) {
       const int t0 = k0 + 32 * u;
       const int j = s + 1 + lane;
       const int pos = (j <= S) ? c.sA[j] - t0 : 64;
@@ -216,133 +290,234 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
       seg[u] = s + __popc(M & below);
       s += __popc(M);
     }
-    int32_t key[kUnroll];
-    int gl[kUnroll];
+    int32_t key[kUnrollShort];
+    int tab[kUnrollShort], gl[kUnrollShort];
 #pragma unroll
-    for (int u = 0; u < kUnroll; ++u) {
+    for (int u = 0; u < kUnrollShort; ++u) {
       const int k = k0 + 32 * u + lane;
       key[u] = 0;
+      tab[u] = 0;
       gl[u] = 0;
       if (k < k1w) {
         key[u] = __ldg(pv.col + c.sB[seg[u]] + k);
         gl[u] = c.sD[seg[u]];
+        tab[u] = c.sInfo[gl[u]];
       }
     }
 #pragma unroll
-    for (int u = 0; u < kUnroll; ++u) {
-      const int k = k0 + 32 * u + lane;
-      if (k < k1w) cnt += probe<kLinear, kHuge>(c.sHash, c.sInfo[gl[u]], key[u], pv, ga + gl[u]);
+    for (int u = 0; u < kUnrollShort; ++u) {
+      // padding lanes have no table of their own: they must not probe (a
+      // linear probe needs a table with an empty slot to terminate)
+      if (k0 + 32 * u + lane >= k1w) continue;
+      if (kHuge && tab[u] < 0) {
+        const int64_t g = ga + gl[u], ib = pv.ins_prefix[g];
+        cnt += global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, key[u]);
+      } else {
+        cnt += table_probe<kLinear>(c.sHash + (tab[u] >> 5), tab[u] & 31, key[u]);
+      }
     }
   }
   return cnt;
 }
 
-__global__ void __launch_bounds__(kMaxBlock, 3)  // 3 CTAs x 16 warps per SM
-    k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
-            unsigned long long* __restrict__ out) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  __shared__ unsigned long long red[kMaxBlock / 32];
-  __shared__ int sFail;
-  const int warp = threadIdx.x >> 5, nw = blockDim.x >> 5, lane = threadIdx.x & 31;
-  unsigned long long acc = 0;
+template <bool kLinear>
+__device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
+                                            const PlanView& pv) {
+  if (h.is_long)
+    return h.huge ? walk_long<kLinear, true>(c, h.S, w0, w1, pv, h.ga)
+                  : walk_long<kLinear, false>(c, h.S, w0, w1, pv, h.ga);
+  return h.huge ? walk_short<kLinear, true>(c, h.S, w0, w1, pv, h.ga)
+                : walk_short<kLinear, false>(c, h.S, w0, w1, pv, h.ga);
+}
 
-  for (int64_t cix = c_begin + blockIdx.x; cix < c_end; cix += gridDim.x) {
-    const int64_t sa = max(pv.chunk_seg[cix], e_begin), sb = min(pv.chunk_seg[cix + 1], e_end);
-    if (sa >= sb) continue;  // uniform over the CTA
-    const bool is_long = cix < pv.n_long_chunks;
-    const int S = (int)(sb - sa);
-    const int64_t ga = pv.seg_group[sa], gb = (int64_t)pv.seg_group[sb - 1] + 1;
-    const int G = (int)(gb - ga);
-    const int64_t slot0 = pv.slot_prefix[ga];
-    const int nslots = (int)(pv.slot_prefix[gb] - slot0);
-    ChunkSmem c;
-    c.sB = reinterpret_cast<int64_t*>(smem);
-    c.sA = reinterpret_cast<int*>(c.sB + S);
-    c.sC = c.sA + S + 1;
-    c.sD = c.sC + S;
-    c.sInfo = c.sD + S;
-    // 16-B aligned start of the slots, as an int offset from the (aligned) base
-    // so the compiler keeps every table access in the shared window (LDS/ATOMS)
-    c.sHash = reinterpret_cast<int*>(smem) + ((2 * S + (S + 1) + S + S + G + 3) & ~3);
+// ------------------------------------------------------------------ producers
+// Stage chunk cix into a slot and build its tables.  pt = producer thread id
+// in [0, PT); the PT producer threads synchronise on named barrier 1.  The
+// header is written by producer 0 before its own mbarrier arrive, so the
+// consumers see it once every producer has arrived.
+__device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
+                                        int64_t e_end, unsigned char* region, SlotHdr& hdr,
+                                        int pt, int PT) {
+  const int64_t sa = max(pv.chunk_seg[cix], e_begin), sb = min(pv.chunk_seg[cix + 1], e_end);
+  if (sa >= sb) {  // empty after clipping to the range
+    if (pt == 0) {
+      hdr.S = 0;
+      hdr.done = 0;
+    }
+    return;
+  }
+  const bool is_long = cix < pv.n_long_chunks;
+  const int S = (int)(sb - sa);
+  const int64_t ga = pv.seg_group[sa], gb = (int64_t)pv.seg_group[sb - 1] + 1;
+  const int G = (int)(gb - ga);
+  const int64_t slot0 = pv.slot_prefix[ga];
+  const int nslots = (int)(pv.slot_prefix[gb] - slot0);
+  ChunkSmem c = slot_view(region, S, G);
 
-    // 1. stage the chunk's edges and table descriptors; empty slots
-    const int64_t kp0 = pv.key_prefix[sa];
-    for (int i = threadIdx.x; i <= S; i += blockDim.x) {
-      const int64_t sg = sa + i;
-      const int rel = (int)(pv.key_prefix[sg] - kp0);
-      c.sA[i] = is_long ? (rel >> 5) : rel;
+  // 1. stage edges and groups; empty slots.  Each producer thread handles
+  //    kB items per batch with all their global loads issued before any
+  //    store, so a batch costs one memory latency.
+  constexpr int kB = 4;
+  const int64_t kp0 = pv.key_prefix[sa];
+  for (int base = pt; base <= S; base += PT * kB) {
+    int64_t kp[kB], st[kB];
+    int ln[kB], gr[kB];
+#pragma unroll
+    for (int r = 0; r < kB; ++r) {
+      const int i = base + r * PT;
+      kp[r] = 0;
+      st[r] = 0;
+      ln[r] = gr[r] = 0;
+      if (i <= S) kp[r] = pv.key_prefix[sa + i];
       if (i < S) {
-        c.sB[i] = is_long ? pv.seg_start[sg] : pv.seg_start[sg] - rel;
-        c.sC[i] = pv.seg_len[sg];
-        c.sD[i] = pv.seg_group[sg] - (int)ga;
+        st[r] = pv.seg_start[sa + i];
+        ln[r] = pv.seg_len[sa + i];
+        gr[r] = pv.seg_group[sa + i];
       }
     }
-    int huge = 0;
-    for (int i = threadIdx.x; i < G; i += blockDim.x) {
-      const int64_t sp = pv.slot_prefix[ga + i], ns = pv.slot_prefix[ga + i + 1] - sp;
-      c.sInfo[i] = ns > 0 ? (((int)(sp - slot0)) << 5) | (32 - (31 - __clz((int)ns))) : -1;
-      huge |= ns == 0;
+#pragma unroll
+    for (int r = 0; r < kB; ++r) {
+      const int i = base + r * PT;
+      const int rel = (int)(kp[r] - kp0);
+      if (i <= S) c.sA[i] = is_long ? (rel >> 5) : rel;
+      if (i < S) {
+        c.sB[i] = is_long ? st[r] : st[r] - rel;
+        c.sC[i] = ln[r];
+        c.sD[i] = gr[r] - (int)ga;
+      }
     }
-    {
-      int4* h4 = reinterpret_cast<int4*>(c.sHash);
-      for (int i = threadIdx.x; i < (nslots >> 2); i += blockDim.x) h4[i] = make_int4(-1, -1, -1, -1);
-      for (int i = (nslots & ~3) + threadIdx.x; i < nslots; i += blockDim.x) c.sHash[i] = -1;
+  }
+  const int64_t ip0 = pv.ins_prefix[ga];
+  int huge = 0;
+  for (int base = pt; base <= G; base += PT * kB) {
+    int64_t ip[kB], sp[kB], sp1[kB], ib[kB];
+#pragma unroll
+    for (int r = 0; r < kB; ++r) {
+      const int i = base + r * PT;
+      ip[r] = sp[r] = sp1[r] = ib[r] = 0;
+      if (i <= G) ip[r] = pv.ins_prefix[ga + i];
+      if (i < G) {
+        sp[r] = pv.slot_prefix[ga + i];
+        sp1[r] = pv.slot_prefix[ga + i + 1];
+        ib[r] = pv.grp_ibase[ga + i];
+      }
     }
-    if (threadIdx.x == 0) sFail = 0;
-    const bool any_huge = __syncthreads_or(huge);
+#pragma unroll
+    for (int r = 0; r < kB; ++r) {
+      const int i = base + r * PT;
+      if (i <= G) c.sGP[i] = (int)(ip[r] - ip0);
+      if (i < G) {
+        const int64_t ns = sp1[r] - sp[r];
+        c.sInfo[i] = ns > 0 ? (((int)(sp[r] - slot0)) << 5) | (32 - (31 - __clz((int)ns))) : -1;
+        huge |= ns == 0;
+        c.sGB[i] = ib[r] + ip0;  // row start - chunk-relative insert prefix
+      }
+    }
+  }
+  {
+    int4* h4 = reinterpret_cast<int4*>(c.sHash);
+    for (int i = pt; i < (nslots >> 2); i += PT) h4[i] = make_int4(-1, -1, -1, -1);
+    for (int i = (nslots & ~3) + pt; i < nslots; i += PT) c.sHash[i] = -1;
+  }
+  const int any_huge = named_sync_or(1, PT, huge);
 
-    // 2. hash N+(v) of every group touched by the chunk
-    bool linear = pv.probe_mode == 1;
-    const int64_t ib = pv.ins_prefix[ga], ilen = pv.ins_prefix[gb] - ib;
-    const int64_t iw0 = ib + ilen * warp / nw, iw1 = ib + ilen * (warp + 1) / nw;
-    if (linear) {
-      warp_walk_global(pv.ins_prefix, ga, gb, iw0, iw1, pv.col, pv.grp_ibase,
-                       [&](int64_t g, int32_t key) {
-                         const int tab = c.sInfo[g - ga];
-                         if (tab >= 0) linear_insert(c.sHash, tab, key);
-                       });
-    } else {
-      bool ok = true;
-      warp_walk_global(pv.ins_prefix, ga, gb, iw0, iw1, pv.col, pv.grp_ibase,
-                       [&](int64_t g, int32_t key) {
-                         const int tab = c.sInfo[g - ga];
-                         if (tab >= 0 && !cuckoo_insert(c.sHash, tab, key)) ok = false;
-                       });
-      if (!ok) sFail = 1;
-    }
-    __syncthreads();
-    if (!linear && sFail) {  // uniform: rebuild this chunk's tables with linear probing
+  // 2. hash N+(v) of every group touched by the chunk (flattened over groups,
+  //    kInsU tiles of N+(v) loads in flight per producer lane)
+  constexpr int kInsU = 4;
+  const int pw = pt >> 5, npw = PT >> 5;
+  const int NI = c.sGP[G];
+  const int i0 = (int)((int64_t)NI * pw / npw), i1 = (int)((int64_t)NI * (pw + 1) / npw);
+  auto load_row = [&](int g, int k) { return __ldg(pv.col + c.sGB[g] + k); };
+  bool linear = pv.probe_mode == 1;
+  if (linear) {
+    warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
+      const int tab = c.sInfo[g];
+      if (tab >= 0) linear_insert(c.sHash, tab, key);
+    });
+  } else {
+    bool ok = true;
+    warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
+      const int tab = c.sInfo[g];
+      if (tab >= 0 && !cuckoo_insert(c.sHash, tab, key)) ok = false;
+    });
+    if (named_sync_or(1, PT, !ok)) {  // uniform over producers: rebuild with linear probing
       linear = true;
-      for (int i = threadIdx.x; i < nslots; i += blockDim.x) c.sHash[i] = -1;
-      __syncthreads();  // (rare path: scalar init is fine)
-      warp_walk_global(pv.ins_prefix, ga, gb, iw0, iw1, pv.col, pv.grp_ibase,
-                       [&](int64_t g, int32_t key) {
-                         const int tab = c.sInfo[g - ga];
-                         if (tab >= 0) linear_insert(c.sHash, tab, key);
-                       });
-      __syncthreads();
+      for (int i = pt; i < nslots; i += PT) c.sHash[i] = -1;
+      named_sync(1, PT);
+      warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
+        const int tab = c.sInfo[g];
+        if (tab >= 0) linear_insert(c.sHash, tab, key);
+      });
     }
+  }
+  if (pt == 0) {
+    hdr.sa = sa;
+    hdr.ga = ga;
+    hdr.S = S;
+    hdr.G = G;
+    hdr.nslots = nslots;
+    hdr.is_long = is_long;
+    hdr.linear = linear;
+    hdr.done = 0;
+    hdr.huge = any_huge;
+  }
+}
 
-    // 3. stream the chunk's suffix keys and probe the heads' tables
-    const int NU = c.sA[S];
-    const int w0 = (int)((int64_t)NU * warp / nw), w1 = (int)((int64_t)NU * (warp + 1) / nw);
-    unsigned cnt;
-    if (is_long) {
-      if (any_huge)
-        cnt = linear ? walk_long<true, true>(c, S, w0, w1, pv, ga) : walk_long<false, true>(c, S, w0, w1, pv, ga);
-      else
-        cnt = linear ? walk_long<true, false>(c, S, w0, w1, pv, ga) : walk_long<false, false>(c, S, w0, w1, pv, ga);
-    } else {
-      if (any_huge)
-        cnt = linear ? walk_short<true, true>(c, S, w0, w1, pv, ga) : walk_short<false, true>(c, S, w0, w1, pv, ga);
-      else
-        cnt = linear ? walk_short<true, false>(c, S, w0, w1, pv, ga) : walk_short<false, false>(c, S, w0, w1, pv, ga);
+__global__ void __launch_bounds__(kMaxBlock, 1)
+    k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
+            int64_t slot_bytes, unsigned long long* __restrict__ out) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ unsigned long long red[kMaxBlock / 32];
+  __shared__ __align__(8) uint64_t full_bar[kSlots];
+  __shared__ __align__(8) uint64_t empty_bar[kSlots];
+  __shared__ SlotHdr hdr[kSlots];
+  const int warp = threadIdx.x >> 5, nw = blockDim.x >> 5, lane = threadIdx.x & 31;
+  const int n_prod = max(1, nw / kProdDiv), n_cons = nw - n_prod;
+  const int PT = n_prod * 32;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kSlots; ++i) {
+      mbar_init(&full_bar[i], PT);       // every producer thread arrives
+      mbar_init(&empty_bar[i], n_cons);  // one lane per consumer warp
     }
-    acc += cnt;
-    __syncthreads();  // SMEM is rebuilt by the next chunk
+  }
+  __syncthreads();
+
+  unsigned long long acc = 0;
+  if (warp < n_prod) {
+    // ------------------------------------------------------------ producers
+    for (int64_t k = 0;; ++k) {
+      const int slot = (int)(k & 1);
+      const uint32_t j = (uint32_t)(k >> 1);  // fill number of this slot
+      if (j > 0) mbar_wait(&empty_bar[slot], (j - 1) & 1);
+      const int64_t cix = c_begin + blockIdx.x + k * gridDim.x;
+      if (cix >= c_end) {
+        if (threadIdx.x == 0) hdr[slot].done = 1;
+        mbar_arrive(&full_bar[slot]);
+        break;
+      }
+      produce(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], threadIdx.x, PT);
+      mbar_arrive(&full_bar[slot]);
+    }
+  } else {
+    // ------------------------------------------------------------ consumers
+    const int cw = warp - n_prod;
+    for (int64_t k = 0;; ++k) {
+      const int slot = (int)(k & 1);
+      mbar_wait(&full_bar[slot], (uint32_t)((k >> 1) & 1));
+      const SlotHdr h = hdr[slot];
+      if (h.done) break;
+      if (h.S > 0) {
+        const ChunkSmem c = slot_view(smem + slot * slot_bytes, h.S, h.G);
+        const int NU = c.sA[h.S];
+        const int w0 = (int)((int64_t)NU * cw / n_cons), w1 = (int)((int64_t)NU * (cw + 1) / n_cons);
+        acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty_bar[slot]);
+    }
   }
 
-  // 4. u64 reduction: warp shuffle -> CTA -> one atomic
+  // u64 reduction: warp shuffle -> CTA -> one atomic
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) acc += __shfl_down_sync(0xffffffffu, acc, o);
   if (lane == 0) red[warp] = acc;
@@ -364,6 +539,8 @@ void ensure_attr() {
   g_attr_set = true;
 }
 
+int64_t slot_bytes_of(int64_t need) { return (need + 15) & ~int64_t(15); }
+
 }  // namespace
 
 int num_sms() {
@@ -382,10 +559,13 @@ int max_smem_per_block() {
   return v - (int)fa.sharedSizeBytes;  // dynamic + static must fit the opt-in limit
 }
 
+int max_chunk_smem() { return (max_smem_per_block() / kSlots) & ~15; }
+
 int count_occupancy(int block, int64_t smem_bytes) {
   ensure_attr();
   int occ = 0;
-  TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_count, block, (size_t)smem_bytes));
+  TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+      &occ, k_count, block, (size_t)(kSlots * slot_bytes_of(smem_bytes))));
   return occ;
 }
 
@@ -408,7 +588,9 @@ void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_b
   pv.n_long_chunks = P.n_long_chunks;
   pv.probe_mode = P.opt.probe_mode;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c_end - c_begin, P.grid));
-  k_count<<<grid, P.block, (size_t)P.smem_bytes, s>>>(pv, c_begin, c_end, e_begin, e_end, d_out);
+  const int64_t sb = slot_bytes_of(P.smem_bytes);
+  k_count<<<grid, P.block, (size_t)(kSlots * sb), s>>>(pv, c_begin, c_end, e_begin, e_end, sb,
+                                                      d_out);
   TC_LAUNCH();
 }
 

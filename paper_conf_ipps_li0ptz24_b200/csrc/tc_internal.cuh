@@ -65,7 +65,7 @@ struct Options {
   int chunk_cost = 16384;
   int seg_cost = 4;
   int huge_degree = 8192;
-  int block_threads = 512;
+  int block_threads = 1024;
   int table_factor = 3;
   int long_min = 32;
   int probe_mode = 0;
@@ -104,10 +104,11 @@ struct PlanView {
 
 // SMEM a chunk needs (bytes): per segment staging + per group descriptor +
 // hash slots.  Shared by the plan (sizing) and the kernel (layout).
-// Layout: sB int64[S] | sA int32[S+1] | sC int32[S] | sD int32[S] | sInfo
-// int32[G] | pad to 16 B | sHash int32[slots].
+// Layout of one chunk slot of the count kernel (tc_count.cu slot_view):
+// sB int64[S] | sGB int64[G] | sA int32[S+1] | sC int32[S] | sD int32[S] |
+// sInfo int32[G] | sGP int32[G+1] | pad to 16 B | sHash int32[slots].
 __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_t slots) {
-  return 8 * S + 4 * (S + 1) + 4 * S + 4 * S + 4 * G + 16 + 4 * slots;
+  return 20 * S + 16 * G + 8 + 16 + 4 * slots;
 }
 
 struct Plan {
@@ -146,6 +147,7 @@ void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_b
                   int64_t e_end, cudaStream_t s, unsigned long long* d_out);
 int count_occupancy(int block, int64_t smem_bytes);  // CTAs per SM (0 = cannot launch)
 int max_smem_per_block();
+int max_chunk_smem();  // SMEM one chunk slot may use (the kernel double-buffers)
 int num_sms();
 
 }  // namespace tc

@@ -70,7 +70,7 @@ def test_bad_arguments_rejected_before_device(tc):
     assert h.value is None
     bad = tc.Options(chunk_cost=8)
     assert L.tc_build_csr(None, None, 0, -1, 0, ctypes.byref(bad), None, ctypes.byref(h)) == 1
-    bad = tc.Options(block_threads=1024)
+    bad = tc.Options(block_threads=2048)
     assert L.tc_build_csr(None, None, 0, -1, 0, ctypes.byref(bad), None, ctypes.byref(h)) == 1
     assert L.tc_count(None, None, None) == 1
     assert L.tc_count_range(None, 0, 0, None, None) == 1

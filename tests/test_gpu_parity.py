@@ -106,6 +106,7 @@ def test_chung_lu_small(tc):
 @pytest.mark.parametrize("opts", [
     dict(chunk_cost=64), dict(chunk_cost=256), dict(chunk_cost=4096), dict(chunk_cost=1 << 20),
     dict(block_threads=64), dict(block_threads=128), dict(block_threads=256),
+    dict(block_threads=512), dict(block_threads=96),
     dict(seg_cost=1), dict(seg_cost=64), dict(table_factor=2), dict(table_factor=16),
     dict(huge_degree=1), dict(huge_degree=16), dict(huge_degree=16, chunk_cost=64),
     dict(long_min=1), dict(long_min=8), dict(long_min=1 << 30), dict(long_min=1 << 30, chunk_cost=64),
