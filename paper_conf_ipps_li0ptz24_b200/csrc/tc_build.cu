@@ -290,7 +290,8 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const int64_t* __re
                            const int32_t* __restrict__ gincl, int64_t S, int64_t S_long,
                            int bits, const int64_t* __restrict__ row_ptr,
                            const int64_t* __restrict__ e_lo, const int32_t* __restrict__ e_len,
-                           int huge_degree, int table_factor, int64_t* __restrict__ seg_start,
+                           int huge_degree, int table_factor, int64_t max_table_slots,
+                           int64_t* __restrict__ seg_start,
                            int32_t* __restrict__ seg_len, int32_t* __restrict__ seg_group,
                            int64_t* __restrict__ units, int64_t* __restrict__ grp_row,
                            int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots) {
@@ -309,12 +310,15 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const int64_t* __re
       const int64_t rs = row_ptr[v], d = row_ptr[v + 1] - rs;
       grp_row[g] = rs;
       grp_d[g] = d;
+      // table_factor * d slots (load <= 1/table_factor, > d so a linear probe
+      // always meets an empty slot), a multiple of 4 for 16-B initialisation;
+      // 0 = huge table (probed in global memory)
       int64_t slots = 0;
       if (d <= huge_degree) {
         int64_t want = d * table_factor;
-        if (want < d + 1) want = d + 1;  // an empty slot always exists
-        slots = 2;
-        while (slots < want) slots <<= 1;
+        if (want < d + 1) want = d + 1;
+        slots = (want + 3) & ~int64_t(3);
+        if (slots > max_table_slots) slots = 0;
       }
       grp_slots[g] = slots;
     }
@@ -372,29 +376,55 @@ __global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t 
   }
 }
 
-__global__ void k_chunk_smem(const int64_t* __restrict__ chunk_seg, int64_t n_chunks, int64_t nL,
-                             const int32_t* __restrict__ seg_group,
-                             const int64_t* __restrict__ slot_prefix,
-                             unsigned long long* out) {  // out[0] long max, out[1] short max
-  typedef cub::BlockReduce<unsigned long long, TPB> BR;
-  __shared__ typename BR::TempStorage tmp;
-  unsigned long long mx[2] = {0, 0};
+// SMEM-capped split of the cost chunks (one thread per chunk, sequential
+// over its edges): a piece grows edge by edge while its slot layout
+// (chunk_smem_bytes: edges, groups, hash slots, long-class tiles) fits
+// `limit`.  Pass 1 (bounds == nullptr) counts pieces per chunk and the
+// largest piece; pass 2 writes each piece's first edge at off[c] + j.
+__global__ void k_split(const int64_t* __restrict__ chunk_seg, int64_t n_chunks, int64_t nL,
+                        const int32_t* __restrict__ seg_group,
+                        const int64_t* __restrict__ slot_prefix,
+                        const int64_t* __restrict__ key_prefix, int64_t limit_long,
+                        int64_t limit_short, int64_t* __restrict__ pieces,
+                        const int64_t* __restrict__ off, int64_t* __restrict__ bounds,
+                        unsigned long long* need_max) {  // need_max[0] long, [1] short
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n_chunks;
        c += (int64_t)gridDim.x * blockDim.x) {
     const int64_t sa = chunk_seg[c], sb = chunk_seg[c + 1];
-    if (sa >= sb) continue;
-    const int64_t ga = seg_group[sa], gb = (int64_t)seg_group[sb - 1] + 1;
-    const int64_t b = chunk_smem_bytes(sb - sa, gb - ga, slot_prefix[gb] - slot_prefix[ga]);
-    mx[c >= nL] = max(mx[c >= nL], (unsigned long long)b);
-  }
-  unsigned long long r0 = BR(tmp).Reduce(mx[0], cub::Max());
-  __syncthreads();
-  unsigned long long r1 = BR(tmp).Reduce(mx[1], cub::Max());
-  if (threadIdx.x == 0) {
-    atomicMax(&out[0], r0);
-    atomicMax(&out[1], r1);
+    int64_t o = bounds ? off[c] : 0, cnt = 0;
+    if (sa >= sb) {  // an empty chunk stays one (empty) piece
+      if (bounds) bounds[o] = sa;
+      else pieces[c] = 1;
+      continue;
+    }
+    const bool is_long = c < nL;
+    const int64_t limit = is_long ? limit_long : limit_short;
+    unsigned long long* nm = need_max ? need_max + (is_long ? 0 : 1) : nullptr;
+    int64_t p0 = sa, g0 = seg_group[sa], ok_need = 0;
+    for (int64_t s = sa; s < sb; ++s) {
+      const int64_t g = seg_group[s];
+      const int64_t tiles = is_long ? (key_prefix[s + 1] - key_prefix[p0]) >> 5 : 0;
+      int64_t need = chunk_smem_bytes(s + 1 - p0, g - g0 + 1, slot_prefix[g + 1] - slot_prefix[g0], tiles);
+      if (need > limit && s > p0) {  // close the piece [p0, s), start a new one at s
+        if (bounds) bounds[o + cnt] = p0;
+        else atomicMax(nm, (unsigned long long)ok_need);
+        ++cnt;
+        p0 = s;
+        g0 = g;
+        const int64_t t1 = is_long ? (key_prefix[s + 1] - key_prefix[s]) >> 5 : 0;
+        need = chunk_smem_bytes(1, 1, slot_prefix[g + 1] - slot_prefix[g], t1);
+      }
+      ok_need = need;
+    }
+    if (bounds) bounds[o + cnt] = p0;
+    else {
+      atomicMax(nm, (unsigned long long)ok_need);
+      pieces[c] = cnt + 1;
+    }
   }
 }
+
+__global__ void k_set_i64(int64_t* p, int64_t v) { *p = v; }
 
 // exclusive prefix of `in` (length n) into out[0..n] (out[0] = 0, out[n] = total)
 void exclusive_prefix(const int64_t* in, int64_t n, int64_t* out, cudaStream_t s) {
@@ -568,6 +598,22 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
   g->ms[5] = tm.ms(0, 5);
 }
 
+Tuning tuning_from_env() {
+  Tuning t;
+  auto get = [](const char* name, int def, int lo, int hi) {
+    const char* v = std::getenv(name);
+    if (!v) return def;
+    int x = std::atoi(v);
+    return x < lo ? lo : (x > hi ? hi : x);
+  };
+  t.slots = get("TC_SLOTS", t.slots, 2, 4);
+  t.grab_long = get("TC_GRAB_LONG", t.grab_long, 0, 1 << 20);
+  t.grab_short = get("TC_GRAB_SHORT", t.grab_short, 0, 1 << 24);
+  t.prod_div = get("TC_PROD_DIV", t.prod_div, 2, 32);
+  t.wait_hint_ns = get("TC_WAIT_HINT", t.wait_hint_ns, 0, 10000000);
+  return t;
+}
+
 // ------------------------------------------------------------------ a6
 void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   Plan& P = g->plan;
@@ -643,13 +689,20 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   }
   const int64_t G = (int64_t)d2h(gincl.get() + (S - 1), s);
   P.G = G;
+  P.tune = tuning_from_env();
+  // SMEM of one chunk slot of the count kernel; a table may use at most half
+  // of it (bigger tables are "huge": probed in global memory)
+  const int64_t slot_limit = max_chunk_smem(P.tune.slots);
+  const int64_t flat_limit = max_flat_chunk_smem();
+  const int64_t max_table_slots = std::min(slot_limit, flat_limit) / 8;
   P.seg_start = DevBuf<int64_t>(S, s);
   P.seg_len = DevBuf<int32_t>(S, s);
   P.seg_group = DevBuf<int32_t>(S, s);
   DevBuf<int64_t> units(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
   k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted.get(), p_sorted.get(), gincl.get(), S, S_long,
                                          g->bits, row_ptr, e_lo.get(), e_len.get(),
-                                         opt.huge_degree, opt.table_factor, P.seg_start.get(),
+                                         opt.huge_degree, opt.table_factor, max_table_slots,
+                                         P.seg_start.get(),
                                          P.seg_len.get(), P.seg_group.get(), units.get(),
                                          grp_row.get(), grp_d.get(), grp_slots.get());
   TC_LAUNCH();
@@ -688,47 +741,47 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   tr("groups + prefixes + costs");
   P.units_total = h_cp[2];
 
-  // Chunking, per class: long chunks start 4x larger (their SMEM is one or
-  // two tables plus a few edges).  A class's chunk cost is halved while its
-  // largest chunk needs more SMEM than one of the count kernel's two chunk
-  // slots can hold.
-  const int64_t hard = max_chunk_smem();  // one of the kernel's two chunk slots
-  const int64_t soft = hard;
-  int64_t CL = std::max<int64_t>(4ll * opt.chunk_cost, 64), CS = std::max<int64_t>(opt.chunk_cost, 64);
-  DevBuf<unsigned long long> mx(2, s);
-  for (;;) {
-    const int64_t nL = (cost_long + CL - 1) / CL, nS = (cost_short + CS - 1) / CS, nc = nL + nS;
-    P.chunk_seg = DevBuf<int64_t>(nc + 1, s);
-    k_chunk_bounds<<<grid_for(nc + 1), TPB, 0, s>>>(cost_prefix.get(), S_long, S, nL, nS, CL, CS,
-                                                    P.chunk_seg.get());
+  // Chunking, per class: cost chunks (long class 4x larger: its edges carry
+  // ~150 keys each), then every chunk is split where its SMEM layout would
+  // exceed one of the count kernel's chunk slots (only outliers split).
+  const int64_t CL = std::max<int64_t>(4ll * opt.chunk_cost, 64), CS = std::max<int64_t>(opt.chunk_cost, 64);
+  {
+    const int64_t nL0 = (cost_long + CL - 1) / CL, nS0 = (cost_short + CS - 1) / CS, nc0 = nL0 + nS0;
+    DevBuf<int64_t> cs0(nc0 + 1, s), pieces(std::max<int64_t>(nc0, 1), s), poff(nc0 + 1, s);
+    k_chunk_bounds<<<grid_for(nc0 + 1), TPB, 0, s>>>(cost_prefix.get(), S_long, S, nL0, nS0, CL, CS,
+                                                     cs0.get());
     TC_LAUNCH();
+    DevBuf<unsigned long long> mx(2, s);
     TC_CUDA(cudaMemsetAsync(mx.get(), 0, 2 * sizeof(unsigned long long), s));
-    k_chunk_smem<<<grid_for(nc), TPB, 0, s>>>(P.chunk_seg.get(), nc, nL, P.seg_group.get(),
-                                              P.slot_prefix.get(), mx.get());
+    k_split<<<grid_for(nc0), TPB, 0, s>>>(cs0.get(), nc0, nL0, P.seg_group.get(), P.slot_prefix.get(),
+                                          P.key_prefix.get(), slot_limit, flat_limit, pieces.get(),
+                                          nullptr, nullptr, mx.get());
     TC_LAUNCH();
-    unsigned long long need[2];
+    exclusive_prefix(pieces.get(), nc0, poff.get(), s);
+    int64_t h_off[2];
+    TC_CUDA(cudaMemcpyAsync(&h_off[0], poff.get() + nL0, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaMemcpyAsync(&h_off[1], poff.get() + nc0, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    unsigned long long need[2] = {0, 0};
     TC_CUDA(cudaMemcpyAsync(need, mx.get(), sizeof(need), cudaMemcpyDeviceToHost, s));
     TC_CUDA(cudaStreamSynchronize(s));
-    auto shrink = [&](int64_t& C, int64_t nd) {
-      if ((nd > (unsigned long long)soft && C > 1024) || (nd > (unsigned long long)hard && C > 64)) {
-        C >>= 1;
-        return true;
-      }
-      return false;
-    };
-    if (tr.on)
-      fprintf(stderr, "[tc]   chunks CL=%lld CS=%lld nL=%lld nS=%lld smem long %llu short %llu\n",
-              (long long)CL, (long long)CS, (long long)nL, (long long)nS, need[0], need[1]);
-    const bool again_l = shrink(CL, (int64_t)need[0]);
-    const bool again_s = shrink(CS, (int64_t)need[1]);
-    if (again_l || again_s) continue;
-    const int64_t nd = (int64_t)std::max(need[0], need[1]);
-    if (nd > hard)
-      fail(TC_ERR_UNSUPPORTED, "a chunk's hash tables exceed shared memory (lower huge_degree)");
+    if ((int64_t)need[0] > slot_limit || (int64_t)need[1] > flat_limit)
+      fail(TC_ERR_UNSUPPORTED, "an edge's hash table exceeds shared memory (lower huge_degree)");
+    const int64_t nc = h_off[1];
+    P.chunk_seg = DevBuf<int64_t>(nc + 1, s);
+    k_split<<<grid_for(nc0), TPB, 0, s>>>(cs0.get(), nc0, nL0, P.seg_group.get(), P.slot_prefix.get(),
+                                          P.key_prefix.get(), slot_limit, flat_limit, nullptr,
+                                          poff.get(), P.chunk_seg.get(), nullptr);
+    TC_LAUNCH();
+    k_set_i64<<<1, 1, 0, s>>>(P.chunk_seg.get() + nc, S);
+    TC_LAUNCH();
     P.n_chunks = nc;
-    P.n_long_chunks = nL;
-    P.smem_bytes = nd;
-    break;
+    P.n_long_chunks = h_off[0];
+    P.smem_bytes = std::max<int64_t>((int64_t)need[0], 16);
+    P.smem_flat = std::max<int64_t>((int64_t)need[1], 16);
+    if (tr.on)
+      fprintf(stderr, "[tc]   chunks CL=%lld CS=%lld cost chunks %lld (long %lld) -> %lld (long %lld), smem long %llu short %llu\n",
+              (long long)CL, (long long)CS, (long long)nc0, (long long)nL0, (long long)nc,
+              (long long)h_off[0], need[0], need[1]);
   }
   P.chunk_cost_long = CL;
   P.chunk_cost_short = CS;
@@ -737,9 +790,13 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   TC_CUDA(cudaMemcpyAsync(P.h_chunk_seg.data(), P.chunk_seg.get(),
                           sizeof(int64_t) * (P.n_chunks + 1), cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));
-  const int occ = count_occupancy(P.block, P.smem_bytes);
-  if (occ < 1) fail(TC_ERR_UNSUPPORTED, "count kernel cannot launch with this SMEM/block size");
-  P.grid = (int)std::min<int64_t>(P.n_chunks, (int64_t)occ * num_sms());
+  const int occ = count_occupancy(P.block, P.smem_bytes, P.tune.slots);
+  const int occ_flat = flat_occupancy(P.smem_flat);
+  if (occ < 1 || occ_flat < 1)
+    fail(TC_ERR_UNSUPPORTED, "count kernel cannot launch with this SMEM/block size");
+  P.grid = (int)std::min<int64_t>(std::max<int64_t>(P.n_long_chunks, 1), (int64_t)occ * num_sms());
+  P.grid_flat = (int)std::min<int64_t>(std::max<int64_t>(P.n_chunks - P.n_long_chunks, 1),
+                                       (int64_t)occ_flat * num_sms());
   tr("chunk copy + occupancy");
 }
 

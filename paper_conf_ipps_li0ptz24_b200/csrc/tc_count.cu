@@ -38,12 +38,12 @@
 namespace tc {
 namespace {
 
-constexpr int kMaxBlock = 1024;
+constexpr int kMaxBlock = 1024;  // warp-specialised kernel (long class)
+constexpr int kFlatBlock = 512;  // flat kernel (short class), 3 CTAs per SM
 constexpr int kUnrollLong = 8;   // tiles in flight per consumer warp (long class)
 constexpr int kUnrollShort = 4;  // tiles in flight per consumer warp (short class)
 constexpr int kMaxKicks = 96;    // cuckoo displacement bound before the linear fallback
-constexpr int kSlots = 2;        // chunk slots (double buffering)
-constexpr int kProdDiv = 4;      // 1/kProdDiv of the warps are producers
+constexpr int kMaxSlots = 4;     // chunk slots in SMEM (runtime count: Tuning::slots)
 
 // ------------------------------------------------------------------ mbarrier (PTX)
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -56,13 +56,22 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* b) {
   asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n\t}" ::"r"(smem_u32(b))
                : "memory");
 }
-__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(b)),
-      "r"(parity)
-      : "memory");
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity, uint32_t hint_ns) {
+  if (hint_ns) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tWAITH_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+        "@!p bra WAITH_%=;\n\t}" ::"r"(smem_u32(b)),
+        "r"(parity), "r"(hint_ns)
+        : "memory");
+  } else {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(b)),
+        "r"(parity)
+        : "memory");
+  }
 }
 __device__ __forceinline__ void named_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
@@ -80,36 +89,34 @@ __device__ __forceinline__ int named_sync_or(int id, int nthreads, int pred) {
 }
 
 // ------------------------------------------------------------------ hashing
-// Table descriptor tab = (slot offset << 5) | sh with sh = 32 - log2(slots):
-// the slot of a key is the top log2(slots) bits of a multiplicative hash.
-__device__ __forceinline__ uint32_t hash1(int32_t key, int sh) {
-  return ((uint32_t)key * 0x9E3779B1u) >> sh;
+// A table is (off, n): n slots starting at sHash[off].  The slot of a key is
+// a multiplicative hash mapped onto [0, n) by a 32x32 -> high-32 multiply
+// (no power-of-two rounding, so the load stays at 1/table_factor).
+__device__ __forceinline__ uint32_t hash1(int32_t key, uint32_t n) {
+  return __umulhi((uint32_t)key * 0x9E3779B1u, n);
 }
-__device__ __forceinline__ uint32_t hash2(int32_t key, int sh) {
-  return ((uint32_t)key * 0x85EBCA77u + 0x7F4A7C15u) >> sh;
+__device__ __forceinline__ uint32_t hash2(int32_t key, uint32_t n) {
+  return __umulhi((uint32_t)key * 0x85EBCA77u + 0x7F4A7C15u, n);
 }
 
-__device__ __forceinline__ bool cuckoo_insert(int* __restrict__ T, int tab, int32_t key) {
-  const int off = tab >> 5, sh = tab & 31;
-  uint32_t pos = hash1(key, sh);
+__device__ __forceinline__ bool cuckoo_insert(int* __restrict__ T, uint32_t n, int32_t key) {
+  uint32_t pos = hash1(key, n);
   for (int i = 0; i < kMaxKicks; ++i) {
-    const int old = atomicExch(&T[off + pos], key);
+    const int old = atomicExch(&T[pos], key);
     if (old < 0) return true;
     key = old;  // displaced: move it to its other slot
-    const uint32_t p1 = hash1(key, sh);
-    pos = (pos == p1) ? hash2(key, sh) : p1;
+    const uint32_t p1 = hash1(key, n);
+    pos = (pos == p1) ? hash2(key, n) : p1;
   }
   return false;  // `key` is homeless: the chunk rebuilds with linear probing
 }
 
-__device__ __forceinline__ void linear_insert(int* __restrict__ T, int tab, int32_t key) {
-  const int off = tab >> 5, sh = tab & 31;
-  const uint32_t mask = 0xffffffffu >> sh;
-  uint32_t h = hash1(key, sh);
+__device__ __forceinline__ void linear_insert(int* __restrict__ T, uint32_t n, int32_t key) {
+  uint32_t h = hash1(key, n);
   for (;;) {
-    const int prev = atomicCAS(&T[off + h], -1, key);
+    const int prev = atomicCAS(&T[h], -1, key);
     if (prev == -1 || prev == key) return;
-    h = (h + 1) & mask;
+    h = (h + 1 == n) ? 0 : h + 1;
   }
 }
 
@@ -124,61 +131,65 @@ __device__ __noinline__ unsigned global_probe(const int32_t* __restrict__ col, i
   return (lo < b + d && __ldg(col + lo) == key) ? 1u : 0u;
 }
 
-// Membership of key in one SMEM table: T = first slot, sh = 32 - log2(slots).
-// Keys are >= 0, empty slots hold -1, and the sentinel -2 (padding lanes)
-// never matches and always terminates.
+// Membership of key in the SMEM table T[0, n).  Keys are >= 0, empty slots
+// hold -1, and the sentinel -2 (padding lanes) never matches and always
+// terminates (a table has more slots than keys).
 template <bool kLinear>
-__device__ __forceinline__ unsigned table_probe(const int* __restrict__ T, int sh, int32_t key) {
+__device__ __forceinline__ unsigned table_probe(const int* __restrict__ T, uint32_t n, int32_t key) {
   if (!kLinear) {
     // two-choice table: a key lives at hash1 or hash2; both reads are issued
-    const int x1 = T[hash1(key, sh)];
-    const int x2 = T[hash2(key, sh)];
+    const int x1 = T[hash1(key, n)];
+    const int x2 = T[hash2(key, n)];
     return (x1 == key) | (x2 == key);
   }
-  const uint32_t mask = 0xffffffffu >> sh;
-  uint32_t h = hash1(key, sh);
+  uint32_t h = hash1(key, n);
   for (;;) {
     const int x = T[h];
     if (x == key) return 1u;
     if (x < 0) return 0u;
-    h = (h + 1) & mask;
+    h = (h + 1 == n) ? 0 : h + 1;
   }
 }
 
+__device__ __forceinline__ unsigned huge_probe(const PlanView& pv, int64_t g, int32_t key) {
+  const int64_t ib = pv.ins_prefix[g];
+  return global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, key);
+}
+
 // ------------------------------------------------------------------ chunk slot
-// One slot = the staged edges, groups and tables of one chunk.  Layout (bytes,
-// region 16-B aligned): sB int64[S] | sGB int64[G] | sA int32[S+1] | sC
-// int32[S] | sD int32[S] | sInfo int32[G] | sGP int32[G+1] | pad | sHash.
-// chunk_smem_bytes (tc_internal.cuh) is the matching size.
+// One slot = the staged edges, groups, tiles and tables of one chunk; layout
+// in chunk_smem_bytes (tc_internal.cuh).
 struct SlotHdr {
   long long sa, ga;
-  int S, G, nslots, is_long, linear, done, huge, pad;
+  int S, G, T, nslots, is_long, linear, done, huge, next, pad;  // next: work-grab counter
 };
 
 struct ChunkSmem {
+  int4* sTile;   // [T] long class: {key pointer lo, hi, table offset (or -1-g), n << 6 | lanes}
   int64_t* sB;   // long: key start in col; short: start - (chunk-relative first key)
   int64_t* sGB;  // group: row start of N+(v) - sGP (so col[sGB[g] + k] is insert k)
+  int2* sInfo;   // [G] table {slot offset, slots}; offset -1 = huge
   int* sA;       // [S+1] long: tile prefix; short: key prefix (chunk-relative)
-  int* sC;       // long: suffix length
+  int* sC;       // suffix length
   int* sD;       // group index (chunk-local)
-  int* sInfo;    // [G] table descriptor (-1: huge)
   int* sGP;      // [G+1] insert prefix (chunk-relative)
   int* sHash;    // slots
 };
 
-__device__ __forceinline__ ChunkSmem slot_view(unsigned char* region, int S, int G) {
+__device__ __forceinline__ ChunkSmem slot_view(unsigned char* region, int S, int G, int T) {
   ChunkSmem c;
-  c.sB = reinterpret_cast<int64_t*>(region);
+  c.sTile = reinterpret_cast<int4*>(region);
+  c.sB = reinterpret_cast<int64_t*>(c.sTile + T);
   c.sGB = c.sB + S;
-  c.sA = reinterpret_cast<int*>(c.sGB + G);
+  c.sInfo = reinterpret_cast<int2*>(c.sGB + G);
+  c.sA = reinterpret_cast<int*>(c.sInfo + G);
   c.sC = c.sA + S + 1;
   c.sD = c.sC + S;
-  c.sInfo = c.sD + S;
-  c.sGP = c.sInfo + G;
+  c.sGP = c.sD + S;
   // 16-B aligned start of the slots as an int offset from the aligned region
   // base, so every table access stays in the shared window (LDS/ATOMS)
   c.sHash = reinterpret_cast<int*>(region) +
-            ((2 * S + 2 * G + (S + 1) + 2 * S + G + (G + 1) + 3) & ~3);
+            ((4 * T + 2 * S + 2 * G + 2 * G + (S + 1) + 2 * S + (G + 1) + 3) & ~3);
   return c;
 }
 
@@ -230,40 +241,40 @@ __device__ __forceinline__ void warp_walk(const int* __restrict__ P, int S, int 
 }
 
 // ------------------------------------------------------------------ consumers
-// LONG class: the warp owns tiles [t0, t1) of the chunk; each tile is 32
-// consecutive keys of one edge.  The warp walks edge by edge (warp-uniform
-// bookkeeping); inside an edge, lane l reads keys l, l+32, ... through one
-// pointer with immediate offsets, kUnrollLong tiles in flight; lanes past
-// the end carry the never-matching sentinel so the probes run unpredicated.
+// LONG class: the warp owns tiles [t0, t1) of the chunk.  Each tile is 32
+// consecutive keys of one edge, described by one 16-B sTile entry the
+// producers wrote (key pointer, valid lanes, table), so kUnrollLong loads are
+// in flight per lane across edge boundaries with no per-edge bookkeeping;
+// padding lanes carry the never-matching sentinel and probe unpredicated.
 template <bool kLinear, bool kHuge>
-__device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int S, int t0, int t1,
+__device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1,
                                               const PlanView& pv, int64_t ga) {
   unsigned cnt = 0;
-  if (t0 >= t1) return cnt;
   const int lane = threadIdx.x & 31;
-  int s = seg_of(c.sA, S, t0);
-  for (int t = t0; t < t1; ++s) {
-    const int ts = c.sA[s], te = min(c.sA[s + 1], t1);
-    const int done = (t - ts) << 5;                             // keys of this edge before tile t
-    const int lim = min(c.sC[s] - done, (te - t) << 5) - lane;  // lane's keys: 32*i < lim
-    const int32_t* __restrict__ p = pv.col + c.sB[s] + done + lane;
-    const int gl = c.sD[s];
-    const int tab = c.sInfo[gl];
-    t = te;
-    if (kHuge && tab < 0) {
-      const int64_t g = ga + gl, ib = pv.ins_prefix[g];
-      for (int i = 0; i < lim; i += 32)
-        cnt += global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, __ldg(p + i));
-      continue;
+  for (int t = t0; t < t1; t += kUnrollLong) {
+    int32_t key[kUnrollLong];
+    int toff[kUnrollLong], tn[kUnrollLong];
+#pragma unroll
+    for (int u = 0; u < kUnrollLong; ++u) {
+      key[u] = -2;
+      toff[u] = 0;
+      tn[u] = 1;
+      if (t + u < t1) {
+        const int4 d = c.sTile[t + u];
+        const int64_t p = (int64_t)(((uint64_t)(uint32_t)d.y << 32) | (uint32_t)d.x);
+        toff[u] = d.z;
+        tn[u] = d.w >> 6;
+        if (lane < (d.w & 63)) key[u] = __ldg(pv.col + p + lane);
+      }
     }
-    const int* __restrict__ T = c.sHash + (tab >> 5);
-    const int sh = tab & 31;
-    for (int i = 0; i < lim; i += 32 * kUnrollLong) {
-      int32_t key[kUnrollLong];
 #pragma unroll
-      for (int u = 0; u < kUnrollLong; ++u) key[u] = (i + 32 * u < lim) ? __ldg(p + i + 32 * u) : -2;
-#pragma unroll
-      for (int u = 0; u < kUnrollLong; ++u) cnt += table_probe<kLinear>(T, sh, key[u]);
+    for (int u = 0; u < kUnrollLong; ++u) {
+      if (kHuge && toff[u] < 0) {
+        if (key[u] >= 0) cnt += huge_probe(pv, ga + (-1 - toff[u]), key[u]);
+      } else if (!kLinear || key[u] >= 0) {  // a linear probe of a padding tile's
+        // dummy 1-slot table might never meet an empty slot: skip sentinels
+        cnt += table_probe<kLinear>(c.sHash + toff[u], (uint32_t)tn[u], key[u]);
+      }
     }
   }
   return cnt;
@@ -291,17 +302,15 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
       s += __popc(M);
     }
     int32_t key[kUnrollShort];
-    int tab[kUnrollShort], gl[kUnrollShort];
+    int gl[kUnrollShort];
 #pragma unroll
     for (int u = 0; u < kUnrollShort; ++u) {
       const int k = k0 + 32 * u + lane;
-      key[u] = 0;
-      tab[u] = 0;
+      key[u] = -2;
       gl[u] = 0;
       if (k < k1w) {
         key[u] = __ldg(pv.col + c.sB[seg[u]] + k);
         gl[u] = c.sD[seg[u]];
-        tab[u] = c.sInfo[gl[u]];
       }
     }
 #pragma unroll
@@ -309,12 +318,9 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
       // padding lanes have no table of their own: they must not probe (a
       // linear probe needs a table with an empty slot to terminate)
       if (k0 + 32 * u + lane >= k1w) continue;
-      if (kHuge && tab[u] < 0) {
-        const int64_t g = ga + gl[u], ib = pv.ins_prefix[g];
-        cnt += global_probe(pv.col, pv.grp_ibase[g] + ib, pv.ins_prefix[g + 1] - ib, key[u]);
-      } else {
-        cnt += table_probe<kLinear>(c.sHash + (tab[u] >> 5), tab[u] & 31, key[u]);
-      }
+      const int2 d = c.sInfo[gl[u]];
+      if (kHuge && d.x < 0) cnt += huge_probe(pv, ga + gl[u], key[u]);
+      else cnt += table_probe<kLinear>(c.sHash + d.x, (uint32_t)d.y, key[u]);
     }
   }
   return cnt;
@@ -324,8 +330,8 @@ template <bool kLinear>
 __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
                                             const PlanView& pv) {
   if (h.is_long)
-    return h.huge ? walk_long<kLinear, true>(c, h.S, w0, w1, pv, h.ga)
-                  : walk_long<kLinear, false>(c, h.S, w0, w1, pv, h.ga);
+    return h.huge ? walk_long<kLinear, true>(c, w0, w1, pv, h.ga)
+                  : walk_long<kLinear, false>(c, w0, w1, pv, h.ga);
   return h.huge ? walk_short<kLinear, true>(c, h.S, w0, w1, pv, h.ga)
                 : walk_short<kLinear, false>(c, h.S, w0, w1, pv, h.ga);
 }
@@ -335,10 +341,11 @@ __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h
 // in [0, PT); the PT producer threads synchronise on named barrier 1.  The
 // header is written by producer 0 before its own mbarrier arrive, so the
 // consumers see it once every producer has arrived.
+template <int kB>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
                                         int pt, int PT) {
-  const int64_t sa = max(pv.chunk_seg[cix], e_begin), sb = min(pv.chunk_seg[cix + 1], e_end);
+  const int64_t sa = max(__ldg(pv.chunk_seg + (cix)), e_begin), sb = min(__ldg(pv.chunk_seg + (cix + 1)), e_end);
   if (sa >= sb) {  // empty after clipping to the range
     if (pt == 0) {
       hdr.S = 0;
@@ -348,17 +355,17 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   }
   const bool is_long = cix < pv.n_long_chunks;
   const int S = (int)(sb - sa);
-  const int64_t ga = pv.seg_group[sa], gb = (int64_t)pv.seg_group[sb - 1] + 1;
+  const int64_t ga = __ldg(pv.seg_group + (sa)), gb = (int64_t)__ldg(pv.seg_group + (sb - 1)) + 1;
   const int G = (int)(gb - ga);
-  const int64_t slot0 = pv.slot_prefix[ga];
-  const int nslots = (int)(pv.slot_prefix[gb] - slot0);
-  ChunkSmem c = slot_view(region, S, G);
+  const int64_t slot0 = __ldg(pv.slot_prefix + (ga));
+  const int nslots = (int)(__ldg(pv.slot_prefix + (gb)) - slot0);
+  const int64_t kp0 = __ldg(pv.key_prefix + (sa));
+  const int T = is_long ? (int)((__ldg(pv.key_prefix + (sb)) - kp0) >> 5) : 0;
+  ChunkSmem c = slot_view(region, S, G, T);
 
   // 1. stage edges and groups; empty slots.  Each producer thread handles
   //    kB items per batch with all their global loads issued before any
   //    store, so a batch costs one memory latency.
-  constexpr int kB = 4;
-  const int64_t kp0 = pv.key_prefix[sa];
   for (int base = pt; base <= S; base += PT * kB) {
     int64_t kp[kB], st[kB];
     int ln[kB], gr[kB];
@@ -368,11 +375,11 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       kp[r] = 0;
       st[r] = 0;
       ln[r] = gr[r] = 0;
-      if (i <= S) kp[r] = pv.key_prefix[sa + i];
+      if (i <= S) kp[r] = __ldg(pv.key_prefix + (sa + i));
       if (i < S) {
-        st[r] = pv.seg_start[sa + i];
-        ln[r] = pv.seg_len[sa + i];
-        gr[r] = pv.seg_group[sa + i];
+        st[r] = __ldg(pv.seg_start + (sa + i));
+        ln[r] = __ldg(pv.seg_len + (sa + i));
+        gr[r] = __ldg(pv.seg_group + (sa + i));
       }
     }
 #pragma unroll
@@ -387,7 +394,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       }
     }
   }
-  const int64_t ip0 = pv.ins_prefix[ga];
+  const int64_t ip0 = __ldg(pv.ins_prefix + (ga));
   int huge = 0;
   for (int base = pt; base <= G; base += PT * kB) {
     int64_t ip[kB], sp[kB], sp1[kB], ib[kB];
@@ -395,11 +402,11 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     for (int r = 0; r < kB; ++r) {
       const int i = base + r * PT;
       ip[r] = sp[r] = sp1[r] = ib[r] = 0;
-      if (i <= G) ip[r] = pv.ins_prefix[ga + i];
+      if (i <= G) ip[r] = __ldg(pv.ins_prefix + (ga + i));
       if (i < G) {
-        sp[r] = pv.slot_prefix[ga + i];
-        sp1[r] = pv.slot_prefix[ga + i + 1];
-        ib[r] = pv.grp_ibase[ga + i];
+        sp[r] = __ldg(pv.slot_prefix + (ga + i));
+        sp1[r] = __ldg(pv.slot_prefix + (ga + i + 1));
+        ib[r] = __ldg(pv.grp_ibase + (ga + i));
       }
     }
 #pragma unroll
@@ -407,8 +414,8 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       const int i = base + r * PT;
       if (i <= G) c.sGP[i] = (int)(ip[r] - ip0);
       if (i < G) {
-        const int64_t ns = sp1[r] - sp[r];
-        c.sInfo[i] = ns > 0 ? (((int)(sp[r] - slot0)) << 5) | (32 - (31 - __clz((int)ns))) : -1;
+        const int ns = (int)(sp1[r] - sp[r]);
+        c.sInfo[i] = ns > 0 ? make_int2((int)(sp[r] - slot0), ns) : make_int2(-1, 0);
         huge |= ns == 0;
         c.sGB[i] = ib[r] + ip0;  // row start - chunk-relative insert prefix
       }
@@ -421,7 +428,22 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   }
   const int any_huge = named_sync_or(1, PT, huge);
 
-  // 2. hash N+(v) of every group touched by the chunk (flattened over groups,
+  // 2. long class: one descriptor per 32-key tile (producer thread per edge)
+  if (is_long) {
+    for (int i = pt; i < S; i += PT) {
+      const int ts = c.sA[i], te = c.sA[i + 1], len = c.sC[i], gl = c.sD[i];
+      const int2 d = c.sInfo[gl];
+      const int toff = d.x >= 0 ? d.x : -1 - gl;
+      const int64_t st = c.sB[i];
+      for (int t = ts; t < te; ++t) {
+        const int64_t p = st + ((int64_t)(t - ts) << 5);
+        const int lanes = min(32, len - ((t - ts) << 5));
+        c.sTile[t] = make_int4((int)(uint32_t)p, (int)(p >> 32), toff, (d.y << 6) | lanes);
+      }
+    }
+  }
+
+  // 3. hash N+(v) of every group touched by the chunk (flattened over groups,
   //    kInsU tiles of N+(v) loads in flight per producer lane)
   constexpr int kInsU = 4;
   const int pw = pt >> 5, npw = PT >> 5;
@@ -431,22 +453,22 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   bool linear = pv.probe_mode == 1;
   if (linear) {
     warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
-      const int tab = c.sInfo[g];
-      if (tab >= 0) linear_insert(c.sHash, tab, key);
+      const int2 d = c.sInfo[g];
+      if (d.x >= 0) linear_insert(c.sHash + d.x, (uint32_t)d.y, key);
     });
   } else {
     bool ok = true;
     warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
-      const int tab = c.sInfo[g];
-      if (tab >= 0 && !cuckoo_insert(c.sHash, tab, key)) ok = false;
+      const int2 d = c.sInfo[g];
+      if (d.x >= 0 && !cuckoo_insert(c.sHash + d.x, (uint32_t)d.y, key)) ok = false;
     });
     if (named_sync_or(1, PT, !ok)) {  // uniform over producers: rebuild with linear probing
       linear = true;
       for (int i = pt; i < nslots; i += PT) c.sHash[i] = -1;
       named_sync(1, PT);
       warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
-        const int tab = c.sInfo[g];
-        if (tab >= 0) linear_insert(c.sHash, tab, key);
+        const int2 d = c.sInfo[g];
+        if (d.x >= 0) linear_insert(c.sHash + d.x, (uint32_t)d.y, key);
       });
     }
   }
@@ -455,27 +477,31 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     hdr.ga = ga;
     hdr.S = S;
     hdr.G = G;
+    hdr.T = T;
     hdr.nslots = nslots;
     hdr.is_long = is_long;
     hdr.linear = linear;
     hdr.done = 0;
     hdr.huge = any_huge;
+    hdr.next = 0;
   }
 }
 
 __global__ void __launch_bounds__(kMaxBlock, 1)
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
-            int64_t slot_bytes, unsigned long long* __restrict__ out) {
+            int64_t slot_bytes, Tuning tu, unsigned long long* __restrict__ out) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ unsigned long long red[kMaxBlock / 32];
-  __shared__ __align__(8) uint64_t full_bar[kSlots];
-  __shared__ __align__(8) uint64_t empty_bar[kSlots];
-  __shared__ SlotHdr hdr[kSlots];
+  __shared__ __align__(8) uint64_t full_bar[kMaxSlots];
+  __shared__ __align__(8) uint64_t empty_bar[kMaxSlots];
+  __shared__ SlotHdr hdr[kMaxSlots];
   const int warp = threadIdx.x >> 5, nw = blockDim.x >> 5, lane = threadIdx.x & 31;
-  const int n_prod = max(1, nw / kProdDiv), n_cons = nw - n_prod;
+  const int n_prod = max(1, min(nw - 1, nw / tu.prod_div)), n_cons = nw - n_prod;
   const int PT = n_prod * 32;
+  const int nslots = tu.slots;
+  const uint32_t hint = (uint32_t)tu.wait_hint_ns;
   if (threadIdx.x == 0) {
-    for (int i = 0; i < kSlots; ++i) {
+    for (int i = 0; i < nslots; ++i) {
       mbar_init(&full_bar[i], PT);       // every producer thread arrives
       mbar_init(&empty_bar[i], n_cons);  // one lane per consumer warp
     }
@@ -486,31 +512,43 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
   if (warp < n_prod) {
     // ------------------------------------------------------------ producers
     for (int64_t k = 0;; ++k) {
-      const int slot = (int)(k & 1);
-      const uint32_t j = (uint32_t)(k >> 1);  // fill number of this slot
-      if (j > 0) mbar_wait(&empty_bar[slot], (j - 1) & 1);
+      const int slot = (int)(k % nslots);
+      const uint32_t j = (uint32_t)(k / nslots);  // fill number of this slot
+      if (j > 0) mbar_wait(&empty_bar[slot], (j - 1) & 1, hint);
       const int64_t cix = c_begin + blockIdx.x + k * gridDim.x;
       if (cix >= c_end) {
         if (threadIdx.x == 0) hdr[slot].done = 1;
         mbar_arrive(&full_bar[slot]);
         break;
       }
-      produce(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], threadIdx.x, PT);
+      produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], threadIdx.x, PT);
       mbar_arrive(&full_bar[slot]);
     }
   } else {
     // ------------------------------------------------------------ consumers
     const int cw = warp - n_prod;
     for (int64_t k = 0;; ++k) {
-      const int slot = (int)(k & 1);
-      mbar_wait(&full_bar[slot], (uint32_t)((k >> 1) & 1));
+      const int slot = (int)(k % nslots);
+      mbar_wait(&full_bar[slot], (uint32_t)((k / nslots) & 1), hint);
       const SlotHdr h = hdr[slot];
       if (h.done) break;
       if (h.S > 0) {
-        const ChunkSmem c = slot_view(smem + slot * slot_bytes, h.S, h.G);
-        const int NU = c.sA[h.S];
-        const int w0 = (int)((int64_t)NU * cw / n_cons), w1 = (int)((int64_t)NU * (cw + 1) / n_cons);
-        acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+        const ChunkSmem c = slot_view(smem + slot * slot_bytes, h.S, h.G, h.T);
+        const int NU = h.is_long ? h.T : c.sA[h.S];
+        const int grab = h.is_long ? tu.grab_long : tu.grab_short;
+        if (grab <= 0) {  // static split: a contiguous share per consumer warp
+          const int w0 = (int)((int64_t)NU * cw / n_cons), w1 = (int)((int64_t)NU * (cw + 1) / n_cons);
+          acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+        } else {  // dynamic: grab `grab` units at a time from the slot's counter
+          for (;;) {
+            int w0 = 0;
+            if (lane == 0) w0 = atomicAdd(&hdr[slot].next, grab);
+            w0 = __shfl_sync(0xffffffffu, w0, 0);
+            if (w0 >= NU) break;
+            const int w1 = min(w0 + grab, NU);
+            acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+          }
+        }
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty_bar[slot]);
@@ -530,51 +568,75 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
   }
 }
 
+// SHORT-class chunks: every warp stages, builds and probes (no producer /
+// consumer split: a short chunk's table building is as much work as its
+// probing), one chunk slot per CTA and 3 CTAs per SM so that one CTA's
+// staging and building latency overlaps the others' probing.
+__global__ void __launch_bounds__(kFlatBlock, 3)
+    k_count_flat(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
+                 unsigned long long* __restrict__ out) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ unsigned long long red[kFlatBlock / 32];
+  __shared__ SlotHdr hdr;
+  const int warp = threadIdx.x >> 5, nw = blockDim.x >> 5, lane = threadIdx.x & 31;
+  unsigned long long acc = 0;
+  for (int64_t cix = c_begin + blockIdx.x; cix < c_end; cix += gridDim.x) {
+    produce<2>(pv, cix, e_begin, e_end, smem, hdr, threadIdx.x, blockDim.x);
+    __syncthreads();
+    const SlotHdr h = hdr;
+    if (h.S > 0) {
+      const ChunkSmem c = slot_view(smem, h.S, h.G, h.T);  // short class only: T = 0
+      const int NU = c.sA[h.S];
+      const int w0 = (int)((int64_t)NU * warp / nw), w1 = (int)((int64_t)NU * (warp + 1) / nw);
+      if (h.linear)
+        acc += h.huge ? walk_short<true, true>(c, h.S, w0, w1, pv, h.ga)
+                      : walk_short<true, false>(c, h.S, w0, w1, pv, h.ga);
+      else
+        acc += h.huge ? walk_short<false, true>(c, h.S, w0, w1, pv, h.ga)
+                      : walk_short<false, false>(c, h.S, w0, w1, pv, h.ga);
+    }
+    __syncthreads();  // the slot is rebuilt by the next chunk
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_down_sync(0xffffffffu, acc, o);
+  if (lane == 0) red[warp] = acc;
+  __syncthreads();
+  if (warp == 0) {
+    unsigned long long v = lane < nw ? red[lane] : 0ull;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+    if (lane == 0 && v) atomicAdd(out, v);
+  }
+}
+
 bool g_attr_set = false;
+
+int optin_smem() {
+  int dev = 0, v = 0;
+  TC_CUDA(cudaGetDevice(&dev));
+  TC_CUDA(cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  return v;
+}
+
+int static_smem(const void* f) {
+  cudaFuncAttributes fa;
+  TC_CUDA(cudaFuncGetAttributes(&fa, f));
+  return (int)fa.sharedSizeBytes;
+}
 
 void ensure_attr() {
   if (g_attr_set) return;
   TC_CUDA(cudaFuncSetAttribute(k_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               max_smem_per_block()));
+                               optin_smem() - static_smem((const void*)k_count)));
+  TC_CUDA(cudaFuncSetAttribute(k_count_flat, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               optin_smem() - static_smem((const void*)k_count_flat)));
   g_attr_set = true;
 }
 
 int64_t slot_bytes_of(int64_t need) { return (need + 15) & ~int64_t(15); }
 
-}  // namespace
-
-int num_sms() {
-  int dev = 0, v = 0;
-  TC_CUDA(cudaGetDevice(&dev));
-  TC_CUDA(cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev));
-  return v;
-}
-
-int max_smem_per_block() {
-  int dev = 0, v = 0;
-  TC_CUDA(cudaGetDevice(&dev));
-  TC_CUDA(cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
-  cudaFuncAttributes fa;
-  TC_CUDA(cudaFuncGetAttributes(&fa, k_count));
-  return v - (int)fa.sharedSizeBytes;  // dynamic + static must fit the opt-in limit
-}
-
-int max_chunk_smem() { return (max_smem_per_block() / kSlots) & ~15; }
-
-int count_occupancy(int block, int64_t smem_bytes) {
-  ensure_attr();
-  int occ = 0;
-  TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-      &occ, k_count, block, (size_t)(kSlots * slot_bytes_of(smem_bytes))));
-  return occ;
-}
-
-void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
-                  int64_t e_end, cudaStream_t s, unsigned long long* d_out) {
-  TC_CUDA(cudaMemsetAsync(d_out, 0, sizeof(unsigned long long), s));
+PlanView plan_view(const tc_graph* g) {
   const Plan& P = g->plan;
-  if (c_end <= c_begin || e_end <= e_begin) return;
-  ensure_attr();
   PlanView pv;
   pv.col = g->col.get();
   pv.key_prefix = P.key_prefix.get();
@@ -587,11 +649,71 @@ void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_b
   pv.chunk_seg = P.chunk_seg.get();
   pv.n_long_chunks = P.n_long_chunks;
   pv.probe_mode = P.opt.probe_mode;
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(c_end - c_begin, P.grid));
-  const int64_t sb = slot_bytes_of(P.smem_bytes);
-  k_count<<<grid, P.block, (size_t)(kSlots * sb), s>>>(pv, c_begin, c_end, e_begin, e_end, sb,
-                                                      d_out);
-  TC_LAUNCH();
+  return pv;
+}
+
+}  // namespace
+
+int num_sms() {
+  int dev = 0, v = 0;
+  TC_CUDA(cudaGetDevice(&dev));
+  TC_CUDA(cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev));
+  return v;
+}
+
+int max_smem_per_block() { return optin_smem() - static_smem((const void*)k_count); }
+
+int max_chunk_smem(int slots) { return (max_smem_per_block() / slots) & ~15; }
+
+// One chunk of the flat kernel must leave room for 3 CTAs per SM.
+int max_flat_chunk_smem() {
+  int dev = 0, per_sm = 0;
+  TC_CUDA(cudaGetDevice(&dev));
+  TC_CUDA(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+  const int per_cta = per_sm / 3 - 1024 - static_smem((const void*)k_count_flat);  // 1 KB reserved per CTA
+  return std::min(per_cta, optin_smem() - static_smem((const void*)k_count_flat)) & ~15;
+}
+
+int count_occupancy(int block, int64_t smem_bytes, int slots) {
+  ensure_attr();
+  int occ = 0;
+  TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+      &occ, k_count, block, (size_t)(slots * slot_bytes_of(smem_bytes))));
+  return occ;
+}
+
+int flat_occupancy(int64_t smem_bytes) {
+  ensure_attr();
+  int occ = 0;
+  TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_count_flat, kFlatBlock,
+                                                        (size_t)slot_bytes_of(smem_bytes)));
+  return occ;
+}
+
+void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
+                  int64_t e_end, cudaStream_t s, unsigned long long* d_out) {
+  TC_CUDA(cudaMemsetAsync(d_out, 0, sizeof(unsigned long long), s));
+  const Plan& P = g->plan;
+  if (c_end <= c_begin || e_end <= e_begin) return;
+  ensure_attr();
+  const PlanView pv = plan_view(g);
+  // long-class chunks [c_begin, min(c_end, nL)): warp-specialised kernel
+  const int64_t l0 = c_begin, l1 = std::min(c_end, P.n_long_chunks);
+  if (l1 > l0) {
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(l1 - l0, P.grid));
+    const int64_t sb = slot_bytes_of(P.smem_bytes);
+    k_count<<<grid, P.block, (size_t)(P.tune.slots * sb), s>>>(pv, l0, l1, e_begin, e_end, sb,
+                                                              P.tune, d_out);
+    TC_LAUNCH();
+  }
+  // short-class chunks: flat kernel
+  const int64_t s0 = std::max(c_begin, P.n_long_chunks), s1 = c_end;
+  if (s1 > s0) {
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(s1 - s0, P.grid_flat));
+    k_count_flat<<<grid, kFlatBlock, (size_t)slot_bytes_of(P.smem_flat), s>>>(pv, s0, s1, e_begin,
+                                                                             e_end, d_out);
+    TC_LAUNCH();
+  }
 }
 
 }  // namespace tc

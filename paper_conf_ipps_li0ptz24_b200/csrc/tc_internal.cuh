@@ -104,23 +104,38 @@ struct PlanView {
 
 // SMEM a chunk needs (bytes): per segment staging + per group descriptor +
 // hash slots.  Shared by the plan (sizing) and the kernel (layout).
-// Layout of one chunk slot of the count kernel (tc_count.cu slot_view):
-// sB int64[S] | sGB int64[G] | sA int32[S+1] | sC int32[S] | sD int32[S] |
-// sInfo int32[G] | sGP int32[G+1] | pad to 16 B | sHash int32[slots].
-__host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_t slots) {
-  return 20 * S + 16 * G + 8 + 16 + 4 * slots;
+// Layout of one chunk slot of the count kernel (tc_count.cu slot_view), all
+// offsets from a 16-B aligned base: sTile int4[T] (long class: one descriptor
+// per 32-key tile) | sB int64[S] | sGB int64[G] | sInfo int2[G] | sA int32[S+1]
+// | sC int32[S] | sD int32[S] | sGP int32[G+1] | pad to 16 B | sHash int32[slots].
+__host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_t slots,
+                                                    int64_t T) {
+  return 16 * T + 20 * S + 20 * G + 8 + 16 + 4 * slots;
 }
+
+// Count-kernel launch tuning (not part of the C-ABI; TC_SLOTS, TC_GRAB_LONG,
+// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT override the defaults for sweeps).
+struct Tuning {
+  int slots = 3;          // chunk slots in SMEM (2..4)
+  int grab_long = 0;      // tiles per consumer grab, long class (0 = static split)
+  int grab_short = 0;     // keys per consumer grab, short class (0 = static split)
+  int prod_div = 8;       // 1/prod_div of the warps are producers
+  int wait_hint_ns = 0;   // mbarrier try_wait suspend hint (0 = none)
+};
+Tuning tuning_from_env();
 
 struct Plan {
   Options opt;
+  Tuning tune;
   int64_t S = 0, S_long = 0, G = 0, n_chunks = 0, n_long_chunks = 0, keys_total = 0;
   int64_t units_total = 0;
   DevBuf<int64_t> key_prefix, seg_start, ins_prefix, grp_ibase, slot_prefix, chunk_seg;
   DevBuf<int32_t> seg_len, seg_group;
   std::vector<int64_t> h_chunk_seg;
   int64_t chunk_cost_long = 0, chunk_cost_short = 0;  // after SMEM-driven halving
-  int64_t smem_bytes = 0;
-  int grid = 0, block = 0;
+  int64_t smem_bytes = 0;  // per chunk slot, long class (warp-specialised kernel)
+  int64_t smem_flat = 0;   // per chunk, short class (flat kernel)
+  int grid = 0, block = 0, grid_flat = 0;
 };
 
 }  // namespace tc
@@ -145,9 +160,11 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s);
 // tc_count.cu
 void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
                   int64_t e_end, cudaStream_t s, unsigned long long* d_out);
-int count_occupancy(int block, int64_t smem_bytes);  // CTAs per SM (0 = cannot launch)
+int count_occupancy(int block, int64_t smem_bytes, int slots);  // CTAs per SM (0 = cannot launch)
 int max_smem_per_block();
-int max_chunk_smem();  // SMEM one chunk slot may use (the kernel double-buffers)
+int max_chunk_smem(int slots);  // SMEM one of the kernel's chunk slots may use
+int max_flat_chunk_smem();      // SMEM one short-class chunk may use (3 CTAs per SM)
+int flat_occupancy(int64_t smem_bytes);
 int num_sms();
 
 }  // namespace tc
