@@ -90,7 +90,10 @@ typedef struct {
                            class (default 32; 1 = all long, 2^30 = all short)     */
   int32_t probe_mode;   /* 0 = two-choice (cuckoo) tables with linear-probing
                            fallback per chunk, 1 = linear probing only (default 0) */
-  int32_t reserved;
+  int32_t bitmap_factor; /* a head v whose window [min N+(v), max N+(v)] needs at most
+                           bitmap_factor * d+(v) 32-bit words gets a bitmap table
+                           (one probe per key) instead of a hash table (two);
+                           default 3 (same SMEM as the hash), -1 = never        */
 } tc_options;
 
 /*

@@ -56,7 +56,7 @@ class Options(ctypes.Structure):
     _fields_ = [("chunk_cost", ctypes.c_int32), ("seg_cost", ctypes.c_int32),
                 ("huge_degree", ctypes.c_int32), ("block_threads", ctypes.c_int32),
                 ("table_factor", ctypes.c_int32), ("long_min", ctypes.c_int32),
-                ("probe_mode", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("probe_mode", ctypes.c_int32), ("bitmap_factor", ctypes.c_int32)]
 
 
 class GraphInfo(ctypes.Structure):

@@ -100,6 +100,7 @@ Options resolve_options(const tc_options* o) {
   if (o->table_factor) r.table_factor = o->table_factor;
   if (o->long_min) r.long_min = o->long_min;
   if (o->probe_mode) r.probe_mode = o->probe_mode;
+  if (o->bitmap_factor) r.bitmap_factor = o->bitmap_factor;
   require(r.chunk_cost >= 64, "chunk_cost must be >= 64");
   require(r.seg_cost >= 1, "seg_cost must be >= 1");
   require(r.huge_degree >= 1, "huge_degree must be >= 1");
@@ -122,7 +123,7 @@ void rebind(tc_graph* g, cudaStream_t s) {
   tc::Plan& P = g->plan;
   P.key_prefix.s = P.seg_start.s = P.ins_prefix.s = P.grp_ibase.s = P.slot_prefix.s =
       P.chunk_seg.s = s;
-  P.seg_len.s = P.seg_group.s = s;
+  P.seg_len.s = P.seg_group.s = P.grp_code.s = s;
 }
 
 tc_status build_impl(const int32_t* src, const int32_t* dst, int64_t num_edges,

@@ -290,8 +290,9 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const int64_t* __re
                            const int32_t* __restrict__ gincl, int64_t S, int64_t S_long,
                            int bits, const int64_t* __restrict__ row_ptr,
                            const int64_t* __restrict__ e_lo, const int32_t* __restrict__ e_len,
-                           int huge_degree, int table_factor, int64_t max_table_slots,
-                           int64_t* __restrict__ seg_start,
+                           int huge_degree, int table_factor, int bitmap_factor,
+                           int64_t max_table_slots, const int32_t* __restrict__ col,
+                           int32_t* __restrict__ grp_code, int64_t* __restrict__ seg_start,
                            int32_t* __restrict__ seg_len, int32_t* __restrict__ seg_group,
                            int64_t* __restrict__ units, int64_t* __restrict__ grp_row,
                            int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots) {
@@ -310,16 +311,30 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const int64_t* __re
       const int64_t rs = row_ptr[v], d = row_ptr[v + 1] - rs;
       grp_row[g] = rs;
       grp_d[g] = d;
-      // table_factor * d slots (load <= 1/table_factor, > d so a linear probe
-      // always meets an empty slot), a multiple of 4 for 16-B initialisation;
-      // 0 = huge table (probed in global memory)
+      // Table of N+(v), in 32-bit words (0 = huge: probed in global memory):
+      //  bitmap: one bit per rank of the window [min N+(v), max N+(v)] at word
+      //    granularity, when that is at most bitmap_factor * d words (one
+      //    probe per key); code = -(first word);
+      //  hash: table_factor * d slots (load <= 1/table_factor, > d so a
+      //    linear probe always meets an empty slot); code = slots.
+      // Sizes are multiples of 4 for 16-B initialisation.
       int64_t slots = 0;
+      int32_t code = 0;
       if (d <= huge_degree) {
-        int64_t want = d * table_factor;
-        if (want < d + 1) want = d + 1;
-        slots = (want + 3) & ~int64_t(3);
+        const int64_t w0 = col[rs] >> 5, w1 = col[rs + d - 1] >> 5;
+        // (the first word must fit the count kernel's 26-bit tile code)
+        if (bitmap_factor > 0 && w0 < (1 << 25) && w1 - w0 + 1 <= (int64_t)bitmap_factor * d) {
+          slots = (w1 - w0 + 1 + 3) & ~int64_t(3);
+          code = -(int32_t)w0;
+        } else {
+          int64_t want = d * table_factor;
+          if (want < d + 1) want = d + 1;
+          slots = (want + 3) & ~int64_t(3);
+          code = (int32_t)slots;
+        }
         if (slots > max_table_slots) slots = 0;
       }
+      grp_code[g] = code;
       grp_slots[g] = slots;
     }
   }
@@ -699,10 +714,11 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P.seg_len = DevBuf<int32_t>(S, s);
   P.seg_group = DevBuf<int32_t>(S, s);
   DevBuf<int64_t> units(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
+  P.grp_code = DevBuf<int32_t>(G, s);
   k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted.get(), p_sorted.get(), gincl.get(), S, S_long,
                                          g->bits, row_ptr, e_lo.get(), e_len.get(),
-                                         opt.huge_degree, opt.table_factor, max_table_slots,
-                                         P.seg_start.get(),
+                                         opt.huge_degree, opt.table_factor, opt.bitmap_factor,
+                                         max_table_slots, col, P.grp_code.get(), P.seg_start.get(),
                                          P.seg_len.get(), P.seg_group.get(), units.get(),
                                          grp_row.get(), grp_d.get(), grp_slots.get());
   TC_LAUNCH();

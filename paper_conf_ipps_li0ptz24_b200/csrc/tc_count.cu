@@ -138,9 +138,10 @@ template <bool kLinear>
 __device__ __forceinline__ unsigned table_probe(const int* __restrict__ T, uint32_t n, int32_t key) {
   if (!kLinear) {
     // two-choice table: a key lives at hash1 or hash2; both reads are issued
+    // unconditionally (a read of hash2 that waits on hash1 measured slower)
     const int x1 = T[hash1(key, n)];
     const int x2 = T[hash2(key, n)];
-    return (x1 == key) | (x2 == key);
+    return (unsigned)(x1 == key) | (unsigned)(x2 == key);
   }
   uint32_t h = hash1(key, n);
   for (;;) {
@@ -149,6 +150,23 @@ __device__ __forceinline__ unsigned table_probe(const int* __restrict__ T, uint3
     if (x < 0) return 0u;
     h = (h + 1 == n) ? 0 : h + 1;
   }
+}
+
+// Membership in a table of either kind: T = its first word, code = n >= 2
+// (hash, n slots) or -(first rank word) <= 0 (bitmap of the rank window,
+// bits inverted so that an initialised word is all ones).  Padding lanes
+// (key < 0) never match and read only inside the table.
+template <bool kLinear>
+__device__ __forceinline__ unsigned any_probe(const int* __restrict__ T, int code, int32_t key) {
+  if (code <= 0) {
+    const int w = max((key >> 5) + code, 0);
+    return (((~(unsigned)T[w]) >> (key & 31)) & 1u) & (unsigned)(key >= 0);
+  }
+  return table_probe<kLinear>(T, (uint32_t)code, key);
+}
+
+__device__ __forceinline__ void bitmap_insert(int* __restrict__ T, int code, int32_t key) {
+  atomicAnd(&T[(key >> 5) + code], ~(1 << (key & 31)));
 }
 
 __device__ __forceinline__ unsigned huge_probe(const PlanView& pv, int64_t g, int32_t key) {
@@ -165,10 +183,10 @@ struct SlotHdr {
 };
 
 struct ChunkSmem {
-  int4* sTile;   // [T] long class: {key pointer lo, hi, table offset (or -1-g), n << 6 | lanes}
+  int4* sTile;   // [T] long class: {key pointer lo, hi, table offset (or -1-g), code << 6 | lanes}
   int64_t* sB;   // long: key start in col; short: start - (chunk-relative first key)
   int64_t* sGB;  // group: row start of N+(v) - sGP (so col[sGB[g] + k] is insert k)
-  int2* sInfo;   // [G] table {slot offset, slots}; offset -1 = huge
+  int2* sInfo;   // [G] table {word offset, code}; offset -1 = huge
   int* sA;       // [S+1] long: tile prefix; short: key prefix (chunk-relative)
   int* sC;       // suffix length
   int* sD;       // group index (chunk-local)
@@ -253,27 +271,23 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   const int lane = threadIdx.x & 31;
   for (int t = t0; t < t1; t += kUnrollLong) {
     int32_t key[kUnrollLong];
-    int toff[kUnrollLong], tn[kUnrollLong];
+    int toff[kUnrollLong], code[kUnrollLong];
 #pragma unroll
     for (int u = 0; u < kUnrollLong; ++u) {
-      key[u] = -2;
-      toff[u] = 0;
-      tn[u] = 1;
-      if (t + u < t1) {
-        const int4 d = c.sTile[t + u];
-        const int64_t p = (int64_t)(((uint64_t)(uint32_t)d.y << 32) | (uint32_t)d.x);
-        toff[u] = d.z;
-        tn[u] = d.w >> 6;
-        if (lane < (d.w & 63)) key[u] = __ldg(pv.col + p + lane);
-      }
+      // tiles past t1 reuse the last tile's (real) table with no lanes
+      const int4 d = c.sTile[min(t + u, t1 - 1)];
+      const int lanes = (t + u < t1) ? (d.w & 63) : 0;
+      const int64_t p = (int64_t)(((uint64_t)(uint32_t)d.y << 32) | (uint32_t)d.x);
+      toff[u] = d.z;
+      code[u] = d.w >> 6;
+      key[u] = lane < lanes ? __ldg(pv.col + p + lane) : -2;
     }
 #pragma unroll
     for (int u = 0; u < kUnrollLong; ++u) {
       if (kHuge && toff[u] < 0) {
         if (key[u] >= 0) cnt += huge_probe(pv, ga + (-1 - toff[u]), key[u]);
-      } else if (!kLinear || key[u] >= 0) {  // a linear probe of a padding tile's
-        // dummy 1-slot table might never meet an empty slot: skip sentinels
-        cnt += table_probe<kLinear>(c.sHash + toff[u], (uint32_t)tn[u], key[u]);
+      } else {
+        cnt += any_probe<kLinear>(c.sHash + toff[u], code[u], key[u]);
       }
     }
   }
@@ -320,7 +334,7 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
       if (k0 + 32 * u + lane >= k1w) continue;
       const int2 d = c.sInfo[gl[u]];
       if (kHuge && d.x < 0) cnt += huge_probe(pv, ga + gl[u], key[u]);
-      else cnt += table_probe<kLinear>(c.sHash + d.x, (uint32_t)d.y, key[u]);
+      else cnt += any_probe<kLinear>(c.sHash + d.x, d.y, key[u]);
     }
   }
   return cnt;
@@ -398,15 +412,18 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   int huge = 0;
   for (int base = pt; base <= G; base += PT * kB) {
     int64_t ip[kB], sp[kB], sp1[kB], ib[kB];
+    int cd[kB];
 #pragma unroll
     for (int r = 0; r < kB; ++r) {
       const int i = base + r * PT;
       ip[r] = sp[r] = sp1[r] = ib[r] = 0;
+      cd[r] = 0;
       if (i <= G) ip[r] = __ldg(pv.ins_prefix + (ga + i));
       if (i < G) {
         sp[r] = __ldg(pv.slot_prefix + (ga + i));
         sp1[r] = __ldg(pv.slot_prefix + (ga + i + 1));
         ib[r] = __ldg(pv.grp_ibase + (ga + i));
+        cd[r] = __ldg(pv.grp_code + (ga + i));
       }
     }
 #pragma unroll
@@ -415,7 +432,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       if (i <= G) c.sGP[i] = (int)(ip[r] - ip0);
       if (i < G) {
         const int ns = (int)(sp1[r] - sp[r]);
-        c.sInfo[i] = ns > 0 ? make_int2((int)(sp[r] - slot0), ns) : make_int2(-1, 0);
+        c.sInfo[i] = ns > 0 ? make_int2((int)(sp[r] - slot0), cd[r]) : make_int2(-1, 0);
         huge |= ns == 0;
         c.sGB[i] = ib[r] + ip0;  // row start - chunk-relative insert prefix
       }
@@ -438,7 +455,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       for (int t = ts; t < te; ++t) {
         const int64_t p = st + ((int64_t)(t - ts) << 5);
         const int lanes = min(32, len - ((t - ts) << 5));
-        c.sTile[t] = make_int4((int)(uint32_t)p, (int)(p >> 32), toff, (d.y << 6) | lanes);
+        c.sTile[t] = make_int4((int)(uint32_t)p, (int)(p >> 32), toff, (int)((unsigned)d.y << 6) | lanes);
       }
     }
   }
@@ -451,25 +468,27 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   const int i0 = (int)((int64_t)NI * pw / npw), i1 = (int)((int64_t)NI * (pw + 1) / npw);
   auto load_row = [&](int g, int k) { return __ldg(pv.col + c.sGB[g] + k); };
   bool linear = pv.probe_mode == 1;
+  auto insert_linear = [&](int g, int32_t key) {
+    const int2 d = c.sInfo[g];
+    if (d.x < 0) return;
+    if (d.y <= 0) bitmap_insert(c.sHash + d.x, d.y, key);
+    else linear_insert(c.sHash + d.x, (uint32_t)d.y, key);
+  };
   if (linear) {
-    warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
-      const int2 d = c.sInfo[g];
-      if (d.x >= 0) linear_insert(c.sHash + d.x, (uint32_t)d.y, key);
-    });
+    warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, insert_linear);
   } else {
     bool ok = true;
     warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
       const int2 d = c.sInfo[g];
-      if (d.x >= 0 && !cuckoo_insert(c.sHash + d.x, (uint32_t)d.y, key)) ok = false;
+      if (d.x < 0) return;
+      if (d.y <= 0) bitmap_insert(c.sHash + d.x, d.y, key);
+      else if (!cuckoo_insert(c.sHash + d.x, (uint32_t)d.y, key)) ok = false;
     });
     if (named_sync_or(1, PT, !ok)) {  // uniform over producers: rebuild with linear probing
       linear = true;
       for (int i = pt; i < nslots; i += PT) c.sHash[i] = -1;
       named_sync(1, PT);
-      warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
-        const int2 d = c.sInfo[g];
-        if (d.x >= 0) linear_insert(c.sHash + d.x, (uint32_t)d.y, key);
-      });
+      warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, insert_linear);
     }
   }
   if (pt == 0) {
@@ -646,6 +665,7 @@ PlanView plan_view(const tc_graph* g) {
   pv.ins_prefix = P.ins_prefix.get();
   pv.grp_ibase = P.grp_ibase.get();
   pv.slot_prefix = P.slot_prefix.get();
+  pv.grp_code = P.grp_code.get();
   pv.chunk_seg = P.chunk_seg.get();
   pv.n_long_chunks = P.n_long_chunks;
   pv.probe_mode = P.opt.probe_mode;

@@ -69,6 +69,7 @@ struct Options {
   int table_factor = 3;
   int long_min = 32;
   int probe_mode = 0;
+  int bitmap_factor = 3;  // <= 0: never
 };
 Options resolve_options(const tc_options* o);
 
@@ -96,7 +97,8 @@ struct PlanView {
   const int32_t* seg_group;    // [S]
   const int64_t* ins_prefix;   // [G+1] prefix of d+(v)
   const int64_t* grp_ibase;    // [G]  = row_ptr[v] - ins_prefix[g]
-  const int64_t* slot_prefix;  // [G+1] prefix of hash slots (0 for huge groups)
+  const int64_t* slot_prefix;  // [G+1] prefix of table words (0 for huge groups)
+  const int32_t* grp_code;     // [G] table kind: n >= 2 hash slots, <= 0 bitmap (-base word)
   const int64_t* chunk_seg;    // [C+1]
   int64_t n_long_chunks;
   int probe_mode;
@@ -130,7 +132,7 @@ struct Plan {
   int64_t S = 0, S_long = 0, G = 0, n_chunks = 0, n_long_chunks = 0, keys_total = 0;
   int64_t units_total = 0;
   DevBuf<int64_t> key_prefix, seg_start, ins_prefix, grp_ibase, slot_prefix, chunk_seg;
-  DevBuf<int32_t> seg_len, seg_group;
+  DevBuf<int32_t> seg_len, seg_group, grp_code;
   std::vector<int64_t> h_chunk_seg;
   int64_t chunk_cost_long = 0, chunk_cost_short = 0;  // after SMEM-driven halving
   int64_t smem_bytes = 0;  // per chunk slot, long class (warp-specialised kernel)

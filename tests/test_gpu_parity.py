@@ -112,6 +112,9 @@ def test_chung_lu_small(tc):
     dict(long_min=1), dict(long_min=8), dict(long_min=1 << 30), dict(long_min=1 << 30, chunk_cost=64),
     dict(probe_mode=1), dict(probe_mode=1, long_min=1), dict(probe_mode=1, long_min=1 << 30),
     dict(table_factor=2, chunk_cost=1 << 20),
+    dict(bitmap_factor=-1), dict(bitmap_factor=1), dict(bitmap_factor=64),
+    dict(bitmap_factor=64, probe_mode=1), dict(bitmap_factor=64, long_min=1 << 30),
+    dict(bitmap_factor=-1, long_min=1),
 ])
 def test_plan_options_never_change_count(tc, opts):
     src, dst, n = tcgen.rmat(13, 16, 11)
