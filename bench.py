@@ -57,6 +57,8 @@ def parse():
                     help="target oracle counting time of the cpu_baseline sample")
     ap.add_argument("--chunk-cost", type=int, default=0)
     ap.add_argument("--block", type=int, default=0)
+    ap.add_argument("--opt", action="append", default=[],
+                    help="plan option key=value (tc_options field), repeatable")
     ap.add_argument("--out", default=None, help="also write the JSON line here")
     return ap.parse_args()
 
@@ -243,6 +245,9 @@ def main():
         opts["chunk_cost"] = a.chunk_cost
     if a.block:
         opts["block_threads"] = a.block
+    for kv in a.opt:
+        k, v = kv.split("=")
+        opts[k] = int(v)
 
     # ---------------------------------------------------------------- build (a1..a6)
     dsrc = torch.from_numpy(src).to(dev)

@@ -223,12 +223,14 @@ __device__ __forceinline__ int64_t upper_bound_i32(const int32_t* __restrict__ a
 // Per oriented edge p = (u, v): the keys are the suffix of N+(u) after v,
 // col[p+1, row_end(u)), trimmed to [min N+(v), max N+(v)] because a
 // key outside that range cannot be in N+(v) (both lists sorted; exact, C-12).
-// Live iff the trimmed suffix is non-empty.  stats: [0] B_ITC edge part
+// Live iff the trimmed suffix is non-empty.  Emits the plan's sort key
+// (class above head v; dead edges get `dead`, which sorts last) and the
+// packed value (trimmed start << 24 | length).  stats: [0] B_ITC edge part
 // (untrimmed), [1] trimmed keys, [2] live, [3] live long.
 __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                            const int32_t* __restrict__ rowid, int64_t m, int long_min,
-                            int64_t* __restrict__ e_lo, int32_t* __restrict__ e_len,
-                            uint8_t* __restrict__ live, unsigned long long* stats) {
+                            const int32_t* __restrict__ rowid, int64_t m, int long_min, int bits,
+                            uint32_t dead, uint32_t* __restrict__ skey, uint64_t* __restrict__ sval,
+                            unsigned long long* stats) {
   typedef cub::BlockReduce<unsigned long long, TPB> BR;
   __shared__ typename BR::TempStorage tmp;
   unsigned long long b = 0, keys = 0, nl = 0, nlong = 0;
@@ -243,9 +245,9 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
       lo = lower_bound_i32(col, p + 1, rend, col[rv]);
       len = upper_bound_i32(col, lo, rend, col[rv + dv - 1]) - lo;
     }
-    e_lo[p] = lo;
-    e_len[p] = (int32_t)len;
-    live[p] = len > 0;
+    const uint32_t cls = len < long_min ? 1u : 0u;
+    skey[p] = len > 0 ? ((cls << bits) | (uint32_t)v) : dead;
+    sval[p] = ((uint64_t)lo << 24) | (uint64_t)len;  // len <= d+(u) < 2^24
     keys += (unsigned long long)len;
     nl += len > 0;
     nlong += len >= long_min;
@@ -265,18 +267,6 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
   }
 }
 
-// sort key of a live edge: class (0 = long, 1 = short) above the head v.
-__global__ void k_class_key(const int64_t* __restrict__ p_live, int64_t S,
-                            const int32_t* __restrict__ col, const int32_t* __restrict__ e_len,
-                            int long_min, int bits, uint32_t* __restrict__ key) {
-  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
-       s += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t p = p_live[s];
-    const uint32_t cls = e_len[p] < long_min ? 1u : 0u;
-    key[s] = (cls << bits) | (uint32_t)col[p];
-  }
-}
-
 __global__ void k_group_mark(const uint32_t* __restrict__ key, int64_t S,
                              int32_t* __restrict__ mark) {
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
@@ -284,26 +274,25 @@ __global__ void k_group_mark(const uint32_t* __restrict__ key, int64_t S,
     mark[s] = (s == 0 || key[s] != key[s - 1]) ? 1 : 0;
 }
 
-// Per segment: start, length, group, work units; per group (at its first
-// segment): row start, d+(v) and hash slots (> d+(v), or 0 for huge tables).
-__global__ void k_seg_fill(const uint32_t* __restrict__ key, const int64_t* __restrict__ p_s,
+// Per segment (sorted live edge): start, length, group, work units; per
+// group (at its first segment): row start, d+(v) and its table.
+__global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val,
                            const int32_t* __restrict__ gincl, int64_t S, int64_t S_long,
                            int bits, const int64_t* __restrict__ row_ptr,
-                           const int64_t* __restrict__ e_lo, const int32_t* __restrict__ e_len,
                            int huge_degree, int table_factor, int bitmap_factor,
                            int64_t max_table_slots, const int32_t* __restrict__ col,
                            int32_t* __restrict__ grp_code, int64_t* __restrict__ seg_start,
                            int32_t* __restrict__ seg_len, int32_t* __restrict__ seg_group,
                            int64_t* __restrict__ units, int64_t* __restrict__ grp_row,
                            int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots) {
-  const uint32_t mask = (1u << bits) - 1u;
+  const uint32_t mask = (uint32_t)((1ull << bits) - 1);
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
        s += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t p = p_s[s];
+    const uint64_t x = val[s];
     const int32_t g = gincl[s] - 1;
-    const int32_t len = e_len[p];
+    const int32_t len = (int32_t)(x & 0xFFFFFFu);
     seg_group[s] = g;
-    seg_start[s] = e_lo[p];
+    seg_start[s] = (int64_t)(x >> 24);
     seg_len[s] = len;
     units[s] = s < S_long ? (int64_t)((len + 31) & ~31) : (int64_t)len;
     if (s == 0 || key[s] != key[s - 1]) {
@@ -641,14 +630,18 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   Trace tr(s);
   DevBuf<unsigned long long> stats(4, s);
   TC_CUDA(cudaMemsetAsync(stats.get(), 0, 4 * sizeof(unsigned long long), s));
-  DevBuf<int32_t> rowid(std::max<int64_t>(m, 1), s), e_len(std::max<int64_t>(m, 1), s);
-  DevBuf<int64_t> e_lo(std::max<int64_t>(m, 1), s);
-  DevBuf<uint8_t> live(std::max<int64_t>(m, 1), s);
+  // sort keys: class bit above the head v; dead edges sort last
+  const int kbits = g->bits + 1;
+  const uint32_t dead = kbits < 32 ? (1u << kbits) : 0xFFFFFFFFu;
+  const int end_bit = kbits < 32 ? kbits + 1 : 32;
+  DevBuf<int32_t> rowid(std::max<int64_t>(m, 1), s);
+  DevBuf<uint32_t> skey(std::max<int64_t>(m, 1), s), skey2(std::max<int64_t>(m, 1), s);
+  DevBuf<uint64_t> sval(std::max<int64_t>(m, 1), s), sval2(std::max<int64_t>(m, 1), s);
   if (m > 0) {
     k_rowid<<<grid_for(n), TPB, 0, s>>>(row_ptr, n, rowid.get());
     TC_LAUNCH();
-    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m, opt.long_min, e_lo.get(),
-                                            e_len.get(), live.get(), stats.get());
+    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m, opt.long_min, g->bits,
+                                            dead, skey.get(), sval.get(), stats.get());
     TC_LAUNCH();
   }
   rowid.reset();
@@ -671,32 +664,21 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     return;
   }
 
-  // live edges ordered by (class, head v, position): radix sort is stable
-  DevBuf<int64_t> p_live(S, s), p_sorted(S, s);
-  DevBuf<uint32_t> key(S, s), key_sorted(S, s);
-  {
-    DevBuf<int64_t> nsel(1, s);
-    cub::CountingInputIterator<int64_t> it(0);
-    cub_run(s, [&](void* t, size_t& b) {
-      return cub::DeviceSelect::Flagged(t, b, it, live.get(), p_live.get(), nsel.get(), m, s);
-    });
-  }
-  live.reset();
-  k_class_key<<<grid_for(S), TPB, 0, s>>>(p_live.get(), S, col, e_len.get(), opt.long_min, g->bits,
-                                          key.get());
-  TC_LAUNCH();
+  // live edges ordered by (class, head v, position): the radix sort is stable
+  // and the edges arrive in position order; dead edges sort past S
+  cub::DoubleBuffer<uint32_t> dk(skey.get(), skey2.get());
+  cub::DoubleBuffer<uint64_t> dv(sval.get(), sval2.get());
   cub_run(s, [&](void* t, size_t& b) {
-    return cub::DeviceRadixSort::SortPairs(t, b, key.get(), key_sorted.get(), p_live.get(),
-                                           p_sorted.get(), S, 0, g->bits + 1, s);
+    return cub::DeviceRadixSort::SortPairs(t, b, dk, dv, m, 0, end_bit, s);
   });
-  key.reset();
-  p_live.reset();
+  const uint32_t* key_sorted = dk.Current();
+  const uint64_t* val_sorted = dv.Current();
   tr("select + class sort");
 
   DevBuf<int32_t> gincl(S, s);
   {
     DevBuf<int32_t> mark(S, s);
-    k_group_mark<<<grid_for(S), TPB, 0, s>>>(key_sorted.get(), S, mark.get());
+    k_group_mark<<<grid_for(S), TPB, 0, s>>>(key_sorted, S, mark.get());
     TC_LAUNCH();
     cub_run(s, [&](void* t, size_t& b) {
       return cub::DeviceScan::InclusiveSum(t, b, mark.get(), gincl.get(), S, s);
@@ -715,18 +697,18 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P.seg_group = DevBuf<int32_t>(S, s);
   DevBuf<int64_t> units(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
   P.grp_code = DevBuf<int32_t>(G, s);
-  k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted.get(), p_sorted.get(), gincl.get(), S, S_long,
-                                         g->bits, row_ptr, e_lo.get(), e_len.get(),
+  k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted, val_sorted, gincl.get(), S, S_long,
+                                         g->bits, row_ptr,
                                          opt.huge_degree, opt.table_factor, opt.bitmap_factor,
                                          max_table_slots, col, P.grp_code.get(), P.seg_start.get(),
                                          P.seg_len.get(), P.seg_group.get(), units.get(),
                                          grp_row.get(), grp_d.get(), grp_slots.get());
   TC_LAUNCH();
   gincl.reset();
-  key_sorted.reset();
-  p_sorted.reset();
-  e_lo.reset();
-  e_len.reset();
+  skey.reset();
+  skey2.reset();
+  sval.reset();
+  sval2.reset();
   exclusive_prefix(units.get(), S, P.key_prefix.get(), s);
   P.ins_prefix = DevBuf<int64_t>(G + 1, s);
   P.slot_prefix = DevBuf<int64_t>(G + 1, s);
