@@ -51,7 +51,22 @@ def main():
     m = raw_metrics(rep)
     dram = to_bytes(*m["dram__bytes_read.sum"]) + to_bytes(*m["dram__bytes_write.sum"])
     ms = to_ms(*m["gpu__time_duration.sum"])
-    entry = {"round_tag": tag, "dram_bytes_per_launch": dram, "kernel_ms_under_ncu": ms,
+    # the short-class kernel of the same count step, if captured
+    rep_flat = os.path.join(ROOT, "gpurun_out", f"{tag}_prof_{low}_flat.ncu-rep")
+    flat = None
+    if os.path.exists(rep_flat):
+        mf = raw_metrics(rep_flat)
+        flat = {"dram_bytes": to_bytes(*mf["dram__bytes_read.sum"]) + to_bytes(*mf["dram__bytes_write.sum"]),
+                "ms": to_ms(*mf["gpu__time_duration.sum"])}
+        summary_flat = subprocess.run([sys.executable, os.path.join(ROOT, "scripts", "ncu_summary.py"),
+                                       rep_flat], capture_output=True, text=True, check=True).stdout
+        with open(os.path.join(OUT, f"{tag}_{low}_count_flat_ncu.txt"), "w") as f:
+            f.write(f"# ncu --set full --clock-control none, one k_count_flat launch, config {cfg} ({tag})\n")
+            f.write(summary_flat)
+    entry = {"round_tag": tag,
+             "dram_bytes_per_launch": dram + (flat["dram_bytes"] if flat else 0.0),
+             "what": "k_count (long class) + k_count_flat (short class) of one count step",
+             "k_count_dram_bytes": dram, "k_count_flat": flat, "kernel_ms_under_ncu": ms,
              "dram_gbs": dram / ms / 1e6, "lts_bytes": to_bytes(*m["lts__t_bytes.sum"]) if "lts__t_bytes.sum" in m else None,
              "issue_active_pct": float(m["smsp__issue_active.avg.pct_of_peak_sustained_active"][0]),
              "warps_active_pct": float(m["sm__warps_active.avg.pct_of_peak_sustained_active"][0]),
