@@ -81,6 +81,32 @@ void* dev_alloc(size_t bytes, cudaStream_t s) {
   return p;
 }
 
+// Grow the default memory pool in one step so that a build's allocations
+// reuse already-mapped memory: mapping physical memory inside the build
+// (pool growth on demand) made identical builds vary by 3-10x in time.
+void reserve_pool(size_t bytes, cudaStream_t s) {
+  if (g_alloc || bytes == 0) return;
+  int dev = 0;
+  cudaMemPool_t pool;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetDefaultMemPool(&pool, dev) != cudaSuccess) {
+    cudaGetLastError();
+    return;
+  }
+  uint64_t reserved = 0, used = 0;
+  cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved);
+  cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used);
+  if (reserved - used >= bytes) return;
+  size_t free_b = 0, total_b = 0;
+  cudaMemGetInfo(&free_b, &total_b);
+  const size_t want = bytes - (size_t)(reserved - used);
+  const size_t cap = free_b > (size_t(4) << 30) ? free_b - (size_t(4) << 30) : 0;
+  const size_t grow = want < cap ? want : cap;
+  if (grow == 0) return;
+  void* p = nullptr;
+  if (cudaMallocAsync(&p, grow, s) == cudaSuccess && p) cudaFreeAsync(p, s);
+  cudaGetLastError();
+}
+
 void dev_free(void* p, size_t bytes, cudaStream_t s) {
   if (!p) return;
   if (g_free) {
@@ -140,6 +166,10 @@ tc_status build_impl(const int32_t* src, const int32_t* dst, int64_t num_edges,
     require((flags & ~TC_KEEP_ISOLATED) == 0, "unknown flag bits");
     const tc::Options opt = tc::resolve_options(opts);
     cudaStream_t s = (cudaStream_t)stream;
+    // peak scratch of a1..a6 is ~72 B per input pair (sort double buffers,
+    // plan arrays) + ~48 B per vertex; the host entry adds the 8-B pair copy
+    const int64_t nv = num_vertices > 0 ? num_vertices : 0;
+    tc::reserve_pool((size_t)num_edges * (host ? 80 : 72) + (size_t)nv * 48, s);
     g = new tc_graph();
     if (host) {
       tc::DevBuf<int32_t> ds(std::max<int64_t>(num_edges, 1), s), dd(std::max<int64_t>(num_edges, 1), s);
