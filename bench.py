@@ -382,7 +382,7 @@ def main():
                                   "(SURVEY.md §8(d)); x this rank's share for N>1",
                      "peak_source": peak_src},
         "e2e": e2e,
-        "gpu_launches": a.steps,
+        "gpu_launches": a.steps * g.launches_per_count,
         "build_ms": {"canon": info.ms_canon, "sort_unique": info.ms_sort_unique,
                      "degree_rank": info.ms_degree_rank, "orient_csr": info.ms_orient_csr,
                      "plan": info.ms_plan, "total_events": info.ms_total,

@@ -143,6 +143,9 @@ typedef struct {
   const int32_t* perm;      /* int32[n], new id -> original id                   */
   /* Build phase times (ms, CUDA events on the build stream): */
   float ms_canon, ms_sort_unique, ms_degree_rank, ms_orient_csr, ms_plan, ms_total;
+  int64_t n_long_chunks;    /* chunks [0, n_long_chunks) are long class (k_count),
+                               the rest short class (k_count_flat): a count launches
+                               one kernel per non-empty class                       */
 } tc_graph_info_t;
 
 TC_API tc_status tc_graph_info(const tc_graph* g, tc_graph_info_t* out);

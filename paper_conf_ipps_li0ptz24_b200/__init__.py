@@ -69,7 +69,8 @@ class GraphInfo(ctypes.Structure):
                 ("col", ctypes.c_void_p), ("perm", ctypes.c_void_p),
                 ("ms_canon", ctypes.c_float), ("ms_sort_unique", ctypes.c_float),
                 ("ms_degree_rank", ctypes.c_float), ("ms_orient_csr", ctypes.c_float),
-                ("ms_plan", ctypes.c_float), ("ms_total", ctypes.c_float)]
+                ("ms_plan", ctypes.c_float), ("ms_total", ctypes.c_float),
+                ("n_long_chunks", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_
@@ -183,6 +184,12 @@ class Graph:
     @property
     def m_live(self) -> int:
         return int(self.info.m_live)
+
+    @property
+    def launches_per_count(self) -> int:
+        """Kernels one count launches: one per non-empty work class."""
+        gi = self.info
+        return int(gi.n_long_chunks > 0) + int(gi.n_chunks - gi.n_long_chunks > 0)
 
     def csr(self):
         """(row_ptr int64[n+1], col int32[m], perm int32[n]) as borrowed CUDA tensors."""

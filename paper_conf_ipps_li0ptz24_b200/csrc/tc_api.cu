@@ -260,6 +260,7 @@ tc_status tc_graph_info(const tc_graph* g, tc_graph_info_t* o) {
     o->ms_orient_csr = g->ms[3];
     o->ms_plan = g->ms[4];
     o->ms_total = g->ms[5];
+    o->n_long_chunks = P.n_long_chunks;
   });
 }
 

@@ -105,3 +105,19 @@ def test_partition_prefix_degenerate(tc):
     assert tc.partition_prefix([0, 10], 3) == [0, 1, 1, 1] or tc.partition_prefix([0, 10], 3)[-1] == 1
     with pytest.raises(tc.InvalidArgument):
         tc.partition_prefix([0, 1], 0)
+
+
+def test_struct_layouts_match_header(tc, tmp_path):
+    """The ctypes mirrors of tc_options / tc_graph_info_t match the C header."""
+    src = tmp_path / "sz.c"
+    src.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "tc.h"\n'
+                   'int main(void){printf("%zu %zu %zu %zu\\n", sizeof(tc_options), '
+                   'sizeof(tc_graph_info_t), offsetof(tc_graph_info_t, row_ptr), '
+                   'offsetof(tc_graph_info_t, n_long_chunks));return 0;}\n')
+    exe = tmp_path / "sz"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    got = [int(x) for x in subprocess.run([str(exe)], capture_output=True, text=True,
+                                          check=True).stdout.split()]
+    want = [ctypes.sizeof(tc.Options), ctypes.sizeof(tc.GraphInfo), tc.GraphInfo.row_ptr.offset,
+            tc.GraphInfo.n_long_chunks.offset]
+    assert got == want
