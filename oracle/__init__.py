@@ -141,3 +141,79 @@ def count(src, dst, n: int = -1, order: int = ORDER_DEGREE, threads: int = 0,
 
 def triangles(src, dst, n: int = -1, **kw) -> int:
     return count(src, dst, n, **kw).triangles
+
+
+# ---------------------------------------------------------------- per-edge support (f1)
+
+def _support_lib():
+    L = lib()
+    if not hasattr(L, "_support_ready"):
+        vp, i64 = ctypes.c_void_p, ctypes.c_int64
+        L.tco_support_build.argtypes = [vp, vp, i64, i64]
+        L.tco_support_build.restype = vp
+        L.tco_support_m.argtypes = [vp]
+        L.tco_support_m.restype = i64
+        L.tco_support_free.argtypes = [vp]
+        L.tco_support_free.restype = None
+        L.tco_support_all.argtypes = [vp, ctypes.c_int, vp, vp, vp]
+        L.tco_support_all.restype = ctypes.c_int
+        L.tco_support_pairs.argtypes = [vp, vp, vp, i64, vp]
+        L.tco_support_pairs.restype = ctypes.c_int
+        L._support_ready = True
+    return L
+
+
+class SupportGraph:
+    """sup(a,b) = |N(a) ∩ N(b)| for the edges {a,b} of the cleaned simple graph
+    (tco_support_* in tc_oracle.cpp)."""
+
+    def __init__(self, src, dst, n: int = -1):
+        src = np.ascontiguousarray(src, dtype=np.int32)
+        dst = np.ascontiguousarray(dst, dtype=np.int32)
+        if src.shape != dst.shape:
+            raise ValueError("src and dst differ in length")
+        self._h = _support_lib().tco_support_build(src.ctypes.data_as(ctypes.c_void_p),
+                                                   dst.ctypes.data_as(ctypes.c_void_p),
+                                                   len(src), int(n))
+        if not self._h:
+            raise ValueError("oracle: invalid input (vertex id out of range)")
+        self.m = int(_support_lib().tco_support_m(self._h))
+
+    def all(self, threads: int = 0):
+        """(a, b, sup): int32, int32, uint32 arrays of length m, ascending (a, b), a < b."""
+        a = np.empty(self.m, np.int32)
+        b = np.empty(self.m, np.int32)
+        s = np.empty(self.m, np.uint32)
+        vp = ctypes.c_void_p
+        if _support_lib().tco_support_all(self._h, int(threads), a.ctypes.data_as(vp),
+                                          b.ctypes.data_as(vp), s.ctypes.data_as(vp)) != 0:
+            raise ValueError("oracle: bad arguments")
+        return a, b, s
+
+    def pairs(self, a, b):
+        """int64 per pair: its support if {a_i, b_i} is an edge, else -1."""
+        a = np.ascontiguousarray(a, dtype=np.int32)
+        b = np.ascontiguousarray(b, dtype=np.int32)
+        out = np.empty(len(a), np.int64)
+        vp = ctypes.c_void_p
+        if _support_lib().tco_support_pairs(self._h, a.ctypes.data_as(vp), b.ctypes.data_as(vp),
+                                            len(a), out.ctypes.data_as(vp)) != 0:
+            raise ValueError("oracle: bad arguments")
+        return out
+
+    def close(self):
+        if self._h:
+            _support_lib().tco_support_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        self.close()
+
+
+def support(src, dst, n: int = -1, threads: int = 0):
+    """Per-edge triangle support of the cleaned simple graph: (a, b, sup) sorted by (a, b)."""
+    g = SupportGraph(src, dst, n)
+    try:
+        return g.all(threads)
+    finally:
+        g.close()

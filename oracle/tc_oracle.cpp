@@ -218,6 +218,129 @@ int tco_count_rows(const tco_graph* g, int threads, int64_t sample_stride, int64
   return 0;
 }
 
+// ---------------------------------------------------------------------------
+// Per-edge support: for every edge {a,b} of the
+// cleaned simple graph, sup(a,b) = the number of triangles that contain it =
+// |N(a) ∩ N(b)| over the FULL undirected neighbourhoods (a triangle {a,b,w}
+// is exactly a common neighbour w; Fig. 1(b) computes the same wSet for
+// one edge).  This is the definition written out: no orientation, no suffix,
+// no hashing.  The k-truss / clustering-coefficient applications P:39 names
+// consume these values.  Pins: tests/test_oracle_pins.py (closed forms such as
+// K_n -> n-2, wheel spokes 2 / rim 1, friendship 1; (A·A)∘A by brute force;
+// sum = 3T).
+struct tco_support_graph {
+  int64_t n = 0, m = 0;
+  std::vector<uint64_t> keys;  // canonical (min << 32 | max), ascending = edge order
+  std::vector<int64_t> off;    // undirected CSR offsets
+  std::vector<int32_t> adj;    // N(x), ascending
+};
+
+// Steps 1-2 of tco_build plus the undirected adjacency.  NULL on invalid input.
+tco_support_graph* tco_support_build(const int32_t* src, const int32_t* dst, int64_t num_pairs,
+                                     int64_t n) {
+  if (num_pairs < 0 || (num_pairs > 0 && (!src || !dst))) return nullptr;
+  if (n < 0) {
+    int64_t mx = -1;
+    for (int64_t i = 0; i < num_pairs; ++i) mx = std::max<int64_t>(mx, std::max(src[i], dst[i]));
+    n = mx + 1;
+  }
+  tco_support_graph* g = new tco_support_graph();
+  std::vector<uint64_t>& keys = g->keys;
+  keys.reserve(num_pairs);
+  for (int64_t i = 0; i < num_pairs; ++i) {
+    int64_t a = src[i], b = dst[i];
+    if (a < 0 || b < 0 || a >= n || b >= n) {
+      delete g;
+      return nullptr;
+    }
+    if (a == b) continue;  // self-loops do not take part in triangles
+    uint64_t lo = (uint64_t)std::min(a, b), hi = (uint64_t)std::max(a, b);
+    keys.push_back((lo << 32) | hi);
+  }
+  std::sort(keys.begin(), keys.end());
+  keys.erase(std::unique(keys.begin(), keys.end()), keys.end());  // merge duplicates
+  g->n = n;
+  g->m = (int64_t)keys.size();
+  g->off.assign(n + 1, 0);
+  for (uint64_t k : keys) {
+    ++g->off[(k >> 32) + 1];
+    ++g->off[(k & 0xffffffffu) + 1];
+  }
+  for (int64_t x = 0; x < n; ++x) g->off[x + 1] += g->off[x];
+  g->adj.resize(2 * g->m);
+  std::vector<int64_t> fill(g->off.begin(), g->off.end() - 1);
+  for (uint64_t k : keys) {  // keys ascending -> each N(x) is filled in ascending order
+    int64_t a = (int64_t)(k >> 32), b = (int64_t)(k & 0xffffffffu);
+    g->adj[fill[a]++] = (int32_t)b;
+  }
+  for (uint64_t k : keys) {
+    int64_t a = (int64_t)(k >> 32), b = (int64_t)(k & 0xffffffffu);
+    g->adj[fill[b]++] = (int32_t)a;
+  }
+  for (int64_t x = 0; x < n; ++x) std::sort(g->adj.begin() + g->off[x], g->adj.begin() + g->off[x + 1]);
+  return g;
+}
+
+int64_t tco_support_m(const tco_support_graph* g) { return g ? g->m : -1; }
+
+void tco_support_free(tco_support_graph* g) { delete g; }
+
+// |N(a) ∩ N(b)| for one pair (the support if {a,b} is an edge).
+static uint64_t common_neighbours(const tco_support_graph* g, int64_t a, int64_t b) {
+  uint64_t c = 0;
+  std::set_intersection(g->adj.begin() + g->off[a], g->adj.begin() + g->off[a + 1],
+                        g->adj.begin() + g->off[b], g->adj.begin() + g->off[b + 1],
+                        CountingIterator{&c});
+  return c;
+}
+
+// All edges: out_a/out_b/out_sup (length m) in ascending (a, b), a < b.
+int tco_support_all(const tco_support_graph* g, int threads, int32_t* out_a, int32_t* out_b,
+                    uint32_t* out_sup) {
+  if (!g || (g->m > 0 && (!out_a || !out_b || !out_sup))) return 1;
+  int nt = threads > 0 ? threads : (int)std::thread::hardware_concurrency();
+  if (nt < 1) nt = 1;
+  std::atomic<int64_t> next{0};
+  const int64_t chunk = 4096;
+  auto worker = [&]() {
+    for (;;) {
+      int64_t b0 = next.fetch_add(chunk);
+      if (b0 >= g->m) break;
+      for (int64_t i = b0; i < std::min(g->m, b0 + chunk); ++i) {
+        const int64_t a = (int64_t)(g->keys[i] >> 32), b = (int64_t)(g->keys[i] & 0xffffffffu);
+        out_a[i] = (int32_t)a;
+        out_b[i] = (int32_t)b;
+        out_sup[i] = (uint32_t)common_neighbours(g, a, b);
+      }
+    }
+  };
+  std::vector<std::thread> pool;
+  for (int w = 0; w < nt; ++w) pool.emplace_back(worker);
+  for (auto& th : pool) th.join();
+  return 0;
+}
+
+// Sampled pairs (any a, b): out[i] = |N(a_i) ∩ N(b_i)| if {a_i, b_i} is an
+// edge, else -1.  Lets a test check sampled outputs at full size.
+int tco_support_pairs(const tco_support_graph* g, const int32_t* a, const int32_t* b, int64_t k,
+                      int64_t* out) {
+  if (!g || (k > 0 && (!a || !b || !out))) return 1;
+  for (int64_t i = 0; i < k; ++i) {
+    int64_t x = std::min(a[i], b[i]), y = std::max(a[i], b[i]);
+    if (x < 0 || y >= g->n || x == y) {
+      out[i] = -1;
+      continue;
+    }
+    const uint64_t key = ((uint64_t)x << 32) | (uint64_t)y;
+    if (!std::binary_search(g->keys.begin(), g->keys.end(), key)) {
+      out[i] = -1;
+      continue;
+    }
+    out[i] = (int64_t)common_neighbours(g, x, y);
+  }
+  return 0;
+}
+
 // Steps 1-5 in one call.  Returns 0 on success, 1 on invalid argument.
 // sample_stride > 1 counts only rows x with x % sample_stride == 0.
 int tco_count(const int32_t* src, const int32_t* dst, int64_t num_pairs, int64_t n, int order,
