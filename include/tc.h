@@ -167,6 +167,29 @@ TC_API tc_status tc_count_range(const tc_graph* g, int64_t e_begin, int64_t e_en
                          uint64_t* d_partial);
 
 /*
+ * Per-edge triangle support (the k-truss and
+ * clustering-coefficient inputs P:39 names): d_support (device uint32[m],
+ * caller-owned, overwritten) receives, for every CSR edge position p in
+ * [0, m), the number of triangles of G that contain the undirected edge
+ * {row(p), col[p]} (= |N(a) ∩ N(b)| over full neighbourhoods).  Every
+ * triangle u<v<w found at oriented edge (u,v) with witness w
+ * adds 1 to (u,v), (u,w) and (v,w), so sum(d_support) = 3T.  Use
+ * tc_edge_list to map positions to original vertex ids.  No sync; needs
+ * 8 B x m_live of stream-ordered scratch.  Errors: NULL graph or output ->
+ * TC_ERR_INVALID_ARGUMENT; tables that would exceed SMEM in support layout
+ * -> TC_ERR_UNSUPPORTED (rebuild with a lower huge_degree).
+ */
+TC_API tc_status tc_support(const tc_graph* g, void* stream, uint32_t* d_support);
+
+/*
+ * Original vertex ids of every CSR edge: d_u[p] = perm[row(p)], d_v[p] =
+ * perm[col[p]] for p in [0, m) (device int32[m] each, caller-owned,
+ * overwritten).  {d_u[p], d_v[p]} runs over the unique undirected edges of
+ * the cleaned input, each once.  No sync.
+ */
+TC_API tc_status tc_edge_list(const tc_graph* g, void* stream, int32_t* d_u, int32_t* d_v);
+
+/*
  * Cost-balanced split of [0, m_live) into world_size contiguous ranges
  * (SURVEY.md §8(e)): h_bounds (host int64[world_size+1]) receives
  * 0 = b_0 <= b_1 <= ... <= b_P = m_live, aligned to work chunks.

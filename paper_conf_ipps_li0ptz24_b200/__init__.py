@@ -32,7 +32,7 @@ TC_KEEP_ISOLATED = 0x1
 EXPORTS = (
     "tc_set_allocator", "tc_build_csr", "tc_build_csr_host", "tc_replan", "tc_graph_info",
     "tc_count", "tc_count_async", "tc_count_range", "tc_partition", "tc_partition_prefix",
-    "tc_free", "tc_last_error", "tc_version",
+    "tc_free", "tc_last_error", "tc_version", "tc_support", "tc_edge_list",
 )
 
 
@@ -100,6 +100,8 @@ def lib():
             "tc_count_range": ([vp, i64, i64, vp, vp], st),
             "tc_partition": ([vp, i32, vp], st),
             "tc_partition_prefix": ([vp, i64, i32, vp], st),
+            "tc_support": ([vp, vp, vp], st),
+            "tc_edge_list": ([vp, vp, vp, vp], st),
             "tc_free": ([vp], None),
             "tc_last_error": ([], ctypes.c_char_p),
             "tc_version": ([], ctypes.c_char_p),
@@ -225,6 +227,26 @@ class Graph:
                                     ctypes.c_void_p(_stream(stream)),
                                     ctypes.c_void_p(out.data_ptr())))
         return out
+
+    # ------------------------------------------------------------ per-edge support (f1)
+    def support(self, out=None, stream=None):
+        """Triangles containing each CSR edge: int32 CUDA tensor [m] holding the
+        uint32 counts (tc_support; stream-ordered).  Pair with edge_list()."""
+        torch = _torch()
+        if out is None:
+            out = torch.empty(self.m, dtype=torch.int32, device="cuda")
+        _check(lib().tc_support(self._h, ctypes.c_void_p(_stream(stream)),
+                                ctypes.c_void_p(out.data_ptr())))
+        return out
+
+    def edge_list(self, stream=None):
+        """(u, v) int32 CUDA tensors [m]: original ids of each CSR edge (tc_edge_list)."""
+        torch = _torch()
+        u = torch.empty(self.m, dtype=torch.int32, device="cuda")
+        v = torch.empty(self.m, dtype=torch.int32, device="cuda")
+        _check(lib().tc_edge_list(self._h, ctypes.c_void_p(_stream(stream)),
+                                  ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(v.data_ptr())))
+        return u, v
 
     def partition(self, world_size: int) -> list:
         b = np.zeros(int(world_size) + 1, dtype=np.int64)

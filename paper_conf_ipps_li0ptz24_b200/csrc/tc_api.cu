@@ -306,6 +306,22 @@ tc_status tc_count_range(const tc_graph* g, int64_t e_begin, int64_t e_end, void
   });
 }
 
+tc_status tc_support(const tc_graph* g, void* stream, uint32_t* d_support) {
+  return guarded([&] {
+    require(g != nullptr, "graph is NULL");
+    require(g->m == 0 || d_support != nullptr, "d_support is NULL");
+    tc::support_all(g, (cudaStream_t)stream, reinterpret_cast<unsigned*>(d_support));
+  });
+}
+
+tc_status tc_edge_list(const tc_graph* g, void* stream, int32_t* d_u, int32_t* d_v) {
+  return guarded([&] {
+    require(g != nullptr, "graph is NULL");
+    require(g->m == 0 || (d_u && d_v), "d_u/d_v is NULL");
+    tc::edge_ends(g, (cudaStream_t)stream, d_u, d_v);
+  });
+}
+
 tc_status tc_partition_prefix(const int64_t* h_prefix, int64_t n_units, int32_t world_size,
                               int64_t* h_bounds) {
   return guarded([&] {

@@ -120,6 +120,32 @@ __device__ __forceinline__ void linear_insert(int* __restrict__ T, uint32_t n, i
   }
 }
 
+// Support mode (8-B entries {key, payload}; empty = all ones).  The same
+// two-choice / linear schemes, moving the payload with its key.
+__device__ __forceinline__ bool cuckoo_insert64(unsigned long long* __restrict__ T, uint32_t n,
+                                                int32_t key, unsigned long long e) {
+  uint32_t pos = hash1(key, n);
+  for (int i = 0; i < kMaxKicks; ++i) {
+    const unsigned long long old = atomicExch(&T[pos], e);
+    if ((int)(uint32_t)old < 0) return true;
+    e = old;
+    key = (int)(uint32_t)old;
+    const uint32_t p1 = hash1(key, n);
+    pos = (pos == p1) ? hash2(key, n) : p1;
+  }
+  return false;
+}
+
+__device__ __forceinline__ void linear_insert64(unsigned long long* __restrict__ T, uint32_t n,
+                                                int32_t key, unsigned long long e) {
+  uint32_t h = hash1(key, n);
+  for (;;) {
+    const unsigned long long prev = atomicCAS(&T[h], ~0ull, e);
+    if (prev == ~0ull || (int)(uint32_t)prev == key) return;
+    h = (h + 1 == n) ? 0 : h + 1;
+  }
+}
+
 // Binary search of key in the sorted list col[b, b+d) (huge tables only).
 __device__ __noinline__ unsigned global_probe(const int32_t* __restrict__ col, int64_t b, int64_t d,
                                               int32_t key) {
@@ -191,7 +217,8 @@ struct ChunkSmem {
   int* sC;       // suffix length
   int* sD;       // group index (chunk-local)
   int* sGP;      // [G+1] insert prefix (chunk-relative)
-  int* sHash;    // slots
+  int* sHash;    // slots (support mode: 8-B entries, see produce)
+  int64_t* sE;   // support mode only: [S] CSR position of each edge (u,v)
 };
 
 __device__ __forceinline__ ChunkSmem slot_view(unsigned char* region, int S, int G, int T) {
@@ -208,6 +235,17 @@ __device__ __forceinline__ ChunkSmem slot_view(unsigned char* region, int S, int
   // base, so every table access stays in the shared window (LDS/ATOMS)
   c.sHash = reinterpret_cast<int*>(region) +
             ((4 * T + 2 * S + 2 * G + 2 * G + (S + 1) + 2 * S + (G + 1) + 3) & ~3);
+  c.sE = nullptr;
+  return c;
+}
+
+// Support mode (f1): every table entry is 8 B (a hash slot {key, index in
+// N+(v)}, a bitmap word {bits, members in earlier words}), followed by the
+// edges' own CSR positions.  Bytes: chunk_smem_bytes + 4*slots + 8*S.
+__device__ __forceinline__ ChunkSmem slot_view_sup(unsigned char* region, int S, int G, int T,
+                                                   int nslots) {
+  ChunkSmem c = slot_view(region, S, G, T);
+  c.sE = reinterpret_cast<int64_t*>(c.sHash + 2 * nslots);
   return c;
 }
 
@@ -226,7 +264,7 @@ __device__ __forceinline__ int seg_of(const int* __restrict__ P, int S, int k) {
 // 32 consecutive flat indices are mapped to their segments with one SMEM
 // load of the next 32 starts, a warp OR-reduce of a position mask and popc.
 // kU tiles are mapped, then load(seg, k) is issued for all of them (kU
-// independent global loads in flight per lane), then proc(seg, value).
+// independent global loads in flight per lane), then proc(seg, k, value).
 template <int kU, class Load, class Proc>
 __device__ __forceinline__ void warp_walk(const int* __restrict__ P, int S, int kbeg, int kend,
                                           Load load, Proc proc) {
@@ -254,7 +292,7 @@ __device__ __forceinline__ void warp_walk(const int* __restrict__ P, int S, int 
     }
 #pragma unroll
     for (int u = 0; u < kU; ++u)
-      if (k0 + 32 * u + lane < kend) proc(seg[u], val[u]);
+      if (k0 + 32 * u + lane < kend) proc(seg[u], k0 + 32 * u + lane, val[u]);
   }
 }
 
@@ -350,12 +388,114 @@ __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h
                 : walk_short<kLinear, false>(c, h.S, w0, w1, pv, h.ga);
 }
 
+// ------------------------------------------------------------------ support mode
+// per-edge triangle counts.  A match of key w (at col
+// position p_uw of u's suffix) in N+(v) closes the triangle {u, v, w}; its
+// three edges are (u,v) (the segment's own CSR position), (u,w) = p_uw and
+// (v,w) = row(v) + index of w in N+(v), which the support tables carry.
+
+// Index of key in N+(v) through its support-mode table, or -1.
+template <bool kLinear>
+__device__ __forceinline__ int sup_find(const int* __restrict__ base, int off, int code,
+                                        int32_t key) {
+  if (code <= 0) {
+    const int2 e = reinterpret_cast<const int2*>(base)[off + max((key >> 5) + code, 0)];
+    const unsigned bits = ~(unsigned)e.x;
+    const int b = key & 31;
+    if (key < 0 || !((bits >> b) & 1u)) return -1;
+    return e.y + __popc(bits & ((1u << b) - 1u));
+  }
+  const unsigned long long* H = reinterpret_cast<const unsigned long long*>(base) + off;
+  const uint32_t n = (uint32_t)code;
+  if (!kLinear) {
+    const unsigned long long x1 = H[hash1(key, n)], x2 = H[hash2(key, n)];
+    if ((int)(uint32_t)x1 == key) return (int)(x1 >> 32);
+    if ((int)(uint32_t)x2 == key) return (int)(x2 >> 32);
+    return -1;
+  }
+  uint32_t h = hash1(key, n);
+  for (;;) {
+    const unsigned long long x = H[h];
+    if ((int)(uint32_t)x == key) return (int)(x >> 32);
+    if ((int)(uint32_t)x < 0) return -1;
+    h = (h + 1 == n) ? 0 : h + 1;
+  }
+}
+
+// Index of key in the sorted list col[b, b+d), or -1 (huge tables).
+__device__ __noinline__ int global_find(const int32_t* __restrict__ col, int64_t b, int64_t d,
+                                        int32_t key) {
+  int64_t lo = b, hi = b + d;
+  while (lo < hi) {
+    int64_t mid = (lo + hi) >> 1;
+    if (__ldg(col + mid) < key) lo = mid + 1; else hi = mid;
+  }
+  return (lo < b + d && __ldg(col + lo) == key) ? (int)(lo - b) : -1;
+}
+
+__device__ __forceinline__ int sup_lookup_any(const ChunkSmem& c, const PlanView& pv, int gl,
+                                              int32_t key, bool linear) {
+  const int2 info = c.sInfo[gl];
+  if (info.x < 0)
+    return global_find(pv.col, c.sGB[gl] + c.sGP[gl], c.sGP[gl + 1] - c.sGP[gl], key);
+  return linear ? sup_find<true>(c.sHash, info.x, info.y, key)
+                : sup_find<false>(c.sHash, info.x, info.y, key);
+}
+
+constexpr int kUnrollSup = 4;
+
+// LONG class, support mode: tiles [t0, t1); a tile's lanes share one edge,
+// whose count is warp-aggregated into one atomic.
+__device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1,
+                                              const PlanView& pv, bool linear) {
+  const int lane = threadIdx.x & 31;
+  for (int t = t0; t < t1; t += kUnrollSup) {
+    int32_t key[kUnrollSup];
+    int64_t p[kUnrollSup];
+    int sl[kUnrollSup];
+#pragma unroll
+    for (int u = 0; u < kUnrollSup; ++u) {
+      const int4 d = c.sTile[min(t + u, t1 - 1)];
+      const int lanes = (t + u < t1) ? d.w : 0;
+      p[u] = (int64_t)(((uint64_t)(uint32_t)d.y << 32) | (uint32_t)d.x);
+      sl[u] = d.z;
+      key[u] = lane < lanes ? __ldg(pv.col + p[u] + lane) : -2;
+    }
+#pragma unroll
+    for (int u = 0; u < kUnrollSup; ++u) {
+      const int gl = c.sD[sl[u]];
+      const int idx = key[u] >= 0 ? sup_lookup_any(c, pv, gl, key[u], linear) : -1;
+      const unsigned bal = __ballot_sync(0xffffffffu, idx >= 0);
+      if (idx >= 0) {
+        atomicAdd(pv.sup + p[u] + lane, 1u);                     // (u, w)
+        atomicAdd(pv.sup + c.sGB[gl] + c.sGP[gl] + idx, 1u);     // (v, w)
+      }
+      if (lane == 0 && bal) atomicAdd(pv.sup + c.sE[sl[u]], (unsigned)__popc(bal));  // (u, v)
+    }
+  }
+}
+
+// SHORT class, support mode: flat keys [k0w, k1w) of the chunk.
+__device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0w, int k1w,
+                                               const PlanView& pv, bool linear) {
+  auto load = [&](int sg, int k) { return __ldg(pv.col + c.sB[sg] + k); };
+  warp_walk<kUnrollSup>(c.sA, S, k0w, k1w, load, [&](int sg, int k, int32_t key) {
+    const int gl = c.sD[sg];
+    const int idx = sup_lookup_any(c, pv, gl, key, linear);
+    if (idx >= 0) {
+      atomicAdd(pv.sup + c.sB[sg] + k, 1u);                  // (u, w)
+      atomicAdd(pv.sup + c.sGB[gl] + c.sGP[gl] + idx, 1u);   // (v, w)
+      atomicAdd(pv.sup + c.sE[sg], 1u);                      // (u, v)
+    }
+  });
+}
+
 // ------------------------------------------------------------------ producers
 // Stage chunk cix into a slot and build its tables.  pt = producer thread id
 // in [0, PT); the PT producer threads synchronise on named barrier 1.  The
 // header is written by producer 0 before its own mbarrier arrive, so the
 // consumers see it once every producer has arrived.
-template <int kB>
+template <int kB, bool kSup = false>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
                                         int pt, int PT) {
@@ -375,7 +515,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   const int nslots = (int)(__ldg(pv.slot_prefix + (gb)) - slot0);
   const int64_t kp0 = __ldg(pv.key_prefix + (sa));
   const int T = is_long ? (int)((__ldg(pv.key_prefix + (sb)) - kp0) >> 5) : 0;
-  ChunkSmem c = slot_view(region, S, G, T);
+  ChunkSmem c = kSup ? slot_view_sup(region, S, G, T, nslots) : slot_view(region, S, G, T);
 
   // 1. stage edges and groups; empty slots.  Each producer thread handles
   //    kB items per batch with all their global loads issued before any
@@ -408,6 +548,8 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       }
     }
   }
+  if (kSup)
+    for (int i = pt; i < S; i += PT) c.sE[i] = __ldg(pv.seg_edge + (sa + i));
   const int64_t ip0 = __ldg(pv.ins_prefix + (ga));
   int huge = 0;
   for (int base = pt; base <= G; base += PT * kB) {
@@ -439,9 +581,11 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     }
   }
   {
+    // support mode: 8-B entries -> twice the words (nslots is a multiple of 4)
+    const int nwords = kSup ? 2 * nslots : nslots;
     int4* h4 = reinterpret_cast<int4*>(c.sHash);
-    for (int i = pt; i < (nslots >> 2); i += PT) h4[i] = make_int4(-1, -1, -1, -1);
-    for (int i = (nslots & ~3) + pt; i < nslots; i += PT) c.sHash[i] = -1;
+    for (int i = pt; i < (nwords >> 2); i += PT) h4[i] = make_int4(-1, -1, -1, -1);
+    for (int i = (nwords & ~3) + pt; i < nwords; i += PT) c.sHash[i] = -1;
   }
   const int any_huge = named_sync_or(1, PT, huge);
 
@@ -455,7 +599,10 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       for (int t = ts; t < te; ++t) {
         const int64_t p = st + ((int64_t)(t - ts) << 5);
         const int lanes = min(32, len - ((t - ts) << 5));
-        c.sTile[t] = make_int4((int)(uint32_t)p, (int)(p >> 32), toff, (int)((unsigned)d.y << 6) | lanes);
+        // support mode: the tile names its edge (chunk-local) instead of its table
+        c.sTile[t] = kSup ? make_int4((int)(uint32_t)p, (int)(p >> 32), i, lanes)
+                          : make_int4((int)(uint32_t)p, (int)(p >> 32), toff,
+                                      (int)((unsigned)d.y << 6) | lanes);
       }
     }
   }
@@ -468,7 +615,42 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   const int i0 = (int)((int64_t)NI * pw / npw), i1 = (int)((int64_t)NI * (pw + 1) / npw);
   auto load_row = [&](int g, int k) { return __ldg(pv.col + c.sGB[g] + k); };
   bool linear = pv.probe_mode == 1;
-  auto insert_linear = [&](int g, int32_t key) {
+  if constexpr (kSup) {
+    // Support mode: entries carry the key's index j in N+(v) (its edge (v,w)
+    // is col position row(v) + j).  Bitmap word x = {bits, members of N+(v)
+    // in words before x}: the inserter of the first key of each word writes
+    // the count of the words it opens (those after its predecessor's word).
+    auto ins_sup = [&](int g, int k, int32_t key, bool lin) {
+      const int2 d = c.sInfo[g];
+      if (d.x < 0) return;
+      const int j = k - c.sGP[g];
+      if (d.y <= 0) {
+        int2* W = reinterpret_cast<int2*>(c.sHash) + d.x;
+        const int w = (key >> 5) + d.y;
+        atomicAnd(&W[w].x, ~(1 << (key & 31)));
+        const int pw = j > 0 ? (__ldg(pv.col + c.sGB[g] + k - 1) >> 5) + d.y : -1;
+        for (int x = pw + 1; x <= w; ++x) W[x].y = j;
+      } else {
+        unsigned long long* H = reinterpret_cast<unsigned long long*>(c.sHash) + d.x;
+        const unsigned long long e = ((unsigned long long)(uint32_t)j << 32) | (uint32_t)key;
+        if (lin) linear_insert64(H, (uint32_t)d.y, key, e);
+        else if (!cuckoo_insert64(H, (uint32_t)d.y, key, e)) linear = true;  // flag, below
+      }
+    };
+    const bool want_linear = linear;
+    linear = false;
+    warp_walk<kInsU>(c.sGP, G, i0, i1, load_row,
+                     [&](int g, int k, int32_t key) { ins_sup(g, k, key, want_linear); });
+    if (!want_linear && named_sync_or(1, PT, linear)) {  // a cuckoo insert failed
+      for (int i = pt; i < 2 * nslots; i += PT) c.sHash[i] = -1;
+      named_sync(1, PT);
+      warp_walk<kInsU>(c.sGP, G, i0, i1, load_row,
+                       [&](int g, int k, int32_t key) { ins_sup(g, k, key, true); });
+      linear = true;
+    }
+    linear = linear || want_linear;
+  } else {
+  auto insert_linear = [&](int g, int, int32_t key) {
     const int2 d = c.sInfo[g];
     if (d.x < 0) return;
     if (d.y <= 0) bitmap_insert(c.sHash + d.x, d.y, key);
@@ -478,7 +660,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, insert_linear);
   } else {
     bool ok = true;
-    warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int32_t key) {
+    warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, [&](int g, int, int32_t key) {
       const int2 d = c.sInfo[g];
       if (d.x < 0) return;
       if (d.y <= 0) bitmap_insert(c.sHash + d.x, d.y, key);
@@ -490,6 +672,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       named_sync(1, PT);
       warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, insert_linear);
     }
+  }
   }
   if (pt == 0) {
     hdr.sa = sa;
@@ -628,6 +811,73 @@ __global__ void __launch_bounds__(kFlatBlock, 3)
   }
 }
 
+// Support mode kernel: one chunk at a time per CTA, all warps build then
+// all warps probe (both classes; 8-B table entries double the SMEM of a chunk).
+__global__ void __launch_bounds__(kMaxBlock, 1)
+    k_support(PlanView pv, int64_t c_begin, int64_t c_end) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ SlotHdr hdr;
+  const int warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  for (int64_t cix = c_begin + blockIdx.x; cix < c_end; cix += gridDim.x) {
+    produce<2, true>(pv, cix, 0, INT64_MAX, smem, hdr, threadIdx.x, blockDim.x);
+    __syncthreads();
+    const SlotHdr h = hdr;
+    if (h.S > 0) {
+      const ChunkSmem c = slot_view_sup(smem, h.S, h.G, h.T, h.nslots);
+      const int NU = h.is_long ? h.T : c.sA[h.S];
+      const int w0 = (int)((int64_t)NU * warp / nw), w1 = (int)((int64_t)NU * (warp + 1) / nw);
+      if (h.is_long) walk_long_sup(c, w0, w1, pv, h.linear);
+      else if (w0 < w1) walk_short_sup(c, h.S, w0, w1, pv, h.linear);
+    }
+    __syncthreads();  // the slot is rebuilt by the next chunk
+  }
+}
+
+// Largest i in [0, len) with a[i] <= x (a non-decreasing, a[0] <= x).
+__device__ __forceinline__ int64_t last_le(const int64_t* __restrict__ a, int64_t len, int64_t x) {
+  int64_t lo = 0, hi = len - 1;
+  while (lo < hi) {
+    const int64_t mid = (lo + hi + 1) >> 1;
+    if (a[mid] <= x) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+// CSR position of every live segment's own edge (u,v): u = the row holding
+// its suffix, v = the head whose row starts at grp_ibase + ins_prefix, and
+// (u,v) = the position of v in N+(u), which precedes the suffix.
+__global__ void k_seg_edge(const int64_t* __restrict__ row_ptr, int64_t n,
+                           const int32_t* __restrict__ col, const int64_t* __restrict__ seg_start,
+                           const int32_t* __restrict__ seg_group,
+                           const int64_t* __restrict__ grp_ibase,
+                           const int64_t* __restrict__ ins_prefix, int64_t S,
+                           int64_t* __restrict__ seg_edge) {
+  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
+       s += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t st = seg_start[s];
+    const int g = seg_group[s];
+    const int64_t u = last_le(row_ptr, n + 1, st);
+    const int32_t v = (int32_t)last_le(row_ptr, n + 1, grp_ibase[g] + ins_prefix[g]);
+    int64_t lo = row_ptr[u], hi = st;
+    while (lo < hi) {
+      const int64_t mid = (lo + hi) >> 1;
+      if (col[mid] < v) lo = mid + 1; else hi = mid;
+    }
+    seg_edge[s] = lo;
+  }
+}
+
+// Original ids of every CSR edge: (perm[row(p)], perm[col[p]]).
+__global__ void k_edge_ends(const int64_t* __restrict__ row_ptr, int64_t n,
+                            const int32_t* __restrict__ col, const int32_t* __restrict__ perm,
+                            int64_t m, int32_t* __restrict__ eu, int32_t* __restrict__ ev) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < m;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    eu[p] = perm[last_le(row_ptr, n + 1, p)];
+    ev[p] = perm[col[p]];
+  }
+}
+
 bool g_attr_set = false;
 
 int optin_smem() {
@@ -649,6 +899,8 @@ void ensure_attr() {
                                optin_smem() - static_smem((const void*)k_count)));
   TC_CUDA(cudaFuncSetAttribute(k_count_flat, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                optin_smem() - static_smem((const void*)k_count_flat)));
+  TC_CUDA(cudaFuncSetAttribute(k_support, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               optin_smem() - static_smem((const void*)k_support)));
   g_attr_set = true;
 }
 
@@ -669,6 +921,8 @@ PlanView plan_view(const tc_graph* g) {
   pv.chunk_seg = P.chunk_seg.get();
   pv.n_long_chunks = P.n_long_chunks;
   pv.probe_mode = P.opt.probe_mode;
+  pv.seg_edge = nullptr;
+  pv.sup = nullptr;
   return pv;
 }
 
@@ -734,6 +988,41 @@ void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_b
                                                                              e_end, d_out);
     TC_LAUNCH();
   }
+}
+
+void support_all(const tc_graph* g, cudaStream_t s, unsigned* d_sup) {
+  if (g->m > 0) TC_CUDA(cudaMemsetAsync(d_sup, 0, sizeof(unsigned) * (size_t)g->m, s));
+  const Plan& P = g->plan;
+  if (P.S == 0 || P.n_chunks == 0) return;
+  ensure_attr();
+  DevBuf<int64_t> seg_edge(P.S, s);
+  const int grid_e = (int)std::min<int64_t>((P.S + 255) / 256, 148 * 16);
+  k_seg_edge<<<grid_e, 256, 0, s>>>(g->row_ptr.get(), g->n, g->col.get(), P.seg_start.get(),
+                                    P.seg_group.get(), P.grp_ibase.get(), P.ins_prefix.get(), P.S,
+                                    seg_edge.get());
+  TC_LAUNCH();
+  PlanView pv = plan_view(g);
+  pv.seg_edge = seg_edge.get();
+  pv.sup = d_sup;
+  // a chunk's support layout is at most twice its count layout (tc_count.cu
+  // slot_view_sup: + 4 B per table word + 8 B per edge)
+  const int64_t bytes = slot_bytes_of(2 * std::max(P.smem_bytes, P.smem_flat) + 16);
+  if (bytes > optin_smem() - static_smem((const void*)k_support))
+    fail(TC_ERR_UNSUPPORTED, "support tables exceed shared memory (lower huge_degree)");
+  int occ = 0;
+  TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_support, kMaxBlock, (size_t)bytes));
+  if (occ < 1) fail(TC_ERR_UNSUPPORTED, "support kernel cannot launch");
+  const int grid = (int)std::min<int64_t>(P.n_chunks, (int64_t)occ * num_sms());
+  k_support<<<grid, kMaxBlock, (size_t)bytes, s>>>(pv, 0, P.n_chunks);
+  TC_LAUNCH();
+}
+
+void edge_ends(const tc_graph* g, cudaStream_t s, int32_t* d_u, int32_t* d_v) {
+  if (g->m == 0) return;
+  const int grid = (int)std::min<int64_t>((g->m + 255) / 256, 148 * 16);
+  k_edge_ends<<<grid, 256, 0, s>>>(g->row_ptr.get(), g->n, g->col.get(), g->perm.get(), g->m, d_u,
+                                   d_v);
+  TC_LAUNCH();
 }
 
 }  // namespace tc

@@ -103,6 +103,9 @@ struct PlanView {
   const int64_t* chunk_seg;    // [C+1]
   int64_t n_long_chunks;
   int probe_mode;
+  // support mode only (tc_support; nullptr when counting)
+  const int64_t* seg_edge;     // [S] CSR position of segment s's own edge (u,v)
+  unsigned* sup;               // [m] per-edge triangle counts (accumulated)
 };
 
 // SMEM a chunk needs (bytes): per segment staging + per group descriptor +
@@ -169,5 +172,7 @@ int max_chunk_smem(int slots);  // SMEM one of the kernel's chunk slots may use
 int max_flat_chunk_smem();      // SMEM one short-class chunk may use (3 CTAs per SM)
 int flat_occupancy(int64_t smem_bytes);
 int num_sms();
+void support_all(const tc_graph* g, cudaStream_t s, unsigned* d_sup);   // f1, tc_support
+void edge_ends(const tc_graph* g, cudaStream_t s, int32_t* d_u, int32_t* d_v);
 
 }  // namespace tc

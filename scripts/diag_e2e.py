@@ -29,3 +29,16 @@ for it in range(2):
     print(f"host-entry iter {it}: build_host {e0.elapsed_time(e1):.1f} ms count {e1.elapsed_time(e2):.1f} ms", flush=True)
     g.close()
 print("mem peak GB", torch.cuda.max_memory_allocated()/1e9, "free/total", [x/1e9 for x in torch.cuda.mem_get_info()])
+# bench-like: a resident graph + flush buffer alive while the host entry runs
+g0 = tc.build_csr(ps.cuda(), pd.cuda(), n)
+flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+for it in range(3):
+    torch.cuda.synchronize(); e0 = ev(); tw = time.perf_counter()
+    g = tc.build_csr_host(ps, pd, n)
+    e1 = ev(); tb = time.perf_counter()
+    b = g.partition(1); o = g.count_range(b[0], b[1]); t = int(o.item())
+    info_ms = {k: v for k, v in g.info.as_dict().items() if k.startswith("ms_")}
+    e2 = ev(); torch.cuda.synchronize(); te = time.perf_counter()
+    g.close(); tc_ = time.perf_counter()
+    print(f"resident-graph iter {it}: build_host {e0.elapsed_time(e1):.1f} ms (wall {1e3*(tb-tw):.1f}) count+item {e1.elapsed_time(e2):.1f} ms  total wall {1e3*(te-tw):.1f}  close {1e3*(tc_-te):.1f}", flush=True)
+    print("   phases", {k: round(v, 1) for k, v in info_ms.items()}, flush=True)

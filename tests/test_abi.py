@@ -76,6 +76,8 @@ def test_bad_arguments_rejected_before_device(tc):
     assert L.tc_count_range(None, 0, 0, None, None) == 1
     assert L.tc_partition(None, 2, None) == 1
     assert L.tc_graph_info(None, None) == 1
+    assert L.tc_support(None, None, None) == 1
+    assert L.tc_edge_list(None, None, None, None) == 1
     L.tc_free(None)  # no-op
 
 
