@@ -60,6 +60,9 @@ def parse():
     ap.add_argument("--opt", action="append", default=[],
                     help="plan option key=value (tc_options field), repeatable")
     ap.add_argument("--out", default=None, help="also write the JSON line here")
+    ap.add_argument("--mode", default="count", choices=["count", "support"],
+                    help="count: T (the headline); support: per-edge triangle counts "
+                         "(tc_support, SURVEY.md §8(f) f1), N = 1 only")
     return ap.parse_args()
 
 
@@ -215,6 +218,91 @@ def cpu_baseline(src, dst, n, a, m_gpu):
     return out
 
 
+def bench_support(a, tc, g, info, src, dst, n, gen_s, build_wall_ms, world, rank):
+    """--mode support: one step = tc_support over the resident graph (all m
+    per-edge counts, zero-init included).  Parity: sum = 3T and 4,000 sampled
+    edges against the oracle's |N(a) ∩ N(b)| (cpu leg)."""
+    import torch
+    if world > 1:
+        if rank == 0:
+            print(json.dumps({"metric": METRIC + " (per-edge support)", "unavailable":
+                              "support mode is single-GPU (replicas only)"}), flush=True)
+        return 0
+    m = int(info.m)
+    stream = torch.cuda.current_stream()
+    sup = torch.empty(max(m, 1), dtype=torch.int32, device="cuda")[:m]
+    flush = torch.empty(a.flush_mb << 20, dtype=torch.uint8, device="cuda")
+    for _ in range(max(1, a.warmup)):
+        g.support(out=sup)
+    torch.cuda.synchronize()
+    sampler = ClockSampler(torch.cuda.current_device())
+    sampler.start()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(a.steps)]
+    for i in range(a.steps):
+        flush.fill_(i & 0xFF)
+        evs[i][0].record(stream)
+        g.support(out=sup)
+        evs[i][1].record(stream)
+    torch.cuda.synchronize()
+    clocks = sampler.stop()
+    step_ms = [x.elapsed_time(y) for x, y in evs]
+    ms = sum(step_ms) / a.steps
+    total = int(sup.to(torch.int64).sum().item())
+    T = g.count()
+    exp = expected_counts(a.config, a.seed)
+    parity = {"sum_is_3T": total == 3 * T,
+              "T_vs_oracle": None if exp is None else exp["triangles"] == T}
+    if not a.no_cpu_baseline:
+        import oracle
+        idx = torch.randint(0, m, (4000,), generator=torch.Generator().manual_seed(1)).cuda()
+        u, v = g.edge_list()
+        su, sv, ss = (x[idx].cpu().numpy() for x in (u, v, sup))
+        og = oracle.SupportGraph(src, dst, n)
+        t0 = time.perf_counter()
+        want = og.pairs(su, sv)
+        cpu_s = time.perf_counter() - t0
+        og.close()
+        parity["sampled_4000_vs_oracle"] = bool(np.array_equal(ss.view(np.uint32).astype(np.int64),
+                                                               want))
+        cpu = {"value": 4000 / max(cpu_s, 1e-9), "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": "4,000 random edges of the same graph, |N(a) ∩ N(b)| one by one "
+                         "(oracle SupportGraph.pairs, 1 thread); build excluded"}
+    else:
+        cpu = None
+    hbm, peak_src = peaks()
+    b = int(info.b_itc) + 4 * m + 24 * T
+    achieved = b / (ms / 1e3) / 1e9
+    line = {
+        "metric": METRIC + " (per-edge support)", "value": m / (ms / 1e3), "unit": UNIT,
+        "n_gpus": 1, "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
+        "data": "synthetic",
+        "config": {"workload": f"{a.config}: {cfg_desc(a.config)}", "seed": a.seed, "n": n,
+                   "m": m, "m_live": int(info.m_live), "mode": "support",
+                   "l2": f"flushed by a {a.flush_mb} MiB write between timed steps"},
+        "triangles": str(T), "parity_vs_oracle": parity,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved / hbm, "traffic": None, "bytes_per_launch": b,
+                     "bytes_def": "B_ITC + 4m (zero-init) + 24T (3 u32 read-modify-writes "
+                                  "per triangle)", "peak_source": peak_src},
+        "gpu_launches": a.steps * 2,
+        "build_ms": {"wall": build_wall_ms, "total_events": info.ms_total},
+        "clocks": clocks, "gen_s": round(gen_s, 2), "step_ms": step_ms,
+    }
+    if cpu:
+        line["cpu_baseline"] = cpu
+    print(json.dumps(line), flush=True)
+    if a.out:
+        open(a.out, "w").write(json.dumps(line) + "\n")
+    g.close()
+    return 0
+
+
+def cfg_desc(name):
+    return tcgen.CONFIGS[name].description
+
+
 def main():
     a = parse()
     if a.impl == "reference":
@@ -262,6 +350,9 @@ def main():
     info = g.info
     del dsrc, dst_t
     m = int(info.m)
+
+    if a.mode == "support":
+        return bench_support(a, tc, g, info, src, dst, n, gen_s, build_wall_ms, world, rank)
 
     bounds = g.partition(world)
     e0, e1 = bounds[rank], bounds[rank + 1]

@@ -53,27 +53,64 @@ void check_cuda(cudaError_t e, const char* what, const char* file, int line) {
   fail(TC_ERR_CUDA, buf);
 }
 
-void* dev_alloc(size_t bytes, cudaStream_t s) {
+namespace {
+constexpr int kMaxDevices = 64;
+
+// Release threshold "never": freed blocks stay mapped across syncs (without
+// this every build re-maps its scratch, tens of ms at config C2).
+void keep_mapped(cudaMemPool_t pool) {
+  uint64_t thr = UINT64_MAX;
+  cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+}
+
+// The device's default pool (persistent buffers) or the library's own scratch
+// pool, created on first use.  nullptr if the device cannot be queried.
+cudaMemPool_t pool_of(bool persistent) {
+  static cudaMemPool_t scratch[kMaxDevices] = {};
+  static bool default_ready[kMaxDevices] = {};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  if (persistent) {
+    cudaMemPool_t p = nullptr;
+    if (cudaDeviceGetDefaultMemPool(&p, dev) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    if (!default_ready[dev]) {
+      keep_mapped(p);
+      default_ready[dev] = true;
+    }
+    return p;
+  }
+  if (!scratch[dev]) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.handleTypes = cudaMemHandleTypeNone;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    if (cudaMemPoolCreate(&scratch[dev], &props) != cudaSuccess) {
+      cudaGetLastError();
+      scratch[dev] = nullptr;
+      return nullptr;
+    }
+    keep_mapped(scratch[dev]);
+  }
+  return scratch[dev];
+}
+}  // namespace
+
+void* dev_alloc(size_t bytes, cudaStream_t s, bool persistent) {
   void* p = nullptr;
   if (g_alloc) {
     p = g_alloc(bytes, (void*)s, g_ctx);
     if (!p) fail(TC_ERR_OUT_OF_MEMORY, "allocator hook returned NULL");
     return p;
   }
-  static bool pool_ready = false;
-  if (!pool_ready) {
-    // Keep freed blocks in the device pool across syncs: without this every
-    // build re-maps its scratch (tens of ms at config C2).
-    int dev = 0;
-    cudaMemPool_t pool;
-    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-      uint64_t thr = UINT64_MAX;
-      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
-    cudaGetLastError();
-    pool_ready = true;
-  }
-  cudaError_t e = cudaMallocAsync(&p, bytes, s);
+  cudaMemPool_t pool = pool_of(persistent);
+  cudaError_t e = pool ? cudaMallocFromPoolAsync(&p, bytes, pool, s) : cudaMallocAsync(&p, bytes, s);
   if (e != cudaSuccess || !p) {
     cudaGetLastError();
     fail(TC_ERR_OUT_OF_MEMORY, "cudaMallocAsync failed (" + std::to_string(bytes) + " bytes)");
@@ -81,17 +118,13 @@ void* dev_alloc(size_t bytes, cudaStream_t s) {
   return p;
 }
 
-// Grow the default memory pool in one step so that a build's allocations
+// Grow the scratch pool in one step so that a build's scratch allocations
 // reuse already-mapped memory: mapping physical memory inside the build
 // (pool growth on demand) made identical builds vary by 3-10x in time.
 void reserve_pool(size_t bytes, cudaStream_t s) {
   if (g_alloc || bytes == 0) return;
-  int dev = 0;
-  cudaMemPool_t pool;
-  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetDefaultMemPool(&pool, dev) != cudaSuccess) {
-    cudaGetLastError();
-    return;
-  }
+  cudaMemPool_t pool = pool_of(false);
+  if (!pool) return;
   uint64_t reserved = 0, used = 0;
   cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved);
   cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used);
@@ -103,7 +136,7 @@ void reserve_pool(size_t bytes, cudaStream_t s) {
   const size_t grow = want < cap ? want : cap;
   if (grow == 0) return;
   void* p = nullptr;
-  if (cudaMallocAsync(&p, grow, s) == cudaSuccess && p) cudaFreeAsync(p, s);
+  if (cudaMallocFromPoolAsync(&p, grow, pool, s) == cudaSuccess && p) cudaFreeAsync(p, s);
   cudaGetLastError();
 }
 

@@ -543,14 +543,14 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
       return cub::DeviceRadixSort::SortKeys(t, b, db, n, 0, 2 * bits + 1, s);
     });
     n_act = (int64_t)d2h(nact.get(), s);
-    g->perm = DevBuf<int32_t>(std::max<int64_t>(n_act, 1), s);
+    g->perm = DevBuf<int32_t>(std::max<int64_t>(n_act, 1), s, true);
     if (n_act > 0) {
       k_perm<<<grid_for(n_act), TPB, 0, s>>>(db.Current(), n_act, bits, g->perm.get(),
                                              rank.get());
       TC_LAUNCH();
     }
   } else {
-    g->perm = DevBuf<int32_t>(1, s);
+    g->perm = DevBuf<int32_t>(1, s, true);
   }
   g->n = n_act;
   deg.reset();
@@ -561,8 +561,8 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
   // a5
   const int bits2 = bits_for(std::max<int64_t>(n_act, 2));
   g->bits = bits2;
-  g->row_ptr = DevBuf<int64_t>(n_act + 1, s);
-  g->col = DevBuf<int32_t>(std::max<int64_t>(m, 1), s);
+  g->row_ptr = DevBuf<int64_t>(n_act + 1, s, true);
+  g->col = DevBuf<int32_t>(std::max<int64_t>(m, 1), s, true);
   if (m > 0) {
     uint64_t* okey_a = (ukey == ka.get()) ? kb.get() : ka.get();  // the free buffer
     k_orient<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank.get(), bits2, okey_a);
@@ -654,10 +654,10 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   const int64_t S = (int64_t)h_stats[2], S_long = (int64_t)h_stats[3];
   P.S = S;
   P.S_long = S_long;
-  P.key_prefix = DevBuf<int64_t>(S + 1, s);
+  P.key_prefix = DevBuf<int64_t>(S + 1, s, true);
   TC_CUDA(cudaMemsetAsync(P.key_prefix.get(), 0, sizeof(int64_t), s));
   if (S == 0) {
-    P.chunk_seg = DevBuf<int64_t>(1, s);
+    P.chunk_seg = DevBuf<int64_t>(1, s, true);
     TC_CUDA(cudaMemsetAsync(P.chunk_seg.get(), 0, sizeof(int64_t), s));
     P.h_chunk_seg.assign(1, 0);
     TC_CUDA(cudaStreamSynchronize(s));
@@ -692,11 +692,11 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   const int64_t slot_limit = max_chunk_smem(P.tune.slots);
   const int64_t flat_limit = max_flat_chunk_smem();
   const int64_t max_table_slots = std::min(slot_limit, flat_limit) / 8;
-  P.seg_start = DevBuf<int64_t>(S, s);
-  P.seg_len = DevBuf<int32_t>(S, s);
-  P.seg_group = DevBuf<int32_t>(S, s);
+  P.seg_start = DevBuf<int64_t>(S, s, true);
+  P.seg_len = DevBuf<int32_t>(S, s, true);
+  P.seg_group = DevBuf<int32_t>(S, s, true);
   DevBuf<int64_t> units(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
-  P.grp_code = DevBuf<int32_t>(G, s);
+  P.grp_code = DevBuf<int32_t>(G, s, true);
   k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted, val_sorted, gincl.get(), S, S_long,
                                          g->bits, row_ptr,
                                          opt.huge_degree, opt.table_factor, opt.bitmap_factor,
@@ -710,11 +710,11 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   sval.reset();
   sval2.reset();
   exclusive_prefix(units.get(), S, P.key_prefix.get(), s);
-  P.ins_prefix = DevBuf<int64_t>(G + 1, s);
-  P.slot_prefix = DevBuf<int64_t>(G + 1, s);
+  P.ins_prefix = DevBuf<int64_t>(G + 1, s, true);
+  P.slot_prefix = DevBuf<int64_t>(G + 1, s, true);
   exclusive_prefix(grp_d.get(), G, P.ins_prefix.get(), s);
   exclusive_prefix(grp_slots.get(), G, P.slot_prefix.get(), s);
-  P.grp_ibase = DevBuf<int64_t>(G, s);
+  P.grp_ibase = DevBuf<int64_t>(G, s, true);
   k_grp_ibase<<<grid_for(G), TPB, 0, s>>>(grp_row.get(), P.ins_prefix.get(), G, P.grp_ibase.get());
   TC_LAUNCH();
   DevBuf<int64_t> cost(S, s), cost_prefix(S + 1, s);
@@ -765,7 +765,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     if ((int64_t)need[0] > slot_limit || (int64_t)need[1] > flat_limit)
       fail(TC_ERR_UNSUPPORTED, "an edge's hash table exceeds shared memory (lower huge_degree)");
     const int64_t nc = h_off[1];
-    P.chunk_seg = DevBuf<int64_t>(nc + 1, s);
+    P.chunk_seg = DevBuf<int64_t>(nc + 1, s, true);
     k_split<<<grid_for(nc0), TPB, 0, s>>>(cs0.get(), nc0, nL0, P.seg_group.get(), P.slot_prefix.get(),
                                           P.key_prefix.get(), slot_limit, flat_limit, nullptr,
                                           poff.get(), P.chunk_seg.get(), nullptr);
