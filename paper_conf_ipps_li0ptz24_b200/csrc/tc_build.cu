@@ -611,7 +611,7 @@ Tuning tuning_from_env() {
     return x < lo ? lo : (x > hi ? hi : x);
   };
   t.slots = get("TC_SLOTS", t.slots, 2, 4);
-  t.grab_long = get("TC_GRAB_LONG", t.grab_long, 0, 1 << 20);
+  t.grab_long = (get("TC_GRAB_LONG", t.grab_long, 0, 1 << 20) + 7) & ~7;  // walk_long: 8-tile batches
   t.grab_short = get("TC_GRAB_SHORT", t.grab_short, 0, 1 << 24);
   t.prod_div = get("TC_PROD_DIV", t.prod_div, 2, 32);
   t.wait_hint_ns = get("TC_WAIT_HINT", t.wait_hint_ns, 0, 10000000);
@@ -625,6 +625,8 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P.opt = opt;
   P.block = opt.block_threads;
   const int64_t m = g->m, n = g->n;
+  // the count kernel's tile descriptors address keys by a 32-bit col index
+  if (m > (int64_t)0xFFFFFFFFll) fail(TC_ERR_UNSUPPORTED, "more than 2^32 - 1 unique edges");
   const int64_t* row_ptr = g->row_ptr.get();
   const int32_t* col = g->col.get();
   Trace tr(s);

@@ -209,7 +209,12 @@ struct SlotHdr {
 };
 
 struct ChunkSmem {
-  int4* sTile;   // [T] long class: {key pointer lo, hi, table offset (or -1-g), code << 6 | lanes}
+  // long class: one descriptor per 32-key tile as four int arrays of T4 =
+  // round4(T) entries (structure of arrays: one LDS.128 reads a field of 4
+  // tiles).  Count mode: sT0 = col index of the tile's first key, sT1 =
+  // valid lanes, sT2/sT3 = table (walk_long); support mode: key position
+  // lo/hi, chunk-local edge, valid lanes (walk_long_sup).
+  int *sT0, *sT1, *sT2, *sT3;
   int64_t* sB;   // long: key start in col; short: start - (chunk-relative first key)
   int64_t* sGB;  // group: row start of N+(v) - sGP (so col[sGB[g] + k] is insert k)
   int2* sInfo;   // [G] table {word offset, code}; offset -1 = huge
@@ -223,8 +228,12 @@ struct ChunkSmem {
 
 __device__ __forceinline__ ChunkSmem slot_view(unsigned char* region, int S, int G, int T) {
   ChunkSmem c;
-  c.sTile = reinterpret_cast<int4*>(region);
-  c.sB = reinterpret_cast<int64_t*>(c.sTile + T);
+  const int T4 = (T + 3) & ~3;
+  c.sT0 = reinterpret_cast<int*>(region);
+  c.sT1 = c.sT0 + T4;
+  c.sT2 = c.sT1 + T4;
+  c.sT3 = c.sT2 + T4;
+  c.sB = reinterpret_cast<int64_t*>(c.sT3 + T4);
   c.sGB = c.sB + S;
   c.sInfo = reinterpret_cast<int2*>(c.sGB + G);
   c.sA = reinterpret_cast<int*>(c.sInfo + G);
@@ -234,7 +243,7 @@ __device__ __forceinline__ ChunkSmem slot_view(unsigned char* region, int S, int
   // 16-B aligned start of the slots as an int offset from the aligned region
   // base, so every table access stays in the shared window (LDS/ATOMS)
   c.sHash = reinterpret_cast<int*>(region) +
-            ((4 * T + 2 * S + 2 * G + 2 * G + (S + 1) + 2 * S + (G + 1) + 3) & ~3);
+            ((4 * T4 + 2 * S + 2 * G + 2 * G + (S + 1) + 2 * S + (G + 1) + 3) & ~3);
   c.sE = nullptr;
   return c;
 }
@@ -299,35 +308,74 @@ __device__ __forceinline__ void warp_walk(const int* __restrict__ P, int S, int 
 // ------------------------------------------------------------------ consumers
 // LONG class: the warp owns tiles [t0, t1) of the chunk.  Each tile is 32
 // consecutive keys of one edge, described by one 16-B sTile entry the
-// producers wrote (key pointer, valid lanes, table), so kUnrollLong loads are
-// in flight per lane across edge boundaries with no per-edge bookkeeping;
-// padding lanes carry the never-matching sentinel and probe unpredicated.
+// producers wrote: {x = col index of the tile's first key (m < 2^32),
+// y = valid lanes (1..32), z/w = its table: w = 0 bitmap whose word for key k
+// is sHash[(k >> 5) + z]; w >= 2 hash of w slots at sHash[z]; w = -1 huge,
+// z = -1 - (chunk-local group)}.  kUnrollLong tiles are loaded per step
+// (kUnrollLong key loads in flight per lane across edge boundaries, no
+// per-edge bookkeeping).  Padding lanes re-load the tile's last valid key
+// (always a legal address and a legal table read) and their hit is masked,
+// so every lane probes unpredicated.
+template <bool kLinear, bool kHuge>
+__device__ __forceinline__ unsigned probe_tile(const ChunkSmem& c, int z, int w, int32_t key,
+                                               unsigned valid, const PlanView& pv, int64_t ga) {
+  if (w == 0) {
+    const unsigned word = (unsigned)c.sHash[(key >> 5) + z];
+    return __funnelshift_r(~word, 0u, (unsigned)key) & valid;  // bit key & 31 of ~word
+  }
+  if (!kHuge || w > 0) return table_probe<kLinear>(c.sHash + z, (uint32_t)w, key) & valid;
+  return valid ? huge_probe(pv, ga + (-1 - z), key) : 0u;
+}
+
+// Tiles [t0, t1), t0 a multiple of kUnrollLong (the consumer split keeps it
+// so) so that each field of a batch is read with aligned LDS.128s.  All of a
+// batch's address fields are read before its first key load is issued: with
+// descriptor reads and key loads interleaved, the compiler let them share a
+// scoreboard and a warp waited out one key load before issuing the next.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1,
                                               const PlanView& pv, int64_t ga) {
+  static_assert(kUnrollLong == 8, "batch = two int4 per descriptor field");
   unsigned cnt = 0;
   const int lane = threadIdx.x & 31;
-  for (int t = t0; t < t1; t += kUnrollLong) {
-    int32_t key[kUnrollLong];
-    int toff[kUnrollLong], code[kUnrollLong];
+  int t = t0;
+  for (; t + 8 <= t1; t += 8) {
+    int x[8], y[8], z[8], w[8];
+    int32_t key[8];
+    *reinterpret_cast<int4*>(x) = *reinterpret_cast<const int4*>(c.sT0 + t);
+    *reinterpret_cast<int4*>(x + 4) = *reinterpret_cast<const int4*>(c.sT0 + t + 4);
+    *reinterpret_cast<int4*>(y) = *reinterpret_cast<const int4*>(c.sT1 + t);
+    *reinterpret_cast<int4*>(y + 4) = *reinterpret_cast<const int4*>(c.sT1 + t + 4);
 #pragma unroll
-    for (int u = 0; u < kUnrollLong; ++u) {
-      // tiles past t1 reuse the last tile's (real) table with no lanes
-      const int4 d = c.sTile[min(t + u, t1 - 1)];
-      const int lanes = (t + u < t1) ? (d.w & 63) : 0;
-      const int64_t p = (int64_t)(((uint64_t)(uint32_t)d.y << 32) | (uint32_t)d.x);
-      toff[u] = d.z;
-      code[u] = d.w >> 6;
-      key[u] = lane < lanes ? __ldg(pv.col + p + lane) : -2;
+    for (int u = 0; u < 8; ++u)
+      key[u] = __ldg(pv.col + ((uint32_t)x[u] + (uint32_t)min(lane, y[u] - 1)));
+    *reinterpret_cast<int4*>(z) = *reinterpret_cast<const int4*>(c.sT2 + t);
+    *reinterpret_cast<int4*>(z + 4) = *reinterpret_cast<const int4*>(c.sT2 + t + 4);
+    *reinterpret_cast<int4*>(w) = *reinterpret_cast<const int4*>(c.sT3 + t);
+    *reinterpret_cast<int4*>(w + 4) = *reinterpret_cast<const int4*>(c.sT3 + t + 4);
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      cnt += probe_tile<kLinear, kHuge>(c, z[u], w[u], key[u], lane < y[u] ? 1u : 0u, pv, ga);
+  }
+  if (t < t1) {  // tail: tiles past t1 repeat the last tile with no valid lanes
+    int y[8], z[8], w[8];
+    int32_t key[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int tt = min(t + u, t1 - 1);
+      y[u] = c.sT1[tt];
+      key[u] = __ldg(pv.col + ((uint32_t)c.sT0[tt] + (uint32_t)min(lane, y[u] - 1)));
+      if (t + u >= t1) y[u] = 0;
     }
 #pragma unroll
-    for (int u = 0; u < kUnrollLong; ++u) {
-      if (kHuge && toff[u] < 0) {
-        if (key[u] >= 0) cnt += huge_probe(pv, ga + (-1 - toff[u]), key[u]);
-      } else {
-        cnt += any_probe<kLinear>(c.sHash + toff[u], code[u], key[u]);
-      }
+    for (int u = 0; u < 8; ++u) {
+      const int tt = min(t + u, t1 - 1);
+      z[u] = c.sT2[tt];
+      w[u] = c.sT3[tt];
     }
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      cnt += probe_tile<kLinear, kHuge>(c, z[u], w[u], key[u], lane < y[u] ? 1u : 0u, pv, ga);
   }
   return cnt;
 }
@@ -455,10 +503,10 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
     int sl[kUnrollSup];
 #pragma unroll
     for (int u = 0; u < kUnrollSup; ++u) {
-      const int4 d = c.sTile[min(t + u, t1 - 1)];
-      const int lanes = (t + u < t1) ? d.w : 0;
-      p[u] = (int64_t)(((uint64_t)(uint32_t)d.y << 32) | (uint32_t)d.x);
-      sl[u] = d.z;
+      const int tt = min(t + u, t1 - 1);
+      const int lanes = (t + u < t1) ? c.sT3[tt] : 0;
+      p[u] = (int64_t)(((uint64_t)(uint32_t)c.sT1[tt] << 32) | (uint32_t)c.sT0[tt]);
+      sl[u] = c.sT2[tt];
       key[u] = lane < lanes ? __ldg(pv.col + p[u] + lane) : -2;
     }
 #pragma unroll
@@ -600,9 +648,16 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         const int64_t p = st + ((int64_t)(t - ts) << 5);
         const int lanes = min(32, len - ((t - ts) << 5));
         // support mode: the tile names its edge (chunk-local) instead of its table
-        c.sTile[t] = kSup ? make_int4((int)(uint32_t)p, (int)(p >> 32), i, lanes)
-                          : make_int4((int)(uint32_t)p, (int)(p >> 32), toff,
-                                      (int)((unsigned)d.y << 6) | lanes);
+        c.sT0[t] = (int)(uint32_t)p;
+        if (kSup) {
+          c.sT1[t] = (int)(p >> 32);
+          c.sT2[t] = i;
+          c.sT3[t] = lanes;
+        } else {  // walk_long: bitmap w = 0, z = word base; hash w = slots; huge w = -1
+          c.sT1[t] = lanes;
+          c.sT2[t] = d.x < 0 ? toff : (d.y <= 0 ? d.x + d.y : d.x);
+          c.sT3[t] = d.x < 0 ? -1 : (d.y <= 0 ? 0 : d.y);
+        }
       }
     }
   }
@@ -739,7 +794,11 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
         const int NU = h.is_long ? h.T : c.sA[h.S];
         const int grab = h.is_long ? tu.grab_long : tu.grab_short;
         if (grab <= 0) {  // static split: a contiguous share per consumer warp
-          const int w0 = (int)((int64_t)NU * cw / n_cons), w1 = (int)((int64_t)NU * (cw + 1) / n_cons);
+          int w0 = (int)((int64_t)NU * cw / n_cons), w1 = (int)((int64_t)NU * (cw + 1) / n_cons);
+          if (h.is_long) {  // walk_long batches start at multiples of 8 tiles
+            w0 = min((w0 + 7) & ~7, NU);
+            w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
+          }
           acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
         } else {  // dynamic: grab `grab` units at a time from the slot's counter
           for (;;) {

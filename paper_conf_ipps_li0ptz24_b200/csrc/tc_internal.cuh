@@ -117,12 +117,13 @@ struct PlanView {
 // SMEM a chunk needs (bytes): per segment staging + per group descriptor +
 // hash slots.  Shared by the plan (sizing) and the kernel (layout).
 // Layout of one chunk slot of the count kernel (tc_count.cu slot_view), all
-// offsets from a 16-B aligned base: sTile int4[T] (long class: one descriptor
-// per 32-key tile) | sB int64[S] | sGB int64[G] | sInfo int2[G] | sA int32[S+1]
-// | sC int32[S] | sD int32[S] | sGP int32[G+1] | pad to 16 B | sHash int32[slots].
+// offsets from a 16-B aligned base: sT0..sT3 int32[round4(T)] each (long
+// class: one descriptor per 32-key tile) | sB int64[S] | sGB int64[G] | sInfo
+// int2[G] | sA int32[S+1] | sC int32[S] | sD int32[S] | sGP int32[G+1] | pad to
+// 16 B | sHash int32[slots].
 __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_t slots,
                                                     int64_t T) {
-  return 16 * T + 20 * S + 20 * G + 8 + 16 + 4 * slots;
+  return 16 * ((T + 3) & ~int64_t(3)) + 20 * S + 20 * G + 8 + 16 + 4 * slots;
 }
 
 // Count-kernel launch tuning (not part of the C-ABI; TC_SLOTS, TC_GRAB_LONG,
