@@ -86,8 +86,9 @@ typedef struct {
   int32_t table_factor; /* hash slots = next_pow2(table_factor * d+(v)), 2..16
                            (default 3, i.e. load <= 1/3)                            */
   int32_t long_min;     /* trimmed suffixes with >= long_min keys go to the
-                           warp-per-edge class, shorter ones to the flattened
-                           class (default 32; 1 = all long, 2^30 = all short)     */
+                           warp-per-edge tile class, shorter ones to the flattened
+                           class (default 32; values below 32 act as 32, since a
+                           tile holds 32 keys of its own edge; 2^30 = all short) */
   int32_t probe_mode;   /* 0 = two-choice (cuckoo) tables with linear-probing
                            fallback per chunk, 1 = linear probing only (default 0) */
   int32_t bitmap_factor; /* a head v whose window [min N+(v), max N+(v)] needs at most

@@ -642,7 +642,10 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   if (m > 0) {
     k_rowid<<<grid_for(n), TPB, 0, s>>>(row_ptr, n, rowid.get());
     TC_LAUNCH();
-    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m, opt.long_min, g->bits,
+    // a long-class tile always holds 32 keys of its own edge (walk_long shifts
+    // a partial last tile back onto the edge), so long_min < 32 acts as 32
+    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m,
+                                            std::max(opt.long_min, 32), g->bits,
                                             dead, skey.get(), sval.get(), stats.get());
     TC_LAUNCH();
   }

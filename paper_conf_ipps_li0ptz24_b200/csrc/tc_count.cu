@@ -328,54 +328,51 @@ __device__ __forceinline__ unsigned probe_tile(const ChunkSmem& c, int z, int w,
 }
 
 // Tiles [t0, t1), t0 a multiple of kUnrollLong (the consumer split keeps it
-// so) so that each field of a batch is read with aligned LDS.128s.  All of a
-// batch's address fields are read before its first key load is issued: with
-// descriptor reads and key loads interleaved, the compiler let them share a
-// scoreboard and a warp waited out one key load before issuing the next.
+// so) so that each field of a batch is read with aligned LDS.128s.  Every
+// lane of a tile loads a key of the tile's own edge (x + lane; a partial last
+// tile was shifted back, its first y lanes masked), so a key address needs
+// only the x field: a batch reads its eight x values, issues its eight key
+// loads, then reads the other fields while the loads are in flight.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1,
                                               const PlanView& pv, int64_t ga) {
   static_assert(kUnrollLong == 8, "batch = two int4 per descriptor field");
   unsigned cnt = 0;
   const int lane = threadIdx.x & 31;
+  const int32_t* colL = pv.col + lane;
   int t = t0;
   for (; t + 8 <= t1; t += 8) {
     int x[8], y[8], z[8], w[8];
     int32_t key[8];
     *reinterpret_cast<int4*>(x) = *reinterpret_cast<const int4*>(c.sT0 + t);
     *reinterpret_cast<int4*>(x + 4) = *reinterpret_cast<const int4*>(c.sT0 + t + 4);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) key[u] = __ldg(colL + (uint32_t)x[u]);
     *reinterpret_cast<int4*>(y) = *reinterpret_cast<const int4*>(c.sT1 + t);
     *reinterpret_cast<int4*>(y + 4) = *reinterpret_cast<const int4*>(c.sT1 + t + 4);
-#pragma unroll
-    for (int u = 0; u < 8; ++u)
-      key[u] = __ldg(pv.col + ((uint32_t)x[u] + (uint32_t)min(lane, y[u] - 1)));
     *reinterpret_cast<int4*>(z) = *reinterpret_cast<const int4*>(c.sT2 + t);
     *reinterpret_cast<int4*>(z + 4) = *reinterpret_cast<const int4*>(c.sT2 + t + 4);
     *reinterpret_cast<int4*>(w) = *reinterpret_cast<const int4*>(c.sT3 + t);
     *reinterpret_cast<int4*>(w + 4) = *reinterpret_cast<const int4*>(c.sT3 + t + 4);
 #pragma unroll
     for (int u = 0; u < 8; ++u)
-      cnt += probe_tile<kLinear, kHuge>(c, z[u], w[u], key[u], lane < y[u] ? 1u : 0u, pv, ga);
+      cnt += probe_tile<kLinear, kHuge>(c, z[u], w[u], key[u], lane >= y[u] ? 1u : 0u, pv, ga);
   }
-  if (t < t1) {  // tail: tiles past t1 repeat the last tile with no valid lanes
+  if (t < t1) {  // tail: tiles past t1 repeat the last tile with every lane masked
     int y[8], z[8], w[8];
     int32_t key[8];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const int tt = min(t + u, t1 - 1);
-      y[u] = c.sT1[tt];
-      key[u] = __ldg(pv.col + ((uint32_t)c.sT0[tt] + (uint32_t)min(lane, y[u] - 1)));
-      if (t + u >= t1) y[u] = 0;
-    }
+    for (int u = 0; u < 8; ++u) key[u] = __ldg(colL + (uint32_t)c.sT0[min(t + u, t1 - 1)]);
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const int tt = min(t + u, t1 - 1);
+      y[u] = t + u < t1 ? c.sT1[tt] : 32;
       z[u] = c.sT2[tt];
       w[u] = c.sT3[tt];
     }
 #pragma unroll
     for (int u = 0; u < 8; ++u)
-      cnt += probe_tile<kLinear, kHuge>(c, z[u], w[u], key[u], lane < y[u] ? 1u : 0u, pv, ga);
+      cnt += probe_tile<kLinear, kHuge>(c, z[u], w[u], key[u], lane >= y[u] ? 1u : 0u, pv, ga);
   }
   return cnt;
 }
@@ -648,13 +645,17 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         const int64_t p = st + ((int64_t)(t - ts) << 5);
         const int lanes = min(32, len - ((t - ts) << 5));
         // support mode: the tile names its edge (chunk-local) instead of its table
-        c.sT0[t] = (int)(uint32_t)p;
         if (kSup) {
+          c.sT0[t] = (int)(uint32_t)p;
           c.sT1[t] = (int)(p >> 32);
           c.sT2[t] = i;
           c.sT3[t] = lanes;
-        } else {  // walk_long: bitmap w = 0, z = word base; hash w = slots; huge w = -1
-          c.sT1[t] = lanes;
+        } else {
+          // walk_long: a partial last tile is shifted back to the edge's last 32
+          // keys (len >= 32 in the long class), its first 32 - lanes lanes
+          // masked; bitmap w = 0, z = word base; hash w = slots; huge w = -1
+          c.sT0[t] = (int)(uint32_t)(p - (32 - lanes));
+          c.sT1[t] = 32 - lanes;
           c.sT2[t] = d.x < 0 ? toff : (d.y <= 0 ? d.x + d.y : d.x);
           c.sT3[t] = d.x < 0 ? -1 : (d.y <= 0 ? 0 : d.y);
         }
