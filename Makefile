@@ -9,7 +9,7 @@ NVCC      ?= /usr/local/cuda/bin/nvcc
 CXX       ?= g++
 PKG       := paper_conf_ipps_li0ptz24_b200
 ARCH      := -gencode arch=compute_100a,code=sm_100a
-NVFLAGS   := -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
+NVFLAGS   := $(NVEXTRA) -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
              -Iinclude --expt-relaxed-constexpr -Xptxas -v
 CXXFLAGS  := -O3 -std=c++17 -fPIC -pthread
 

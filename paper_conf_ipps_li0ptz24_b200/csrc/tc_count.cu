@@ -40,7 +40,11 @@ namespace {
 
 constexpr int kMaxBlock = 1024;  // warp-specialised kernel (long class)
 constexpr int kFlatBlock = 512;  // flat kernel (short class), 3 CTAs per SM
-constexpr int kUnrollLong = 8;   // tiles in flight per consumer warp (long class)
+constexpr int kUnrollLong = 8;   // tail batch of the long class
+#ifndef TC_BATCH_LONG
+#define TC_BATCH_LONG 8
+#endif
+constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
 constexpr int kUnrollShort = 4;  // tiles in flight per consumer warp (short class)
 constexpr int kMaxKicks = 96;    // cuckoo displacement bound before the linear fallback
 constexpr int kMaxSlots = 4;     // chunk slots in SMEM (runtime count: Tuning::slots)
@@ -72,6 +76,14 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity, uint32_t
         "r"(parity)
         : "memory");
   }
+}
+// The two waits of the count kernel as separate functions, so profiles
+// attribute consumer (slot full) and producer (slot empty) waiting apart.
+__device__ __noinline__ void wait_full(uint64_t* b, uint32_t parity, uint32_t hint_ns) {
+  mbar_wait(b, parity, hint_ns);
+}
+__device__ __noinline__ void wait_empty(uint64_t* b, uint32_t parity, uint32_t hint_ns) {
+  mbar_wait(b, parity, hint_ns);
 }
 __device__ __forceinline__ void named_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
@@ -316,9 +328,13 @@ __device__ __forceinline__ void warp_walk(const int* __restrict__ P, int S, int 
 // per-edge bookkeeping).  Padding lanes re-load the tile's last valid key
 // (always a legal address and a legal table read) and their hit is masked,
 // so every lane probes unpredicated.
+// zw = (code << 6) | first valid lane (see produce): code 0 bitmap, >= 2 hash
+// slots, -1 huge; first valid lane 32 = none.
 template <bool kLinear, bool kHuge>
-__device__ __forceinline__ unsigned probe_tile(const ChunkSmem& c, int z, int w, int32_t key,
-                                               unsigned valid, const PlanView& pv, int64_t ga) {
+__device__ __forceinline__ unsigned probe_tile(const ChunkSmem& c, int z, int zw, int32_t key,
+                                               int lane, const PlanView& pv, int64_t ga) {
+  const unsigned valid = lane >= (zw & 63) ? 1u : 0u;
+  const int w = zw >> 6;
   if (w == 0) {
     const unsigned word = (unsigned)c.sHash[(key >> 5) + z];
     return __funnelshift_r(~word, 0u, (unsigned)key) & valid;  // bit key & 31 of ~word
@@ -327,52 +343,58 @@ __device__ __forceinline__ unsigned probe_tile(const ChunkSmem& c, int z, int w,
   return valid ? huge_probe(pv, ga + (-1 - z), key) : 0u;
 }
 
-// Tiles [t0, t1), t0 a multiple of kUnrollLong (the consumer split keeps it
-// so) so that each field of a batch is read with aligned LDS.128s.  Every
-// lane of a tile loads a key of the tile's own edge (x + lane; a partial last
-// tile was shifted back, its first y lanes masked), so a key address needs
-// only the x field: a batch reads its eight x values, issues its eight key
-// loads, then reads the other fields while the loads are in flight.
+// Tiles [t0, t1), t0 a multiple of 8 (the consumer split keeps it so): each
+// descriptor field of an 8-tile batch is two aligned LDS.128.  Every lane of a
+// tile loads a key of the tile's own edge (x + lane; a partial last tile was
+// shifted back and its first lanes are masked), so a key address needs only
+// the x field.  (Software-pipelining batch b+1's loads under batch b's probes
+// measured slower: 4-tile batches 66 ms, 8-tile batches spill, vs 62.5 ms.)
+template <int kB>
+__device__ __forceinline__ void load_batch(const ChunkSmem& c, const int32_t* colL, int t,
+                                           int32_t (&key)[kB]) {
+  int x[kB];
+#pragma unroll
+  for (int q = 0; q < kB; q += 4)
+    *reinterpret_cast<int4*>(x + q) = *reinterpret_cast<const int4*>(c.sT0 + t + q);
+#pragma unroll
+  for (int u = 0; u < kB; ++u) key[u] = __ldg(colL + (uint32_t)x[u]);
+}
+
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1,
                                               const PlanView& pv, int64_t ga) {
-  static_assert(kUnrollLong == 8, "batch = two int4 per descriptor field");
+  constexpr int kB = kBatchLong;
+  static_assert(kB % 4 == 0 && 8 % kB == 0, "batches of 4 or 8 tiles, 8-aligned splits");
   unsigned cnt = 0;
   const int lane = threadIdx.x & 31;
   const int32_t* colL = pv.col + lane;
   int t = t0;
-  for (; t + 8 <= t1; t += 8) {
-    int x[8], y[8], z[8], w[8];
-    int32_t key[8];
-    *reinterpret_cast<int4*>(x) = *reinterpret_cast<const int4*>(c.sT0 + t);
-    *reinterpret_cast<int4*>(x + 4) = *reinterpret_cast<const int4*>(c.sT0 + t + 4);
+  for (; t + kB <= t1; t += kB) {
+    int32_t key[kB];
+    load_batch<kB>(c, colL, t, key);
+    int z[kB], zw[kB];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) key[u] = __ldg(colL + (uint32_t)x[u]);
-    *reinterpret_cast<int4*>(y) = *reinterpret_cast<const int4*>(c.sT1 + t);
-    *reinterpret_cast<int4*>(y + 4) = *reinterpret_cast<const int4*>(c.sT1 + t + 4);
-    *reinterpret_cast<int4*>(z) = *reinterpret_cast<const int4*>(c.sT2 + t);
-    *reinterpret_cast<int4*>(z + 4) = *reinterpret_cast<const int4*>(c.sT2 + t + 4);
-    *reinterpret_cast<int4*>(w) = *reinterpret_cast<const int4*>(c.sT3 + t);
-    *reinterpret_cast<int4*>(w + 4) = *reinterpret_cast<const int4*>(c.sT3 + t + 4);
+    for (int q = 0; q < kB; q += 4) {
+      *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
+      *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
+    }
 #pragma unroll
-    for (int u = 0; u < 8; ++u)
-      cnt += probe_tile<kLinear, kHuge>(c, z[u], w[u], key[u], lane >= y[u] ? 1u : 0u, pv, ga);
+    for (int u = 0; u < kB; ++u)
+      cnt += probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
   }
   if (t < t1) {  // tail: tiles past t1 repeat the last tile with every lane masked
-    int y[8], z[8], w[8];
+    int z[8], zw[8];
     int32_t key[8];
 #pragma unroll
     for (int u = 0; u < 8; ++u) key[u] = __ldg(colL + (uint32_t)c.sT0[min(t + u, t1 - 1)]);
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const int tt = min(t + u, t1 - 1);
-      y[u] = t + u < t1 ? c.sT1[tt] : 32;
-      z[u] = c.sT2[tt];
-      w[u] = c.sT3[tt];
+      z[u] = c.sT1[tt];
+      zw[u] = c.sT2[tt] | (t + u < t1 ? 0 : 32);  // first valid lane 32: none
     }
 #pragma unroll
-    for (int u = 0; u < 8; ++u)
-      cnt += probe_tile<kLinear, kHuge>(c, z[u], w[u], key[u], lane >= y[u] ? 1u : 0u, pv, ga);
+    for (int u = 0; u < 8; ++u) cnt += probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
   }
   return cnt;
 }
@@ -653,11 +675,12 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         } else {
           // walk_long: a partial last tile is shifted back to the edge's last 32
           // keys (len >= 32 in the long class), its first 32 - lanes lanes
-          // masked; bitmap w = 0, z = word base; hash w = slots; huge w = -1
+          // masked.  sT1 = z, sT2 = (code << 5) | first valid lane, code:
+          // bitmap 0 (z = word base), hash = slots (z = offset), huge -1.
+          // (6-bit lane field: 32 = no valid lane)
           c.sT0[t] = (int)(uint32_t)(p - (32 - lanes));
-          c.sT1[t] = 32 - lanes;
-          c.sT2[t] = d.x < 0 ? toff : (d.y <= 0 ? d.x + d.y : d.x);
-          c.sT3[t] = d.x < 0 ? -1 : (d.y <= 0 ? 0 : d.y);
+          c.sT1[t] = d.x < 0 ? toff : (d.y <= 0 ? d.x + d.y : d.x);
+          c.sT2[t] = ((d.x < 0 ? -1 : (d.y <= 0 ? 0 : d.y)) * 64) | (32 - lanes);
         }
       }
     }
@@ -772,7 +795,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     for (int64_t k = 0;; ++k) {
       const int slot = (int)(k % nslots);
       const uint32_t j = (uint32_t)(k / nslots);  // fill number of this slot
-      if (j > 0) mbar_wait(&empty_bar[slot], (j - 1) & 1, hint);
+      if (j > 0) wait_empty(&empty_bar[slot], (j - 1) & 1, hint);
       const int64_t cix = c_begin + blockIdx.x + k * gridDim.x;
       if (cix >= c_end) {
         if (threadIdx.x == 0) hdr[slot].done = 1;
@@ -787,7 +810,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     const int cw = warp - n_prod;
     for (int64_t k = 0;; ++k) {
       const int slot = (int)(k % nslots);
-      mbar_wait(&full_bar[slot], (uint32_t)((k / nslots) & 1), hint);
+      wait_full(&full_bar[slot], (uint32_t)((k / nslots) & 1), hint);
       const SlotHdr h = hdr[slot];
       if (h.done) break;
       if (h.S > 0) {
