@@ -60,6 +60,9 @@ def parse():
     ap.add_argument("--opt", action="append", default=[],
                     help="plan option key=value (tc_options field), repeatable")
     ap.add_argument("--out", default=None, help="also write the JSON line here")
+    ap.add_argument("--variant", default=None, choices=["polak", "trust"],
+                    help="count with one of the paper's surveyed kernels (tc_count_variant, "
+                         "SURVEY.md §8(f) f3) instead of the grouped path; N = 1 only")
     ap.add_argument("--mode", default="count", choices=["count", "support"],
                     help="count: T (the headline); support: per-edge triangle counts "
                          "(tc_support, SURVEY.md §8(f) f1), N = 1 only")
@@ -364,8 +367,14 @@ def main():
     flush = torch.empty(a.flush_mb << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
 
+    if a.variant and world > 1:
+        raise SystemExit("--variant runs on one GPU")
+
     def step(ev_mid=None):
-        g.count_range(e0, e1, out=out)
+        if a.variant:
+            g.count_variant(a.variant, out=out)
+        else:
+            g.count_range(e0, e1, out=out)
         if ev_mid is not None:
             ev_mid.record(stream)
         if world > 1:
@@ -464,7 +473,8 @@ def main():
                    "m_live": int(info.m_live), "keys_total": int(info.keys_total),
                    "parallelism": f"edge-range x{world} (replicated CSR, 1 NCCL all_reduce)",
                    "l2": f"flushed by a {a.flush_mb} MiB write between timed steps; CSR "
-                         f"{(info.m * 4 + (info.n + 1) * 8) / 2**20:.0f} MiB"},
+                         f"{(info.m * 4 + (info.n + 1) * 8) / 2**20:.0f} MiB",
+                   "kernel": a.variant or "grouped (k_count + k_count_flat)"},
         "triangles": str(T), "parity_vs_oracle": parity,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                      "frac": achieved / hbm, "traffic": traffic,
@@ -473,7 +483,8 @@ def main():
                                   "(SURVEY.md §8(d)); x this rank's share for N>1",
                      "peak_source": peak_src},
         "e2e": e2e,
-        "gpu_launches": a.steps * g.launches_per_count,
+        "gpu_launches": a.steps * (g.launches_per_count if not a.variant else
+                                   (1 if a.variant == "polak" else 3)),
         "build_ms": {"canon": info.ms_canon, "sort_unique": info.ms_sort_unique,
                      "degree_rank": info.ms_degree_rank, "orient_csr": info.ms_orient_csr,
                      "plan": info.ms_plan, "total_events": info.ms_total,

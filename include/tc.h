@@ -191,6 +191,22 @@ TC_API tc_status tc_support(const tc_graph* g, void* stream, uint32_t* d_support
 TC_API tc_status tc_edge_list(const tc_graph* g, void* stream, int32_t* d_u, int32_t* d_v);
 
 /*
+ * T by one of the paper's surveyed kernels instead of
+ * the grouped path, on the same oriented CSR, for the paper's comparison
+ * on B200.  Writes T into device uint64 *d_count (no sync).
+ *   TC_VARIANT_POLAK : edge-centric, one thread per oriented edge, sequential
+ *                      merge of N+(u) and N+(v) (Fig. 3).
+ *   TC_VARIANT_TRUST : vertex-centric, N+(u) hashed, 2-hop neighbours as
+ *                      queries; d+(u) > 100 -> a 1024-thread block with 1024
+ *                      buckets, 2..100 -> a warp with 32 buckets.
+ * Errors: unknown variant or NULL pointer -> TC_ERR_INVALID_ARGUMENT.
+ */
+#define TC_VARIANT_POLAK 1
+#define TC_VARIANT_TRUST 2
+TC_API tc_status tc_count_variant(const tc_graph* g, int32_t variant, void* stream,
+                                  uint64_t* d_count);
+
+/*
  * Cost-balanced split of [0, m_live) into world_size contiguous ranges
  * (SURVEY.md §8(e)): h_bounds (host int64[world_size+1]) receives
  * 0 = b_0 <= b_1 <= ... <= b_P = m_live, aligned to work chunks.

@@ -33,7 +33,9 @@ EXPORTS = (
     "tc_set_allocator", "tc_build_csr", "tc_build_csr_host", "tc_replan", "tc_graph_info",
     "tc_count", "tc_count_async", "tc_count_range", "tc_partition", "tc_partition_prefix",
     "tc_free", "tc_last_error", "tc_version", "tc_support", "tc_edge_list",
+    "tc_count_variant",
 )
+VARIANTS = {"polak": 1, "trust": 2}  # tc_count_variant
 
 
 class TCError(RuntimeError):
@@ -102,6 +104,7 @@ def lib():
             "tc_partition_prefix": ([vp, i64, i32, vp], st),
             "tc_support": ([vp, vp, vp], st),
             "tc_edge_list": ([vp, vp, vp, vp], st),
+            "tc_count_variant": ([vp, i32, vp, vp], st),
             "tc_free": ([vp], None),
             "tc_last_error": ([], ctypes.c_char_p),
             "tc_version": ([], ctypes.c_char_p),
@@ -216,6 +219,16 @@ class Graph:
             out = torch.empty(1, dtype=torch.int64, device="cuda")
         _check(lib().tc_count_async(self._h, ctypes.c_void_p(_stream(stream)),
                                     ctypes.c_void_p(out.data_ptr())))
+        return out
+
+    def count_variant(self, variant: str, out=None, stream=None):
+        """T by the paper's Polak or TRUST kernel (tc_count_variant), stream-ordered
+        into a 1-element int64 CUDA tensor (u64 bit pattern)."""
+        torch = _torch()
+        if out is None:
+            out = torch.empty(1, dtype=torch.int64, device="cuda")
+        _check(lib().tc_count_variant(self._h, VARIANTS[variant], ctypes.c_void_p(_stream(stream)),
+                                      ctypes.c_void_p(out.data_ptr())))
         return out
 
     def count_range(self, e_begin: int, e_end: int, out=None, stream=None):

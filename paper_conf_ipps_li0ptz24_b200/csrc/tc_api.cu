@@ -339,6 +339,15 @@ tc_status tc_count_range(const tc_graph* g, int64_t e_begin, int64_t e_end, void
   });
 }
 
+tc_status tc_count_variant(const tc_graph* g, int32_t variant, void* stream, uint64_t* d_count) {
+  return guarded([&] {
+    require(g && d_count, "NULL argument");
+    require(variant == TC_VARIANT_POLAK || variant == TC_VARIANT_TRUST, "unknown variant");
+    tc::count_variant(g, variant, (cudaStream_t)stream,
+                      reinterpret_cast<unsigned long long*>(d_count));
+  });
+}
+
 tc_status tc_support(const tc_graph* g, void* stream, uint32_t* d_support) {
   return guarded([&] {
     require(g != nullptr, "graph is NULL");

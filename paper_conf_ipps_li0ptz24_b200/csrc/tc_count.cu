@@ -364,7 +364,7 @@ template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1,
                                               const PlanView& pv, int64_t ga) {
   constexpr int kB = kBatchLong;
-  static_assert(kB % 4 == 0 && 8 % kB == 0, "batches of 4 or 8 tiles, 8-aligned splits");
+  static_assert(kB % 4 == 0, "batches of whole int4 reads");
   unsigned cnt = 0;
   const int lane = threadIdx.x & 31;
   const int32_t* colL = pv.col + lane;
@@ -382,7 +382,7 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
     for (int u = 0; u < kB; ++u)
       cnt += probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
   }
-  if (t < t1) {  // tail: tiles past t1 repeat the last tile with every lane masked
+  for (; t < t1; t += 8) {  // tail: tiles past t1 repeat the last tile with every lane masked
     int z[8], zw[8];
     int32_t key[8];
 #pragma unroll

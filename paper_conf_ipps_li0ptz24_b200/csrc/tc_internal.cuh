@@ -182,4 +182,7 @@ int num_sms();
 void support_all(const tc_graph* g, cudaStream_t s, unsigned* d_sup);   // f1, tc_support
 void edge_ends(const tc_graph* g, cudaStream_t s, int32_t* d_u, int32_t* d_v);
 
+// tc_variants.cu (f3: the paper's Polak / TRUST kernels on this CSR)
+void count_variant(const tc_graph* g, int variant, cudaStream_t s, unsigned long long* d_out);
+
 }  // namespace tc

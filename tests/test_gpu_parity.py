@@ -96,6 +96,29 @@ def test_c5_lattice_full(tc):
     assert gpu_count(tc, src, dst, n) == oracle.triangles(src, dst, n)
 
 
+@pytest.mark.parametrize("cfg", ["C3", "C4"])
+def test_full_size_vs_stored_oracle(tc, cfg):
+    """C3 (260M edges) and C4 (1.57B edges, the 8-GPU config, here on one GPU)
+    at BASELINE size and in bench.py's launch configuration, against the
+    oracle's exact count stored by tests/golden/make_config_counts.py (the
+    input is regenerated and its checksum must match the stored one)."""
+    import json, os
+    stored = json.load(open(os.path.join(os.path.dirname(__file__), "golden",
+                                         "config_counts.json")))[f"{cfg}/seed1"]
+    src, dst, n = tcgen.CONFIGS[cfg].generate(1)
+    assert tcgen.checksum(src, dst) == stored["checksum"]
+    ds, dd = dev(src), dev(dst)
+    del src, dst
+    with tc.build_csr(ds, dd, n) as g:
+        del ds, dd
+        assert g.m == stored["m"] and g.n == stored["n_active"]
+        assert g.info.max_out_degree == stored["max_out_degree"]
+        assert g.count() == stored["triangles"]
+        b = g.partition(8)  # the 8-rank split of the multi-GPU run, emulated on one GPU
+        parts = [int(g.count_range(b[r], b[r + 1]).item()) for r in range(8)]
+        assert sum(parts) == stored["triangles"]
+
+
 def test_chung_lu_small(tc):
     src, dst, n = tcgen.chung_lu(200_000, 1_500_000, 3)
     assert gpu_count(tc, src, dst, n) == oracle.triangles(src, dst, n)
@@ -301,3 +324,42 @@ def test_huge_table_path_on_clique(tc):
     """K_1200 with huge_degree=100: most tables go through the global probe."""
     (src, dst, n), t = graphs.complete(1200)
     assert gpu_count(tc, src, dst, n, options=dict(huge_degree=100)) == t
+
+
+# ------------------------------------------------------------------ f3: the paper's Polak / TRUST kernels
+
+def variant_counts(tc, src, dst, n):
+    with tc.build_csr(dev(src), dev(dst), n) as g:
+        return {v: int(g.count_variant(v).item()) for v in ("polak", "trust")}, g.count()
+
+
+@pytest.mark.parametrize("name", ["K3", "K10", "K100", "W10", "F300", "K5,6,7,8", "Q10", "star1000"])
+def test_variants_closed_forms(tc, name):
+    (src, dst, n), t = graphs.closed_form_cases()[name]
+    got, grouped = variant_counts(tc, src, dst, n)
+    assert got == {"polak": t, "trust": t} and grouped == t
+
+
+@pytest.mark.parametrize("cfg_seed", [("C1", 1), ("C1", 2), ("rmat16", 3), ("skew15", 4), ("C5", 1)])
+def test_variants_vs_oracle(tc, cfg_seed):
+    name, seed = cfg_seed
+    if name == "rmat16":
+        src, dst, n = tcgen.rmat(16, 16, seed)
+    elif name == "skew15":
+        src, dst, n = tcgen.rmat(15, 24, seed, abc=(0.65, 0.15, 0.15))
+    else:
+        src, dst, n = tcgen.CONFIGS[name].generate(seed)
+    want = oracle.triangles(src, dst, n)
+    got, grouped = variant_counts(tc, src, dst, n)
+    assert got == {"polak": want, "trust": want} and grouped == want
+
+
+def test_trust_bucket_overflow_fallback(tc, monkeypatch):
+    """TC_TRUST_CAP=1 makes almost every TRUST bucket overflow, so both the warp
+    and the block kernels take the binary-search fallback; T must not change."""
+    src, dst, n = tcgen.rmat(14, 16, 5)
+    want = oracle.triangles(src, dst, n)
+    monkeypatch.setenv("TC_TRUST_CAP", "1")
+    with tc.build_csr(dev(src), dev(dst), n) as g:
+        assert g.info.max_out_degree > 100  # the block path runs too
+        assert int(g.count_variant("trust").item()) == want
