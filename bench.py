@@ -63,6 +63,8 @@ def parse():
     ap.add_argument("--variant", default=None, choices=["polak", "trust"],
                     help="count with one of the paper's surveyed kernels (tc_count_variant, "
                          "SURVEY.md §8(f) f3) instead of the grouped path; N = 1 only")
+    ap.add_argument("--no-sharded", action="store_true",
+                    help="skip the sharded-build measurement (tc_shard_*, SURVEY.md §8(f) f2)")
     ap.add_argument("--mode", default="count", choices=["count", "support"],
                     help="count: T (the headline); support: per-edge triangle counts "
                          "(tc_support, SURVEY.md §8(f) f1), N = 1 only")
@@ -411,6 +413,40 @@ def main():
     ms_per_step = total_ms / a.steps
     value = m / (ms_per_step / 1e3)
 
+    # ---------------------------------------------------------------- sharded build (f2)
+    # Every rank holds the contiguous 1/world slice of the raw pairs and the
+    # ranks build the identical replicated graph (tc_shard_* + NCCL
+    # all_reduce / all_to_all / broadcast); wall time after a device sync,
+    # max over ranks.  At N = 1 it runs the same steps without collectives.
+    lo, hi = rank * len(src) // world, (rank + 1) * len(src) // world
+    sharded = None
+    if not a.no_sharded:
+        s_dev = torch.from_numpy(src[lo:hi]).to(dev)
+        d_dev = torch.from_numpy(dst[lo:hi]).to(dev)
+        g3 = tc.build_csr_sharded(s_dev, d_dev, n, options=opts or None)  # warm
+        g3.close()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        phases = {}
+        t3 = time.perf_counter()
+        g3 = tc.build_csr_sharded(s_dev, d_dev, n, options=opts or None, timings=phases)
+        torch.cuda.synchronize()
+        sh_ms = (time.perf_counter() - t3) * 1e3
+        same = int(g3.m == m and g3.m_live == info.m_live and g3.info.b_itc == info.b_itc)
+        g3.close()
+        del s_dev, d_dev
+        x = torch.tensor([sh_ms, float(1 - same)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(x, op=dist.ReduceOp.MAX)
+        sharded = {"wall_ms": float(x[0]), "same_graph_as_full_build": bool(x[1] == 0),
+                   "phases_ms_rank0": {k: round(v, 3) for k, v in phases.items()},
+                   "pairs_per_rank": int(hi - lo),
+                   "what": "build_csr_sharded: tc_shard_canon, key-range all_to_all, "
+                           "tc_shard_unique + degree all_reduce, tc_rank_vertices, tc_shard_orient, "
+                           "row-range all_to_all + tc_sort_keys, ordered all-gather, "
+                           "tc_build_from_oriented (max over ranks)"}
+
     # ---------------------------------------------------------------- e2e (public API, host data)
     e2e = None
     if not a.no_e2e:
@@ -426,7 +462,12 @@ def main():
             x0 = torch.cuda.Event(enable_timing=True)
             x1 = torch.cuda.Event(enable_timing=True)
             x0.record(stream)
-            g2 = tc.build_csr_host(ps, pd, n, options=opts or None)
+            if world > 1:  # each rank copies and sorts only its slice (f2)
+                g2 = tc.build_csr_sharded(ps[lo:hi].to(dev, non_blocking=True),
+                                          pd[lo:hi].to(dev, non_blocking=True), n,
+                                          options=opts or None)
+            else:
+                g2 = tc.build_csr_host(ps, pd, n, options=opts or None)
             b = g2.partition(world)
             o2 = g2.count_range(b[rank], b[rank + 1])
             if world > 1:
@@ -444,10 +485,11 @@ def main():
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
         e2e_ms = float(et[0]) / max(1, len(ts))
         e2e = {"value": m / (e2e_ms / 1e3), "unit": UNIT, "ms_per_step": e2e_ms,
-               "h2d_bytes_per_step": int(src.nbytes + dst.nbytes),
+               "h2d_bytes_per_step": int(src.nbytes + dst.nbytes) * (hi - lo) // max(1, len(src)),
                "d2h_bytes_per_step": 8 + 8 * (n_chunks + 1) + 96,
-               "what": "tc_build_csr_host (H2D of the raw pinned edge list + a1..a6) + "
-                       "tc_count_range + all_reduce + 8-B D2H of T"}
+               "what": ("tc_build_csr_host (H2D of the raw pinned edge list + a1..a6)" if world == 1
+                        else "H2D of this rank's 1/N pinned slice + build_csr_sharded (f2)")
+                       + " + tc_count_range + all_reduce + 8-B D2H of T"}
 
     if rank != 0:
         if world > 1:
@@ -488,7 +530,7 @@ def main():
         "build_ms": {"canon": info.ms_canon, "sort_unique": info.ms_sort_unique,
                      "degree_rank": info.ms_degree_rank, "orient_csr": info.ms_orient_csr,
                      "plan": info.ms_plan, "total_events": info.ms_total,
-                     "wall": build_wall_ms},
+                     "wall": build_wall_ms, "sharded": sharded},
         "plan": {"n_chunks": int(info.n_chunks), "grid": int(info.count_grid),
                  "block": int(info.count_block), "smem_bytes": int(info.smem_bytes),
                  "groups": int(info.n_groups)},

@@ -222,6 +222,133 @@ TC_API tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_
 TC_API tc_status tc_partition_prefix(const int64_t* h_prefix, int64_t n_units, int32_t world_size,
                               int64_t* h_bounds);
 
+/*
+ * ------------------------------------------------------------------------
+ * SHARDED preprocessing.  The same a1..a6 pipeline
+ * split into stateless steps so that P ranks, each holding 1/P of the raw
+ * pairs, build the identical replicated graph while the heavy sorts run on
+ * 1/P of the keys each.  The exchange steps between them are collectives of
+ * the caller (torch.distributed over NCCL; paper_conf_ipps_li0ptz24_b200.
+ * sharded.build_csr_sharded drives them):
+ *
+ *   tc_shard_canon      a1 + a2 on the local pairs -> sorted unique keys
+ *   tc_shard_histogram  per-bucket key counts (top bits)   -> all_reduce
+ *   tc_shard_cuts       host: bucket cuts with near-equal key counts
+ *   tc_shard_bounds     positions of the cuts in the local sorted keys
+ *                                                            -> all_to_all
+ *   tc_shard_unique     a2 (global dedup: equal keys meet on one rank) + a3
+ *                       partial degrees                      -> all_reduce
+ *   tc_rank_vertices    a4 (replicated: same degrees -> same ranking)
+ *   tc_shard_orient     a5 relabel + orient + local sort
+ *   (histogram / cuts / bounds again on the oriented keys)  -> all_to_all
+ *   tc_sort_keys        local sort of the received row range
+ *                       (rank r's slice precedes rank r+1's) -> all-gather
+ *   tc_build_from_oriented  CSR + plan (a5, a6) from all m sorted keys
+ *
+ * KEY FORMAT: a key over a vertex bound n is (a << b) | c with a, c in
+ * [0, n) and b = tc_key_bits(n) = max(1, ceil(log2 n)); canonical keys have
+ * a < c (original ids), oriented keys a = rank u < c = rank v.
+ * Keys are uint64 in device memory, caller-owned.  None of these calls keeps
+ * state between calls; scratch is stream-ordered and freed before return.
+ * ------------------------------------------------------------------------
+ */
+
+/* b = bits of one vertex field for a vertex bound n (n >= 0). */
+TC_API int32_t tc_key_bits(int64_t n);
+
+/*
+ * a1 + a2 on one shard: canonical keys of the valid non-loop pairs of
+ * (d_src, d_dst) (device int32[num_edges], caller-owned, unmodified), sorted
+ * ascending and unique, into d_keys (device uint64, capacity >= num_edges;
+ * may not alias the inputs).  *h_count = number written.  num_vertices >= 0
+ * is REQUIRED (all ranks must agree on it).  Errors: id < 0 or >=
+ * num_vertices -> TC_ERR_INVALID_ARGUMENT.  Synchronises.
+ */
+TC_API tc_status tc_shard_canon(const int32_t* d_src, const int32_t* d_dst, int64_t num_edges,
+                                int64_t num_vertices, void* stream, uint64_t* d_keys,
+                                int64_t* h_count);
+
+/*
+ * Key counts per bucket of the top `hist_bits` bits of the 2*tc_key_bits(n)
+ * bit key space: d_hist[b] (device int64[2^hist_bits], overwritten) = number
+ * of the `count` sorted keys whose bucket is b.  1 <= hist_bits <=
+ * min(24, 2*tc_key_bits(n)).  Stream-ordered, no sync.
+ */
+TC_API tc_status tc_shard_histogram(const uint64_t* d_keys, int64_t count, int64_t n,
+                                    int32_t hist_bits, void* stream, int64_t* d_hist);
+
+/*
+ * Host only: cut the buckets [0, n_buckets) into world_size contiguous
+ * ranges of near-equal total count (h_hist: host int64[n_buckets], the
+ * GLOBAL histogram).  h_cuts (host int64[world_size+1]) receives 0 = c_0 <=
+ * ... <= c_P = n_buckets; rank r owns buckets [c_r, c_{r+1}).
+ */
+TC_API tc_status tc_shard_cuts(const int64_t* h_hist, int64_t n_buckets, int32_t world_size,
+                               int64_t* h_cuts);
+
+/*
+ * Positions of the bucket cuts in `count` sorted keys: h_bounds (host
+ * int64[world_size+1]) receives p_r = first key whose bucket >= c_r
+ * (p_0 = 0, p_P = count), so keys [p_r, p_{r+1}) go to rank r.  Synchronises.
+ */
+TC_API tc_status tc_shard_bounds(const uint64_t* d_keys, int64_t count, int64_t n,
+                                 int32_t hist_bits, const int64_t* h_cuts, int32_t world_size,
+                                 void* stream, int64_t* h_bounds);
+
+/*
+ * a2 + a3 after the first exchange: sort d_keys[0, count) (canonical keys,
+ * any order, device uint64, in place), drop duplicates (*h_count = unique
+ * count, compacted to the front), and ADD each unique key's two endpoints to
+ * d_degree (device int32[n], caller-zeroed; the all_reduce of the ranks'
+ * arrays is the undirected degree).  Synchronises.
+ */
+TC_API tc_status tc_shard_unique(uint64_t* d_keys, int64_t count, int64_t n, void* stream,
+                                 int64_t* h_count, int32_t* d_degree);
+
+/*
+ * a3 alone: ADD each of `count` keys' two endpoints to d_degree (device
+ * int32[n], caller-zeroed).  For a single rank, whose tc_shard_canon output
+ * is already globally sorted and unique.  Stream-ordered.
+ */
+TC_API tc_status tc_shard_degree(const uint64_t* d_keys, int64_t count, int64_t n, void* stream,
+                                 int32_t* d_degree);
+
+/*
+ * a4: rank vertices by (degree ascending, id ascending), dropping
+ * degree-0 vertices unless TC_KEEP_ISOLATED.  d_degree: device int32[n]
+ * (global degrees).  Writes d_rank[v] (device int32[n]) for every kept v and
+ * d_perm[r] = v (device int32, capacity n) for r < *h_n_active.  Identical
+ * inputs give identical outputs on every rank.  Synchronises.
+ */
+TC_API tc_status tc_rank_vertices(const int32_t* d_degree, int64_t n, uint32_t flags,
+                                  void* stream, int32_t* d_rank, int32_t* d_perm,
+                                  int64_t* h_n_active);
+
+/*
+ * a5 (first half): relabel canonical keys (over n) to ranks and orient low
+ * -> high rank: d_okeys[i] (device uint64[count], caller-owned, may
+ * not alias d_keys) = (min(ra, rc) << tc_key_bits(n_active)) | max(ra, rc),
+ * sorted ascending.  Stream-ordered.
+ */
+TC_API tc_status tc_shard_orient(const uint64_t* d_keys, int64_t count, int64_t n,
+                                 const int32_t* d_rank, int64_t n_active, void* stream,
+                                 uint64_t* d_okeys);
+
+/* Sort count keys over vertex bound n (device uint64, in place).  Stream-ordered. */
+TC_API tc_status tc_sort_keys(uint64_t* d_keys, int64_t count, int64_t n, void* stream);
+
+/*
+ * a5 (second half) + a6: a graph from ALL m oriented keys, globally sorted
+ * and unique (device uint64[m] over n_active, caller-owned, unmodified), the
+ * ranking's d_perm (device int32[n_active]; copied) and the original vertex
+ * bound n_input.  Equal to what tc_build_csr builds from the union of the
+ * shards (tests compare the CSR byte for byte).  Synchronises.
+ */
+TC_API tc_status tc_build_from_oriented(const uint64_t* d_okeys, int64_t m,
+                                        const int32_t* d_perm, int64_t n_active,
+                                        int64_t n_input, const tc_options* opts, void* stream,
+                                        tc_graph** out);
+
 /* Release a graph (NULL is a no-op).  Stream-ordered frees on the build stream. */
 TC_API void tc_free(tc_graph* g);
 

@@ -33,7 +33,9 @@ EXPORTS = (
     "tc_set_allocator", "tc_build_csr", "tc_build_csr_host", "tc_replan", "tc_graph_info",
     "tc_count", "tc_count_async", "tc_count_range", "tc_partition", "tc_partition_prefix",
     "tc_free", "tc_last_error", "tc_version", "tc_support", "tc_edge_list",
-    "tc_count_variant",
+    "tc_count_variant", "tc_key_bits", "tc_shard_canon", "tc_shard_histogram", "tc_shard_cuts",
+    "tc_shard_bounds", "tc_shard_unique", "tc_shard_degree", "tc_rank_vertices", "tc_shard_orient", "tc_sort_keys",
+    "tc_build_from_oriented",
 )
 VARIANTS = {"polak": 1, "trust": 2}  # tc_count_variant
 
@@ -105,6 +107,17 @@ def lib():
             "tc_support": ([vp, vp, vp], st),
             "tc_edge_list": ([vp, vp, vp, vp], st),
             "tc_count_variant": ([vp, i32, vp, vp], st),
+            "tc_key_bits": ([i64], i32),
+            "tc_shard_canon": ([vp, vp, i64, i64, vp, vp, vp], st),
+            "tc_shard_histogram": ([vp, i64, i64, i32, vp, vp], st),
+            "tc_shard_cuts": ([vp, i64, i32, vp], st),
+            "tc_shard_bounds": ([vp, i64, i64, i32, vp, i32, vp, vp], st),
+            "tc_shard_unique": ([vp, i64, i64, vp, vp, vp], st),
+            "tc_shard_degree": ([vp, i64, i64, vp, vp], st),
+            "tc_rank_vertices": ([vp, i64, u32, vp, vp, vp, vp], st),
+            "tc_shard_orient": ([vp, i64, i64, vp, i64, vp, vp], st),
+            "tc_sort_keys": ([vp, i64, i64, vp], st),
+            "tc_build_from_oriented": ([vp, i64, vp, i64, i64, vp, vp, ctypes.POINTER(vp)], st),
             "tc_free": ([vp], None),
             "tc_last_error": ([], ctypes.c_char_p),
             "tc_version": ([], ctypes.c_char_p),
@@ -355,6 +368,8 @@ def count_partitioned(graph, group=None, stream=None) -> int:
     return int(partial.item()) & (2**64 - 1)
 
 
-__all__ = ["Graph", "Options", "GraphInfo", "build_csr", "build_csr_host", "count_partitioned",
+from .sharded import build_csr_sharded, shard_cuts  # noqa: E402  (f2)
+
+__all__ = ["build_csr_sharded", "shard_cuts", "Graph", "Options", "GraphInfo", "build_csr", "build_csr_host", "count_partitioned",
            "partition_prefix", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
            "EXPORTS", "LIB_PATH"]

@@ -5,6 +5,7 @@
 #include <cstdio>
 #include <cstring>
 #include <new>
+#include <vector>
 
 #include "tc_internal.cuh"
 
@@ -398,6 +399,141 @@ tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds)
       h_bounds[r] = (r == world_size) ? P.S : P.h_chunk_seg[c];
     }
   });
+}
+
+// ---------------------------------------------------------------- f2 sharded build
+int32_t tc_key_bits(int64_t n) { return tc::key_bits(n < 0 ? 0 : n); }
+
+tc_status tc_shard_canon(const int32_t* d_src, const int32_t* d_dst, int64_t num_edges,
+                         int64_t num_vertices, void* stream, uint64_t* d_keys, int64_t* h_count) {
+  return guarded([&] {
+    require(h_count != nullptr, "h_count is NULL");
+    require(num_edges >= 0, "num_edges < 0");
+    require(num_edges == 0 || (d_src && d_dst && d_keys), "NULL device pointer");
+    require(num_vertices >= 0 && num_vertices <= 0x7fffffffLL,
+            "num_vertices must be in [0, 2^31-1] for a sharded build");
+    cudaStream_t s = (cudaStream_t)stream;
+    tc::reserve_pool((size_t)num_edges * 16, s);
+    *h_count = tc::shard_canon(d_src, d_dst, num_edges, num_vertices, s, d_keys);
+  });
+}
+
+tc_status tc_shard_histogram(const uint64_t* d_keys, int64_t count, int64_t n, int32_t hist_bits,
+                             void* stream, int64_t* d_hist) {
+  return guarded([&] {
+    require(count >= 0 && n >= 0, "count/n < 0");
+    require(d_hist && (count == 0 || d_keys), "NULL device pointer");
+    require(hist_bits >= 1 && hist_bits <= 24 && hist_bits <= 2 * tc::key_bits(n),
+            "hist_bits must be in [1, min(24, 2*tc_key_bits(n))]");
+    tc::shard_histogram(d_keys, count, n, hist_bits, (cudaStream_t)stream, d_hist);
+  });
+}
+
+tc_status tc_shard_cuts(const int64_t* h_hist, int64_t n_buckets, int32_t world_size,
+                        int64_t* h_cuts) {
+  return guarded([&] {
+    require(h_hist && h_cuts, "NULL argument");
+    require(n_buckets >= 1, "n_buckets < 1");
+    require(world_size >= 1, "world_size < 1");
+    std::vector<int64_t> prefix(n_buckets + 1, 0);
+    for (int64_t b = 0; b < n_buckets; ++b) {
+      require(h_hist[b] >= 0, "negative bucket count");
+      prefix[b + 1] = prefix[b] + h_hist[b];
+    }
+    tc_status st = tc_partition_prefix(prefix.data(), n_buckets, world_size, h_cuts);
+    if (st != TC_OK) tc::fail(st, t_last_error);
+  });
+}
+
+tc_status tc_shard_bounds(const uint64_t* d_keys, int64_t count, int64_t n, int32_t hist_bits,
+                          const int64_t* h_cuts, int32_t world_size, void* stream,
+                          int64_t* h_bounds) {
+  return guarded([&] {
+    require(h_cuts && h_bounds && (count == 0 || d_keys), "NULL argument");
+    require(count >= 0 && n >= 0, "count/n < 0");
+    require(world_size >= 1, "world_size < 1");
+    require(hist_bits >= 1 && hist_bits <= 24 && hist_bits <= 2 * tc::key_bits(n),
+            "hist_bits must be in [1, min(24, 2*tc_key_bits(n))]");
+    for (int32_t r = 0; r < world_size; ++r)
+      require(h_cuts[r] <= h_cuts[r + 1], "cuts must be non-decreasing");
+    tc::shard_bounds(d_keys, count, n, hist_bits, h_cuts, world_size, (cudaStream_t)stream,
+                     h_bounds);
+  });
+}
+
+tc_status tc_shard_unique(uint64_t* d_keys, int64_t count, int64_t n, void* stream,
+                          int64_t* h_count, int32_t* d_degree) {
+  return guarded([&] {
+    require(h_count != nullptr, "h_count is NULL");
+    require(count >= 0 && n >= 0, "count/n < 0");
+    require(count == 0 || (d_keys && d_degree), "NULL device pointer");
+    *h_count = tc::shard_unique(d_keys, count, n, (cudaStream_t)stream, d_degree);
+  });
+}
+
+tc_status tc_shard_degree(const uint64_t* d_keys, int64_t count, int64_t n, void* stream,
+                          int32_t* d_degree) {
+  return guarded([&] {
+    require(count >= 0 && n >= 0, "count/n < 0");
+    require(count == 0 || (d_keys && d_degree), "NULL device pointer");
+    tc::shard_degree(d_keys, count, n, (cudaStream_t)stream, d_degree);
+  });
+}
+
+tc_status tc_rank_vertices(const int32_t* d_degree, int64_t n, uint32_t flags, void* stream,
+                           int32_t* d_rank, int32_t* d_perm, int64_t* h_n_active) {
+  return guarded([&] {
+    require(h_n_active != nullptr, "h_n_active is NULL");
+    require(n >= 0 && n <= 0x7fffffffLL, "n must be in [0, 2^31-1]");
+    require(n == 0 || (d_degree && d_rank && d_perm), "NULL device pointer");
+    require((flags & ~TC_KEEP_ISOLATED) == 0, "unknown flag bits");
+    *h_n_active = tc::shard_rank(d_degree, n, flags, (cudaStream_t)stream, d_rank, d_perm);
+  });
+}
+
+tc_status tc_shard_orient(const uint64_t* d_keys, int64_t count, int64_t n, const int32_t* d_rank,
+                          int64_t n_active, void* stream, uint64_t* d_okeys) {
+  return guarded([&] {
+    require(count >= 0 && n >= 0 && n_active >= 0 && n_active <= n, "bad sizes");
+    require(count == 0 || (d_keys && d_rank && d_okeys), "NULL device pointer");
+    require(count == 0 || d_keys != d_okeys, "d_okeys may not alias d_keys");
+    tc::shard_orient(d_keys, count, n, d_rank, n_active, (cudaStream_t)stream, d_okeys);
+  });
+}
+
+tc_status tc_sort_keys(uint64_t* d_keys, int64_t count, int64_t n, void* stream) {
+  return guarded([&] {
+    require(count >= 0 && n >= 0, "count/n < 0");
+    require(count == 0 || d_keys, "NULL device pointer");
+    tc::sort_keys(d_keys, count, n, (cudaStream_t)stream);
+  });
+}
+
+tc_status tc_build_from_oriented(const uint64_t* d_okeys, int64_t m, const int32_t* d_perm,
+                                 int64_t n_active, int64_t n_input, const tc_options* opts,
+                                 void* stream, tc_graph** out) {
+  if (out) *out = nullptr;
+  tc_graph* g = nullptr;
+  tc_status st = guarded([&] {
+    require(out != nullptr, "out is NULL");
+    require(m >= 0 && n_active >= 0 && n_input >= n_active && n_input <= 0x7fffffffLL, "bad sizes");
+    require(m == 0 || d_okeys, "d_okeys is NULL");
+    require(n_active == 0 || d_perm, "d_perm is NULL");
+    const tc::Options opt = tc::resolve_options(opts);
+    cudaStream_t s = (cudaStream_t)stream;
+    tc::reserve_pool((size_t)m * 40, s);
+    g = new tc_graph();
+    tc::build_from_oriented(d_okeys, m, d_perm, n_active, n_input, opt, s, g);
+  });
+  if (st != TC_OK) {
+    if (g) {
+      cudaStreamSynchronize((cudaStream_t)stream);
+      delete g;
+    }
+    return st;
+  }
+  *out = g;
+  return TC_OK;
 }
 
 void tc_free(tc_graph* g) {

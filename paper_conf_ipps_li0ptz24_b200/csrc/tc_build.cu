@@ -428,6 +428,37 @@ __global__ void k_split(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
   }
 }
 
+// ------------------------------------------------------------------ f2
+// Sharded preprocessing: range split of sorted keys.
+__device__ __forceinline__ int64_t lower_bound_u64(const uint64_t* __restrict__ a, int64_t n,
+                                                   uint64_t x) {
+  int64_t lo = 0, hi = n;
+  while (lo < hi) {
+    int64_t mid = (lo + hi) >> 1;
+    if (a[mid] < x) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+// hist[b] = #keys with key >> shift == b, by two binary searches per bucket
+// (the keys are sorted: no atomics, deterministic).
+__global__ void k_key_hist(const uint64_t* __restrict__ keys, int64_t cnt, int shift, int64_t nb,
+                           int64_t* __restrict__ hist) {
+  for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nb;
+       b += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t lo = lower_bound_u64(keys, cnt, (uint64_t)b << shift);
+    const int64_t hi = b + 1 < nb ? lower_bound_u64(keys, cnt, (uint64_t)(b + 1) << shift) : cnt;
+    hist[b] = hi - lo;
+  }
+}
+
+// pos[r] = first key whose bucket >= cut[r] (cut[r] == nb -> cnt).
+__global__ void k_key_bounds(const uint64_t* __restrict__ keys, int64_t cnt, int shift, int64_t nb,
+                             const int64_t* __restrict__ cut, int np, int64_t* __restrict__ pos) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r < np) pos[r] = cut[r] >= nb ? cnt : lower_bound_u64(keys, cnt, (uint64_t)cut[r] << shift);
+}
+
 __global__ void k_set_i64(int64_t* p, int64_t v) { *p = v; }
 
 // exclusive prefix of `in` (length n) into out[0..n] (out[0] = 0, out[n] = total)
@@ -457,6 +488,98 @@ struct Timer {
   }
 };
 
+// a1 + a2: canonical keys of the valid non-loop pairs, radix sorted on
+// 2*bits(n) bits, unique.  ka/kb: capacity max(m_gen, 1) each; returns the
+// one holding the *m_out unique keys (the SENT key of loops is dropped).
+uint64_t* canon_unique(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
+                       cudaStream_t s, uint64_t* ka, uint64_t* kb, int64_t* m_out, Timer* tm) {
+  const int bits = bits_for(std::max<int64_t>(n, 2));
+  const uint64_t sent = (uint64_t(1) << (2 * bits)) - 1;  // never a valid (lo < hi) key
+  DevBuf<int> err(1, s);
+  DevBuf<int64_t> nsel(1, s);
+  DevBuf<UniqTail> tail(1, s);
+  TC_CUDA(cudaMemsetAsync(err.get(), 0, sizeof(int), s));
+  TC_CUDA(cudaMemsetAsync(nsel.get(), 0, sizeof(int64_t), s));
+  if (m_gen > 0) {
+    k_canon<<<grid_for(m_gen), TPB, 0, s>>>(d_src, d_dst, m_gen, n, bits, sent, ka, err.get());
+    TC_LAUNCH();
+  }
+  if (tm) tm->mark();
+  uint64_t* ukey = ka;
+  if (m_gen > 0) {
+    cub::DoubleBuffer<uint64_t> db(ka, kb);
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceRadixSort::SortKeys(t, b, db, m_gen, 0, 2 * bits, s);
+    });
+    uint64_t* sorted = db.Current();
+    uint64_t* other = sorted == ka ? kb : ka;
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceSelect::Unique(t, b, sorted, other, nsel.get(), m_gen, s);
+    });
+    ukey = other;
+  }
+  k_uniq_tail<<<1, 1, 0, s>>>(err.get(), nsel.get(), ukey, tail.get());
+  TC_LAUNCH();
+  UniqTail ut = d2h(tail.get(), s);
+  if (ut.err) fail(TC_ERR_INVALID_ARGUMENT, "vertex id < 0 or >= num_vertices in the edge list");
+  *m_out = ut.nsel - ((ut.nsel > 0 && ut.last == sent) ? 1 : 0);
+  return ukey;
+}
+
+// a4: rank by (deg, id) ascending, isolated vertices last (dropped unless
+// keep).  rank[v] for kept v; perm = perm_at(n_act) receives rank -> v.
+template <class PermAt>
+int64_t rank_vertices(const int32_t* deg, int64_t n, int keep, cudaStream_t s, int32_t* rank,
+                      PermAt perm_at) {
+  if (n <= 0) {
+    perm_at(0);
+    return 0;
+  }
+  const int bits = bits_for(std::max<int64_t>(n, 2));
+  const uint64_t sentv = (uint64_t(1) << (2 * bits + 1)) - 1;
+  DevBuf<uint64_t> va(n, s), vb(n, s);
+  DevBuf<unsigned long long> nact(1, s);
+  TC_CUDA(cudaMemsetAsync(nact.get(), 0, sizeof(unsigned long long), s));
+  k_vkey<<<grid_for(n), TPB, 0, s>>>(deg, n, bits, keep, sentv, va.get(), nact.get());
+  TC_LAUNCH();
+  cub::DoubleBuffer<uint64_t> db(va.get(), vb.get());
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceRadixSort::SortKeys(t, b, db, n, 0, 2 * bits + 1, s);
+  });
+  const int64_t n_act = (int64_t)d2h(nact.get(), s);
+  int32_t* perm = perm_at(n_act);
+  if (n_act > 0) {
+    k_perm<<<grid_for(n_act), TPB, 0, s>>>(db.Current(), n_act, bits, perm, rank);
+    TC_LAUNCH();
+  }
+  return n_act;
+}
+
+// a5 (second half): CSR of m sorted unique oriented keys over n_act rows.
+void csr_from_sorted(const uint64_t* okey, int64_t m, int64_t n_act, cudaStream_t s,
+                     tc_graph* g) {
+  const int bits2 = bits_for(std::max<int64_t>(n_act, 2));
+  g->bits = bits2;
+  g->m = m;
+  g->n = n_act;
+  g->row_ptr = DevBuf<int64_t>(n_act + 1, s, true);
+  g->col = DevBuf<int32_t>(std::max<int64_t>(m, 1), s, true);
+  if (m > 0) {
+    k_csr<<<grid_for(m), TPB, 0, s>>>(okey, m, n_act, bits2, g->col.get(), g->row_ptr.get());
+    TC_LAUNCH();
+  } else {
+    k_fill_i64<<<grid_for(n_act + 1), TPB, 0, s>>>(g->row_ptr.get(), n_act + 1, 0);
+    TC_LAUNCH();
+  }
+  DevBuf<unsigned long long> mx(1, s);
+  TC_CUDA(cudaMemsetAsync(mx.get(), 0, sizeof(unsigned long long), s));
+  if (n_act > 0) {
+    k_max_outdeg<<<grid_for(n_act), TPB, 0, s>>>(g->row_ptr.get(), n_act, mx.get());
+    TC_LAUNCH();
+  }
+  g->max_out = (int64_t)d2h(mx.get(), s);
+}
+
 }  // namespace
 
 // ------------------------------------------------------------------ a1..a5
@@ -484,40 +607,11 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
   }
   g->n_input = n;
   const int bits = bits_for(std::max<int64_t>(n, 2));
-  const uint64_t sent = (uint64_t(1) << (2 * bits)) - 1;  // never a valid (lo < hi) key
 
   // a1 + a2
   DevBuf<uint64_t> ka(std::max<int64_t>(m_gen, 1), s), kb(std::max<int64_t>(m_gen, 1), s);
-  DevBuf<int> err(1, s);
-  DevBuf<int64_t> nsel(1, s);
-  DevBuf<UniqTail> tail(1, s);
-  TC_CUDA(cudaMemsetAsync(err.get(), 0, sizeof(int), s));
-  TC_CUDA(cudaMemsetAsync(nsel.get(), 0, sizeof(int64_t), s));
-  if (m_gen > 0) {
-    k_canon<<<grid_for(m_gen), TPB, 0, s>>>(d_src, d_dst, m_gen, n, bits, sent, ka.get(),
-                                            err.get());
-    TC_LAUNCH();
-  }
-  tm.mark();
   int64_t m = 0;
-  uint64_t* ukey = ka.get();
-  if (m_gen > 0) {
-    cub::DoubleBuffer<uint64_t> db(ka.get(), kb.get());
-    cub_run(s, [&](void* t, size_t& b) {
-      return cub::DeviceRadixSort::SortKeys(t, b, db, m_gen, 0, 2 * bits, s);
-    });
-    uint64_t* sorted = db.Current();
-    uint64_t* other = sorted == ka.get() ? kb.get() : ka.get();
-    cub_run(s, [&](void* t, size_t& b) {
-      return cub::DeviceSelect::Unique(t, b, sorted, other, nsel.get(), m_gen, s);
-    });
-    ukey = other;
-  }
-  k_uniq_tail<<<1, 1, 0, s>>>(err.get(), nsel.get(), ukey, tail.get());
-  TC_LAUNCH();
-  UniqTail ut = d2h(tail.get(), s);
-  if (ut.err) fail(TC_ERR_INVALID_ARGUMENT, "vertex id < 0 or >= num_vertices in the edge list");
-  m = ut.nsel - ((ut.nsel > 0 && ut.last == sent) ? 1 : 0);
+  uint64_t* ukey = canon_unique(d_src, d_dst, m_gen, n, s, ka.get(), kb.get(), &m, &tm);
   g->m = m;
   tm.mark();
 
@@ -529,40 +623,17 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
     TC_LAUNCH();
   }
   const int keep = (flags & TC_KEEP_ISOLATED) ? 1 : 0;
-  const uint64_t sentv = (uint64_t(1) << (2 * bits + 1)) - 1;
-  DevBuf<uint64_t> va(std::max<int64_t>(n, 1), s), vb(std::max<int64_t>(n, 1), s);
-  DevBuf<unsigned long long> nact(1, s);
-  TC_CUDA(cudaMemsetAsync(nact.get(), 0, sizeof(unsigned long long), s));
-  int64_t n_act = 0;
   DevBuf<int32_t> rank(std::max<int64_t>(n, 1), s);
-  if (n > 0) {
-    k_vkey<<<grid_for(n), TPB, 0, s>>>(deg.get(), n, bits, keep, sentv, va.get(), nact.get());
-    TC_LAUNCH();
-    cub::DoubleBuffer<uint64_t> db(va.get(), vb.get());
-    cub_run(s, [&](void* t, size_t& b) {
-      return cub::DeviceRadixSort::SortKeys(t, b, db, n, 0, 2 * bits + 1, s);
-    });
-    n_act = (int64_t)d2h(nact.get(), s);
-    g->perm = DevBuf<int32_t>(std::max<int64_t>(n_act, 1), s, true);
-    if (n_act > 0) {
-      k_perm<<<grid_for(n_act), TPB, 0, s>>>(db.Current(), n_act, bits, g->perm.get(),
-                                             rank.get());
-      TC_LAUNCH();
-    }
-  } else {
-    g->perm = DevBuf<int32_t>(1, s, true);
-  }
+  const int64_t n_act = rank_vertices(deg.get(), n, keep, s, rank.get(), [&](int64_t na) {
+    g->perm = DevBuf<int32_t>(std::max<int64_t>(na, 1), s, true);
+    return g->perm.get();
+  });
   g->n = n_act;
   deg.reset();
-  va.reset();
-  vb.reset();
   tm.mark();
 
   // a5
   const int bits2 = bits_for(std::max<int64_t>(n_act, 2));
-  g->bits = bits2;
-  g->row_ptr = DevBuf<int64_t>(n_act + 1, s, true);
-  g->col = DevBuf<int32_t>(std::max<int64_t>(m, 1), s, true);
   if (m > 0) {
     uint64_t* okey_a = (ukey == ka.get()) ? kb.get() : ka.get();  // the free buffer
     k_orient<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank.get(), bits2, okey_a);
@@ -571,25 +642,13 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
     cub_run(s, [&](void* t, size_t& b) {
       return cub::DeviceRadixSort::SortKeys(t, b, db, m, 0, 2 * bits2, s);
     });
-    k_csr<<<grid_for(m), TPB, 0, s>>>(db.Current(), m, n_act, bits2, g->col.get(),
-                                      g->row_ptr.get());
-    TC_LAUNCH();
+    csr_from_sorted(db.Current(), m, n_act, s, g);
   } else {
-    k_fill_i64<<<grid_for(n_act + 1), TPB, 0, s>>>(g->row_ptr.get(), n_act + 1, 0);
-    TC_LAUNCH();
+    csr_from_sorted(nullptr, 0, n_act, s, g);
   }
   ka.reset();
   kb.reset();
   rank.reset();
-  {
-    DevBuf<unsigned long long> mx(1, s);
-    TC_CUDA(cudaMemsetAsync(mx.get(), 0, sizeof(unsigned long long), s));
-    if (n_act > 0) {
-      k_max_outdeg<<<grid_for(n_act), TPB, 0, s>>>(g->row_ptr.get(), n_act, mx.get());
-      TC_LAUNCH();
-    }
-    g->max_out = (int64_t)d2h(mx.get(), s);
-  }
   tm.mark();
   build_plan(g, opt, s);
   tm.mark();
@@ -600,6 +659,115 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
   g->ms[3] = tm.ms(3, 4);
   g->ms[4] = tm.ms(4, 5);
   g->ms[5] = tm.ms(0, 5);
+}
+
+// ------------------------------------------------------------------ f2
+int key_bits(int64_t n) { return bits_for(std::max<int64_t>(n, 2)); }
+
+int64_t shard_canon(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
+                    cudaStream_t s, uint64_t* out) {
+  DevBuf<uint64_t> ka(std::max<int64_t>(m_gen, 1), s), kb(std::max<int64_t>(m_gen, 1), s);
+  int64_t m = 0;
+  uint64_t* u = canon_unique(d_src, d_dst, m_gen, n, s, ka.get(), kb.get(), &m, nullptr);
+  if (m > 0) TC_CUDA(cudaMemcpyAsync(out, u, sizeof(uint64_t) * m, cudaMemcpyDeviceToDevice, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  return m;
+}
+
+void shard_histogram(const uint64_t* keys, int64_t cnt, int64_t n, int hist_bits, cudaStream_t s,
+                     int64_t* d_hist) {
+  const int shift = 2 * key_bits(n) - hist_bits;
+  const int64_t nb = int64_t(1) << hist_bits;
+  k_key_hist<<<grid_for(nb), TPB, 0, s>>>(keys, cnt, shift, nb, d_hist);
+  TC_LAUNCH();
+}
+
+void shard_bounds(const uint64_t* keys, int64_t cnt, int64_t n, int hist_bits,
+                  const int64_t* h_cuts, int P, cudaStream_t s, int64_t* h_bounds) {
+  const int shift = 2 * key_bits(n) - hist_bits;
+  const int64_t nb = int64_t(1) << hist_bits;
+  DevBuf<int64_t> cut(P + 1, s), pos(P + 1, s);
+  TC_CUDA(cudaMemcpyAsync(cut.get(), h_cuts, sizeof(int64_t) * (P + 1), cudaMemcpyHostToDevice, s));
+  k_key_bounds<<<1, 64 * ((P + 64) / 64), 0, s>>>(keys, cnt, shift, nb, cut.get(), P + 1, pos.get());
+  TC_LAUNCH();
+  TC_CUDA(cudaMemcpyAsync(h_bounds, pos.get(), sizeof(int64_t) * (P + 1), cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  h_bounds[0] = 0;
+  h_bounds[P] = cnt;
+}
+
+void sort_keys(uint64_t* keys, int64_t cnt, int64_t n, cudaStream_t s) {
+  if (cnt <= 1) return;
+  DevBuf<uint64_t> kb(cnt, s);
+  cub::DoubleBuffer<uint64_t> db(keys, kb.get());
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceRadixSort::SortKeys(t, b, db, cnt, 0, 2 * key_bits(n), s);
+  });
+  if (db.Current() != keys)
+    TC_CUDA(cudaMemcpyAsync(keys, db.Current(), sizeof(uint64_t) * cnt, cudaMemcpyDeviceToDevice, s));
+}
+
+int64_t shard_unique(uint64_t* keys, int64_t cnt, int64_t n, cudaStream_t s, int32_t* d_deg) {
+  if (cnt <= 0) return 0;
+  const int bits = key_bits(n);
+  DevBuf<uint64_t> kb(cnt, s);
+  DevBuf<int64_t> nsel(1, s);
+  cub::DoubleBuffer<uint64_t> db(keys, kb.get());
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceRadixSort::SortKeys(t, b, db, cnt, 0, 2 * bits, s);
+  });
+  uint64_t* sorted = db.Current();
+  uint64_t* other = sorted == keys ? kb.get() : keys;
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceSelect::Unique(t, b, sorted, other, nsel.get(), cnt, s);
+  });
+  const int64_t m = d2h(nsel.get(), s);
+  if (other != keys)
+    TC_CUDA(cudaMemcpyAsync(keys, other, sizeof(uint64_t) * m, cudaMemcpyDeviceToDevice, s));
+  if (m > 0) {
+    k_degree<<<grid_for(m), TPB, 0, s>>>(keys, m, bits, d_deg);
+    TC_LAUNCH();
+  }
+  TC_CUDA(cudaStreamSynchronize(s));
+  return m;
+}
+
+void shard_degree(const uint64_t* keys, int64_t cnt, int64_t n, cudaStream_t s, int32_t* d_deg) {
+  if (cnt <= 0) return;
+  k_degree<<<grid_for(cnt), TPB, 0, s>>>(keys, cnt, key_bits(n), d_deg);
+  TC_LAUNCH();
+}
+
+int64_t shard_rank(const int32_t* deg, int64_t n, uint32_t flags, cudaStream_t s, int32_t* rank,
+                   int32_t* perm) {
+  const int keep = (flags & TC_KEEP_ISOLATED) ? 1 : 0;
+  return rank_vertices(deg, n, keep, s, rank, [&](int64_t) { return perm; });
+}
+
+void shard_orient(const uint64_t* keys, int64_t cnt, int64_t n, const int32_t* rank,
+                  int64_t n_act, cudaStream_t s, uint64_t* okeys) {
+  if (cnt <= 0) return;
+  k_orient<<<grid_for(cnt), TPB, 0, s>>>(keys, cnt, key_bits(n), rank, key_bits(n_act), okeys);
+  TC_LAUNCH();
+  sort_keys(okeys, cnt, n_act, s);
+}
+
+void build_from_oriented(const uint64_t* okeys, int64_t m, const int32_t* perm, int64_t n_act,
+                         int64_t n_input, const Options& opt, cudaStream_t s, tc_graph* g) {
+  Timer tm(s);
+  tm.mark();
+  g->n_input = n_input;
+  g->perm = DevBuf<int32_t>(std::max<int64_t>(n_act, 1), s, true);
+  if (n_act > 0)
+    TC_CUDA(cudaMemcpyAsync(g->perm.get(), perm, sizeof(int32_t) * n_act, cudaMemcpyDeviceToDevice, s));
+  csr_from_sorted(m > 0 ? okeys : nullptr, m, n_act, s, g);
+  tm.mark();
+  build_plan(g, opt, s);
+  tm.mark();
+  TC_CUDA(cudaStreamSynchronize(s));
+  g->ms[3] = tm.ms(0, 1);
+  g->ms[4] = tm.ms(1, 2);
+  g->ms[5] = tm.ms(0, 2);
 }
 
 Tuning tuning_from_env() {
@@ -615,6 +783,7 @@ Tuning tuning_from_env() {
   t.grab_short = get("TC_GRAB_SHORT", t.grab_short, 0, 1 << 24);
   t.prod_div = get("TC_PROD_DIV", t.prod_div, 2, 32);
   t.wait_hint_ns = get("TC_WAIT_HINT", t.wait_hint_ns, 0, 10000000);
+  t.prefetch = get("TC_PREFETCH", t.prefetch, 0, 1);
   return t;
 }
 

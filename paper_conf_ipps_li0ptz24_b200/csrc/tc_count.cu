@@ -565,7 +565,7 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
 template <int kB, bool kSup = false>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
-                                        int pt, int PT) {
+                                        int pt, int PT, int prefetch = 0) {
   const int64_t sa = max(__ldg(pv.chunk_seg + (cix)), e_begin), sb = min(__ldg(pv.chunk_seg + (cix + 1)), e_end);
   if (sa >= sb) {  // empty after clipping to the range
     if (pt == 0) {
@@ -663,6 +663,14 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       const int2 d = c.sInfo[gl];
       const int toff = d.x >= 0 ? d.x : -1 - gl;
       const int64_t st = c.sB[i];
+      if (!kSup && prefetch) {
+        // Pull the edge's keys toward L2 now, one chunk before the consumers
+        // load them (a bulk prefetch: no registers, no SMEM; 16-B granules).
+        const uintptr_t lo = reinterpret_cast<uintptr_t>(pv.col + st) & ~uintptr_t(15);
+        const uintptr_t hi = (reinterpret_cast<uintptr_t>(pv.col + st + len) + 15) & ~uintptr_t(15);
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(lo), "r"((uint32_t)(hi - lo))
+                     : "memory");
+      }
       for (int t = ts; t < te; ++t) {
         const int64_t p = st + ((int64_t)(t - ts) << 5);
         const int lanes = min(32, len - ((t - ts) << 5));
@@ -802,7 +810,8 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
         mbar_arrive(&full_bar[slot]);
         break;
       }
-      produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], threadIdx.x, PT);
+      produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], threadIdx.x, PT,
+                 tu.prefetch);
       mbar_arrive(&full_bar[slot]);
     }
   } else {

@@ -127,13 +127,14 @@ __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_
 }
 
 // Count-kernel launch tuning (not part of the C-ABI; TC_SLOTS, TC_GRAB_LONG,
-// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT override the defaults for sweeps).
+// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_PREFETCH override the defaults for sweeps).
 struct Tuning {
   int slots = 3;          // chunk slots in SMEM (2..4)
   int grab_long = 0;      // tiles per consumer grab, long class (0 = static split)
   int grab_short = 0;     // keys per consumer grab, short class (0 = static split)
   int prod_div = 8;       // 1/prod_div of the warps are producers
   int wait_hint_ns = 0;   // mbarrier try_wait suspend hint (0 = none)
+  int prefetch = 0;       // long class: L2 bulk prefetch of each edge's keys at staging
 };
 Tuning tuning_from_env();
 
@@ -169,6 +170,24 @@ namespace tc {
 void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
                  uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g);
 void build_plan(tc_graph* g, const Options& opt, cudaStream_t s);
+
+// tc_build.cu, f2 sharded preprocessing (tc_shard_* in tc.h)
+int key_bits(int64_t n);
+int64_t shard_canon(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
+                    cudaStream_t s, uint64_t* out);
+void shard_histogram(const uint64_t* keys, int64_t cnt, int64_t n, int hist_bits, cudaStream_t s,
+                     int64_t* d_hist);
+void shard_bounds(const uint64_t* keys, int64_t cnt, int64_t n, int hist_bits,
+                  const int64_t* h_cuts, int P, cudaStream_t s, int64_t* h_bounds);
+void sort_keys(uint64_t* keys, int64_t cnt, int64_t n, cudaStream_t s);
+int64_t shard_unique(uint64_t* keys, int64_t cnt, int64_t n, cudaStream_t s, int32_t* d_deg);
+void shard_degree(const uint64_t* keys, int64_t cnt, int64_t n, cudaStream_t s, int32_t* d_deg);
+int64_t shard_rank(const int32_t* deg, int64_t n, uint32_t flags, cudaStream_t s, int32_t* rank,
+                   int32_t* perm);
+void shard_orient(const uint64_t* keys, int64_t cnt, int64_t n, const int32_t* rank,
+                  int64_t n_act, cudaStream_t s, uint64_t* okeys);
+void build_from_oriented(const uint64_t* okeys, int64_t m, const int32_t* perm, int64_t n_act,
+                         int64_t n_input, const Options& opt, cudaStream_t s, tc_graph* g);
 
 // tc_count.cu
 void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
