@@ -349,6 +349,44 @@ TC_API tc_status tc_build_from_oriented(const uint64_t* d_okeys, int64_t m,
                                         int64_t n_input, const tc_options* opts, void* stream,
                                         tc_graph** out);
 
+/*
+ * ------------------------------------------------------------------------
+ * the cross-GPU sum of the partial counts done by
+ * the library over NVLink peer memory (no NCCL).  After this rank's count of
+ * [e_begin, e_end) (as tc_count_range), one thread adds the partial into a
+ * SYMMETRIC buffer on every rank and waits for every rank's contribution:
+ *   - d_mc != NULL: through an NVLS multicast address (one
+ *     multimem.red.add.u64; the NVSwitch updates every replica);
+ *   - else through the world unicast peer addresses h_peers[0..world) (one
+ *     red.add.u64 per peer over NVLink P2P; h_peers[rank] == d_own).
+ * d_own : this rank's unicast address of the buffer (device uint64[3],
+ *         zero-initialised once, same layout on every rank; do not touch it
+ *         between calls).  epoch: 1 for the first call on a buffer, +1 per
+ *         call, equal on all ranks.  world <= TC_MAX_PEERS.
+ * d_total (device uint64) receives T on every rank.  Stream-ordered; the
+ * finishing kernel spins until all ranks arrive, so every rank must make the
+ * call; if some rank has not arrived within 20 s the kernel gives up and
+ * writes UINT64_MAX to d_total instead of hanging the stream.
+ * The multicast / peer mappings are the caller's plumbing (e.g. torch
+ * symmetric memory); tc_mc_buffer_create makes a single-device one.
+ */
+#define TC_MAX_PEERS 16
+TC_API tc_status tc_count_range_fused(const tc_graph* g, int64_t e_begin, int64_t e_end,
+                                      uint64_t* d_own, uint64_t* d_mc, uint64_t* const* h_peers,
+                                      int32_t world, uint64_t epoch, void* stream,
+                                      uint64_t* d_total);
+
+/*
+ * A multicast object whose only member is the current device, its memory
+ * mapped at a unicast (*d_uc) and a multicast (*d_mc) address, >= bytes,
+ * zeroed.  For single-process use (tests, one-GPU runs of the f4 path);
+ * TC_ERR_UNSUPPORTED where the device or driver has no multicast objects.
+ * Synchronises the device.  Release with tc_mc_buffer_destroy.
+ */
+TC_API tc_status tc_mc_buffer_create(size_t bytes, void** handle, uint64_t** d_uc,
+                                     uint64_t** d_mc);
+TC_API void tc_mc_buffer_destroy(void* handle);
+
 /* Release a graph (NULL is a no-op).  Stream-ordered frees on the build stream. */
 TC_API void tc_free(tc_graph* g);
 

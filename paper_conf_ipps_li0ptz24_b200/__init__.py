@@ -35,8 +35,10 @@ EXPORTS = (
     "tc_free", "tc_last_error", "tc_version", "tc_support", "tc_edge_list",
     "tc_count_variant", "tc_key_bits", "tc_shard_canon", "tc_shard_histogram", "tc_shard_cuts",
     "tc_shard_bounds", "tc_shard_unique", "tc_shard_degree", "tc_rank_vertices", "tc_shard_orient", "tc_sort_keys",
-    "tc_build_from_oriented",
+    "tc_build_from_oriented", "tc_count_range_fused", "tc_mc_buffer_create",
+    "tc_mc_buffer_destroy",
 )
+TC_MAX_PEERS = 16
 VARIANTS = {"polak": 1, "trust": 2}  # tc_count_variant
 
 
@@ -118,6 +120,10 @@ def lib():
             "tc_shard_orient": ([vp, i64, i64, vp, i64, vp, vp], st),
             "tc_sort_keys": ([vp, i64, i64, vp], st),
             "tc_build_from_oriented": ([vp, i64, vp, i64, i64, vp, vp, ctypes.POINTER(vp)], st),
+            "tc_count_range_fused": ([vp, i64, i64, vp, vp, vp, i32, ctypes.c_uint64, vp, vp], st),
+            "tc_mc_buffer_create": ([ctypes.c_size_t, ctypes.POINTER(vp), ctypes.POINTER(vp),
+                                     ctypes.POINTER(vp)], st),
+            "tc_mc_buffer_destroy": ([vp], None),
             "tc_free": ([vp], None),
             "tc_last_error": ([], ctypes.c_char_p),
             "tc_version": ([], ctypes.c_char_p),
@@ -350,26 +356,127 @@ def partition_prefix(prefix: Sequence[int], world_size: int) -> list:
     return [int(x) for x in b]
 
 
-def count_partitioned(graph, group=None, stream=None) -> int:
+class FusedSum:
+    """the symmetric buffer of the library's own
+    cross-GPU sum (tc_count_range_fused) — no NCCL on the counting path.
+
+    mode "multicast": an NVLS multicast address (one multimem.red per rank);
+    mode "peers": every rank's unicast address (one P2P red per peer);
+    "auto": multicast when available, else peers.  With more than one rank
+    the mapping comes from torch symmetric memory (plumbing: allocation and
+    handle exchange); a single process gets a one-device multicast object
+    from tc_mc_buffer_create, or a plain device buffer in peers mode.
+    """
+
+    def __init__(self, group=None, mode: str = "auto", peers=None, own=None):
+        import torch
+        import torch.distributed as dist
+        if mode not in ("auto", "multicast", "peers"):
+            raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, f"unknown mode {mode!r}")
+        self.group, self.epoch, self._handle, self._keep = group, 0, None, []
+        on = dist.is_available() and dist.is_initialized()
+        self.world = dist.get_world_size(group) if on else 1
+        self.rank = dist.get_rank(group) if on else 0
+        if self.world > TC_MAX_PEERS:
+            raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, f"at most {TC_MAX_PEERS} ranks")
+        self.mc, self.own, self.peers = 0, 0, None
+        if peers is not None:  # caller-provided mapping (tests: IPC-shared buffers)
+            self._keep = list(peers)
+            self.peers = [int(t.data_ptr()) for t in peers]
+            self.own = int(own.data_ptr()) if own is not None else self.peers[self.rank]
+            self.mode = "peers"
+            return
+        if self.world == 1:
+            if mode in ("auto", "multicast"):
+                h, uc, mc = ctypes.c_void_p(0), ctypes.c_void_p(0), ctypes.c_void_p(0)
+                st = lib().tc_mc_buffer_create(64, ctypes.byref(h), ctypes.byref(uc), ctypes.byref(mc))
+                if st == TC_OK:
+                    self._handle, self.own, self.mc, self.mode = h, uc.value, mc.value, "multicast"
+                    return
+                if mode == "multicast":
+                    _check(st)
+            buf = torch.zeros(4, dtype=torch.int64, device="cuda")
+            self._keep = [buf]
+            self.own = int(buf.data_ptr())
+            self.peers = [self.own]
+            self.mode = "peers"
+            return
+        import torch.distributed._symmetric_memory as symm
+        buf = symm.empty(4, dtype=torch.int64, device=torch.device("cuda", torch.cuda.current_device()))
+        buf.zero_()
+        torch.cuda.synchronize()
+        gname = group.group_name if group is not None else dist.group.WORLD.group_name
+        h = symm.rendezvous(buf, gname)
+        self._keep = [buf, h]
+        self.own = int(buf.data_ptr())
+        if mode != "peers" and int(getattr(h, "multicast_ptr", 0) or 0):
+            self.mc, self.mode = int(h.multicast_ptr), "multicast"
+        elif mode == "multicast":
+            raise TCError(TC_ERR_UNSUPPORTED, "no multicast address from symmetric memory")
+        else:
+            self.peers = [int(p) for p in h.buffer_ptrs]
+            self.mode = "peers"
+        dist.barrier(group=group)
+
+    def count_range(self, graph, e_begin: int, e_end: int, out=None, stream=None):
+        """This rank's partial over [e_begin, e_end) summed over all ranks, into
+        a 1-element int64 CUDA tensor (u64 bits; UINT64_MAX if a rank never
+        arrived).  Every rank must call it, in the same order."""
+        torch = _torch()
+        if out is None:
+            out = torch.empty(1, dtype=torch.int64, device="cuda")
+        self.epoch += 1
+        peers = None
+        if self.peers is not None:
+            peers = (ctypes.c_void_p * len(self.peers))(*self.peers)
+        _check(lib().tc_count_range_fused(graph._h, int(e_begin), int(e_end),
+                                          ctypes.c_void_p(self.own),
+                                          ctypes.c_void_p(self.mc or None), peers,
+                                          int(self.world), int(self.epoch),
+                                          ctypes.c_void_p(_stream(stream)),
+                                          ctypes.c_void_p(out.data_ptr())))
+        return out
+
+    def close(self):
+        if self._handle is not None:
+            lib().tc_mc_buffer_destroy(self._handle)
+            self._handle = None
+        self._keep = []
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] = None) -> int:
     """T over a torch.distributed process group.
 
     Every rank holds the same replicated graph; rank r counts the live
     oriented edges [b_r, b_{r+1}) of tc_partition's cost-balanced split and a
     single all_reduce(SUM) of the 8-byte partials (ProcessGroupNCCL over
     NVLink on the GPU box) gives T on every rank.  Two's-complement int64
-    addition is bit-identical to uint64 addition mod 2^64.
+    addition is bit-identical to uint64 addition mod 2^64.  With ``fused`` (a
+    :class:`FusedSum`), the sum is the library's own over NVLink peer memory
+    (f4) instead of the NCCL all_reduce.
     """
     import torch.distributed as dist
-    world = dist.get_world_size(group)
-    rank = dist.get_rank(group)
+    on = dist.is_available() and dist.is_initialized()
+    world = dist.get_world_size(group) if on else 1
+    rank = dist.get_rank(group) if on else 0
     bounds = graph.partition(world)
+    if fused is not None:  # f4: the library's own sum over NVLink peer memory
+        total = fused.count_range(graph, bounds[rank], bounds[rank + 1], stream=stream)
+        return int(total.item()) & (2**64 - 1)
     partial = graph.count_range(bounds[rank], bounds[rank + 1], stream=stream)
-    dist.all_reduce(partial, op=dist.ReduceOp.SUM, group=group)
+    if on:
+        dist.all_reduce(partial, op=dist.ReduceOp.SUM, group=group)
     return int(partial.item()) & (2**64 - 1)
 
 
 from .sharded import build_csr_sharded, shard_cuts  # noqa: E402  (f2)
 
-__all__ = ["build_csr_sharded", "shard_cuts", "Graph", "Options", "GraphInfo", "build_csr", "build_csr_host", "count_partitioned",
+__all__ = ["FusedSum", "build_csr_sharded", "shard_cuts", "Graph", "Options", "GraphInfo", "build_csr", "build_csr_host", "count_partitioned",
            "partition_prefix", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
            "EXPORTS", "LIB_PATH"]

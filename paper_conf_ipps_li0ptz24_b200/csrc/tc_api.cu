@@ -340,6 +340,34 @@ tc_status tc_count_range(const tc_graph* g, int64_t e_begin, int64_t e_end, void
   });
 }
 
+tc_status tc_count_range_fused(const tc_graph* g, int64_t e_begin, int64_t e_end, uint64_t* d_own,
+                               uint64_t* d_mc, uint64_t* const* h_peers, int32_t world,
+                               uint64_t epoch, void* stream, uint64_t* d_total) {
+  return guarded([&] {
+    require(g && d_total && d_own, "NULL argument");
+    require(world >= 1 && world <= TC_MAX_PEERS, "world must be in [1, TC_MAX_PEERS]");
+    require(epoch >= 1, "epoch must be >= 1");
+    require(d_mc || h_peers, "need a multicast address or the peer addresses");
+    if (!d_mc)
+      for (int r = 0; r < world; ++r) require(h_peers[r] != nullptr, "NULL peer address");
+    tc_status st = tc_count_range(g, e_begin, e_end, stream, d_total);
+    if (st != TC_OK) tc::fail(st, t_last_error);
+    tc::fused_finish(reinterpret_cast<unsigned long long*>(d_total), d_own, d_mc, h_peers, world,
+                     epoch, (cudaStream_t)stream);
+  });
+}
+
+tc_status tc_mc_buffer_create(size_t bytes, void** handle, uint64_t** d_uc, uint64_t** d_mc) {
+  if (handle) *handle = nullptr;
+  return guarded([&] {
+    require(handle && d_uc && d_mc, "NULL argument");
+    require(bytes > 0, "bytes must be > 0");
+    *handle = tc::mc_create(bytes, d_uc, d_mc);
+  });
+}
+
+void tc_mc_buffer_destroy(void* handle) { tc::mc_destroy(handle); }
+
 tc_status tc_count_variant(const tc_graph* g, int32_t variant, void* stream, uint64_t* d_count) {
   return guarded([&] {
     require(g && d_count, "NULL argument");

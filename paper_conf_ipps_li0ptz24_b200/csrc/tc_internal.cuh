@@ -201,6 +201,12 @@ int num_sms();
 void support_all(const tc_graph* g, cudaStream_t s, unsigned* d_sup);   // f1, tc_support
 void edge_ends(const tc_graph* g, cudaStream_t s, int32_t* d_u, int32_t* d_v);
 
+// tc_fused.cu (f4: fused cross-GPU sum over NVLink peer memory)
+void fused_finish(unsigned long long* d_total, uint64_t* own, uint64_t* mc,
+                  uint64_t* const* peers, int world, uint64_t epoch, cudaStream_t s);
+void* mc_create(size_t bytes, uint64_t** uc, uint64_t** mc);
+void mc_destroy(void* h);
+
 // tc_variants.cu (f3: the paper's Polak / TRUST kernels on this CSR)
 void count_variant(const tc_graph* g, int variant, cudaStream_t s, unsigned long long* d_out);
 
