@@ -63,6 +63,9 @@ def parse():
     ap.add_argument("--variant", default=None, choices=["polak", "trust"],
                     help="count with one of the paper's surveyed kernels (tc_count_variant, "
                          "SURVEY.md §8(f) f3) instead of the grouped path; N = 1 only")
+    ap.add_argument("--reduce", default="nccl", choices=["nccl", "fused"],
+                    help="cross-GPU sum of the partial counts: NCCL all_reduce, or the library's "
+                         "own over NVLink peer memory (tc_count_range_fused, SURVEY.md §8(f) f4)")
     ap.add_argument("--no-sharded", action="store_true",
                     help="skip the sharded-build measurement (tc_shard_*, SURVEY.md §8(f) f2)")
     ap.add_argument("--mode", default="count", choices=["count", "support"],
@@ -372,14 +375,18 @@ def main():
     if a.variant and world > 1:
         raise SystemExit("--variant runs on one GPU")
 
+    fused = tc.FusedSum() if a.reduce == "fused" and not a.variant else None
+
     def step(ev_mid=None):
         if a.variant:
             g.count_variant(a.variant, out=out)
+        elif fused is not None:  # count + the library's own cross-GPU sum (f4)
+            fused.count_range(g, e0, e1, out=out)
         else:
             g.count_range(e0, e1, out=out)
         if ev_mid is not None:
             ev_mid.record(stream)
-        if world > 1:
+        if world > 1 and fused is None:
             dist.all_reduce(out)
 
     for _ in range(max(1, a.warmup)):
@@ -513,7 +520,9 @@ def main():
         "config": {"workload": f"{a.config}: {cfg.description}", "seed": a.seed, "n": n,
                    "n_active": int(info.n), "m": m, "max_out_degree": int(info.max_out_degree),
                    "m_live": int(info.m_live), "keys_total": int(info.keys_total),
-                   "parallelism": f"edge-range x{world} (replicated CSR, 1 NCCL all_reduce)",
+                   "parallelism": f"edge-range x{world} (replicated CSR, " + (
+                       "1 NCCL all_reduce)" if fused is None else
+                       f"fused sum over NVLink peer memory, {fused.mode})"),
                    "l2": f"flushed by a {a.flush_mb} MiB write between timed steps; CSR "
                          f"{(info.m * 4 + (info.n + 1) * 8) / 2**20:.0f} MiB",
                    "kernel": a.variant or "grouped (k_count + k_count_flat)"},
@@ -525,8 +534,8 @@ def main():
                                   "(SURVEY.md §8(d)); x this rank's share for N>1",
                      "peak_source": peak_src},
         "e2e": e2e,
-        "gpu_launches": a.steps * (g.launches_per_count if not a.variant else
-                                   (1 if a.variant == "polak" else 3)),
+        "gpu_launches": a.steps * (g.launches_per_count + (fused is not None) if not a.variant
+                                   else (1 if a.variant == "polak" else 3)),
         "build_ms": {"canon": info.ms_canon, "sort_unique": info.ms_sort_unique,
                      "degree_rank": info.ms_degree_rank, "orient_csr": info.ms_orient_csr,
                      "plan": info.ms_plan, "total_events": info.ms_total,

@@ -330,17 +330,21 @@ __device__ __forceinline__ void warp_walk(const int* __restrict__ P, int S, int 
 // so every lane probes unpredicated.
 // zw = (code << 6) | first valid lane (see produce): code 0 bitmap, >= 2 hash
 // slots, -1 huge; first valid lane 32 = none.
+// Returns the lane's hit WITHOUT the valid-lane mask (the caller adds it
+// under `lane >= first valid lane`: one ISETP + a predicated IADD).
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned probe_tile(const ChunkSmem& c, int z, int zw, int32_t key,
                                                int lane, const PlanView& pv, int64_t ga) {
-  const unsigned valid = lane >= (zw & 63) ? 1u : 0u;
+  // z of a staged table is relative to the slot base c.sT0 (the producer
+  // added the table area's offset), so an address is ((key >> 5) + z) * 4 +
+  // slot base
   const int w = zw >> 6;
   if (w == 0) {
-    const unsigned word = (unsigned)c.sHash[(key >> 5) + z];
-    return __funnelshift_r(~word, 0u, (unsigned)key) & valid;  // bit key & 31 of ~word
+    const unsigned word = (unsigned)c.sT0[(key >> 5) + z];
+    return (__funnelshift_r(word, 0u, (unsigned)key) & 1u) ^ 1u;  // bit key & 31 of ~word
   }
-  if (!kHuge || w > 0) return table_probe<kLinear>(c.sHash + z, (uint32_t)w, key) & valid;
-  return valid ? huge_probe(pv, ga + (-1 - z), key) : 0u;
+  if (!kHuge || w > 0) return table_probe<kLinear>(c.sT0 + z, (uint32_t)w, key);
+  return lane >= (zw & 63) ? huge_probe(pv, ga + (-1 - z), key) : 0u;
 }
 
 // Tiles [t0, t1), t0 a multiple of 8 (the consumer split keeps it so): each
@@ -356,8 +360,18 @@ __device__ __forceinline__ void load_batch(const ChunkSmem& c, const int32_t* co
 #pragma unroll
   for (int q = 0; q < kB; q += 4)
     *reinterpret_cast<int4*>(x + q) = *reinterpret_cast<const int4*>(c.sT0 + t + q);
+  // colL = col + lane, opaque to the compiler (lane_base): each key address is
+  // ONE IMAD.WIDE.U32 x * 4 + colL (left to itself, nvcc re-associates it into
+  // a 64-bit add-with-carry + LEA pair, 4 instructions per key)
 #pragma unroll
   for (int u = 0; u < kB; ++u) key[u] = __ldg(colL + (uint32_t)x[u]);
+}
+
+// col + lane in a register the compiler cannot see through.
+__device__ __forceinline__ const int32_t* lane_base(const int32_t* col, int lane) {
+  const int32_t* p = col + lane;
+  asm volatile("" : "+l"(p));
+  return p;
 }
 
 template <bool kLinear, bool kHuge>
@@ -367,7 +381,7 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   static_assert(kB % 4 == 0, "batches of whole int4 reads");
   unsigned cnt = 0;
   const int lane = threadIdx.x & 31;
-  const int32_t* colL = pv.col + lane;
+  const int32_t* colL = lane_base(pv.col, lane);
   int t = t0;
   for (; t + kB <= t1; t += kB) {
     int32_t key[kB];
@@ -378,9 +392,26 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
       *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
       *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
     }
+    int code_or = 0;
 #pragma unroll
-    for (int u = 0; u < kB; ++u)
-      cnt += probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
+    for (int u = 0; u < kB; ++u) code_or |= zw[u] >> 6;
+    if (code_or == 0) {
+      // warp-uniform fast path, every tile of the batch probes a bitmap (most
+      // batches: ~94% of RMAT keys meet a bitmap table): straight-line code,
+      // no per-tile branch; zw is then just the first valid lane
+#pragma unroll
+      for (int u = 0; u < kB; ++u) {
+        const unsigned word = (unsigned)c.sT0[(key[u] >> 5) + z[u]];
+        const unsigned hit = (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
+        if (lane >= zw[u]) cnt += hit;
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < kB; ++u) {
+        const unsigned hit = probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
+        if (lane >= (zw[u] & 63)) cnt += hit;
+      }
+    }
   }
   for (; t < t1; t += 8) {  // tail: tiles past t1 repeat the last tile with every lane masked
     int z[8], zw[8];
@@ -394,7 +425,10 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
       zw[u] = c.sT2[tt] | (t + u < t1 ? 0 : 32);  // first valid lane 32: none
     }
 #pragma unroll
-    for (int u = 0; u < 8; ++u) cnt += probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
+    for (int u = 0; u < 8; ++u) {
+      const unsigned hit = probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
+      if (lane >= (zw[u] & 63)) cnt += hit;
+    }
   }
   return cnt;
 }
@@ -687,7 +721,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
           // bitmap 0 (z = word base), hash = slots (z = offset), huge -1.
           // (6-bit lane field: 32 = no valid lane)
           c.sT0[t] = (int)(uint32_t)(p - (32 - lanes));
-          c.sT1[t] = d.x < 0 ? toff : (d.y <= 0 ? d.x + d.y : d.x);
+          c.sT1[t] = d.x < 0 ? toff : (int)(c.sHash - c.sT0) + (d.y <= 0 ? d.x + d.y : d.x);
           c.sT2[t] = ((d.x < 0 ? -1 : (d.y <= 0 ? 0 : d.y)) * 64) | (32 - lanes);
         }
       }

@@ -153,23 +153,42 @@ void* mc_create(size_t bytes, uint64_t** uc, uint64_t** mcp) {
   McBuffer* b = new McBuffer();
   b->dev = ordinal;
   try {
-  CUmulticastObjectProp mp;
-  std::memset(&mp, 0, sizeof(mp));
-  mp.numDevices = 1;
-  mp.size = bytes;
-  mp.handleTypes = 0;
+  // The driver wants a shareable handle type on the multicast object (and the
+  // bound memory) even when it is never exported; try POSIX fd, then fabric.
+  const CUmemAllocationHandleType kinds[2] = {CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR,
+                                              CU_MEM_HANDLE_TYPE_FABRIC};
   size_t gran = 0;
-  cu_check(driver_fn<FnGran>("cuMulticastGetGranularity")(&gran, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED),
-           "cuMulticastGetGranularity");
-  b->size = (bytes + gran - 1) / gran * gran;
-  mp.size = b->size;
-  cu_check(driver_fn<FnCreate>("cuMulticastCreate")(&b->mc, &mp), "cuMulticastCreate");
+  CUresult r = CUDA_ERROR_NOT_SUPPORTED;
+  CUmemAllocationHandleType kind = kinds[0];
+  for (CUmemAllocationHandleType k : kinds) {
+    CUmulticastObjectProp mp;
+    std::memset(&mp, 0, sizeof(mp));
+    mp.numDevices = 1;
+    mp.size = bytes;
+    mp.handleTypes = (unsigned long long)k;
+    r = driver_fn<FnGran>("cuMulticastGetGranularity")(&gran, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED);
+    if (r != CUDA_SUCCESS) continue;
+    b->size = (bytes + gran - 1) / gran * gran;
+    mp.size = b->size;
+    r = driver_fn<FnCreate>("cuMulticastCreate")(&b->mc, &mp);
+    if (r == CUDA_SUCCESS) {
+      kind = k;
+      break;
+    }
+  }
+  if (r == CUDA_ERROR_INVALID_VALUE || r == CUDA_ERROR_NOT_PERMITTED || r == CUDA_ERROR_NOT_SUPPORTED)
+    // seen on a one-GPU container whose process has no NVSwitch fabric access
+    // (every handle type / device count refused, MULTICAST_SUPPORTED = 1)
+    fail(TC_ERR_UNSUPPORTED, "cuMulticastCreate refused (CUresult " + std::to_string((int)r) +
+                                 "): no NVLS multicast for this process");
+  cu_check(r, "cuMulticastCreate");
   cu_check(driver_fn<FnAdd>("cuMulticastAddDevice")(b->mc, dev), "cuMulticastAddDevice");
   CUmemAllocationProp ap;
   std::memset(&ap, 0, sizeof(ap));
   ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
   ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
   ap.location.id = ordinal;
+  ap.requestedHandleTypes = kind;
   cu_check(driver_fn<FnMemCreate>("cuMemCreate")(&b->mem, b->size, &ap, 0), "cuMemCreate");
   cu_check(driver_fn<FnBind>("cuMulticastBindMem")(b->mc, 0, b->mem, 0, b->size, 0),
            "cuMulticastBindMem");

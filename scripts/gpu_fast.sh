@@ -1,0 +1,7 @@
+TAG=${1:-r19g}
+O=gpurun_out
+timeout 600 python -m pytest tests/test_gpu_parity.py tests/test_gpu_fused.py -q -x > $O/${TAG}_pytest.txt 2>&1; echo "rc=$?" >> $O/${TAG}_pytest.txt
+for c in C3 C2 C3 C5 C1; do
+  timeout 300 python bench.py --config $c --no-cpu-baseline --no-e2e --no-sharded --steps 5 2>/dev/null | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$c', round(d['ms_per_step'],4), d['parity_vs_oracle'])" >> $O/${TAG}_ab.txt
+done
+echo done > $O/${TAG}_done.txt
