@@ -392,10 +392,10 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
       *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
       *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
     }
-    int code_or = 0;
+    int zw_or = 0;  // first-lane fields are < 64, so the OR's code bits are the OR of the codes
 #pragma unroll
-    for (int u = 0; u < kB; ++u) code_or |= zw[u] >> 6;
-    if (code_or == 0) {
+    for (int u = 0; u < kB; ++u) zw_or |= zw[u];
+    if ((zw_or >> 6) == 0) {
       // warp-uniform fast path, every tile of the batch probes a bitmap (most
       // batches: ~94% of RMAT keys meet a bitmap table): straight-line code,
       // no per-tile branch; zw is then just the first valid lane
@@ -462,7 +462,10 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
       key[u] = -2;
       gl[u] = 0;
       if (k < k1w) {
-        key[u] = __ldg(pv.col + c.sB[seg[u]] + k);
+        // col index sB + k < m < 2^32: a 32-bit add on the low word of sB
+        // (two's complement wraps correctly) and one IMAD.WIDE
+        const uint32_t lo = reinterpret_cast<const uint32_t*>(c.sB)[2 * seg[u]];
+        key[u] = __ldg(pv.col + (lo + (uint32_t)k));
         gl[u] = c.sD[seg[u]];
       }
     }
@@ -472,8 +475,16 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
       // linear probe needs a table with an empty slot to terminate)
       if (k0 + 32 * u + lane >= k1w) continue;
       const int2 d = c.sInfo[gl[u]];
-      if (kHuge && d.x < 0) cnt += huge_probe(pv, ga + gl[u], key[u]);
-      else cnt += any_probe<kLinear>(c.sHash + d.x, d.y, key[u]);
+      if (kHuge && d.x < 0) {
+        cnt += huge_probe(pv, ga + gl[u], key[u]);
+      } else if (d.y <= 0) {
+        // bitmap of the rank window: the trimmed key lies inside it (C-21),
+        // so the word index (key >> 5) + code is in range
+        const unsigned word = (unsigned)c.sHash[d.x + (key[u] >> 5) + d.y];
+        cnt += (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
+      } else {
+        cnt += table_probe<kLinear>(c.sHash + d.x, (uint32_t)d.y, key[u]);
+      }
     }
   }
   return cnt;
