@@ -203,7 +203,10 @@ tc_status build_impl(const int32_t* src, const int32_t* dst, int64_t num_edges,
     // peak scratch of a1..a6 is ~72 B per input pair (sort double buffers,
     // plan arrays) + ~48 B per vertex; the host entry adds the 8-B pair copy
     const int64_t nv = num_vertices > 0 ? num_vertices : 0;
-    tc::reserve_pool((size_t)num_edges * (host ? 80 : 72) + (size_t)nv * 48, s);
+    // + the a2 hash set (u64, capacity the power of two >= 2 num_edges)
+    size_t cap = 1024;
+    while ((int64_t)cap < 2 * num_edges && num_edges <= (int64_t(1) << 25)) cap <<= 1;
+    tc::reserve_pool((size_t)num_edges * (host ? 80 : 72) + (size_t)nv * 48 + cap * 8, s);
     g = new tc_graph();
     if (host) {
       tc::DevBuf<int32_t> ds(std::max<int64_t>(num_edges, 1), s), dd(std::max<int64_t>(num_edges, 1), s);

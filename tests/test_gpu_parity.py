@@ -5,6 +5,7 @@ seeded input from tcgen/; neither side's numbers come from the other.
 Sizes span many work chunks and ragged tails; the plan options are varied
 because they must never change a count.
 """
+import os
 from math import comb
 
 import numpy as np
@@ -13,6 +14,8 @@ import pytest
 import oracle
 import tcgen
 from tests import graphs
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
@@ -241,10 +244,14 @@ def reference_csr(src, dst, n):
     return row_ptr, hi.astype(np.int32), order.astype(np.int32)
 
 
-@pytest.mark.parametrize("case", ["rmat", "lattice", "karate"])
+@pytest.mark.parametrize("case", ["rmat", "lattice", "karate", "dups"])
 def test_csr_exact(tc, golden, case):
     if case == "rmat":
         src, dst, n = tcgen.rmat(12, 16, 2)
+    elif case == "dups":  # every pair 3x, half reversed, plus self-loops: a2's dedup
+        s0, d0, n = tcgen.rmat(14, 8, 4)
+        src = np.concatenate([s0, d0, s0, np.arange(0, n, 7, dtype=np.int32)])
+        dst = np.concatenate([d0, s0, d0, np.arange(0, n, 7, dtype=np.int32)])
     elif case == "lattice":
         src, dst, n = tcgen.lattice(50, 3)
     else:
@@ -363,3 +370,27 @@ def test_trust_bucket_overflow_fallback(tc, monkeypatch):
     with tc.build_csr(dev(src), dev(dst), n) as g:
         assert g.info.max_out_degree > 100  # the block path runs too
         assert int(g.count_variant("trust").item()) == want
+
+
+def test_dedup_paths_agree(tc):
+    """a2 by hashing and by radix sort + unique (forced with TC_DEDUP in child
+    processes) build the same CSR and count."""
+    import hashlib
+    import subprocess
+    import sys
+    src, dst, n = tcgen.rmat(16, 16, 9)
+    code = ("import sys, hashlib, numpy as np, torch; sys.path.insert(0, %r); import tcgen;"
+            "import paper_conf_ipps_li0ptz24_b200 as tc;"
+            "s, d, n = tcgen.rmat(16, 16, 9);"
+            "g = tc.build_csr(torch.from_numpy(s).cuda(), torch.from_numpy(d).cuda(), n);"
+            "h = hashlib.sha256(); [h.update(x.cpu().numpy().tobytes()) for x in g.csr()];"
+            "print(h.hexdigest(), g.count())") % ROOT
+    out = {}
+    for mode in ("sort", "hash"):
+        env = dict(os.environ, TC_DEDUP=mode)
+        r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                           timeout=300)
+        assert r.returncode == 0, r.stderr[-2000:]
+        out[mode] = r.stdout.split()[-2:]
+    assert out["sort"] == out["hash"]
+    assert int(out["sort"][1]) == oracle.triangles(src, dst)
