@@ -888,6 +888,7 @@ Tuning tuning_from_env() {
   t.prod_div = get("TC_PROD_DIV", t.prod_div, 2, 32);
   t.wait_hint_ns = get("TC_WAIT_HINT", t.wait_hint_ns, 0, 10000000);
   t.prefetch = get("TC_PREFETCH", t.prefetch, 0, 1);
+  t.ring = get("TC_RING", t.ring, 0, 1);
   return t;
 }
 
@@ -967,7 +968,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P.tune = tuning_from_env();
   // SMEM of one chunk slot of the count kernel; a table may use at most half
   // of it (bigger tables are "huge": probed in global memory)
-  const int64_t slot_limit = max_chunk_smem(P.tune.slots);
+  const int64_t slot_limit = max_chunk_smem(P.tune);
   const int64_t flat_limit = max_flat_chunk_smem();
   const int64_t max_table_slots = std::min(slot_limit, flat_limit) / 8;
   P.seg_start = DevBuf<int64_t>(S, s, true);
@@ -1066,7 +1067,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   TC_CUDA(cudaMemcpyAsync(P.h_chunk_seg.data(), P.chunk_seg.get(),
                           sizeof(int64_t) * (P.n_chunks + 1), cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));
-  const int occ = count_occupancy(P.block, P.smem_bytes, P.tune.slots);
+  const int occ = count_occupancy(P.block, P.smem_bytes, P.tune);
   const int occ_flat = flat_occupancy(P.smem_flat);
   if (occ < 1 || occ_flat < 1)
     fail(TC_ERR_UNSUPPORTED, "count kernel cannot launch with this SMEM/block size");

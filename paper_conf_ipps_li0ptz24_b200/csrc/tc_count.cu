@@ -46,6 +46,10 @@ constexpr int kUnrollLong = 8;   // tail batch of the long class
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
 constexpr int kUnrollShort = 4;  // tiles in flight per consumer warp (short class)
+#ifndef TC_RING_DEPTH
+#define TC_RING_DEPTH 2
+#endif
+constexpr int kRingDepth = TC_RING_DEPTH;  // batches in flight per consumer warp (Tuning::ring)
 constexpr int kMaxKicks = 96;    // cuckoo displacement bound before the linear fallback
 constexpr int kMaxSlots = 4;     // chunk slots in SMEM (runtime count: Tuning::slots)
 
@@ -433,6 +437,82 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   return cnt;
 }
 
+// Same walk with the key loads as asynchronous global->shared copies
+// (`cp.async` 4 B per lane, one commit group per 8-tile batch) into a
+// per-warp ring of kD batch buffers: batch b+kD is in flight while batch b
+// is probed, and in-flight keys occupy SMEM instead of registers (the
+// register-resident walk keeps only 8 loads per lane in flight: 64 registers
+// per thread at 1024 threads).  Each lane copies and later reads only its own
+// words, so no warp barrier is needed: cp.async.wait_group orders them.
+template <int kD>
+__device__ __forceinline__ void ring_issue(const ChunkSmem& c, const int32_t* colL, int t,
+                                           uint32_t dst) {
+  constexpr int kB = kBatchLong;
+  int x[kB];
+#pragma unroll
+  for (int q = 0; q < kB; q += 4)
+    *reinterpret_cast<int4*>(x + q) = *reinterpret_cast<const int4*>(c.sT0 + t + q);
+#pragma unroll
+  for (int u = 0; u < kB; ++u)
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst + 128u * u),
+                 "l"(colL + (uint32_t)x[u])
+                 : "memory");
+}
+
+template <bool kLinear, bool kHuge, int kD>
+__device__ __forceinline__ unsigned walk_long_ring(const ChunkSmem& c, int t0, int t1,
+                                                   const PlanView& pv, int64_t ga,
+                                                   int* __restrict__ ring) {
+  constexpr int kB = kBatchLong;
+  unsigned cnt = 0;
+  const int lane = threadIdx.x & 31;
+  const int32_t* colL = lane_base(pv.col, lane);
+  const int* ringL = ring + lane;
+  const uint32_t rs = smem_u32(ring) + 4u * lane;
+  constexpr uint32_t kSlotBytes = kB * 32 * 4;
+  const int nb = (t1 - t0) / kB;
+#pragma unroll
+  for (int b = 0; b < kD; ++b) {
+    if (b < nb) ring_issue<kD>(c, colL, t0 + b * kB, rs + kSlotBytes * b);
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  }
+  for (int b = 0; b < nb; ++b) {
+    const int t = t0 + b * kB, r = b % kD;
+    asm volatile("cp.async.wait_group %0;" ::"n"(kD - 1) : "memory");
+    int32_t key[kB];
+#pragma unroll
+    for (int u = 0; u < kB; ++u) key[u] = ringL[r * (kB * 32) + 32 * u];
+    if (b + kD < nb) ring_issue<kD>(c, colL, t + kD * kB, rs + kSlotBytes * r);
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    int z[kB], zw[kB];
+#pragma unroll
+    for (int q = 0; q < kB; q += 4) {
+      *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
+      *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
+    }
+    int zw_or = 0;
+#pragma unroll
+    for (int u = 0; u < kB; ++u) zw_or |= zw[u];
+    if ((zw_or >> 6) == 0) {
+#pragma unroll
+      for (int u = 0; u < kB; ++u) {
+        const unsigned word = (unsigned)c.sT0[(key[u] >> 5) + z[u]];
+        const unsigned hit = (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
+        if (lane >= zw[u]) cnt += hit;
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < kB; ++u) {
+        const unsigned hit = probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
+        if (lane >= (zw[u] & 63)) cnt += hit;
+      }
+    }
+  }
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
+  // the < 8 tiles left: the register walk's tail
+  return cnt + walk_long<kLinear, kHuge>(c, t0 + nb * kB, t1, pv, ga);
+}
+
 // SHORT class: the warp owns the flat keys [k0w, k1w) of the chunk.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0w, int k1w,
@@ -492,7 +572,10 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
 
 template <bool kLinear>
 __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
-                                            const PlanView& pv) {
+                                            const PlanView& pv, int* ring = nullptr) {
+  if (h.is_long && ring)
+    return h.huge ? walk_long_ring<kLinear, true, kRingDepth>(c, w0, w1, pv, h.ga, ring)
+                  : walk_long_ring<kLinear, false, kRingDepth>(c, w0, w1, pv, h.ga, ring);
   if (h.is_long)
     return h.huge ? walk_long<kLinear, true>(c, w0, w1, pv, h.ga)
                   : walk_long<kLinear, false>(c, w0, w1, pv, h.ga);
@@ -862,6 +945,9 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
   } else {
     // ------------------------------------------------------------ consumers
     const int cw = warp - n_prod;
+    int* ring = tu.ring ? reinterpret_cast<int*>(smem + nslots * slot_bytes) +
+                              cw * (kRingDepth * kBatchLong * 32)
+                        : nullptr;
     for (int64_t k = 0;; ++k) {
       const int slot = (int)(k % nslots);
       wait_full(&full_bar[slot], (uint32_t)((k / nslots) & 1), hint);
@@ -877,7 +963,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = min((w0 + 7) & ~7, NU);
             w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
           }
-          acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+          acc += h.linear ? consume<true>(c, h, w0, w1, pv, ring) : consume<false>(c, h, w0, w1, pv, ring);
         } else {  // dynamic: grab `grab` units at a time from the slot's counter
           for (;;) {
             int w0 = 0;
@@ -885,7 +971,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = __shfl_sync(0xffffffffu, w0, 0);
             if (w0 >= NU) break;
             const int w1 = min(w0 + grab, NU);
-            acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+            acc += h.linear ? consume<true>(c, h, w0, w1, pv, ring) : consume<false>(c, h, w0, w1, pv, ring);
           }
         }
       }
@@ -1074,7 +1160,14 @@ int num_sms() {
 
 int max_smem_per_block() { return optin_smem() - static_smem((const void*)k_count); }
 
-int max_chunk_smem(int slots) { return (max_smem_per_block() / slots) & ~15; }
+// The consumers' cp.async rings (Tuning::ring), sized for all 32 warps.
+int64_t ring_bytes(const Tuning& tu) {
+  return tu.ring ? (int64_t)(kMaxBlock / 32) * kRingDepth * kBatchLong * 32 * 4 : 0;
+}
+
+int max_chunk_smem(const Tuning& tu) {
+  return (int)((max_smem_per_block() - ring_bytes(tu)) / tu.slots) & ~15;
+}
 
 // One chunk of the flat kernel must leave room for 3 CTAs per SM.
 int max_flat_chunk_smem() {
@@ -1085,11 +1178,11 @@ int max_flat_chunk_smem() {
   return std::min(per_cta, optin_smem() - static_smem((const void*)k_count_flat)) & ~15;
 }
 
-int count_occupancy(int block, int64_t smem_bytes, int slots) {
+int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu) {
   ensure_attr();
   int occ = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-      &occ, k_count, block, (size_t)(slots * slot_bytes_of(smem_bytes))));
+      &occ, k_count, block, (size_t)(tu.slots * slot_bytes_of(smem_bytes) + ring_bytes(tu))));
   return occ;
 }
 
@@ -1113,8 +1206,8 @@ void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_b
   if (l1 > l0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(l1 - l0, P.grid));
     const int64_t sb = slot_bytes_of(P.smem_bytes);
-    k_count<<<grid, P.block, (size_t)(P.tune.slots * sb), s>>>(pv, l0, l1, e_begin, e_end, sb,
-                                                              P.tune, d_out);
+    k_count<<<grid, P.block, (size_t)(P.tune.slots * sb + ring_bytes(P.tune)), s>>>(
+        pv, l0, l1, e_begin, e_end, sb, P.tune, d_out);
     TC_LAUNCH();
   }
   // short-class chunks: flat kernel

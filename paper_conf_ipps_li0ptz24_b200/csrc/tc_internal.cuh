@@ -127,7 +127,7 @@ __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_
 }
 
 // Count-kernel launch tuning (not part of the C-ABI; TC_SLOTS, TC_GRAB_LONG,
-// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_PREFETCH override the defaults for sweeps).
+// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_PREFETCH, TC_RING override the defaults for sweeps).
 struct Tuning {
   int slots = 3;          // chunk slots in SMEM (2..4)
   int grab_long = 0;      // tiles per consumer grab, long class (0 = static split)
@@ -135,6 +135,7 @@ struct Tuning {
   int prod_div = 5;       // 1/prod_div of the warps are producers (C3 sweep: 8 -> 57.7 ms, 6 -> 55.0, 5 -> 53.5, 4 -> 54.0)
   int wait_hint_ns = 0;   // mbarrier try_wait suspend hint (0 = none)
   int prefetch = 0;       // long class: L2 bulk prefetch of each edge's keys at staging
+  int ring = 0;           // long class: key loads as cp.async into per-warp SMEM rings
 };
 Tuning tuning_from_env();
 
@@ -192,9 +193,9 @@ void build_from_oriented(const uint64_t* okeys, int64_t m, const int32_t* perm, 
 // tc_count.cu
 void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
                   int64_t e_end, cudaStream_t s, unsigned long long* d_out);
-int count_occupancy(int block, int64_t smem_bytes, int slots);  // CTAs per SM (0 = cannot launch)
+int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu);  // CTAs per SM (0 = cannot launch)
 int max_smem_per_block();
-int max_chunk_smem(int slots);  // SMEM one of the kernel's chunk slots may use
+int max_chunk_smem(const Tuning& tu);  // SMEM one of the kernel's chunk slots may use
 int max_flat_chunk_smem();      // SMEM one short-class chunk may use (3 CTAs per SM)
 int flat_occupancy(int64_t smem_bytes);
 int num_sms();
