@@ -639,33 +639,57 @@ __device__ __forceinline__ int sup_lookup_any(const ChunkSmem& c, const PlanView
 
 constexpr int kUnrollSup = 4;
 
+// Support-mode lookup of key in group gl's table; kHuge = the chunk has
+// groups probed in global memory (otherwise that path is not compiled in).
+template <bool kLinear, bool kHuge>
+__device__ __forceinline__ int sup_lookup(const ChunkSmem& c, const PlanView& pv, int gl,
+                                          uint32_t vrow, int32_t key) {
+  const int2 info = c.sInfo[gl];
+  if (kHuge && info.x < 0) return global_find(pv.col, vrow, c.sGP[gl + 1] - c.sGP[gl], key);
+  return sup_find<kLinear>(c.sHash, info.x, info.y, key);
+}
+
+// col + lane / sup + lane in a register the compiler cannot see through.
+__device__ __forceinline__ unsigned* lane_base_u(unsigned* p, int lane) {
+  unsigned* q = p + lane;
+  asm volatile("" : "+l"(q));
+  return q;
+}
+
 // LONG class, support mode: tiles [t0, t1); a tile's lanes share one edge,
-// whose count is warp-aggregated into one atomic.
+// whose count is warp-aggregated into one atomic.  Tile descriptors (see
+// produce): sT0 = col position of the tile's first key, sT1 = row_ptr[v]
+// (so (v, w) is sT1 + index of w in N+(v)), sT2 = the CSR position of the
+// tile's own edge (u, v), sT3 = chunk-local group << 6 | valid lanes; every
+// position < m < 2^32.
+template <bool kLinear, bool kHuge>
 __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1,
-                                              const PlanView& pv, bool linear) {
+                                              const PlanView& pv) {
   const int lane = threadIdx.x & 31;
+  const int32_t* colL = lane_base(pv.col, lane);
+  unsigned* supL = lane_base_u(pv.sup, lane);
   for (int t = t0; t < t1; t += kUnrollSup) {
     int32_t key[kUnrollSup];
-    int64_t p[kUnrollSup];
-    int sl[kUnrollSup];
+    uint32_t p[kUnrollSup], vr[kUnrollSup], own[kUnrollSup];
+    int g6[kUnrollSup];
 #pragma unroll
     for (int u = 0; u < kUnrollSup; ++u) {
       const int tt = min(t + u, t1 - 1);
-      const int lanes = (t + u < t1) ? c.sT3[tt] : 0;
-      p[u] = (int64_t)(((uint64_t)(uint32_t)c.sT1[tt] << 32) | (uint32_t)c.sT0[tt]);
-      sl[u] = c.sT2[tt];
-      key[u] = lane < lanes ? __ldg(pv.col + p[u] + lane) : -2;
+      p[u] = (uint32_t)c.sT0[tt];
+      vr[u] = (uint32_t)c.sT1[tt];
+      own[u] = (uint32_t)c.sT2[tt];
+      g6[u] = (t + u < t1) ? c.sT3[tt] : 0;
+      key[u] = lane < (g6[u] & 63) ? __ldg(colL + p[u]) : -2;
     }
 #pragma unroll
     for (int u = 0; u < kUnrollSup; ++u) {
-      const int gl = c.sD[sl[u]];
-      const int idx = key[u] >= 0 ? sup_lookup_any(c, pv, gl, key[u], linear) : -1;
+      const int idx = key[u] >= 0 ? sup_lookup<kLinear, kHuge>(c, pv, g6[u] >> 6, vr[u], key[u]) : -1;
       const unsigned bal = __ballot_sync(0xffffffffu, idx >= 0);
       if (idx >= 0) {
-        atomicAdd(pv.sup + p[u] + lane, 1u);                     // (u, w)
-        atomicAdd(pv.sup + c.sGB[gl] + c.sGP[gl] + idx, 1u);     // (v, w)
+        atomicAdd(supL + p[u], 1u);                        // (u, w)
+        atomicAdd(pv.sup + (vr[u] + (uint32_t)idx), 1u);   // (v, w)
       }
-      if (lane == 0 && bal) atomicAdd(pv.sup + c.sE[sl[u]], (unsigned)__popc(bal));  // (u, v)
+      if (lane == 0 && bal) atomicAdd(pv.sup + own[u], (unsigned)__popc(bal));  // (u, v)
     }
   }
 }
@@ -803,11 +827,11 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         const int64_t p = st + ((int64_t)(t - ts) << 5);
         const int lanes = min(32, len - ((t - ts) << 5));
         // support mode: the tile names its edge (chunk-local) instead of its table
-        if (kSup) {
+        if (kSup) {  // walk_long_sup's descriptor (positions < m < 2^32)
           c.sT0[t] = (int)(uint32_t)p;
-          c.sT1[t] = (int)(p >> 32);
-          c.sT2[t] = i;
-          c.sT3[t] = lanes;
+          c.sT1[t] = (int)(uint32_t)(c.sGB[gl] + c.sGP[gl]);  // row_ptr[v]
+          c.sT2[t] = (int)(uint32_t)c.sE[i];
+          c.sT3[t] = (gl << 6) | lanes;
         } else {
           // walk_long: a partial last tile is shifted back to the edge's last 32
           // keys (len >= 32 in the long class), its first 32 - lanes lanes
@@ -1049,7 +1073,12 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
       const ChunkSmem c = slot_view_sup(smem, h.S, h.G, h.T, h.nslots);
       const int NU = h.is_long ? h.T : c.sA[h.S];
       const int w0 = (int)((int64_t)NU * warp / nw), w1 = (int)((int64_t)NU * (warp + 1) / nw);
-      if (h.is_long) walk_long_sup(c, w0, w1, pv, h.linear);
+      if (h.is_long) {
+        if (h.huge)
+          h.linear ? walk_long_sup<true, true>(c, w0, w1, pv) : walk_long_sup<false, true>(c, w0, w1, pv);
+        else
+          h.linear ? walk_long_sup<true, false>(c, w0, w1, pv) : walk_long_sup<false, false>(c, w0, w1, pv);
+      }
       else if (w0 < w1) walk_short_sup(c, h.S, w0, w1, pv, h.linear);
     }
     __syncthreads();  // the slot is rebuilt by the next chunk

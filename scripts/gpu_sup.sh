@@ -1,0 +1,6 @@
+TAG=${1:-r19m}
+O=gpurun_out
+timeout 900 python -m pytest tests/test_gpu_support.py -q -x > $O/${TAG}_pytest.txt 2>&1; echo "rc=$?" >> $O/${TAG}_pytest.txt
+timeout 600 python bench.py --mode support --no-sharded --out $O/${TAG}_bench_support_c3.json > /dev/null 2>&1
+timeout 600 python bench.py --mode support --config C2 --no-sharded --out $O/${TAG}_bench_support_c2.json > /dev/null 2>&1
+echo done > $O/${TAG}_done.txt
