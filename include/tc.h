@@ -83,8 +83,8 @@ typedef struct {
                            binary search instead of an SMEM hash (default 8192)    */
   int32_t block_threads;/* threads per CTA of the count kernel, 64..1024; 1/8 of
                            the warps build tables, the rest probe (default 1024)   */
-  int32_t table_factor; /* hash slots = next_pow2(table_factor * d+(v)), 2..16
-                           (default 3, i.e. load <= 1/3)                            */
+  int32_t table_factor; /* hash slots = table_factor * d+(v) (rounded up to a
+                           multiple of 4), 2..16 (default 6, i.e. load <= 1/6)     */
   int32_t long_min;     /* trimmed suffixes with >= long_min keys go to the
                            warp-per-edge tile class, shorter ones to the flattened
                            class (default 32; values below 32 act as 32, since a
@@ -94,7 +94,7 @@ typedef struct {
   int32_t bitmap_factor; /* a head v whose window [min N+(v), max N+(v)] needs at most
                            bitmap_factor * d+(v) 32-bit words gets a bitmap table
                            (one probe per key) instead of a hash table (two);
-                           default 3 (same SMEM as the hash), -1 = never        */
+                           default 12, -1 = never                                */
 } tc_options;
 
 /*

@@ -853,7 +853,10 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   const int NI = c.sGP[G];
   const int i0 = (int)((int64_t)NI * pw / npw), i1 = (int)((int64_t)NI * (pw + 1) / npw);
   auto load_row = [&](int g, int k) { return __ldg(pv.col + c.sGB[g] + k); };
-  bool linear = pv.probe_mode == 1;
+  // short class: linear probing from the start when the plan says so (its
+  // tables are tiny — a few keys each — and a chunk whose cuckoo insert fails
+  // builds all its tables twice)
+  bool linear = pv.probe_mode == 1 || (!is_long && pv.short_linear);
   if constexpr (kSup) {
     // Support mode: entries carry the key's index j in N+(v) (its edge (v,w)
     // is col position row(v) + j).  Bitmap word x = {bits, members of N+(v)
@@ -1173,6 +1176,7 @@ PlanView plan_view(const tc_graph* g) {
   pv.chunk_seg = P.chunk_seg.get();
   pv.n_long_chunks = P.n_long_chunks;
   pv.probe_mode = P.opt.probe_mode;
+  pv.short_linear = P.tune.short_linear;
   pv.seg_edge = nullptr;
   pv.sup = nullptr;
   return pv;

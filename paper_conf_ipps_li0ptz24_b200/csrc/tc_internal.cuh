@@ -73,10 +73,10 @@ struct Options {
   int seg_cost = 4;
   int huge_degree = 8192;
   int block_threads = 1024;
-  int table_factor = 3;
+  int table_factor = 6;   // C3/C2/C5 sweep (r19o/r19p): 3 -> 6 with bitmap_factor 12: -7% / -18% / -23%
   int long_min = 32;
   int probe_mode = 0;
-  int bitmap_factor = 3;  // <= 0: never
+  int bitmap_factor = 12;  // <= 0: never
 };
 Options resolve_options(const tc_options* o);
 
@@ -109,6 +109,7 @@ struct PlanView {
   const int64_t* chunk_seg;    // [C+1]
   int64_t n_long_chunks;
   int probe_mode;
+  int short_linear;            // short class always probes linearly (Tuning::short_linear)
   // support mode only (tc_support; nullptr when counting)
   const int64_t* seg_edge;     // [S] CSR position of segment s's own edge (u,v)
   unsigned* sup;               // [m] per-edge triangle counts (accumulated)
@@ -127,7 +128,7 @@ __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_
 }
 
 // Count-kernel launch tuning (not part of the C-ABI; TC_SLOTS, TC_GRAB_LONG,
-// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_PREFETCH, TC_RING override the defaults for sweeps).
+// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_PREFETCH, TC_RING, TC_CS_DIV, TC_SHORT_LINEAR override the defaults for sweeps).
 struct Tuning {
   int slots = 3;          // chunk slots in SMEM (2..4)
   int grab_long = 0;      // tiles per consumer grab, long class (0 = static split)
@@ -136,6 +137,8 @@ struct Tuning {
   int wait_hint_ns = 0;   // mbarrier try_wait suspend hint (0 = none)
   int prefetch = 0;       // long class: L2 bulk prefetch of each edge's keys at staging
   int ring = 0;           // long class: key loads as cp.async into per-warp SMEM rings
+  int cs_div = 1;         // short-class chunk cost = chunk_cost / cs_div
+  int short_linear = 0;   // short class: linear-probing tables (no cuckoo attempt)
 };
 Tuning tuning_from_env();
 
