@@ -209,14 +209,7 @@ tc_status build_impl(const int32_t* src, const int32_t* dst, int64_t num_edges,
     tc::reserve_pool((size_t)num_edges * (host ? 80 : 72) + (size_t)nv * 48 + cap * 8, s);
     g = new tc_graph();
     if (host) {
-      tc::DevBuf<int32_t> ds(std::max<int64_t>(num_edges, 1), s), dd(std::max<int64_t>(num_edges, 1), s);
-      if (num_edges) {
-        TC_CUDA(cudaMemcpyAsync(ds.get(), src, sizeof(int32_t) * num_edges,
-                                cudaMemcpyHostToDevice, s));
-        TC_CUDA(cudaMemcpyAsync(dd.get(), dst, sizeof(int32_t) * num_edges,
-                                cudaMemcpyHostToDevice, s));
-      }
-      tc::build_graph(ds.get(), dd.get(), num_edges, num_vertices, flags, opt, s, g);
+      tc::build_graph_host(src, dst, num_edges, num_vertices, flags, opt, s, g);
     } else {
       tc::build_graph(src, dst, num_edges, num_vertices, flags, opt, s, g);
     }

@@ -672,50 +672,12 @@ void csr_from_sorted(const uint64_t* okey, int64_t m, int64_t n_act, cudaStream_
 
 }  // namespace
 
-// ------------------------------------------------------------------ a1..a5
-void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
-                 uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g) {
-  Timer tm(s);
-  tm.mark();
-  if (n < 0) {  // num_vertices = max id + 1
-    if (m_gen == 0) {
-      n = 0;
-    } else {
-      DevBuf<int32_t> mx(2, s);
-      cub_run(s, [&](void* t, size_t& b) {
-        return cub::DeviceReduce::Max(t, b, d_src, mx.get(), m_gen, s);
-      });
-      cub_run(s, [&](void* t, size_t& b) {
-        return cub::DeviceReduce::Max(t, b, d_dst, mx.get() + 1, m_gen, s);
-      });
-      int32_t h[2];
-      TC_CUDA(cudaMemcpyAsync(h, mx.get(), sizeof(h), cudaMemcpyDeviceToHost, s));
-      TC_CUDA(cudaStreamSynchronize(s));
-      n = (int64_t)std::max(h[0], h[1]) + 1;
-      if (n < 0) n = 0;
-    }
-  }
-  g->n_input = n;
+// a3..a6 from the m unique canonical keys `ukey` (in ka or kb; the other
+// buffer is free), shared by the device and the pipelined host builds.
+static void build_tail(uint64_t* ukey, int64_t m, DevBuf<uint64_t>& ka, DevBuf<uint64_t>& kb,
+                       int64_t n, uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g,
+                       Timer& tm) {
   const int bits = bits_for(std::max<int64_t>(n, 2));
-
-  // a1 + a2
-  DevBuf<uint64_t> ka(std::max<int64_t>(m_gen, 1), s), kb(std::max<int64_t>(m_gen, 1), s);
-  int64_t m = 0;
-  // a2 by hash set for up to 2^25 pairs (table <= 512 MB; measured C5 2.45
-  // -> 1.89 ms, C1 launch-bound 0.10 -> 0.06), by radix sort above (C3: hash
-  // 21.7 ms vs sort 18.5: random CAS into a 4.3 GB table loses to 6 streaming
-  // passes).  TC_DEDUP=sort|hash forces one (tests compare the two).
-  static const int dedup_force = [] {
-    const char* v = std::getenv("TC_DEDUP");
-    if (!v) return 0;
-    return std::string(v) == "sort" ? 1 : (std::string(v) == "hash" ? 2 : 0);
-  }();
-  const bool dedup_sort = dedup_force ? dedup_force == 1 : m_gen > (int64_t(1) << 25);
-  uint64_t* ukey = ka.get();
-  if (dedup_sort)
-    ukey = canon_unique(d_src, d_dst, m_gen, n, s, ka.get(), kb.get(), &m, &tm);
-  else
-    m = canon_unique_hash(d_src, d_dst, m_gen, n, s, ka.get(), &tm);
   g->m = m;
   tm.mark();
 
@@ -763,6 +725,158 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
   g->ms[3] = tm.ms(3, 4);
   g->ms[4] = tm.ms(4, 5);
   g->ms[5] = tm.ms(0, 5);
+}
+
+
+// ------------------------------------------------------------------ a1..a5
+void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
+                 uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g) {
+  Timer tm(s);
+  tm.mark();
+  if (n < 0) {  // num_vertices = max id + 1
+    if (m_gen == 0) {
+      n = 0;
+    } else {
+      DevBuf<int32_t> mx(2, s);
+      cub_run(s, [&](void* t, size_t& b) {
+        return cub::DeviceReduce::Max(t, b, d_src, mx.get(), m_gen, s);
+      });
+      cub_run(s, [&](void* t, size_t& b) {
+        return cub::DeviceReduce::Max(t, b, d_dst, mx.get() + 1, m_gen, s);
+      });
+      int32_t h[2];
+      TC_CUDA(cudaMemcpyAsync(h, mx.get(), sizeof(h), cudaMemcpyDeviceToHost, s));
+      TC_CUDA(cudaStreamSynchronize(s));
+      n = (int64_t)std::max(h[0], h[1]) + 1;
+      if (n < 0) n = 0;
+    }
+  }
+  g->n_input = n;
+
+  // a1 + a2
+  DevBuf<uint64_t> ka(std::max<int64_t>(m_gen, 1), s), kb(std::max<int64_t>(m_gen, 1), s);
+  int64_t m = 0;
+  // a2 by hash set for up to 2^25 pairs (table <= 512 MB; measured C5 2.45
+  // -> 1.89 ms, C1 launch-bound 0.10 -> 0.06), by radix sort above (C3: hash
+  // 21.7 ms vs sort 18.5: random CAS into a 4.3 GB table loses to 6 streaming
+  // passes).  TC_DEDUP=sort|hash forces one (tests compare the two).
+  static const int dedup_force = [] {
+    const char* v = std::getenv("TC_DEDUP");
+    if (!v) return 0;
+    return std::string(v) == "sort" ? 1 : (std::string(v) == "hash" ? 2 : 0);
+  }();
+  const bool dedup_sort = dedup_force ? dedup_force == 1 : m_gen > (int64_t(1) << 25);
+  uint64_t* ukey = ka.get();
+  if (dedup_sort)
+    ukey = canon_unique(d_src, d_dst, m_gen, n, s, ka.get(), kb.get(), &m, &tm);
+  else
+    m = canon_unique_hash(d_src, d_dst, m_gen, n, s, ka.get(), &tm);
+  build_tail(ukey, m, ka, kb, n, flags, opt, s, g, tm);
+}
+
+// The host entry point (tc_build_csr_host) for large inputs: the H2D copy of
+// the raw pairs is split into K pieces on a copy stream, and piece i is
+// canonicalised and radix-sorted on the build stream while piece i+1 is
+// still crossing PCIe; the K sorted runs are then merged pairwise
+// (cub::DeviceMerge) and deduplicated.  Only the last piece's sort, the
+// merges and the unique follow the copy (C3 K = 4: ~1/4 of the a2 sort plus
+// two merge passes instead of the whole sort).  Same unique keys as
+// canon_unique, so the same graph (tests compare the CSR).
+void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen, int64_t n,
+                      uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g) {
+  static const int pieces = [] {
+    const char* v = std::getenv("TC_H2D_PIECES");
+    const int k = v ? std::atoi(v) : 4;
+    return k == 1 || k == 2 || k == 4 || k == 8 ? k : 4;
+  }();
+  DevBuf<int32_t> ds(std::max<int64_t>(m_gen, 1), s), dd(std::max<int64_t>(m_gen, 1), s);
+  if (n < 0 || pieces == 1 || m_gen <= (int64_t(1) << 25) ||
+      m_gen / pieces > (int64_t)0x7fffffff) {  // (cub merge counts are int)
+    if (m_gen) {
+      TC_CUDA(cudaMemcpyAsync(ds.get(), h_src, sizeof(int32_t) * m_gen, cudaMemcpyHostToDevice, s));
+      TC_CUDA(cudaMemcpyAsync(dd.get(), h_dst, sizeof(int32_t) * m_gen, cudaMemcpyHostToDevice, s));
+    }
+    build_graph(ds.get(), dd.get(), m_gen, n, flags, opt, s, g);
+    return;
+  }
+  Timer tm(s);
+  tm.mark();
+  g->n_input = n;
+  const int bits = bits_for(std::max<int64_t>(n, 2));
+  const uint64_t sent = (uint64_t(1) << (2 * bits)) - 1;
+  DevBuf<uint64_t> ka(m_gen, s), kb(m_gen, s);
+  DevBuf<int> err(1, s);
+  DevBuf<int64_t> nsel(1, s);
+  DevBuf<UniqTail> tail(1, s);
+  TC_CUDA(cudaMemsetAsync(err.get(), 0, sizeof(int), s));
+  TC_CUDA(cudaMemsetAsync(nsel.get(), 0, sizeof(int64_t), s));
+  struct Res {
+    cudaStream_t cs = nullptr;
+    cudaEvent_t ready = nullptr, ev[8] = {};
+    ~Res() {
+      if (cs) {
+        cudaStreamSynchronize(cs);  // no copy may outlive the buffers it writes
+        cudaStreamDestroy(cs);
+      }
+      if (ready) cudaEventDestroy(ready);
+      for (auto e : ev)
+        if (e) cudaEventDestroy(e);
+    }
+  } r;
+  TC_CUDA(cudaStreamCreateWithFlags(&r.cs, cudaStreamNonBlocking));
+  TC_CUDA(cudaEventCreateWithFlags(&r.ready, cudaEventDisableTiming));
+  for (int i = 0; i < pieces; ++i) TC_CUDA(cudaEventCreateWithFlags(&r.ev[i], cudaEventDisableTiming));
+  TC_CUDA(cudaEventRecord(r.ready, s));  // the device buffers exist (stream-ordered allocs)
+  TC_CUDA(cudaStreamWaitEvent(r.cs, r.ready, 0));
+  int64_t lo[9];
+  for (int i = 0; i <= pieces; ++i) lo[i] = m_gen * i / pieces;
+  for (int i = 0; i < pieces; ++i) {
+    const size_t b = sizeof(int32_t) * (lo[i + 1] - lo[i]);
+    TC_CUDA(cudaMemcpyAsync(ds.get() + lo[i], h_src + lo[i], b, cudaMemcpyHostToDevice, r.cs));
+    TC_CUDA(cudaMemcpyAsync(dd.get() + lo[i], h_dst + lo[i], b, cudaMemcpyHostToDevice, r.cs));
+    TC_CUDA(cudaEventRecord(r.ev[i], r.cs));
+  }
+  // piece i: canon + sort into ka[lo_i, lo_i+1) (copied back from kb if the
+  // radix sort ends there), overlapping the copy of piece i + 1
+  for (int i = 0; i < pieces; ++i) {
+    TC_CUDA(cudaStreamWaitEvent(s, r.ev[i], 0));
+    const int64_t c = lo[i + 1] - lo[i];
+    k_canon<<<grid_for(c), TPB, 0, s>>>(ds.get() + lo[i], dd.get() + lo[i], c, n, bits, sent,
+                                        ka.get() + lo[i], err.get());
+    TC_LAUNCH();
+    cub::DoubleBuffer<uint64_t> db(ka.get() + lo[i], kb.get() + lo[i]);
+    cub_run(s, [&](void* t, size_t& b) {
+      return cub::DeviceRadixSort::SortKeys(t, b, db, c, 0, 2 * bits, s);
+    });
+    if (db.Current() != ka.get() + lo[i])
+      TC_CUDA(cudaMemcpyAsync(ka.get() + lo[i], db.Current(), sizeof(uint64_t) * c,
+                              cudaMemcpyDeviceToDevice, s));
+  }
+  tm.mark();
+  ds.reset();
+  dd.reset();
+  // pairwise merge rounds: runs of `w` pieces in `src` -> runs of 2w in `dst`
+  uint64_t* src = ka.get();
+  uint64_t* dst = kb.get();
+  for (int w = 1; w < pieces; w *= 2) {
+    for (int i = 0; i < pieces; i += 2 * w) {
+      const int64_t a = lo[i], b = lo[i + w], e = lo[i + 2 * w];
+      cub_run(s, [&](void* t, size_t& bytes) {
+        return cub::DeviceMerge::MergeKeys(t, bytes, src + a, (int)(b - a), src + b, (int)(e - b),
+                                           dst + a, cuda::std::less<uint64_t>{}, s);
+      });
+    }
+    std::swap(src, dst);
+  }
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceSelect::Unique(t, b, src, dst, nsel.get(), m_gen, s);
+  });
+  k_uniq_tail<<<1, 1, 0, s>>>(err.get(), nsel.get(), dst, tail.get());
+  TC_LAUNCH();
+  const UniqTail ut = d2h(tail.get(), s);
+  if (ut.err) fail(TC_ERR_INVALID_ARGUMENT, "vertex id < 0 or >= num_vertices in the edge list");
+  const int64_t m = ut.nsel - ((ut.nsel > 0 && ut.last == sent) ? 1 : 0);
+  build_tail(dst, m, ka, kb, n, flags, opt, s, g, tm);
 }
 
 // ------------------------------------------------------------------ f2

@@ -174,6 +174,8 @@ namespace tc {
 void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
                  uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g);
 void build_plan(tc_graph* g, const Options& opt, cudaStream_t s);
+void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen, int64_t n,
+                      uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g);
 
 // tc_build.cu, f2 sharded preprocessing (tc_shard_* in tc.h)
 int key_bits(int64_t n);

@@ -394,3 +394,18 @@ def test_dedup_paths_agree(tc):
         out[mode] = r.stdout.split()[-2:]
     assert out["sort"] == out["hash"]
     assert int(out["sort"][1]) == oracle.triangles(src, dst)
+
+
+def test_host_pipelined_build_equals_device(tc):
+    """Above 2^25 pairs tc_build_csr_host overlaps the H2D copy of piece i+1
+    with the sort of piece i and merges the sorted runs: the graph must be
+    the one tc_build_csr builds from device arrays."""
+    src, dst, n = tcgen.rmat(21, 20, 6)  # 41.9 M pairs
+    assert len(src) > (1 << 25)
+    ps = torch.from_numpy(src).pin_memory()
+    pd = torch.from_numpy(dst).pin_memory()
+    with tc.build_csr(dev(src), dev(dst), n) as g0, tc.build_csr_host(ps, pd, n) as g1:
+        for a, b in zip(g0.csr(), g1.csr()):
+            assert torch.equal(a, b)
+        assert g1.count() == g0.count()
+        assert g1.info.b_itc == g0.info.b_itc
