@@ -779,15 +779,15 @@ void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int6
 // canonicalised and radix-sorted on the build stream while piece i+1 is
 // still crossing PCIe; the K sorted runs are then merged pairwise
 // (cub::DeviceMerge) and deduplicated.  Only the last piece's sort, the
-// merges and the unique follow the copy (C3 K = 4: ~1/4 of the a2 sort plus
-// two merge passes instead of the whole sort).  Same unique keys as
+// merges and the unique follow the copy (C3 K = 8: ~1/8 of the a2 sort plus
+// three merge passes instead of the whole sort; K = 8 by default).  Same unique keys as
 // canon_unique, so the same graph (tests compare the CSR).
 void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen, int64_t n,
                       uint32_t flags, const Options& opt, cudaStream_t s, tc_graph* g) {
   static const int pieces = [] {
     const char* v = std::getenv("TC_H2D_PIECES");
-    const int k = v ? std::atoi(v) : 4;
-    return k == 1 || k == 2 || k == 4 || k == 8 ? k : 4;
+    const int k = v ? std::atoi(v) : 8;  // C3 e2e: 1 piece 157.6 ms, 2 148.9, 4 148.5, 8 144.8
+    return k == 1 || k == 2 || k == 4 || k == 8 ? k : 8;
   }();
   DevBuf<int32_t> ds(std::max<int64_t>(m_gen, 1), s), dd(std::max<int64_t>(m_gen, 1), s);
   if (n < 0 || pieces == 1 || m_gen <= (int64_t(1) << 25) ||

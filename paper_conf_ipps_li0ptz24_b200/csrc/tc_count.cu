@@ -955,9 +955,10 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
   unsigned long long acc = 0;
   if (warp < n_prod) {
     // ------------------------------------------------------------ producers
-    for (int64_t k = 0;; ++k) {
-      const int slot = (int)(k % nslots);
-      const uint32_t j = (uint32_t)(k / nslots);  // fill number of this slot
+    // slot / fill number kept incrementally (no 64-bit division per chunk)
+    int slot = 0;
+    uint32_t j = 0;  // fill number of this slot
+    for (int64_t k = 0;; ++k, slot = (slot + 1 == nslots) ? (++j, 0) : slot + 1) {
       if (j > 0) wait_empty(&empty_bar[slot], (j - 1) & 1, hint);
       const int64_t cix = c_begin + blockIdx.x + k * gridDim.x;
       if (cix >= c_end) {
@@ -975,9 +976,10 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     int* ring = tu.ring ? reinterpret_cast<int*>(smem + nslots * slot_bytes) +
                               cw * (kRingDepth * kBatchLong * 32)
                         : nullptr;
-    for (int64_t k = 0;; ++k) {
-      const int slot = (int)(k % nslots);
-      wait_full(&full_bar[slot], (uint32_t)((k / nslots) & 1), hint);
+    int slot = 0;
+    uint32_t fill = 0;
+    for (;; slot = (slot + 1 == nslots) ? (++fill, 0) : slot + 1) {
+      wait_full(&full_bar[slot], fill & 1u, hint);
       const SlotHdr h = hdr[slot];
       if (h.done) break;
       if (h.S > 0) {
@@ -985,7 +987,9 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
         const int NU = h.is_long ? h.T : c.sA[h.S];
         const int grab = h.is_long ? tu.grab_long : tu.grab_short;
         if (grab <= 0) {  // static split: a contiguous share per consumer warp
-          int w0 = (int)((int64_t)NU * cw / n_cons), w1 = (int)((int64_t)NU * (cw + 1) / n_cons);
+          // 32-bit: NU * n_cons < 2^31 (a chunk slot holds < 2^16 tiles / keys)
+          int w0 = (int)((unsigned)NU * (unsigned)cw / (unsigned)n_cons),
+              w1 = (int)((unsigned)NU * (unsigned)(cw + 1) / (unsigned)n_cons);
           if (h.is_long) {  // walk_long batches start at multiples of 8 tiles
             w0 = min((w0 + 7) & ~7, NU);
             w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
@@ -1039,7 +1043,8 @@ __global__ void __launch_bounds__(kFlatBlock, 3)
     if (h.S > 0) {
       const ChunkSmem c = slot_view(smem, h.S, h.G, h.T);  // short class only: T = 0
       const int NU = c.sA[h.S];
-      const int w0 = (int)((int64_t)NU * warp / nw), w1 = (int)((int64_t)NU * (warp + 1) / nw);
+      const int w0 = (int)((unsigned)NU * (unsigned)warp / (unsigned)nw),
+                w1 = (int)((unsigned)NU * (unsigned)(warp + 1) / (unsigned)nw);
       if (h.linear)
         acc += h.huge ? walk_short<true, true>(c, h.S, w0, w1, pv, h.ga)
                       : walk_short<true, false>(c, h.S, w0, w1, pv, h.ga);
@@ -1075,7 +1080,8 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     if (h.S > 0) {
       const ChunkSmem c = slot_view_sup(smem, h.S, h.G, h.T, h.nslots);
       const int NU = h.is_long ? h.T : c.sA[h.S];
-      const int w0 = (int)((int64_t)NU * warp / nw), w1 = (int)((int64_t)NU * (warp + 1) / nw);
+      const int w0 = (int)((unsigned)NU * (unsigned)warp / (unsigned)nw),
+                w1 = (int)((unsigned)NU * (unsigned)(warp + 1) / (unsigned)nw);
       if (h.is_long) {
         if (h.huge)
           h.linear ? walk_long_sup<true, true>(c, w0, w1, pv) : walk_long_sup<false, true>(c, w0, w1, pv);
