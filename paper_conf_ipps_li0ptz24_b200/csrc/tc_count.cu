@@ -848,10 +848,14 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
 
   // 3. hash N+(v) of every group touched by the chunk (flattened over groups,
   //    kInsU tiles of N+(v) loads in flight per producer lane)
-  constexpr int kInsU = 4;
+#ifndef TC_INS_UNROLL
+#define TC_INS_UNROLL 4
+#endif
+  constexpr int kInsU = TC_INS_UNROLL;  // N+(v) row loads in flight per producer lane
   const int pw = pt >> 5, npw = PT >> 5;
   const int NI = c.sGP[G];
-  const int i0 = (int)((int64_t)NI * pw / npw), i1 = (int)((int64_t)NI * (pw + 1) / npw);
+  const int i0 = (int)((unsigned)NI * (unsigned)pw / (unsigned)npw),
+            i1 = (int)((unsigned)NI * (unsigned)(pw + 1) / (unsigned)npw);  // NI * npw < 2^31
   auto load_row = [&](int g, int k) { return __ldg(pv.col + c.sGB[g] + k); };
   // short class: linear probing from the start when the plan says so (its
   // tables are tiny — a few keys each — and a chunk whose cuckoo insert fails
