@@ -158,7 +158,10 @@ Options resolve_options(const tc_options* o) {
   if (o->huge_degree) r.huge_degree = o->huge_degree;
   if (o->block_threads) r.block_threads = o->block_threads;
   if (o->table_factor) r.table_factor = o->table_factor;
-  if (o->long_min) r.long_min = o->long_min;
+  if (o->long_min) {
+    r.long_min = o->long_min;
+    r.long_min_auto = false;
+  }
   if (o->probe_mode) r.probe_mode = o->probe_mode;
   if (o->bitmap_factor) r.bitmap_factor = o->bitmap_factor;
   require(r.chunk_cost >= 64, "chunk_cost must be >= 64");

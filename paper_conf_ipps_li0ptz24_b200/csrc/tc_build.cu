@@ -1034,8 +1034,13 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     TC_LAUNCH();
     // a long-class tile always holds 32 keys of its own edge (walk_long shifts
     // a partial last tile back onto the edge), so long_min < 32 acts as 32
-    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m,
-                                            std::max(opt.long_min, 32), g->bits,
+    // Small graphs (C1: 10 K edges) count faster with every edge in the
+    // short class: one launch of the flat kernel instead of also starting the
+    // persistent warp-specialised one (C1 0.041 -> 0.023 ms); an explicit
+    // long_min keeps the split.
+    constexpr int64_t kSmallGraph = int64_t(1) << 20;
+    const int long_min = (opt.long_min_auto && m < kSmallGraph) ? (1 << 30) : std::max(opt.long_min, 32);
+    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m, long_min, g->bits,
                                             dead, skey.get(), sval.get(), stats.get());
     TC_LAUNCH();
   }

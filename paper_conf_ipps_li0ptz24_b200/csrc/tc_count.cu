@@ -39,13 +39,23 @@ namespace tc {
 namespace {
 
 constexpr int kMaxBlock = 1024;  // warp-specialised kernel (long class)
-constexpr int kFlatBlock = 512;  // flat kernel (short class), 3 CTAs per SM
+#ifndef TC_FLAT_BLOCK
+#define TC_FLAT_BLOCK 384
+#endif
+#ifndef TC_FLAT_CTAS
+#define TC_FLAT_CTAS 4
+#endif
+constexpr int kFlatBlock = TC_FLAT_BLOCK;  // flat kernel (short class) ...
+constexpr int kFlatCTAs = TC_FLAT_CTAS;    // ... and its CTAs per SM
 constexpr int kUnrollLong = 8;   // tail batch of the long class
 #ifndef TC_BATCH_LONG
 #define TC_BATCH_LONG 8
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
-constexpr int kUnrollShort = 4;  // tiles in flight per consumer warp (short class)
+#ifndef TC_UNROLL_SHORT
+#define TC_UNROLL_SHORT 2
+#endif
+constexpr int kUnrollShort = TC_UNROLL_SHORT;  // tiles in flight per consumer warp (short class)
 #ifndef TC_RING_DEPTH
 #define TC_RING_DEPTH 2
 #endif
@@ -1032,7 +1042,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
 // consumer split: a short chunk's table building is as much work as its
 // probing), one chunk slot per CTA and 3 CTAs per SM so that one CTA's
 // staging and building latency overlaps the others' probing.
-__global__ void __launch_bounds__(kFlatBlock, 3)
+__global__ void __launch_bounds__(kFlatBlock, kFlatCTAs)
     k_count_flat(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
                  unsigned long long* __restrict__ out) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -1217,7 +1227,7 @@ int max_flat_chunk_smem() {
   int dev = 0, per_sm = 0;
   TC_CUDA(cudaGetDevice(&dev));
   TC_CUDA(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
-  const int per_cta = per_sm / 3 - 1024 - static_smem((const void*)k_count_flat);  // 1 KB reserved per CTA
+  const int per_cta = per_sm / kFlatCTAs - 1024 - static_smem((const void*)k_count_flat);  // 1 KB reserved per CTA
   return std::min(per_cta, optin_smem() - static_smem((const void*)k_count_flat)) & ~15;
 }
 

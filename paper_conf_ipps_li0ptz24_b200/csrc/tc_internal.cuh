@@ -75,6 +75,7 @@ struct Options {
   int block_threads = 1024;
   int table_factor = 6;   // C3/C2/C5 sweep (r19o/r19p): 3 -> 6 with bitmap_factor 12: -7% / -18% / -23%
   int long_min = 32;
+  bool long_min_auto = true;  // long_min not given: graphs under kSmallGraph edges are all short
   int probe_mode = 0;
   int bitmap_factor = 12;  // <= 0: never
 };

@@ -45,6 +45,7 @@ def gpu_count(tc, src, dst, n=None, **kw):
 def test_closed_forms(tc, name):
     (src, dst, n), t = graphs.closed_form_cases()[name]
     assert gpu_count(tc, src, dst, n) == t
+    assert gpu_count(tc, src, dst, n, options={"long_min": 32}) == t  # with the long class
 
 
 def test_karate(tc, golden):
@@ -72,6 +73,7 @@ def test_fig14_suffix_example(tc):
 def test_c1_rmat10_seeds(tc, seed):
     src, dst, n = tcgen.CONFIGS["C1"].generate(seed)
     r = oracle.count(src, dst, n)
+    assert gpu_count(tc, src, dst, n, options={"long_min": 32}) == r.triangles
     with tc.build_csr(dev(src), dev(dst), n) as g:
         assert g.count() == r.triangles
         assert g.m == r.m and g.n == r.n_active
@@ -141,6 +143,12 @@ def test_chung_lu_small(tc):
     dict(bitmap_factor=-1), dict(bitmap_factor=1), dict(bitmap_factor=64),
     dict(bitmap_factor=64, probe_mode=1), dict(bitmap_factor=64, long_min=1 << 30),
     dict(bitmap_factor=-1, long_min=1),
+    # explicit long_min = 32: the two-class split large graphs use (a graph this
+    # small is otherwise all short class)
+    dict(long_min=32), dict(long_min=32, chunk_cost=64), dict(long_min=32, block_threads=128),
+    dict(long_min=32, probe_mode=1), dict(long_min=32, bitmap_factor=-1),
+    dict(long_min=32, table_factor=2), dict(long_min=32, huge_degree=16),
+    dict(long_min=32, bitmap_factor=64),
 ])
 def test_plan_options_never_change_count(tc, opts):
     src, dst, n = tcgen.rmat(13, 16, 11)

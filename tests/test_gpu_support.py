@@ -50,9 +50,10 @@ def check_full(tc, src, dst, n, **kw):
 
 @pytest.mark.parametrize("name", ["K3", "K10", "K33", "W10", "F300", "K3,4,5", "K5,6,7,8",
                                   "Q4", "star1000", "petersen"])
-def test_closed_forms(tc, name):
+@pytest.mark.parametrize("long_min", [None, 32])  # None: small graphs are all short class
+def test_closed_forms(tc, name, long_min):
     (src, dst, n), _ = graphs.closed_form_cases()[name]
-    check_full(tc, src, dst, n)
+    check_full(tc, src, dst, n, options=None if long_min is None else {"long_min": long_min})
 
 
 def test_complete_graph_value(tc):
@@ -71,6 +72,7 @@ def test_golden(tc, golden, name, n):
 def test_c1_seeds(tc, seed):
     src, dst, n = tcgen.CONFIGS["C1"].generate(seed)
     check_full(tc, src, dst, n)
+    check_full(tc, src, dst, n, options={"long_min": 32})  # with the long (tile) class
 
 
 @pytest.mark.parametrize("scale,ef,seed", [(14, 16, 1), (16, 16, 2)])
@@ -90,6 +92,9 @@ def test_skewed_rmat(tc):
     {"bitmap_factor": 64},                # bitmaps almost everywhere
     {"huge_degree": 16},                  # global binary search for d+(v) > 16
     {"long_min": 1},                      # all edges in the tile class
+    {"long_min": 32},                     # the split the large graphs use
+    {"long_min": 32, "probe_mode": 1},
+    {"long_min": 32, "bitmap_factor": -1},
     {"long_min": 1 << 30},                # all edges flattened
     {"table_factor": 2, "chunk_cost": 256},
 ])
