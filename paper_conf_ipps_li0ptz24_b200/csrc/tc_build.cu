@@ -1003,7 +1003,7 @@ Tuning tuning_from_env() {
   t.wait_hint_ns = get("TC_WAIT_HINT", t.wait_hint_ns, 0, 10000000);
   t.prefetch = get("TC_PREFETCH", t.prefetch, 0, 1);
   t.ring = get("TC_RING", t.ring, 0, 1);
-  t.cs_div = get("TC_CS_DIV", t.cs_div, 1, 64);
+  t.cs_div = get("TC_CS_DIV", t.cs_div, 0, 64);
   t.short_linear = get("TC_SHORT_LINEAR", t.short_linear, 0, 1);
   return t;
 }
@@ -1142,8 +1142,11 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   // Chunking, per class: cost chunks (long class 4x larger: its edges carry
   // ~150 keys each), then every chunk is split where its SMEM layout would
   // exceed one of the count kernel's chunk slots (only outliers split).
+  // short chunks of half the cost when edges carry ~1 key (C5 road lattice:
+  // 1.05 keys per live edge, 0.114 -> 0.073 ms; C2 at 5.4 keys: neutral)
+  const int cs_div = P.tune.cs_div ? P.tune.cs_div : (P.keys_total < 2 * S ? 2 : 1);
   const int64_t CL = std::max<int64_t>(4ll * opt.chunk_cost, 64),
-                CS = std::max<int64_t>(opt.chunk_cost / P.tune.cs_div, 64);
+                CS = std::max<int64_t>(opt.chunk_cost / cs_div, 64);
   {
     const int64_t nL0 = (cost_long + CL - 1) / CL, nS0 = (cost_short + CS - 1) / CS, nc0 = nL0 + nS0;
     DevBuf<int64_t> cs0(nc0 + 1, s), pieces(std::max<int64_t>(nc0, 1), s), poff(nc0 + 1, s);

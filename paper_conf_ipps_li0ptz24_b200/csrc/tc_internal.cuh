@@ -138,8 +138,9 @@ struct Tuning {
   int wait_hint_ns = 0;   // mbarrier try_wait suspend hint (0 = none)
   int prefetch = 0;       // long class: L2 bulk prefetch of each edge's keys at staging
   int ring = 0;           // long class: key loads as cp.async into per-warp SMEM rings
-  int cs_div = 1;         // short-class chunk cost = chunk_cost / cs_div
-  int short_linear = 0;   // short class: linear-probing tables (no cuckoo attempt)
+  int cs_div = 0;         // short-class chunk cost = chunk_cost / cs_div (0: auto, 2 when the live
+                          // edges carry < 2 keys on average, e.g. road graphs, else 1)
+  int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
 };
 Tuning tuning_from_env();
 

@@ -394,8 +394,8 @@ def test_dedup_paths_agree(tc):
             "h = hashlib.sha256(); [h.update(x.cpu().numpy().tobytes()) for x in g.csr()];"
             "print(h.hexdigest(), g.count())") % ROOT
     out = {}
-    for mode in ("sort", "hash"):
-        env = dict(os.environ, TC_DEDUP=mode)
+    for mode, env_kv in (("sort", {"TC_DEDUP": "sort"}), ("hash", {"TC_DEDUP": "hash"})):
+        env = dict(os.environ, **env_kv)
         r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
                            timeout=300)
         assert r.returncode == 0, r.stderr[-2000:]
