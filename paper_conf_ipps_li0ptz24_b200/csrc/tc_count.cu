@@ -647,7 +647,10 @@ __device__ __forceinline__ int sup_lookup_any(const ChunkSmem& c, const PlanView
                 : sup_find<false>(c.sHash, info.x, info.y, key);
 }
 
-constexpr int kUnrollSup = 4;
+#ifndef TC_UNROLL_SUP
+#define TC_UNROLL_SUP 6
+#endif
+constexpr int kUnrollSup = TC_UNROLL_SUP;  // tiles in flight per warp (support mode)
 
 // Support-mode lookup of key in group gl's table; kHuge = the chunk has
 // groups probed in global memory (otherwise that path is not compiled in).
