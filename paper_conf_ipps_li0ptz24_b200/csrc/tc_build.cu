@@ -324,7 +324,8 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint64_t* __r
                            const int32_t* __restrict__ gincl, int64_t S, int64_t S_long,
                            int bits, const int64_t* __restrict__ row_ptr,
                            int huge_degree, int table_factor, int bitmap_factor,
-                           int64_t max_table_slots, const int32_t* __restrict__ col,
+                           int64_t max_slots_long, int64_t max_slots_short,
+                           const int32_t* __restrict__ col,
                            int32_t* __restrict__ grp_code, int64_t* __restrict__ seg_start,
                            int32_t* __restrict__ seg_len, int32_t* __restrict__ seg_group,
                            int64_t* __restrict__ units, int64_t* __restrict__ grp_row,
@@ -351,21 +352,31 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint64_t* __r
       //  hash: table_factor * d slots (load <= 1/table_factor, > d so a
       //    linear probe always meets an empty slot); code = slots.
       // Sizes are multiples of 4 for 16-B initialisation.
+      // The cap is the SMEM of the class's own kernel (a long group's table
+      // lives in a k_count slot, a short group's in a k_count_flat chunk); a
+      // hash table that would exceed it at table_factor falls back to load
+      // 1/3, then 1/2, before the group is declared huge (C4's hubs, d+ up to
+      // 4,218: with one cap for both classes they went to global binary search).
+      const int64_t maxs = s < S_long ? max_slots_long : max_slots_short;
       int64_t slots = 0;
       int32_t code = 0;
       if (d <= huge_degree) {
         const int64_t w0 = col[rs] >> 5, w1 = col[rs + d - 1] >> 5;
+        const int64_t bw = (w1 - w0 + 1 + 3) & ~int64_t(3);
         // (the first word must fit the count kernel's 26-bit tile code)
-        if (bitmap_factor > 0 && w0 < (1 << 25) && w1 - w0 + 1 <= (int64_t)bitmap_factor * d) {
-          slots = (w1 - w0 + 1 + 3) & ~int64_t(3);
+        if (bitmap_factor > 0 && w0 < (1 << 25) && w1 - w0 + 1 <= (int64_t)bitmap_factor * d &&
+            bw <= maxs) {
+          slots = bw;
           code = -(int32_t)w0;
         } else {
           int64_t want = d * table_factor;
+          if (want > maxs) want = 3 * d;  // load 1/3: two-choice inserts still rarely fail
+          if (want > maxs) want = 2 * d;
           if (want < d + 1) want = d + 1;
           slots = (want + 3) & ~int64_t(3);
           code = (int32_t)slots;
+          if (slots > maxs) slots = code = 0;
         }
-        if (slots > max_table_slots) slots = 0;
       }
       grp_code[g] = code;
       grp_slots[g] = slots;
@@ -1091,7 +1102,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   // of it (bigger tables are "huge": probed in global memory)
   const int64_t slot_limit = max_chunk_smem(P.tune);
   const int64_t flat_limit = max_flat_chunk_smem();
-  const int64_t max_table_slots = std::min(slot_limit, flat_limit) / 8;
+  const int64_t max_slots_long = slot_limit / 8, max_slots_short = flat_limit / 8;  // half a slot
   P.seg_start = DevBuf<int64_t>(S, s, true);
   P.seg_len = DevBuf<int32_t>(S, s, true);
   P.seg_group = DevBuf<int32_t>(S, s, true);
@@ -1100,7 +1111,8 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted, val_sorted, gincl.get(), S, S_long,
                                          g->bits, row_ptr,
                                          opt.huge_degree, opt.table_factor, opt.bitmap_factor,
-                                         max_table_slots, col, P.grp_code.get(), P.seg_start.get(),
+                                         max_slots_long, max_slots_short, col, P.grp_code.get(),
+                                         P.seg_start.get(),
                                          P.seg_len.get(), P.seg_group.get(), units.get(),
                                          grp_row.get(), grp_d.get(), grp_slots.get());
   TC_LAUNCH();
