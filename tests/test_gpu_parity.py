@@ -417,3 +417,16 @@ def test_host_pipelined_build_equals_device(tc):
             assert torch.equal(a, b)
         assert g1.count() == g0.count()
         assert g1.info.b_itc == g0.info.b_itc
+
+
+@pytest.mark.parametrize("n,opts", [
+    (1500, dict(table_factor=16, bitmap_factor=-1, long_min=32)),   # 16 d+ > the cap -> load 1/3
+    (3000, dict(table_factor=16, bitmap_factor=-1, long_min=32)),   # -> load 1/3 (long) and 1/2 (short)
+    (3000, dict(table_factor=16, bitmap_factor=-1, long_min=1 << 30)),
+])
+def test_table_cap_fallbacks(tc, n, opts):
+    """Hash tables that would exceed their class's SMEM cap at table_factor
+    fall back to load 1/3, then 1/2, before going to global binary search;
+    the count is unchanged (K_n: C(n, 3), > 2^32 at n = 3000)."""
+    (src, dst, nn), t = graphs.complete(n)
+    assert gpu_count(tc, src, dst, nn, options=opts) == t
