@@ -1016,6 +1016,7 @@ Tuning tuning_from_env() {
   t.ring = get("TC_RING", t.ring, 0, 1);
   t.cs_div = get("TC_CS_DIV", t.cs_div, 0, 64);
   t.short_linear = get("TC_SHORT_LINEAR", t.short_linear, 0, 1);
+  t.interleave = get("TC_INTERLEAVE", t.interleave, 0, 1);
   return t;
 }
 

@@ -975,9 +975,16 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     // slot / fill number kept incrementally (no 64-bit division per chunk)
     int slot = 0;
     uint32_t j = 0;  // fill number of this slot
+    // This CTA's chunks are c_begin + b + i * grid, i < nk.  Plan order runs
+    // from many small tables (producer-heavy) to hub tables with many tiles
+    // (consumer-heavy); with tu.interleave the CTA alternates between the
+    // front and the back of its list so both sides stay busy.
+    const int64_t mine = c_end - c_begin - (int64_t)blockIdx.x;
+    const int64_t nk = mine > 0 ? (mine + gridDim.x - 1) / gridDim.x : 0;
     for (int64_t k = 0;; ++k, slot = (slot + 1 == nslots) ? (++j, 0) : slot + 1) {
       if (j > 0) wait_empty(&empty_bar[slot], (j - 1) & 1, hint);
-      const int64_t cix = c_begin + blockIdx.x + k * gridDim.x;
+      const int64_t i = !tu.interleave ? k : ((k & 1) ? nk - 1 - (k >> 1) : (k >> 1));
+      const int64_t cix = k < nk ? c_begin + blockIdx.x + i * gridDim.x : c_end;
       if (cix >= c_end) {
         if (threadIdx.x == 0) hdr[slot].done = 1;
         mbar_arrive(&full_bar[slot]);

@@ -129,7 +129,7 @@ __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_
 }
 
 // Count-kernel launch tuning (not part of the C-ABI; TC_SLOTS, TC_GRAB_LONG,
-// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_PREFETCH, TC_RING, TC_CS_DIV, TC_SHORT_LINEAR override the defaults for sweeps).
+// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_PREFETCH, TC_RING, TC_CS_DIV, TC_SHORT_LINEAR, TC_INTERLEAVE override the defaults for sweeps).
 struct Tuning {
   int slots = 3;          // chunk slots in SMEM (2..4)
   int grab_long = 0;      // tiles per consumer grab, long class (0 = static split)
@@ -141,6 +141,7 @@ struct Tuning {
   int cs_div = 0;         // short-class chunk cost = chunk_cost / cs_div (0: auto, 2 when the live
                           // edges carry < 2 keys on average, e.g. road graphs, else 1)
   int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
+  int interleave = 0;     // long class: each CTA alternates the front and back of its chunk list
 };
 Tuning tuning_from_env();
 
