@@ -651,6 +651,9 @@ __device__ __forceinline__ int sup_lookup_any(const ChunkSmem& c, const PlanView
 #define TC_UNROLL_SUP 6
 #endif
 constexpr int kUnrollSup = TC_UNROLL_SUP;  // tiles in flight per warp (support mode)
+#ifndef TC_SUP_AGG
+#define TC_SUP_AGG 1
+#endif
 
 // Support-mode lookup of key in group gl's table; kHuge = the chunk has
 // groups probed in global memory (otherwise that path is not compiled in).
@@ -681,6 +684,12 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
   const int lane = threadIdx.x & 31;
   const int32_t* colL = lane_base(pv.col, lane);
   unsigned* supL = lane_base_u(pv.sup, lane);
+#if TC_SUP_AGG
+  // consecutive tiles of one long suffix share their edge (u, v): its count
+  // is summed over the run and added once when the edge changes
+  unsigned run = 0;
+  uint32_t cur = 0u;
+#endif
   for (int t = t0; t < t1; t += kUnrollSup) {
     int32_t key[kUnrollSup];
     uint32_t p[kUnrollSup], vr[kUnrollSup], own[kUnrollSup];
@@ -702,9 +711,21 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
         atomicAdd(supL + p[u], 1u);                        // (u, w)
         atomicAdd(pv.sup + (vr[u] + (uint32_t)idx), 1u);   // (v, w)
       }
+#if TC_SUP_AGG
+      if (own[u] != cur) {
+        if (lane == 0 && run) atomicAdd(pv.sup + cur, run);  // (u, v)
+        run = 0;
+        cur = own[u];
+      }
+      run += (unsigned)__popc(bal);
+#else
       if (lane == 0 && bal) atomicAdd(pv.sup + own[u], (unsigned)__popc(bal));  // (u, v)
+#endif
     }
   }
+#if TC_SUP_AGG
+  if (lane == 0 && run) atomicAdd(pv.sup + cur, run);  // (u, v)
+#endif
 }
 
 // SHORT class, support mode: flat keys [k0w, k1w) of the chunk.
