@@ -654,6 +654,9 @@ constexpr int kUnrollSup = TC_UNROLL_SUP;  // tiles in flight per warp (support 
 #ifndef TC_SUP_AGG
 #define TC_SUP_AGG 1
 #endif
+#ifndef TC_SUP_FAST
+#define TC_SUP_FAST 1
+#endif
 
 // Support-mode lookup of key in group gl's table; kHuge = the chunk has
 // groups probed in global memory (otherwise that path is not compiled in).
@@ -703,13 +706,44 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
       g6[u] = (t + u < t1) ? c.sT3[tt] : 0;
       key[u] = lane < (g6[u] & 63) ? __ldg(colL + p[u]) : -2;
     }
+#if TC_SUP_FAST
+    // warp-uniform fast path when every tile of the batch meets a bitmap
+    // table (most batches on RMAT): all table reads issued before any use
+    int2 inf[kUnrollSup];
+    bool all_bm = true;
 #pragma unroll
     for (int u = 0; u < kUnrollSup; ++u) {
-      const int idx = key[u] >= 0 ? sup_lookup<kLinear, kHuge>(c, pv, g6[u] >> 6, vr[u], key[u]) : -1;
-      const unsigned bal = __ballot_sync(0xffffffffu, idx >= 0);
-      if (idx >= 0) {
-        atomicAdd(supL + p[u], 1u);                        // (u, w)
-        atomicAdd(pv.sup + (vr[u] + (uint32_t)idx), 1u);   // (v, w)
+      inf[u] = c.sInfo[g6[u] >> 6];
+      all_bm &= inf[u].y <= 0 && (!kHuge || inf[u].x >= 0);
+    }
+    int idx[kUnrollSup];
+    if (all_bm) {
+      const int2* H2 = reinterpret_cast<const int2*>(c.sHash);
+      int2 e[kUnrollSup];
+#pragma unroll
+      for (int u = 0; u < kUnrollSup; ++u) e[u] = H2[inf[u].x + max((key[u] >> 5) + inf[u].y, 0)];
+#pragma unroll
+      for (int u = 0; u < kUnrollSup; ++u) {
+        const unsigned bits = ~(unsigned)e[u].x, b = (unsigned)key[u] & 31u;
+        idx[u] = (key[u] >= 0 && ((bits >> b) & 1u)) ? e[u].y + __popc(bits & ((1u << b) - 1u)) : -1;
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < kUnrollSup; ++u)
+        idx[u] = key[u] >= 0 ? sup_lookup<kLinear, kHuge>(c, pv, g6[u] >> 6, vr[u], key[u]) : -1;
+    }
+#endif
+#pragma unroll
+    for (int u = 0; u < kUnrollSup; ++u) {
+#if TC_SUP_FAST
+      const int id = idx[u];
+#else
+      const int id = key[u] >= 0 ? sup_lookup<kLinear, kHuge>(c, pv, g6[u] >> 6, vr[u], key[u]) : -1;
+#endif
+      const unsigned bal = __ballot_sync(0xffffffffu, id >= 0);
+      if (id >= 0) {
+        atomicAdd(supL + p[u], 1u);                       // (u, w)
+        atomicAdd(pv.sup + (vr[u] + (uint32_t)id), 1u);   // (v, w)
       }
 #if TC_SUP_AGG
       if (own[u] != cur) {
