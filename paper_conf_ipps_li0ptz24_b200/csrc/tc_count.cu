@@ -657,6 +657,9 @@ constexpr int kUnrollSup = TC_UNROLL_SUP;  // tiles in flight per warp (support 
 #ifndef TC_SUP_FAST
 #define TC_SUP_FAST 1
 #endif
+#ifndef TC_SUP_SHORT_AGG
+#define TC_SUP_SHORT_AGG 0
+#endif
 
 // Support-mode lookup of key in group gl's table; kHuge = the chunk has
 // groups probed in global memory (otherwise that path is not compiled in).
@@ -765,6 +768,58 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
 // SHORT class, support mode: flat keys [k0w, k1w) of the chunk.
 __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0w, int k1w,
                                                const PlanView& pv, bool linear) {
+#if TC_SUP_SHORT_AGG
+  // warp_walk's loop with the (u, v) count summed per segment: the lanes of
+  // one segment are contiguous, so its first lane adds the hits of the lanes
+  // up to the next segment's first lane in one atomic
+  if (k0w >= k1w) return;
+  const int lane = threadIdx.x & 31;
+  const unsigned below = (1u << lane) - 1u;
+  int s = seg_of(c.sA, S, k0w);
+  for (int k0 = k0w; k0 < k1w; k0 += 32 * kUnrollSup) {
+    int seg[kUnrollSup];
+#pragma unroll
+    for (int u = 0; u < kUnrollSup; ++u) {
+      const int t0 = k0 + 32 * u;
+      const int j = s + 1 + lane;
+      const int pos = (j <= S) ? c.sA[j] - t0 : 64;
+      const unsigned bit = (pos >= 1 && pos <= 32) ? (1u << (pos - 1)) : 0u;
+      const unsigned M = __reduce_or_sync(0xffffffffu, bit);
+      seg[u] = s + __popc(M & below);
+      s += __popc(M);
+    }
+    int32_t key[kUnrollSup];
+#pragma unroll
+    for (int u = 0; u < kUnrollSup; ++u) {
+      const int k = k0 + 32 * u + lane;
+      key[u] = k < k1w ? __ldg(pv.col + c.sB[seg[u]] + k) : -1;
+    }
+#pragma unroll
+    for (int u = 0; u < kUnrollSup; ++u) {
+      const int k = k0 + 32 * u + lane;
+      const int sg = seg[u];
+      int idx = -1;
+      if (k < k1w) {
+        const int gl = c.sD[sg];
+        idx = sup_lookup_any(c, pv, gl, key[u], linear);
+        if (idx >= 0) {
+          atomicAdd(pv.sup + c.sB[sg] + k, 1u);                  // (u, w)
+          atomicAdd(pv.sup + c.sGB[gl] + c.sGP[gl] + idx, 1u);   // (v, w)
+        }
+      }
+      const unsigned H = __ballot_sync(0xffffffffu, idx >= 0);
+      const int prev = __shfl_up_sync(0xffffffffu, sg, 1);
+      const bool first = k < k1w && (lane == 0 || prev != sg);
+      const unsigned F = __ballot_sync(0xffffffffu, first);
+      if (first) {
+        const unsigned after = F & ~(below | (1u << lane));  // later segment starts
+        const unsigned span = (after ? (after & (0u - after)) - 1u : 0xffffffffu) & ~below;
+        const int n = __popc(H & span);
+        if (n) atomicAdd(pv.sup + c.sE[sg], (unsigned)n);     // (u, v)
+      }
+    }
+  }
+#else
   auto load = [&](int sg, int k) { return __ldg(pv.col + c.sB[sg] + k); };
   warp_walk<kUnrollSup>(c.sA, S, k0w, k1w, load, [&](int sg, int k, int32_t key) {
     const int gl = c.sD[sg];
@@ -775,6 +830,7 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
       atomicAdd(pv.sup + c.sE[sg], 1u);                      // (u, v)
     }
   });
+#endif
 }
 
 // ------------------------------------------------------------------ producers
