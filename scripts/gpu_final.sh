@@ -6,3 +6,6 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/${TAG}_smoke
 timeout 900 python bench.py --out $O/${TAG}_bench_c3.json > $O/${TAG}_bench_c3.log 2>&1
 timeout 900 python bench.py --impl reference --out $O/${TAG}_reference_c3.json > /dev/null 2>&1
 echo done > $O/${TAG}_done.txt
+timeout 600 python bench.py --mode support --no-sharded --out $O/${TAG}_bench_support_c3.json > /dev/null 2>&1
+timeout 600 python bench.py --mode support --config C2 --no-sharded --out $O/${TAG}_bench_support_c2.json > /dev/null 2>&1
+echo done2 >> $O/${TAG}_done.txt
