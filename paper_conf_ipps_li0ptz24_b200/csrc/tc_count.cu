@@ -648,7 +648,7 @@ __device__ __forceinline__ int sup_lookup_any(const ChunkSmem& c, const PlanView
 }
 
 #ifndef TC_UNROLL_SUP
-#define TC_UNROLL_SUP 6
+#define TC_UNROLL_SUP 5
 #endif
 constexpr int kUnrollSup = TC_UNROLL_SUP;  // tiles in flight per warp (support mode)
 #ifndef TC_SUP_AGG
