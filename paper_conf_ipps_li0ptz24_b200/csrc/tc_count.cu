@@ -660,6 +660,9 @@ constexpr int kUnrollSup = TC_UNROLL_SUP;  // tiles in flight per warp (support 
 #ifndef TC_SUP_SHORT_AGG
 #define TC_SUP_SHORT_AGG 0
 #endif
+#ifndef TC_SUP_MIX
+#define TC_SUP_MIX 0
+#endif
 
 // Support-mode lookup of key in group gl's table; kHuge = the chunk has
 // groups probed in global memory (otherwise that path is not compiled in).
@@ -713,12 +716,14 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
     // warp-uniform fast path when every tile of the batch meets a bitmap
     // table (most batches on RMAT): all table reads issued before any use
     int2 inf[kUnrollSup];
-    bool all_bm = true;
+    bool all_bm = true, no_huge = true;
 #pragma unroll
     for (int u = 0; u < kUnrollSup; ++u) {
       inf[u] = c.sInfo[g6[u] >> 6];
-      all_bm &= inf[u].y <= 0 && (!kHuge || inf[u].x >= 0);
+      no_huge &= !kHuge || inf[u].x >= 0;
+      all_bm &= inf[u].y <= 0;
     }
+    all_bm &= no_huge;
     int idx[kUnrollSup];
     if (all_bm) {
       const int2* H2 = reinterpret_cast<const int2*>(c.sHash);
@@ -730,6 +735,31 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
         const unsigned bits = ~(unsigned)e[u].x, b = (unsigned)key[u] & 31u;
         idx[u] = (key[u] >= 0 && ((bits >> b) & 1u)) ? e[u].y + __popc(bits & ((1u << b) - 1u)) : -1;
       }
+#if TC_SUP_MIX
+    } else if (!kLinear && no_huge) {
+      // bitmaps and two-choice hash tables mixed: both candidate entries of
+      // every tile read before any use (a bitmap tile reads its word twice)
+      const int2* H2 = reinterpret_cast<const int2*>(c.sHash);
+      int2 e1[kUnrollSup], e2[kUnrollSup];
+#pragma unroll
+      for (int u = 0; u < kUnrollSup; ++u) {
+        const int code = inf[u].y;
+        const uint32_t n = (uint32_t)code;
+        const int i1 = code <= 0 ? max((key[u] >> 5) + code, 0) : (int)hash1(key[u], n);
+        const int i2 = code <= 0 ? i1 : (int)hash2(key[u], n);
+        e1[u] = H2[inf[u].x + i1];
+        e2[u] = H2[inf[u].x + i2];
+      }
+#pragma unroll
+      for (int u = 0; u < kUnrollSup; ++u) {
+        if (inf[u].y <= 0) {
+          const unsigned bits = ~(unsigned)e1[u].x, b = (unsigned)key[u] & 31u;
+          idx[u] = (key[u] >= 0 && ((bits >> b) & 1u)) ? e1[u].y + __popc(bits & ((1u << b) - 1u)) : -1;
+        } else {
+          idx[u] = key[u] < 0 ? -1 : e1[u].x == key[u] ? e1[u].y : e2[u].x == key[u] ? e2[u].y : -1;
+        }
+      }
+#endif
     } else {
 #pragma unroll
       for (int u = 0; u < kUnrollSup; ++u)
