@@ -651,6 +651,10 @@ __device__ __forceinline__ int sup_lookup_any(const ChunkSmem& c, const PlanView
 #define TC_UNROLL_SUP 5
 #endif
 constexpr int kUnrollSup = TC_UNROLL_SUP;  // tiles in flight per warp (support mode)
+#ifndef TC_UNROLL_SUP_SHORT
+#define TC_UNROLL_SUP_SHORT 3
+#endif
+constexpr int kUnrollSupShort = TC_UNROLL_SUP_SHORT;  // 32-key steps in flight (short class)
 #ifndef TC_SUP_AGG
 #define TC_SUP_AGG 1
 #endif
@@ -851,7 +855,7 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
   }
 #else
   auto load = [&](int sg, int k) { return __ldg(pv.col + c.sB[sg] + k); };
-  warp_walk<kUnrollSup>(c.sA, S, k0w, k1w, load, [&](int sg, int k, int32_t key) {
+  warp_walk<kUnrollSupShort>(c.sA, S, k0w, k1w, load, [&](int sg, int k, int32_t key) {
     const int gl = c.sD[sg];
     const int idx = sup_lookup_any(c, pv, gl, key, linear);
     if (idx >= 0) {
