@@ -66,6 +66,8 @@ def parse():
     ap.add_argument("--reduce", default="nccl", choices=["nccl", "fused"],
                     help="cross-GPU sum of the partial counts: NCCL all_reduce, or the library's "
                          "own over NVLink peer memory (tc_count_range_fused, SURVEY.md §8(f) f4)")
+    ap.add_argument("--no-balance", action="store_true",
+                    help="skip the N = 1 emulated multi-GPU balance measurement")
     ap.add_argument("--no-sharded", action="store_true",
                     help="skip the sharded-build measurement (tc_shard_*, SURVEY.md §8(f) f2)")
     ap.add_argument("--mode", default="count", choices=["count", "support"],
@@ -101,13 +103,41 @@ def peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def profile_traffic(cfg):
-    """dram bytes per launch of the count kernel from the committed ncu summary."""
+SRC_GLOBS = ("paper_conf_ipps_li0ptz24_b200/csrc", "include", "Makefile")
+
+
+def src_hash():
+    """sha256 (16 hex) over the sources that make libtc.so: the key that ties a
+    committed ncu capture (profiles/ncu_summary.json) to the benched tree."""
+    import hashlib
+    h = hashlib.sha256()
+    files = []
+    for g in SRC_GLOBS:
+        p = os.path.join(ROOT, g)
+        if os.path.isdir(p):
+            files += [os.path.join(p, f) for f in sorted(os.listdir(p))
+                      if f.endswith((".cu", ".cuh", ".h"))]
+        elif os.path.exists(p):
+            files.append(p)
+    for f in files:
+        h.update(os.path.relpath(f, ROOT).encode())
+        h.update(open(f, "rb").read())
+    return h.hexdigest()[:16]
+
+
+def profile_kernel(cfg, kernel):
+    """ncu counters of `kernel` for this config from the committed summary, or
+    (None, why) when it was not captured from these exact sources."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if not os.path.exists(p):
-        return None
+        return None, "no profiles/ncu_summary.json"
     d = json.load(open(p)).get(cfg)
-    return None if not d else d.get("dram_bytes_per_launch")
+    if not d or "kernels" not in d:
+        return None, f"no capture for {cfg}"
+    if d.get("src_hash") != src_hash():
+        return None, f"capture {d.get('tag')} is of other sources ({d.get('src_hash')} != {src_hash()})"
+    k = d["kernels"].get(kernel)
+    return (k, d.get("tag")) if k else (None, f"{kernel} not in capture {d.get('tag')}")
 
 
 class ClockSampler:
@@ -362,13 +392,18 @@ def main():
     if a.mode == "support":
         return bench_support(a, tc, g, info, src, dst, n, gen_s, build_wall_ms, world, rank)
 
-    bounds = g.partition(world)
+    # cost-balanced ranges: at N > 1 every rank calibrates the per-class cost
+    # weights and the ranks agree on their average (one all_reduce)
+    weights = tc.agreed_weights(g) if world > 1 else None
+    bounds = g.partition(world, weights) if weights else g.partition(world)
     e0, e1 = bounds[rank], bounds[rank + 1]
-    keys_share = 1.0
-    if world > 1:
-        # this rank's share of the probe keys, for its roofline bytes
-        keys_share = (e1 - e0) / max(1, info.m_live)
-    out = torch.zeros(1, dtype=torch.int64, device=dev)
+    # the rank's range split at the class boundary: the long class is k_count
+    # (a8), the short class k_count_flat (a7); one step = both calls, with an
+    # event between them so the dominant kernel is timed on its own
+    mlong = int(info.m_live_long)
+    l0, l1 = e0, max(e0, min(e1, mlong))
+    s0, s1 = max(e0, min(e1, mlong)), e1
+    out = torch.zeros(2, dtype=torch.int64, device=dev)
     flush = torch.empty(a.flush_mb << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
 
@@ -376,49 +411,88 @@ def main():
         raise SystemExit("--variant runs on one GPU")
 
     fused = tc.FusedSum() if a.reduce == "fused" and not a.variant else None
+    split = fused is None and not a.variant
 
-    def step(ev_mid=None):
+    def step(ev_mid=None, ev_cnt=None):
         if a.variant:
-            g.count_variant(a.variant, out=out)
-        elif fused is not None:  # count + the library's own cross-GPU sum (f4)
-            fused.count_range(g, e0, e1, out=out)
+            g.count_variant(a.variant, out=out[0:1])
+        elif fused is not None:  # count + the library's own cross-GPU sum in the last CTA (f4)
+            fused.count_range(g, e0, e1, out=out[0:1])
         else:
-            g.count_range(e0, e1, out=out)
-        if ev_mid is not None:
-            ev_mid.record(stream)
+            g.count_range(l0, l1, out=out[0:1])
+            if ev_mid is not None:
+                ev_mid.record(stream)
+            g.count_range(s0, s1, out=out[1:2])
+        if ev_cnt is not None:
+            ev_cnt.record(stream)
         if world > 1 and fused is None:
             dist.all_reduce(out)
+
+    def total():
+        return int(out[0].item() + (out[1].item() if split else 0)) & (2**64 - 1)
 
     for _ in range(max(1, a.warmup)):
         step()
     torch.cuda.synchronize()
-    T = int(out.item()) & (2**64 - 1)
+    T = total()
 
     sampler = ClockSampler(torch.cuda.current_device())
     sampler.start()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
-            torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(a.steps)]
     for i in range(a.steps):
         flush.fill_(i & 0xFF)  # L2 flush between timed steps (outside the events)
-        s0, sm, s1 = evs[i]
-        s0.record(stream)
-        step(sm)
-        s1.record(stream)
+        x0, xm, xc, x1 = evs[i]
+        x0.record(stream)
+        step(xm, xc)
+        x1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clocks = sampler.stop()
-    step_ms = [s0.elapsed_time(s1) for s0, _, s1 in evs]
-    kern_ms = [s0.elapsed_time(sm) for s0, sm, _ in evs]
-    tot = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
+    step_ms = [x0.elapsed_time(x1) for x0, _, _, x1 in evs]
+    kern_ms = [x0.elapsed_time(xc) for x0, _, xc, _ in evs]
+    long_ms = [x0.elapsed_time(xm) for x0, xm, _, _ in evs] if split else kern_ms
+    tot = torch.tensor([sum(step_ms), sum(kern_ms), sum(long_ms)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(tot, op=dist.ReduceOp.MAX)
-    total_ms, kern_total_ms = float(tot[0]), float(tot[1])
+    total_ms, kern_total_ms, long_total_ms = float(tot[0]), float(tot[1]), float(tot[2])
     ms_per_step = total_ms / a.steps
     value = m / (ms_per_step / 1e3)
+
+    # ---------------------------------------------------------------- emulated multi-GPU balance
+    # N = 1: the P-rank splits of tc_partition (built-in weights) and of
+    # tc_partition_weighted with this device's calibrated weights, every
+    # range timed alone (L2 flushed, median of 3): max/mean per P
+    balance = None
+    if world == 1 and not a.variant and not a.no_balance:
+        w = tuple(x if x > 0 else 1.0 for x in g.calibrate())
+        balance = {"weights_ns_per_unit": {"long": w[0], "short": w[1]},
+                   "what": "each rank's tc_count_range timed alone on this GPU (CUDA events, "
+                           "L2 flushed, median of 3); max/mean over ranks"}
+        tmp = torch.zeros(1, dtype=torch.int64, device=dev)
+
+        def range_ms(b, e):
+            ts = []
+            for r in range(3):
+                flush.fill_(r)
+                y0, y1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                y0.record(stream)
+                g.count_range(b, e, out=tmp)
+                y1.record(stream)
+                torch.cuda.synchronize()
+                ts.append(y0.elapsed_time(y1))
+            return statistics.median(ts), int(tmp.item())
+
+        for P in (2, 4, 8):
+            for label, bb in (("calibrated", g.partition(P, w)), ("builtin", g.partition(P))):
+                res = [range_ms(bb[r], bb[r + 1]) for r in range(P)]
+                ms = [x for x, _ in res]
+                balance[f"P{P}_{label}"] = {
+                    "max_over_mean": max(ms) / (sum(ms) / P), "range_ms": [round(x, 3) for x in ms],
+                    "partials_sum_to_T": (sum(p for _, p in res) & (2**64 - 1)) == T}
 
     # ---------------------------------------------------------------- sharded build (f2)
     # Every rank holds the contiguous 1/world slice of the raw pairs and the
@@ -475,7 +549,7 @@ def main():
                                           options=opts or None)
             else:
                 g2 = tc.build_csr_host(ps, pd, n, options=opts or None)
-            b = g2.partition(world)
+            b = g2.partition(world, weights) if weights else g2.partition(world)
             o2 = g2.count_range(b[rank], b[rank + 1])
             if world > 1:
                 dist.all_reduce(o2)
@@ -508,10 +582,51 @@ def main():
     parity = None if exp is None else (exp["triangles"] == T and exp["m"] == m)
 
     hbm, peak_src = peaks()
-    kern_avg_s = kern_total_ms / a.steps / 1e3
-    b_launch = info.b_itc * keys_share
-    achieved = b_launch / kern_avg_s / 1e9
-    traffic = profile_traffic(a.config) if world == 1 else None
+    # Roofline of the dominant kernel, k_count (the long class, a8): the
+    # method's own bytes (4 B per trimmed key + the plan
+    # entries + N+(v) once per (chunk, group)) over its CUDA-event time in
+    # the timed region.  For N > 1: this rank's share of the long class, by
+    # the plan cost of its chunks.
+    seg, cost = g.chunks()
+    nl = int(info.n_long_chunks)
+    share = 1.0
+    if world > 1 and cost[nl] > 0:
+        c0, c1 = (int(np.searchsorted(seg[:nl + 1], x, side="left")) for x in (l0, l1))
+        share = float(cost[c1] - cost[c0]) / float(cost[nl])
+    long_s = long_total_ms / a.steps / 1e3
+    kern_s = kern_total_ms / a.steps / 1e3
+    if split:
+        b_launch = float(info.method_bytes_long) * share
+        kname, kdesc = "k_count", "k_count (long class, a8), timed alone between its events"
+    else:  # variant / fused: one call, whole-step bytes
+        b_launch = float(info.method_bytes) * (share if world > 1 else 1.0)
+        kname, kdesc = "k_count", "whole count step (variant or fused: one call)"
+    achieved = b_launch / long_s / 1e9
+    frac = achieved / hbm
+    prof, why = profile_kernel(a.config, kname) if world == 1 and not a.variant else (None, "N>1 or variant")
+    step_bytes = float(info.method_bytes) * (1.0 if world == 1 else (e1 - e0) / max(1, info.m_live))
+    roof = {"bound": "hbm", "kernel": kdesc, "achieved": achieved, "peak": hbm, "unit": "GB/s",
+            "frac": frac,
+            "traffic": None if prof is None else prof["dram_bytes"] * share,
+            "traffic_source": (f"ncu --set full, capture {why}, same sources (src_hash {src_hash()})"
+                               if prof is not None else f"none: {why}"),
+            "bytes_per_launch": b_launch, "kernel_ms": long_s * 1e3,
+            "bytes_def": "method bytes = 4*keys + 24 B plan entries per live edge + "
+                         "(4*d+(v) + 28 B) per (chunk, group) + 40 B per chunk, long class "
+                         "(info.method_bytes_long); x this rank's cost share for N>1",
+            "peak_source": peak_src,
+            "step": {"bytes": step_bytes, "ms": kern_s * 1e3,
+                     "frac": step_bytes / kern_s / 1e9 / hbm,
+                     "what": "both count kernels (k_count + k_count_flat), whole-step method bytes"},
+            "merge_equiv": {"bytes": float(info.b_itc), "frac": float(info.b_itc) / kern_s / 1e9 / hbm,
+                            "what": "B_ITC (SURVEY.md §8(d), both operand lists per edge): context "
+                                    "only, not a roofline - this design reads N+(v) once per group"}}
+    if prof is not None:
+        roof["ncu"] = {k: prof.get(k) for k in ("dram_bytes", "lts_bytes", "l2_hit_pct", "l1_hit_pct",
+                                                "dram_pct", "l1tex_pct", "issue_pct",
+                                                "warps_active_pct", "long_scoreboard")}
+    if frac > 1.2:
+        raise SystemExit(f"roofline frac {frac:.2f} > 1.2: the bytes do not describe the timed kernel")
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
         "warmup": a.warmup, "ms_per_step": ms_per_step, "tc_ms": ms_per_step,
@@ -525,17 +640,14 @@ def main():
                        f"fused sum over NVLink peer memory, {fused.mode})"),
                    "l2": f"flushed by a {a.flush_mb} MiB write between timed steps; CSR "
                          f"{(info.m * 4 + (info.n + 1) * 8) / 2**20:.0f} MiB",
-                   "kernel": a.variant or "grouped (k_count + k_count_flat)"},
+                   "kernel": a.variant or "grouped (k_count + k_count_flat)",
+                   "src_hash": src_hash()},
         "triangles": str(T), "parity_vs_oracle": parity,
-        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                     "frac": achieved / hbm, "traffic": traffic,
-                     "bytes_per_launch": b_launch, "kernel_ms": kern_avg_s * 1e3,
-                     "bytes_def": "B_ITC = sum_e [4(suf_e + d+(v_e)) + 12] + 8(n'+1) "
-                                  "(SURVEY.md §8(d)); x this rank's share for N>1",
-                     "peak_source": peak_src},
+        "roofline": roof,
         "e2e": e2e,
-        "gpu_launches": a.steps * (g.launches_per_count + (fused is not None) if not a.variant
-                                   else (1 if a.variant == "polak" else 3)),
+        "emulated_balance": balance,
+        "gpu_launches": a.steps * (((l1 > l0) + (s1 > s0) if split else g.launches_per_count)
+                                   if not a.variant else (1 if a.variant == "polak" else 3)),
         "build_ms": {"canon": info.ms_canon, "sort_unique": info.ms_sort_unique,
                      "degree_rank": info.ms_degree_rank, "orient_csr": info.ms_orient_csr,
                      "plan": info.ms_plan, "total_events": info.ms_total,

@@ -81,8 +81,9 @@ typedef struct {
   int32_t seg_cost;     /* fixed cost per live oriented edge (default 4)          */
   int32_t huge_degree;  /* d+(v) above which N+(v) is probed in global memory by
                            binary search instead of an SMEM hash (default 8192)    */
-  int32_t block_threads;/* threads per CTA of the count kernel, 64..1024; 1/8 of
-                           the warps build tables, the rest probe (default 1024)   */
+  int32_t block_threads;/* threads per CTA of the long-class count kernel,
+                           64..1024; 1/5 of the warps build tables, the rest probe
+                           (default 1024)                                          */
   int32_t table_factor; /* hash slots = table_factor * d+(v) (rounded up to a
                            multiple of 4), 2..16 (default 6, i.e. load <= 1/6)     */
   int32_t long_min;     /* trimmed suffixes with >= long_min keys go to the
@@ -147,6 +148,17 @@ typedef struct {
   int64_t n_long_chunks;    /* chunks [0, n_long_chunks) are long class (k_count),
                                the rest short class (k_count_flat): a count launches
                                one kernel per non-empty class                       */
+  /* The method's own bytes: what one full count reads from
+   * memory as designed, every element once per use — the 4-B key of every
+   * trimmed suffix position (4 * keys_total), the plan entries of every live
+   * edge, and per (chunk, group) pair the head's row N+(v) (4 * d+(v)) and its
+   * group entries, plus the chunk bounds.  The count step's roofline bytes. */
+  uint64_t method_bytes;
+  int64_t table_words;      /* sum over (chunk, group) pairs of d+(v)             */
+  int64_t group_visits;     /* number of (chunk, group) pairs                     */
+  int64_t m_live_long;      /* live edges [0, m_live_long) are long class         */
+  uint64_t method_bytes_long; /* the long class's part of method_bytes            */
+  int64_t keys_long;        /* trimmed keys of the long class                      */
 } tc_graph_info_t;
 
 TC_API tc_status tc_graph_info(const tc_graph* g, tc_graph_info_t* out);
@@ -208,10 +220,52 @@ TC_API tc_status tc_count_variant(const tc_graph* g, int32_t variant, void* stre
 
 /*
  * Cost-balanced split of [0, m_live) into world_size contiguous ranges
- * (SURVEY.md §8(e)): h_bounds (host int64[world_size+1]) receives
- * 0 = b_0 <= b_1 <= ... <= b_P = m_live, aligned to work chunks.
+ * (per-edge intersections are independent, and edge
+ * chunks are the unit of work): h_bounds (host int64[world_size+1])
+ * receives 0 = b_0 <= b_1 <= ... <= b_P = m_live, aligned to work chunks.
+ * The cut points are binary-searched on the weighted prefix of the plan's
+ * per-chunk cost (a6: key lanes + seg_cost per edge + d+(v) and table words
+ * per group), long-class cost units weighted w_long and short-class units
+ * w_short (any positive doubles, e.g. the ns per unit of tc_calibrate):
+ * rank r gets the chunks whose weighted prefix lies in [r/P, (r+1)/P) of the
+ * total (rounded to the nearer chunk boundary).  tc_partition uses the
+ * plan's built-in weights (TC_PARTITION_W_LONG/SHORT below).  Every rank of a
+ * multi-GPU run must pass the same weights.  Host only (no GPU call).
+ * Errors: NULL, world_size < 1, non-positive weight -> TC_ERR_INVALID_ARGUMENT.
  */
+#define TC_PARTITION_W_LONG 1.0
+#define TC_PARTITION_W_SHORT 1.0
 TC_API tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds);
+TC_API tc_status tc_partition_weighted(const tc_graph* g, int32_t world_size, double w_long,
+                                       double w_short, int64_t* h_bounds);
+
+/*
+ * Host-only form of the weighted split (no GPU; CPU-tested): h_seg / h_cost
+ * (host int64[n_chunks+1], non-decreasing) are the chunks' first edges and
+ * cost prefix as tc_plan_chunks returns them, chunks [0, n_long_chunks) long.
+ * Writes h_bounds[0..world_size] as tc_partition_weighted does.
+ */
+TC_API tc_status tc_partition_chunks(const int64_t* h_seg, const int64_t* h_cost, int64_t n_chunks,
+                                     int64_t n_long_chunks, int32_t world_size, double w_long,
+                                     double w_short, int64_t* h_bounds);
+
+/*
+ * Measure the per-class cost weights on this device: one warm-up count, then
+ * one timed launch of each class over all its chunks (CUDA events on
+ * `stream`).  *h_ns_long / *h_ns_short (host double) receive the ns per plan
+ * cost unit of the long / short class (0 if the class is empty).
+ * Synchronises.  Feed the ranks' average to tc_partition_weighted.
+ */
+TC_API tc_status tc_calibrate(const tc_graph* g, void* stream, double* h_ns_long,
+                              double* h_ns_short);
+
+/*
+ * The plan's work chunks, host copies: h_seg (host int64[n_chunks+1], or
+ * NULL) receives each chunk's first live edge (h_seg[n_chunks] = m_live);
+ * h_cost (host int64[n_chunks+1], or NULL) the plan cost prefix at those
+ * edges (h_cost[n_long_chunks] = the long class's total).  Host only.
+ */
+TC_API tc_status tc_plan_chunks(const tc_graph* g, int64_t* h_seg, int64_t* h_cost);
 
 /*
  * Host-only form of the same split (no GPU needed; tested on CPU):

@@ -36,9 +36,11 @@ EXPORTS = (
     "tc_count_variant", "tc_key_bits", "tc_shard_canon", "tc_shard_histogram", "tc_shard_cuts",
     "tc_shard_bounds", "tc_shard_unique", "tc_shard_degree", "tc_rank_vertices", "tc_shard_orient", "tc_sort_keys",
     "tc_build_from_oriented", "tc_count_range_fused", "tc_mc_buffer_create",
-    "tc_mc_buffer_destroy",
+    "tc_mc_buffer_destroy", "tc_partition_weighted", "tc_calibrate", "tc_plan_chunks",
+    "tc_partition_chunks",
 )
 TC_MAX_PEERS = 16
+FUSED_WORDS = 8  # u64 words of the f4 symmetric buffer (tc_fused.cuh: sums, arrivals, poison, ticket)
 VARIANTS = {"polak": 1, "trust": 2}  # tc_count_variant
 
 
@@ -76,7 +78,10 @@ class GraphInfo(ctypes.Structure):
                 ("ms_canon", ctypes.c_float), ("ms_sort_unique", ctypes.c_float),
                 ("ms_degree_rank", ctypes.c_float), ("ms_orient_csr", ctypes.c_float),
                 ("ms_plan", ctypes.c_float), ("ms_total", ctypes.c_float),
-                ("n_long_chunks", ctypes.c_int64)]
+                ("n_long_chunks", ctypes.c_int64), ("method_bytes", ctypes.c_uint64),
+                ("table_words", ctypes.c_int64), ("group_visits", ctypes.c_int64),
+                ("m_live_long", ctypes.c_int64), ("method_bytes_long", ctypes.c_uint64),
+                ("keys_long", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_
@@ -106,6 +111,12 @@ def lib():
             "tc_count_range": ([vp, i64, i64, vp, vp], st),
             "tc_partition": ([vp, i32, vp], st),
             "tc_partition_prefix": ([vp, i64, i32, vp], st),
+            "tc_partition_weighted": ([vp, i32, ctypes.c_double, ctypes.c_double, vp], st),
+            "tc_calibrate": ([vp, vp, ctypes.POINTER(ctypes.c_double),
+                              ctypes.POINTER(ctypes.c_double)], st),
+            "tc_plan_chunks": ([vp, vp, vp], st),
+            "tc_partition_chunks": ([vp, vp, i64, i64, i32, ctypes.c_double, ctypes.c_double, vp],
+                                    st),
             "tc_support": ([vp, vp, vp], st),
             "tc_edge_list": ([vp, vp, vp, vp], st),
             "tc_count_variant": ([vp, i32, vp, vp], st),
@@ -280,10 +291,35 @@ class Graph:
                                   ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(v.data_ptr())))
         return u, v
 
-    def partition(self, world_size: int) -> list:
+    def partition(self, world_size: int, weights=None) -> list:
+        """Cost-balanced chunk-aligned cut of [0, m_live) (tc_partition, or
+        tc_partition_weighted with (w_long, w_short), e.g. from calibrate())."""
         b = np.zeros(int(world_size) + 1, dtype=np.int64)
-        _check(lib().tc_partition(self._h, int(world_size), b.ctypes.data_as(ctypes.c_void_p)))
+        if weights is None:
+            _check(lib().tc_partition(self._h, int(world_size), b.ctypes.data_as(ctypes.c_void_p)))
+        else:
+            wl, ws = (float(x) for x in weights)
+            _check(lib().tc_partition_weighted(self._h, int(world_size), wl, ws,
+                                               b.ctypes.data_as(ctypes.c_void_p)))
         return [int(x) for x in b]
+
+    def calibrate(self, stream=None):
+        """(ns per cost unit of the long class, of the short class) measured on
+        this device (tc_calibrate; 0.0 for an empty class)."""
+        wl, ws = ctypes.c_double(0), ctypes.c_double(0)
+        _check(lib().tc_calibrate(self._h, ctypes.c_void_p(_stream(stream)), ctypes.byref(wl),
+                                  ctypes.byref(ws)))
+        return float(wl.value), float(ws.value)
+
+    def chunks(self):
+        """(first live edge of every chunk, plan cost prefix at it): two int64
+        numpy arrays of n_chunks + 1 entries (tc_plan_chunks)."""
+        nc = int(self.info.n_chunks)
+        seg = np.zeros(nc + 1, dtype=np.int64)
+        cost = np.zeros(nc + 1, dtype=np.int64)
+        _check(lib().tc_plan_chunks(self._h, seg.ctypes.data_as(ctypes.c_void_p),
+                                    cost.ctypes.data_as(ctypes.c_void_p)))
+        return seg, cost
 
     def replan(self, options=None, stream=None):
         _check(lib().tc_replan(self._h, _options(options), ctypes.c_void_p(_stream(stream))))
@@ -356,6 +392,22 @@ def partition_prefix(prefix: Sequence[int], world_size: int) -> list:
     return [int(x) for x in b]
 
 
+def partition_chunks(seg, cost, n_long_chunks: int, world_size: int, w_long: float = 1.0,
+                     w_short: float = 1.0) -> list:
+    """Host-only weighted chunk split (tc_partition_chunks): seg/cost are the
+    n_chunks+1 first-edge and cost-prefix arrays of Graph.chunks()."""
+    sg = np.ascontiguousarray(seg, dtype=np.int64)
+    cs = np.ascontiguousarray(cost, dtype=np.int64)
+    if sg.shape != cs.shape or sg.size < 1:
+        raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, "seg/cost must have n_chunks + 1 entries")
+    b = np.zeros(int(world_size) + 1, dtype=np.int64)
+    _check(lib().tc_partition_chunks(sg.ctypes.data_as(ctypes.c_void_p),
+                                     cs.ctypes.data_as(ctypes.c_void_p), sg.size - 1,
+                                     int(n_long_chunks), int(world_size), float(w_long),
+                                     float(w_short), b.ctypes.data_as(ctypes.c_void_p)))
+    return [int(x) for x in b]
+
+
 class FusedSum:
     """the symmetric buffer of the library's own
     cross-GPU sum (tc_count_range_fused) — no NCCL on the counting path.
@@ -374,6 +426,7 @@ class FusedSum:
         if mode not in ("auto", "multicast", "peers"):
             raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, f"unknown mode {mode!r}")
         self.group, self.epoch, self._handle, self._keep = group, 0, None, []
+        self.poisoned = False
         on = dist.is_available() and dist.is_initialized()
         self.world = dist.get_world_size(group) if on else 1
         self.rank = dist.get_rank(group) if on else 0
@@ -389,20 +442,22 @@ class FusedSum:
         if self.world == 1:
             if mode in ("auto", "multicast"):
                 h, uc, mc = ctypes.c_void_p(0), ctypes.c_void_p(0), ctypes.c_void_p(0)
-                st = lib().tc_mc_buffer_create(64, ctypes.byref(h), ctypes.byref(uc), ctypes.byref(mc))
+                st = lib().tc_mc_buffer_create(8 * FUSED_WORDS, ctypes.byref(h), ctypes.byref(uc),
+                                           ctypes.byref(mc))
                 if st == TC_OK:
                     self._handle, self.own, self.mc, self.mode = h, uc.value, mc.value, "multicast"
                     return
                 if mode == "multicast":
                     _check(st)
-            buf = torch.zeros(4, dtype=torch.int64, device="cuda")
+            buf = torch.zeros(FUSED_WORDS, dtype=torch.int64, device="cuda")
             self._keep = [buf]
             self.own = int(buf.data_ptr())
             self.peers = [self.own]
             self.mode = "peers"
             return
         import torch.distributed._symmetric_memory as symm
-        buf = symm.empty(4, dtype=torch.int64, device=torch.device("cuda", torch.cuda.current_device()))
+        buf = symm.empty(FUSED_WORDS, dtype=torch.int64,
+                         device=torch.device("cuda", torch.cuda.current_device()))
         buf.zero_()
         torch.cuda.synchronize()
         gname = group.group_name if group is not None else dist.group.WORLD.group_name
@@ -421,8 +476,12 @@ class FusedSum:
     def count_range(self, graph, e_begin: int, e_end: int, out=None, stream=None):
         """This rank's partial over [e_begin, e_end) summed over all ranks, into
         a 1-element int64 CUDA tensor (u64 bits; UINT64_MAX if a rank never
-        arrived).  Every rank must call it, in the same order."""
+        arrived — check with :meth:`check`).  Every rank must call it, in the
+        same order.  The count kernel's last CTA does the sum (no extra launch
+        unless the range is empty)."""
         torch = _torch()
+        if self.poisoned:
+            raise TCError(TC_ERR_CUDA, "FusedSum poisoned by an earlier arrival timeout: recreate it")
         if out is None:
             out = torch.empty(1, dtype=torch.int64, device="cuda")
         self.epoch += 1
@@ -437,6 +496,19 @@ class FusedSum:
                                           ctypes.c_void_p(out.data_ptr())))
         return out
 
+    def check(self, value: int) -> int:
+        """Raise if the sum of this epoch timed out (a rank never arrived): the
+        kernel then wrote UINT64_MAX and set the buffer's POISON word; the
+        buffer stays unusable (a late partial may still land in it)."""
+        if value & (2**64 - 1) != 2**64 - 1:
+            return value
+        torch = _torch()
+        word = torch.as_tensor(_DevArray(self.own + 8 * 3, 1, "<i8", self), device="cuda")
+        if int(word.item()) != 0:
+            self.poisoned = True
+            raise TCError(TC_ERR_CUDA, "fused sum: a rank did not arrive within 20 s (buffer poisoned)")
+        return value
+
     def close(self):
         if self._handle is not None:
             lib().tc_mc_buffer_destroy(self._handle)
@@ -450,14 +522,33 @@ class FusedSum:
             pass
 
 
-def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] = None) -> int:
+def agreed_weights(graph, group=None, stream=None):
+    """Per-class cost weights every rank agrees on: each rank calibrates
+    (tc_calibrate) and the ranks' values are averaged with one all_reduce
+    (the bounds must be identical on every rank).  None when not distributed."""
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
+        return None
+    w = graph.calibrate(stream=stream)
+    dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
+    t = torch.tensor(w, dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    wl, ws = (float(x) / dist.get_world_size(group) for x in t.cpu())
+    return (wl if wl > 0 else 1.0, ws if ws > 0 else 1.0)
+
+
+def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] = None,
+                      weights=None) -> int:
     """T over a torch.distributed process group.
 
     Every rank holds the same replicated graph; rank r counts the live
-    oriented edges [b_r, b_{r+1}) of tc_partition's cost-balanced split and a
-    single all_reduce(SUM) of the 8-byte partials (ProcessGroupNCCL over
-    NVLink on the GPU box) gives T on every rank.  Two's-complement int64
-    addition is bit-identical to uint64 addition mod 2^64.  With ``fused`` (a
+    oriented edges [b_r, b_{r+1}) of the cost-balanced split
+    (tc_partition_weighted with ``weights``, the same on every rank — e.g.
+    :func:`agreed_weights` — or tc_partition's built-in weights) and a single
+    all_reduce(SUM) of the 8-byte partials (ProcessGroupNCCL over NVLink on
+    the GPU box) gives T on every rank.  Two's-complement int64 addition is
+    bit-identical to uint64 addition mod 2^64.  With ``fused`` (a
     :class:`FusedSum`), the sum is the library's own over NVLink peer memory
     (f4) instead of the NCCL all_reduce.
     """
@@ -465,10 +556,10 @@ def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] 
     on = dist.is_available() and dist.is_initialized()
     world = dist.get_world_size(group) if on else 1
     rank = dist.get_rank(group) if on else 0
-    bounds = graph.partition(world)
+    bounds = graph.partition(world) if weights is None else graph.partition(world, weights)
     if fused is not None:  # f4: the library's own sum over NVLink peer memory
         total = fused.count_range(graph, bounds[rank], bounds[rank + 1], stream=stream)
-        return int(total.item()) & (2**64 - 1)
+        return fused.check(int(total.item()) & (2**64 - 1))
     partial = graph.count_range(bounds[rank], bounds[rank + 1], stream=stream)
     if on:
         dist.all_reduce(partial, op=dist.ReduceOp.SUM, group=group)
@@ -478,5 +569,5 @@ def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] 
 from .sharded import build_csr_sharded, shard_cuts  # noqa: E402  (f2)
 
 __all__ = ["FusedSum", "build_csr_sharded", "shard_cuts", "Graph", "Options", "GraphInfo", "build_csr", "build_csr_host", "count_partitioned",
-           "partition_prefix", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
+           "partition_prefix", "partition_chunks", "agreed_weights", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
            "EXPORTS", "LIB_PATH"]

@@ -189,6 +189,18 @@ void rebind(tc_graph* g, cudaStream_t s) {
   P.seg_len.s = P.seg_group.s = P.grp_code.s = s;
 }
 
+// Chunks overlapping the live edges [e_begin, e_end): the first whose end is
+// > e_begin up to the last whose start is < e_end.
+void chunk_range(const tc_graph* g, int64_t e_begin, int64_t e_end, int64_t* c_begin,
+                 int64_t* c_end) {
+  const tc::Plan& P = g->plan;
+  const auto& cs = P.h_chunk_seg;
+  *c_begin = *c_end = 0;
+  if (e_end <= e_begin) return;
+  *c_begin = std::max<int64_t>(std::upper_bound(cs.begin(), cs.end(), e_begin) - cs.begin() - 1, 0);
+  *c_end = std::min<int64_t>(std::lower_bound(cs.begin(), cs.end(), e_end) - cs.begin(), P.n_chunks);
+}
+
 tc_status build_impl(const int32_t* src, const int32_t* dst, int64_t num_edges,
                      int64_t num_vertices, uint32_t flags, const tc_options* opts, void* stream,
                      tc_graph** out, bool host) {
@@ -294,6 +306,12 @@ tc_status tc_graph_info(const tc_graph* g, tc_graph_info_t* o) {
     o->ms_plan = g->ms[4];
     o->ms_total = g->ms[5];
     o->n_long_chunks = P.n_long_chunks;
+    o->method_bytes = P.method_bytes;
+    o->table_words = P.table_words;
+    o->group_visits = P.group_visits;
+    o->m_live_long = P.S_long;
+    o->method_bytes_long = P.method_bytes_long;
+    o->keys_long = P.keys_long;
   });
 }
 
@@ -325,15 +343,8 @@ tc_status tc_count_range(const tc_graph* g, int64_t e_begin, int64_t e_end, void
     const tc::Plan& P = g->plan;
     require(0 <= e_begin && e_begin <= e_end && e_end <= P.S,
             "need 0 <= e_begin <= e_end <= m_live");
-    const auto& cs = P.h_chunk_seg;
-    // first chunk whose end is > e_begin, last chunk whose start is < e_end
     int64_t c_begin = 0, c_end = 0;
-    if (e_end > e_begin) {
-      c_begin = std::upper_bound(cs.begin(), cs.end(), e_begin) - cs.begin() - 1;
-      c_end = std::lower_bound(cs.begin(), cs.end(), e_end) - cs.begin();
-      c_begin = std::max<int64_t>(c_begin, 0);
-      c_end = std::min<int64_t>(c_end, P.n_chunks);
-    }
+    chunk_range(g, e_begin, e_end, &c_begin, &c_end);
     tc::count_chunks(g, c_begin, c_end, e_begin, e_end, (cudaStream_t)stream,
                      reinterpret_cast<unsigned long long*>(d_partial));
   });
@@ -347,12 +358,18 @@ tc_status tc_count_range_fused(const tc_graph* g, int64_t e_begin, int64_t e_end
     require(world >= 1 && world <= TC_MAX_PEERS, "world must be in [1, TC_MAX_PEERS]");
     require(epoch >= 1, "epoch must be >= 1");
     require(d_mc || h_peers, "need a multicast address or the peer addresses");
+    require(0 <= e_begin && e_begin <= e_end && e_end <= g->plan.S,
+            "need 0 <= e_begin <= e_end <= m_live");
     if (!d_mc)
       for (int r = 0; r < world; ++r) require(h_peers[r] != nullptr, "NULL peer address");
-    tc_status st = tc_count_range(g, e_begin, e_end, stream, d_total);
-    if (st != TC_OK) tc::fail(st, t_last_error);
-    tc::fused_finish(reinterpret_cast<unsigned long long*>(d_total), d_own, d_mc, h_peers, world,
-                     epoch, (cudaStream_t)stream);
+    const tc::FuseArgs f = tc::fuse_args(d_own, d_mc, h_peers, world, epoch);
+    int64_t c_begin = 0, c_end = 0;
+    chunk_range(g, e_begin, e_end, &c_begin, &c_end);
+    // the count kernel's last CTA runs the cross-rank sum; a rank whose range
+    // launches no kernel still takes part through the finishing kernel
+    unsigned long long* tot = reinterpret_cast<unsigned long long*>(d_total);
+    if (tc::count_chunks(g, c_begin, c_end, e_begin, e_end, (cudaStream_t)stream, tot, &f) == 0)
+      tc::fused_finish(tot, f, (cudaStream_t)stream);
   });
 }
 
@@ -413,18 +430,98 @@ tc_status tc_partition_prefix(const int64_t* h_prefix, int64_t n_units, int32_t 
   });
 }
 
-tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds) {
+tc_status tc_partition_chunks(const int64_t* h_seg, const int64_t* h_cost, int64_t n_chunks,
+                              int64_t n_long_chunks, int32_t world_size, double w_long,
+                              double w_short, int64_t* h_bounds) {
+  return guarded([&] {
+    require(h_seg && h_cost && h_bounds, "NULL argument");
+    require(n_chunks >= 0 && n_long_chunks >= 0 && n_long_chunks <= n_chunks, "bad chunk counts");
+    require(world_size >= 1, "world_size < 1");
+    require(w_long > 0 && w_short > 0, "weights must be > 0");
+    for (int64_t c = 0; c < n_chunks; ++c)
+      require(h_seg[c] <= h_seg[c + 1] && h_cost[c] <= h_cost[c + 1], "prefixes must be non-decreasing");
+    // Weighted cost prefix over chunks: long chunks [0, nL) come first, so
+    // W(c) = w_long * cost[c] up to nL, then the short class's units at
+    // w_short.  Cut r is the chunk boundary nearest to r/P of W(nc).
+    const int64_t nc = n_chunks, nL = n_long_chunks;
+    const long double CL = (long double)h_cost[nL];
+    auto W = [&](int64_t c) -> long double {
+      return c <= nL ? w_long * (long double)h_cost[c]
+                     : w_long * CL + w_short * ((long double)h_cost[c] - CL);
+    };
+    const long double total = W(nc);
+    h_bounds[0] = h_seg[0];
+    int64_t prev = 0;
+    for (int32_t r = 1; r < world_size; ++r) {
+      const long double t = total * r / world_size;
+      int64_t lo = prev, hi = nc;  // first chunk boundary c >= prev with W(c) >= t
+      while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (W(mid) < t) lo = mid + 1; else hi = mid;
+      }
+      if (lo > prev && t - W(lo - 1) < W(lo) - t) --lo;  // the nearer boundary
+      prev = lo;
+      h_bounds[r] = h_seg[lo];
+    }
+    h_bounds[world_size] = h_seg[nc];
+  });
+}
+
+tc_status tc_partition_weighted(const tc_graph* g, int32_t world_size, double w_long,
+                                double w_short, int64_t* h_bounds) {
   return guarded([&] {
     require(g && h_bounds, "NULL argument");
-    require(world_size >= 1, "world_size < 1");
     const tc::Plan& P = g->plan;
-    // Chunks carry near-equal cost (a6), so a split by chunk count is a
-    // split by cost; bounds are the chunks' first live edges.
-    const int64_t nc = P.n_chunks;
-    for (int32_t r = 0; r <= world_size; ++r) {
-      const int64_t c = nc * r / world_size;
-      h_bounds[r] = (r == world_size) ? P.S : P.h_chunk_seg[c];
-    }
+    const tc_status st = tc_partition_chunks(P.h_chunk_seg.data(), P.h_chunk_cost.data(), P.n_chunks,
+                                             P.n_long_chunks, world_size, w_long, w_short, h_bounds);
+    if (st != TC_OK) tc::fail(st, t_last_error);
+  });
+}
+
+tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds) {
+  return tc_partition_weighted(g, world_size, TC_PARTITION_W_LONG, TC_PARTITION_W_SHORT, h_bounds);
+}
+
+tc_status tc_plan_chunks(const tc_graph* g, int64_t* h_seg, int64_t* h_cost) {
+  return guarded([&] {
+    require(g != nullptr, "graph is NULL");
+    const tc::Plan& P = g->plan;
+    if (h_seg) std::copy(P.h_chunk_seg.begin(), P.h_chunk_seg.end(), h_seg);
+    if (h_cost) std::copy(P.h_chunk_cost.begin(), P.h_chunk_cost.end(), h_cost);
+  });
+}
+
+tc_status tc_calibrate(const tc_graph* g, void* stream, double* h_ns_long, double* h_ns_short) {
+  return guarded([&] {
+    require(g && h_ns_long && h_ns_short, "NULL argument");
+    const tc::Plan& P = g->plan;
+    cudaStream_t s = (cudaStream_t)stream;
+    *h_ns_long = *h_ns_short = 0;
+    if (P.n_chunks == 0) return;
+    const int64_t nc = P.n_chunks, nL = P.n_long_chunks;
+    tc::DevBuf<unsigned long long> d(1, s);
+    cudaEvent_t ev[3] = {};
+    struct Guard {
+      cudaEvent_t* e;
+      ~Guard() {
+        for (int i = 0; i < 3; ++i)
+          if (e[i]) cudaEventDestroy(e[i]);
+      }
+    } guard{ev};
+    for (auto& e : ev) TC_CUDA(cudaEventCreate(&e));
+    tc::count_chunks(g, 0, nc, 0, P.S, s, d.get());  // warm-up
+    TC_CUDA(cudaEventRecord(ev[0], s));
+    if (nL > 0) tc::count_chunks(g, 0, nL, 0, P.S, s, d.get());
+    TC_CUDA(cudaEventRecord(ev[1], s));
+    if (nc > nL) tc::count_chunks(g, nL, nc, 0, P.S, s, d.get());
+    TC_CUDA(cudaEventRecord(ev[2], s));
+    TC_CUDA(cudaEventSynchronize(ev[2]));
+    float ms_l = 0, ms_s = 0;
+    TC_CUDA(cudaEventElapsedTime(&ms_l, ev[0], ev[1]));
+    TC_CUDA(cudaEventElapsedTime(&ms_s, ev[1], ev[2]));
+    const int64_t cl = P.h_chunk_cost[nL], cs = P.h_chunk_cost[nc] - cl;
+    if (nL > 0 && cl > 0) *h_ns_long = 1e6 * ms_l / (double)cl;
+    if (nc > nL && cs > 0) *h_ns_short = 1e6 * ms_s / (double)cs;
   });
 }
 

@@ -270,14 +270,15 @@ __device__ __forceinline__ int64_t upper_bound_i32(const int32_t* __restrict__ a
 // Live iff the trimmed suffix is non-empty.  Emits the plan's sort key
 // (class above head v; dead edges get `dead`, which sorts last) and the
 // packed value (trimmed start << 24 | length).  stats: [0] B_ITC edge part
-// (untrimmed), [1] trimmed keys, [2] live, [3] live long.
+// (untrimmed), [1] trimmed keys, [2] live, [3] live long,
+// [4] trimmed keys of the long class.
 __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
                             const int32_t* __restrict__ rowid, int64_t m, int long_min, int bits,
                             uint32_t dead, uint32_t* __restrict__ skey, uint64_t* __restrict__ sval,
                             unsigned long long* stats) {
   typedef cub::BlockReduce<unsigned long long, TPB> BR;
   __shared__ typename BR::TempStorage tmp;
-  unsigned long long b = 0, keys = 0, nl = 0, nlong = 0;
+  unsigned long long b = 0, keys = 0, nl = 0, nlong = 0, klong = 0;
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < m;
        p += (int64_t)gridDim.x * blockDim.x) {
     const int32_t u = rowid[p], v = col[p];
@@ -295,6 +296,7 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
     keys += (unsigned long long)len;
     nl += len > 0;
     nlong += len >= long_min;
+    klong += len >= long_min ? (unsigned long long)len : 0ull;
   }
   unsigned long long r0 = BR(tmp).Sum(b);
   __syncthreads();
@@ -303,11 +305,14 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
   unsigned long long r2 = BR(tmp).Sum(nl);
   __syncthreads();
   unsigned long long r3 = BR(tmp).Sum(nlong);
+  __syncthreads();
+  unsigned long long r4 = BR(tmp).Sum(klong);
   if (threadIdx.x == 0) {
     atomicAdd(&stats[0], r0);
     atomicAdd(&stats[1], r1);
     atomicAdd(&stats[2], r2);
     atomicAdd(&stats[3], r3);
+    atomicAdd(&stats[4], r4);
   }
 }
 
@@ -495,6 +500,43 @@ __global__ void k_split(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
       atomicMax(nm, (unsigned long long)ok_need);
       pieces[c] = cnt + 1;
     }
+  }
+}
+
+// Per chunk: the plan cost prefix at its first edge (the host copy drives
+// tc_partition's cost split), and the table rows / group visits its producers
+// read (the method's own bytes).  stats: [0] sum of d+(v)
+// over (chunk, group) pairs, [1] number of such pairs.
+__global__ void k_chunk_meta(const int64_t* __restrict__ chunk_seg, int64_t nc, int64_t nL,
+                             const int32_t* __restrict__ seg_group,
+                             const int64_t* __restrict__ ins_prefix,
+                             const int64_t* __restrict__ cost_prefix,
+                             int64_t* __restrict__ chunk_cost, unsigned long long* stats) {
+  typedef cub::BlockReduce<unsigned long long, TPB> BR;
+  __shared__ typename BR::TempStorage tmp;
+  unsigned long long tw = 0, gv = 0, twl = 0, gvl = 0;
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= nc;
+       c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t sa = chunk_seg[c];
+    chunk_cost[c] = cost_prefix[sa];
+    if (c == nc) continue;
+    const int64_t sb = chunk_seg[c + 1];
+    if (sa >= sb) continue;
+    const int64_t ga = seg_group[sa], gb = seg_group[sb - 1];
+    const unsigned long long w = (unsigned long long)(ins_prefix[gb + 1] - ins_prefix[ga]);
+    const unsigned long long v = (unsigned long long)(gb - ga + 1);
+    tw += w;
+    gv += v;
+    if (c < nL) {
+      twl += w;
+      gvl += v;
+    }
+  }
+  unsigned long long r[4] = {tw, gv, twl, gvl};
+  for (int i = 0; i < 4; ++i) {
+    const unsigned long long x = BR(tmp).Sum(r[i]);
+    __syncthreads();
+    if (threadIdx.x == 0) atomicAdd(&stats[i], x);
   }
 }
 
@@ -1012,11 +1054,11 @@ Tuning tuning_from_env() {
   t.grab_short = get("TC_GRAB_SHORT", t.grab_short, 0, 1 << 24);
   t.prod_div = get("TC_PROD_DIV", t.prod_div, 2, 32);
   t.wait_hint_ns = get("TC_WAIT_HINT", t.wait_hint_ns, 0, 10000000);
-  t.prefetch = get("TC_PREFETCH", t.prefetch, 0, 1);
-  t.ring = get("TC_RING", t.ring, 0, 1);
   t.cs_div = get("TC_CS_DIV", t.cs_div, 0, 64);
   t.short_linear = get("TC_SHORT_LINEAR", t.short_linear, 0, 1);
-  t.interleave = get("TC_INTERLEAVE", t.interleave, 0, 1);
+  t.l2_meta = get("TC_L2_META", t.l2_meta, 0, 1);
+  t.l2_keys = get("TC_L2_KEYS", t.l2_keys, 0, 2);
+  t.l2_persist_mb = get("TC_L2_PERSIST_MB", t.l2_persist_mb, 0, 1 << 16);
   return t;
 }
 
@@ -1032,8 +1074,8 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   const int64_t* row_ptr = g->row_ptr.get();
   const int32_t* col = g->col.get();
   Trace tr(s);
-  DevBuf<unsigned long long> stats(4, s);
-  TC_CUDA(cudaMemsetAsync(stats.get(), 0, 4 * sizeof(unsigned long long), s));
+  DevBuf<unsigned long long> stats(5, s);
+  TC_CUDA(cudaMemsetAsync(stats.get(), 0, 5 * sizeof(unsigned long long), s));
   // sort keys: class bit above the head v; dead edges sort last
   const int kbits = g->bits + 1;
   const uint32_t dead = kbits < 32 ? (1u << kbits) : 0xFFFFFFFFu;
@@ -1058,11 +1100,12 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   }
   rowid.reset();
   tr("rowid + edge trim");
-  unsigned long long h_stats[4];
+  unsigned long long h_stats[5];
   TC_CUDA(cudaMemcpyAsync(h_stats, stats.get(), sizeof(h_stats), cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));
   g->b_itc = h_stats[0] + 8ull * (unsigned long long)(n + 1);
   P.keys_total = (int64_t)h_stats[1];
+  P.keys_long = (int64_t)h_stats[4];
   const int64_t S = (int64_t)h_stats[2], S_long = (int64_t)h_stats[3];
   P.S = S;
   P.S_long = S_long;
@@ -1072,6 +1115,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     P.chunk_seg = DevBuf<int64_t>(1, s, true);
     TC_CUDA(cudaMemsetAsync(P.chunk_seg.get(), 0, sizeof(int64_t), s));
     P.h_chunk_seg.assign(1, 0);
+    P.h_chunk_cost.assign(1, 0);
     TC_CUDA(cudaStreamSynchronize(s));
     return;
   }
@@ -1201,10 +1245,34 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P.chunk_cost_long = CL;
   P.chunk_cost_short = CS;
   tr("chunking");
-  P.h_chunk_seg.resize(P.n_chunks + 1);
-  TC_CUDA(cudaMemcpyAsync(P.h_chunk_seg.data(), P.chunk_seg.get(),
-                          sizeof(int64_t) * (P.n_chunks + 1), cudaMemcpyDeviceToHost, s));
-  TC_CUDA(cudaStreamSynchronize(s));
+  {
+    DevBuf<int64_t> ccost(P.n_chunks + 1, s);
+    DevBuf<unsigned long long> st2(4, s);
+    TC_CUDA(cudaMemsetAsync(st2.get(), 0, 4 * sizeof(unsigned long long), s));
+    k_chunk_meta<<<grid_for(P.n_chunks + 1), TPB, 0, s>>>(P.chunk_seg.get(), P.n_chunks,
+                                                          P.n_long_chunks,
+                                                          P.seg_group.get(), P.ins_prefix.get(),
+                                                          cost_prefix.get(), ccost.get(), st2.get());
+    TC_LAUNCH();
+    P.h_chunk_seg.resize(P.n_chunks + 1);
+    P.h_chunk_cost.resize(P.n_chunks + 1);
+    unsigned long long h_st2[4];
+    TC_CUDA(cudaMemcpyAsync(P.h_chunk_seg.data(), P.chunk_seg.get(),
+                            sizeof(int64_t) * (P.n_chunks + 1), cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaMemcpyAsync(P.h_chunk_cost.data(), ccost.get(), sizeof(int64_t) * (P.n_chunks + 1),
+                            cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaMemcpyAsync(h_st2, st2.get(), sizeof(h_st2), cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaStreamSynchronize(s));
+    P.table_words = (int64_t)h_st2[0];
+    P.group_visits = (int64_t)h_st2[1];
+    auto bytes = [](int64_t keys, int64_t edges, int64_t words, int64_t visits, int64_t chunks) {
+      return 4ull * (uint64_t)keys + (uint64_t)(kPlanEdgeBytes * edges) + 4ull * (uint64_t)words +
+             (uint64_t)(kPlanGroupBytes * visits) + (uint64_t)(kPlanChunkBytes * chunks);
+    };
+    P.method_bytes = bytes(P.keys_total, S, P.table_words, P.group_visits, P.n_chunks);
+    P.method_bytes_long = bytes(P.keys_long, S_long, (int64_t)h_st2[2], (int64_t)h_st2[3],
+                                P.n_long_chunks);
+  }
   const int occ = count_occupancy(P.block, P.smem_bytes, P.tune);
   const int occ_flat = flat_occupancy(P.smem_flat);
   if (occ < 1 || occ_flat < 1)

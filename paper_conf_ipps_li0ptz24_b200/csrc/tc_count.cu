@@ -8,30 +8,34 @@
 //
 // How.  Live edges are grouped by their head v.  Work comes
 // in chunks = runs of consecutive live edges of one class and near-equal
-// cost, covering a run of groups.  One persistent CTA per SM, warp-specialised,
-// with two chunk slots in shared memory:
-//   PRODUCER warps (the first 1/4 of the CTA) take the CTA's chunk k+1 while
-//     the consumers work on chunk k: they stage the chunk's edges and table
-//     descriptors into the free slot and build one hash table per group from
-//     N+(v) (the GroupTC idea of a table shared by a block of edges, P:349,
-//     hashed as in TRUST, instead of binary search, the cost
-//     P:369/P:379 name on large graphs).  Tables are two-choice (cuckoo): a
-//     probe reads exactly two slots, so no warp waits on the longest of 32
-//     probe chains; if an insert ever fails the chunk falls back to linear
-//     probing.  They hand the slot over with an mbarrier.
-//   CONSUMER warps stream the chunk's suffix keys and probe the heads' tables:
-//     LONG class (suffix >= long_min keys): a warp walks one edge at a time
-//       in 32-key tiles, coalesced, with warp-uniform bookkeeping;
-//     SHORT class: the keys of all the chunk's edges are flattened over the
-//       lanes (the flattened walk of P:349 / Alg. 1 with the `>=` boundary
-//       of DESIGN.md reading C-7), 32 consecutive keys mapped to their edges
-//       with one SMEM load, a warp OR-reduce and popc
-//     (degree-bucketed dispatch, the TRUST/Fox idea of P:176/P:254), then
-//     release the slot with an mbarrier.
-//   Counts go thread u32 -> u64 -> warp shuffle -> CTA -> one atomic.
+// cost, covering a run of groups.  Two kernels, one per class:
+//   k_count (LONG class, suffix >= long_min keys): one persistent 1024-thread
+//   CTA per SM, warp-specialised, with three chunk slots in shared memory.
+//   PRODUCER warps (1/5 of the CTA) stage the CTA's next chunk into a free
+//     slot: its edges, its per-32-key tile descriptors, and one table per
+//     group built from N+(v) (the GroupTC idea of a table shared by a block
+//     of edges): a bitmap of N+(v)'s rank window (one probe per key)
+//     or a two-choice (cuckoo) hash, as in TRUST, instead of the
+//     binary search P:369/P:379 name as the cost on large graphs; a failed
+//     cuckoo insert rebuilds the chunk's tables with linear probing.  They
+//     hand the slot over with an mbarrier.
+//   CONSUMER warps walk the chunk's tiles (32 consecutive keys of one edge,
+//     coalesced, 8 tiles per batch in flight per lane), probe the heads'
+//     tables and release the slot with an mbarrier.
+//   k_count_flat (SHORT class): 4 CTAs x 384 threads per SM, every warp
+//     stages, builds and probes one chunk per CTA; the keys of all the chunk's
+//     edges are flattened over the lanes (the flattened walk of P:349 / Alg. 1
+//     with the `>=` boundary of DESIGN.md reading C-7), 32 consecutive keys
+//     mapped to their edges with one SMEM load, a warp OR-reduce and popc
+//     (degree-bucketed dispatch, the TRUST/Fox idea of P:176/P:254).
+//   Counts go thread u32 -> u64 -> warp shuffle -> CTA -> one atomic;
+//   with the fused cross-GPU sum (f4) the last CTA of the last launch adds the
+//   partial into every rank's symmetric buffer (tc_fused.cuh).
 // Tables whose N+(v) exceeds huge_degree are not staged; their keys are
 // binary-searched in global memory (the TriCore-style probe).
 #include <algorithm>
+#include <cstring>
+#include <mutex>
 
 #include "tc_internal.cuh"
 
@@ -56,10 +60,6 @@ constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flig
 #define TC_UNROLL_SHORT 2
 #endif
 constexpr int kUnrollShort = TC_UNROLL_SHORT;  // tiles in flight per consumer warp (short class)
-#ifndef TC_RING_DEPTH
-#define TC_RING_DEPTH 2
-#endif
-constexpr int kRingDepth = TC_RING_DEPTH;  // batches in flight per consumer warp (Tuning::ring)
 constexpr int kMaxKicks = 96;    // cuckoo displacement bound before the linear fallback
 constexpr int kMaxSlots = 4;     // chunk slots in SMEM (runtime count: Tuning::slots)
 
@@ -112,6 +112,31 @@ __device__ __forceinline__ int named_sync_or(int id, int nthreads, int pred) {
       : "r"(pred), "r"(id), "r"(nthreads)
       : "memory");
   return r;
+}
+
+// ------------------------------------------------------------------ L2 policy
+// Cache-policy loads (PTX createpolicy + ld.global.nc.L2::cache_hint; the
+// policy lives in a uniform descriptor, so a hinted load costs no extra
+// instruction).  kind: 0 evict_normal, 1 evict_first, 2 evict_last.
+__device__ __forceinline__ uint64_t l2_policy(int kind) {
+  uint64_t p;
+  if (kind == 1)
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  else if (kind == 2)
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  else
+    asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ int32_t ldp(const int32_t* a, uint64_t pol) {
+  int32_t v;
+  asm("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ int64_t ldp(const int64_t* a, uint64_t pol) {
+  int64_t v;
+  asm("ld.global.nc.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(v) : "l"(a), "l"(pol));
+  return v;
 }
 
 // ------------------------------------------------------------------ hashing
@@ -369,7 +394,7 @@ __device__ __forceinline__ unsigned probe_tile(const ChunkSmem& c, int z, int zw
 // measured slower: 4-tile batches 66 ms, 8-tile batches spill, vs 62.5 ms.)
 template <int kB>
 __device__ __forceinline__ void load_batch(const ChunkSmem& c, const int32_t* colL, int t,
-                                           int32_t (&key)[kB]) {
+                                           int32_t (&key)[kB], uint64_t pk) {
   int x[kB];
 #pragma unroll
   for (int q = 0; q < kB; q += 4)
@@ -378,7 +403,7 @@ __device__ __forceinline__ void load_batch(const ChunkSmem& c, const int32_t* co
   // ONE IMAD.WIDE.U32 x * 4 + colL (left to itself, nvcc re-associates it into
   // a 64-bit add-with-carry + LEA pair, 4 instructions per key)
 #pragma unroll
-  for (int u = 0; u < kB; ++u) key[u] = __ldg(colL + (uint32_t)x[u]);
+  for (int u = 0; u < kB; ++u) key[u] = ldp(colL + (uint32_t)x[u], pk);
 }
 
 // col + lane in a register the compiler cannot see through.
@@ -396,10 +421,11 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   unsigned cnt = 0;
   const int lane = threadIdx.x & 31;
   const int32_t* colL = lane_base(pv.col, lane);
+  const uint64_t pk = l2_policy(pv.l2_keys);
   int t = t0;
   for (; t + kB <= t1; t += kB) {
     int32_t key[kB];
-    load_batch<kB>(c, colL, t, key);
+    load_batch<kB>(c, colL, t, key, pk);
     int z[kB], zw[kB];
 #pragma unroll
     for (int q = 0; q < kB; q += 4) {
@@ -431,7 +457,7 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
     int z[8], zw[8];
     int32_t key[8];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) key[u] = __ldg(colL + (uint32_t)c.sT0[min(t + u, t1 - 1)]);
+    for (int u = 0; u < 8; ++u) key[u] = ldp(colL + (uint32_t)c.sT0[min(t + u, t1 - 1)], pk);
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const int tt = min(t + u, t1 - 1);
@@ -447,82 +473,6 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   return cnt;
 }
 
-// Same walk with the key loads as asynchronous global->shared copies
-// (`cp.async` 4 B per lane, one commit group per 8-tile batch) into a
-// per-warp ring of kD batch buffers: batch b+kD is in flight while batch b
-// is probed, and in-flight keys occupy SMEM instead of registers (the
-// register-resident walk keeps only 8 loads per lane in flight: 64 registers
-// per thread at 1024 threads).  Each lane copies and later reads only its own
-// words, so no warp barrier is needed: cp.async.wait_group orders them.
-template <int kD>
-__device__ __forceinline__ void ring_issue(const ChunkSmem& c, const int32_t* colL, int t,
-                                           uint32_t dst) {
-  constexpr int kB = kBatchLong;
-  int x[kB];
-#pragma unroll
-  for (int q = 0; q < kB; q += 4)
-    *reinterpret_cast<int4*>(x + q) = *reinterpret_cast<const int4*>(c.sT0 + t + q);
-#pragma unroll
-  for (int u = 0; u < kB; ++u)
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst + 128u * u),
-                 "l"(colL + (uint32_t)x[u])
-                 : "memory");
-}
-
-template <bool kLinear, bool kHuge, int kD>
-__device__ __forceinline__ unsigned walk_long_ring(const ChunkSmem& c, int t0, int t1,
-                                                   const PlanView& pv, int64_t ga,
-                                                   int* __restrict__ ring) {
-  constexpr int kB = kBatchLong;
-  unsigned cnt = 0;
-  const int lane = threadIdx.x & 31;
-  const int32_t* colL = lane_base(pv.col, lane);
-  const int* ringL = ring + lane;
-  const uint32_t rs = smem_u32(ring) + 4u * lane;
-  constexpr uint32_t kSlotBytes = kB * 32 * 4;
-  const int nb = (t1 - t0) / kB;
-#pragma unroll
-  for (int b = 0; b < kD; ++b) {
-    if (b < nb) ring_issue<kD>(c, colL, t0 + b * kB, rs + kSlotBytes * b);
-    asm volatile("cp.async.commit_group;" ::: "memory");
-  }
-  for (int b = 0; b < nb; ++b) {
-    const int t = t0 + b * kB, r = b % kD;
-    asm volatile("cp.async.wait_group %0;" ::"n"(kD - 1) : "memory");
-    int32_t key[kB];
-#pragma unroll
-    for (int u = 0; u < kB; ++u) key[u] = ringL[r * (kB * 32) + 32 * u];
-    if (b + kD < nb) ring_issue<kD>(c, colL, t + kD * kB, rs + kSlotBytes * r);
-    asm volatile("cp.async.commit_group;" ::: "memory");
-    int z[kB], zw[kB];
-#pragma unroll
-    for (int q = 0; q < kB; q += 4) {
-      *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
-      *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
-    }
-    int zw_or = 0;
-#pragma unroll
-    for (int u = 0; u < kB; ++u) zw_or |= zw[u];
-    if ((zw_or >> 6) == 0) {
-#pragma unroll
-      for (int u = 0; u < kB; ++u) {
-        const unsigned word = (unsigned)c.sT0[(key[u] >> 5) + z[u]];
-        const unsigned hit = (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
-        if (lane >= zw[u]) cnt += hit;
-      }
-    } else {
-#pragma unroll
-      for (int u = 0; u < kB; ++u) {
-        const unsigned hit = probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
-        if (lane >= (zw[u] & 63)) cnt += hit;
-      }
-    }
-  }
-  asm volatile("cp.async.wait_group 0;" ::: "memory");
-  // the < 8 tiles left: the register walk's tail
-  return cnt + walk_long<kLinear, kHuge>(c, t0 + nb * kB, t1, pv, ga);
-}
-
 // SHORT class: the warp owns the flat keys [k0w, k1w) of the chunk.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0w, int k1w,
@@ -531,6 +481,7 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
   if (k0w >= k1w) return cnt;
   const int lane = threadIdx.x & 31;
   const unsigned below = (1u << lane) - 1u;
+  const uint64_t pk = l2_policy(pv.l2_keys);
   int s = seg_of(c.sA, S, k0w);
   for (int k0 = k0w; k0 < k1w; k0 += 32 * kUnrollShort) {
     int seg[kUnrollShort];
@@ -555,7 +506,7 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
         // col index sB + k < m < 2^32: a 32-bit add on the low word of sB
         // (two's complement wraps correctly) and one IMAD.WIDE
         const uint32_t lo = reinterpret_cast<const uint32_t*>(c.sB)[2 * seg[u]];
-        key[u] = __ldg(pv.col + (lo + (uint32_t)k));
+        key[u] = ldp(pv.col + (lo + (uint32_t)k), pk);
         gl[u] = c.sD[seg[u]];
       }
     }
@@ -582,10 +533,7 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
 
 template <bool kLinear>
 __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
-                                            const PlanView& pv, int* ring = nullptr) {
-  if (h.is_long && ring)
-    return h.huge ? walk_long_ring<kLinear, true, kRingDepth>(c, w0, w1, pv, h.ga, ring)
-                  : walk_long_ring<kLinear, false, kRingDepth>(c, w0, w1, pv, h.ga, ring);
+                                            const PlanView& pv) {
   if (h.is_long)
     return h.huge ? walk_long<kLinear, true>(c, w0, w1, pv, h.ga)
                   : walk_long<kLinear, false>(c, w0, w1, pv, h.ga);
@@ -661,12 +609,6 @@ constexpr int kUnrollSupShort = TC_UNROLL_SUP_SHORT;  // 32-key steps in flight 
 #ifndef TC_SUP_FAST
 #define TC_SUP_FAST 1
 #endif
-#ifndef TC_SUP_SHORT_AGG
-#define TC_SUP_SHORT_AGG 0
-#endif
-#ifndef TC_SUP_MIX
-#define TC_SUP_MIX 0
-#endif
 
 // Support-mode lookup of key in group gl's table; kHuge = the chunk has
 // groups probed in global memory (otherwise that path is not compiled in).
@@ -739,31 +681,6 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
         const unsigned bits = ~(unsigned)e[u].x, b = (unsigned)key[u] & 31u;
         idx[u] = (key[u] >= 0 && ((bits >> b) & 1u)) ? e[u].y + __popc(bits & ((1u << b) - 1u)) : -1;
       }
-#if TC_SUP_MIX
-    } else if (!kLinear && no_huge) {
-      // bitmaps and two-choice hash tables mixed: both candidate entries of
-      // every tile read before any use (a bitmap tile reads its word twice)
-      const int2* H2 = reinterpret_cast<const int2*>(c.sHash);
-      int2 e1[kUnrollSup], e2[kUnrollSup];
-#pragma unroll
-      for (int u = 0; u < kUnrollSup; ++u) {
-        const int code = inf[u].y;
-        const uint32_t n = (uint32_t)code;
-        const int i1 = code <= 0 ? max((key[u] >> 5) + code, 0) : (int)hash1(key[u], n);
-        const int i2 = code <= 0 ? i1 : (int)hash2(key[u], n);
-        e1[u] = H2[inf[u].x + i1];
-        e2[u] = H2[inf[u].x + i2];
-      }
-#pragma unroll
-      for (int u = 0; u < kUnrollSup; ++u) {
-        if (inf[u].y <= 0) {
-          const unsigned bits = ~(unsigned)e1[u].x, b = (unsigned)key[u] & 31u;
-          idx[u] = (key[u] >= 0 && ((bits >> b) & 1u)) ? e1[u].y + __popc(bits & ((1u << b) - 1u)) : -1;
-        } else {
-          idx[u] = key[u] < 0 ? -1 : e1[u].x == key[u] ? e1[u].y : e2[u].x == key[u] ? e2[u].y : -1;
-        }
-      }
-#endif
     } else {
 #pragma unroll
       for (int u = 0; u < kUnrollSup; ++u)
@@ -802,58 +719,6 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
 // SHORT class, support mode: flat keys [k0w, k1w) of the chunk.
 __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0w, int k1w,
                                                const PlanView& pv, bool linear) {
-#if TC_SUP_SHORT_AGG
-  // warp_walk's loop with the (u, v) count summed per segment: the lanes of
-  // one segment are contiguous, so its first lane adds the hits of the lanes
-  // up to the next segment's first lane in one atomic
-  if (k0w >= k1w) return;
-  const int lane = threadIdx.x & 31;
-  const unsigned below = (1u << lane) - 1u;
-  int s = seg_of(c.sA, S, k0w);
-  for (int k0 = k0w; k0 < k1w; k0 += 32 * kUnrollSup) {
-    int seg[kUnrollSup];
-#pragma unroll
-    for (int u = 0; u < kUnrollSup; ++u) {
-      const int t0 = k0 + 32 * u;
-      const int j = s + 1 + lane;
-      const int pos = (j <= S) ? c.sA[j] - t0 : 64;
-      const unsigned bit = (pos >= 1 && pos <= 32) ? (1u << (pos - 1)) : 0u;
-      const unsigned M = __reduce_or_sync(0xffffffffu, bit);
-      seg[u] = s + __popc(M & below);
-      s += __popc(M);
-    }
-    int32_t key[kUnrollSup];
-#pragma unroll
-    for (int u = 0; u < kUnrollSup; ++u) {
-      const int k = k0 + 32 * u + lane;
-      key[u] = k < k1w ? __ldg(pv.col + c.sB[seg[u]] + k) : -1;
-    }
-#pragma unroll
-    for (int u = 0; u < kUnrollSup; ++u) {
-      const int k = k0 + 32 * u + lane;
-      const int sg = seg[u];
-      int idx = -1;
-      if (k < k1w) {
-        const int gl = c.sD[sg];
-        idx = sup_lookup_any(c, pv, gl, key[u], linear);
-        if (idx >= 0) {
-          atomicAdd(pv.sup + c.sB[sg] + k, 1u);                  // (u, w)
-          atomicAdd(pv.sup + c.sGB[gl] + c.sGP[gl] + idx, 1u);   // (v, w)
-        }
-      }
-      const unsigned H = __ballot_sync(0xffffffffu, idx >= 0);
-      const int prev = __shfl_up_sync(0xffffffffu, sg, 1);
-      const bool first = k < k1w && (lane == 0 || prev != sg);
-      const unsigned F = __ballot_sync(0xffffffffu, first);
-      if (first) {
-        const unsigned after = F & ~(below | (1u << lane));  // later segment starts
-        const unsigned span = (after ? (after & (0u - after)) - 1u : 0xffffffffu) & ~below;
-        const int n = __popc(H & span);
-        if (n) atomicAdd(pv.sup + c.sE[sg], (unsigned)n);     // (u, v)
-      }
-    }
-  }
-#else
   auto load = [&](int sg, int k) { return __ldg(pv.col + c.sB[sg] + k); };
   warp_walk<kUnrollSupShort>(c.sA, S, k0w, k1w, load, [&](int sg, int k, int32_t key) {
     const int gl = c.sD[sg];
@@ -864,7 +729,6 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
       atomicAdd(pv.sup + c.sE[sg], 1u);                      // (u, v)
     }
   });
-#endif
 }
 
 // ------------------------------------------------------------------ producers
@@ -875,8 +739,9 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
 template <int kB, bool kSup = false>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
-                                        int pt, int PT, int prefetch = 0) {
-  const int64_t sa = max(__ldg(pv.chunk_seg + (cix)), e_begin), sb = min(__ldg(pv.chunk_seg + (cix + 1)), e_end);
+                                        int pt, int PT) {
+  const uint64_t pm = l2_policy(pv.l2_meta);  // plan metadata: read once per count
+  const int64_t sa = max(ldp(pv.chunk_seg + (cix), pm), e_begin), sb = min(ldp(pv.chunk_seg + (cix + 1), pm), e_end);
   if (sa >= sb) {  // empty after clipping to the range
     if (pt == 0) {
       hdr.S = 0;
@@ -886,12 +751,12 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   }
   const bool is_long = cix < pv.n_long_chunks;
   const int S = (int)(sb - sa);
-  const int64_t ga = __ldg(pv.seg_group + (sa)), gb = (int64_t)__ldg(pv.seg_group + (sb - 1)) + 1;
+  const int64_t ga = ldp(pv.seg_group + (sa), pm), gb = (int64_t)ldp(pv.seg_group + (sb - 1), pm) + 1;
   const int G = (int)(gb - ga);
-  const int64_t slot0 = __ldg(pv.slot_prefix + (ga));
-  const int nslots = (int)(__ldg(pv.slot_prefix + (gb)) - slot0);
-  const int64_t kp0 = __ldg(pv.key_prefix + (sa));
-  const int T = is_long ? (int)((__ldg(pv.key_prefix + (sb)) - kp0) >> 5) : 0;
+  const int64_t slot0 = ldp(pv.slot_prefix + (ga), pm);
+  const int nslots = (int)(ldp(pv.slot_prefix + (gb), pm) - slot0);
+  const int64_t kp0 = ldp(pv.key_prefix + (sa), pm);
+  const int T = is_long ? (int)((ldp(pv.key_prefix + (sb), pm) - kp0) >> 5) : 0;
   ChunkSmem c = kSup ? slot_view_sup(region, S, G, T, nslots) : slot_view(region, S, G, T);
 
   // 1. stage edges and groups; empty slots.  Each producer thread handles
@@ -906,11 +771,11 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       kp[r] = 0;
       st[r] = 0;
       ln[r] = gr[r] = 0;
-      if (i <= S) kp[r] = __ldg(pv.key_prefix + (sa + i));
+      if (i <= S) kp[r] = ldp(pv.key_prefix + (sa + i), pm);
       if (i < S) {
-        st[r] = __ldg(pv.seg_start + (sa + i));
-        ln[r] = __ldg(pv.seg_len + (sa + i));
-        gr[r] = __ldg(pv.seg_group + (sa + i));
+        st[r] = ldp(pv.seg_start + (sa + i), pm);
+        ln[r] = ldp(pv.seg_len + (sa + i), pm);
+        gr[r] = ldp(pv.seg_group + (sa + i), pm);
       }
     }
 #pragma unroll
@@ -926,8 +791,8 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     }
   }
   if (kSup)
-    for (int i = pt; i < S; i += PT) c.sE[i] = __ldg(pv.seg_edge + (sa + i));
-  const int64_t ip0 = __ldg(pv.ins_prefix + (ga));
+    for (int i = pt; i < S; i += PT) c.sE[i] = ldp(pv.seg_edge + (sa + i), pm);
+  const int64_t ip0 = ldp(pv.ins_prefix + (ga), pm);
   int huge = 0;
   for (int base = pt; base <= G; base += PT * kB) {
     int64_t ip[kB], sp[kB], sp1[kB], ib[kB];
@@ -937,12 +802,12 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       const int i = base + r * PT;
       ip[r] = sp[r] = sp1[r] = ib[r] = 0;
       cd[r] = 0;
-      if (i <= G) ip[r] = __ldg(pv.ins_prefix + (ga + i));
+      if (i <= G) ip[r] = ldp(pv.ins_prefix + (ga + i), pm);
       if (i < G) {
-        sp[r] = __ldg(pv.slot_prefix + (ga + i));
-        sp1[r] = __ldg(pv.slot_prefix + (ga + i + 1));
-        ib[r] = __ldg(pv.grp_ibase + (ga + i));
-        cd[r] = __ldg(pv.grp_code + (ga + i));
+        sp[r] = ldp(pv.slot_prefix + (ga + i), pm);
+        sp1[r] = ldp(pv.slot_prefix + (ga + i + 1), pm);
+        ib[r] = ldp(pv.grp_ibase + (ga + i), pm);
+        cd[r] = ldp(pv.grp_code + (ga + i), pm);
       }
     }
 #pragma unroll
@@ -973,14 +838,6 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       const int2 d = c.sInfo[gl];
       const int toff = d.x >= 0 ? d.x : -1 - gl;
       const int64_t st = c.sB[i];
-      if (!kSup && prefetch) {
-        // Pull the edge's keys toward L2 now, one chunk before the consumers
-        // load them (a bulk prefetch: no registers, no SMEM; 16-B granules).
-        const uintptr_t lo = reinterpret_cast<uintptr_t>(pv.col + st) & ~uintptr_t(15);
-        const uintptr_t hi = (reinterpret_cast<uintptr_t>(pv.col + st + len) + 15) & ~uintptr_t(15);
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(lo), "r"((uint32_t)(hi - lo))
-                     : "memory");
-      }
       for (int t = ts; t < te; ++t) {
         const int64_t p = st + ((int64_t)(t - ts) << 5);
         const int lanes = min(32, len - ((t - ts) << 5));
@@ -1095,7 +952,8 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
 
 __global__ void __launch_bounds__(kMaxBlock, 1)
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
-            int64_t slot_bytes, Tuning tu, unsigned long long* __restrict__ out) {
+            int64_t slot_bytes, Tuning tu, unsigned long long* __restrict__ out,
+            const FuseArgs fuse) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ unsigned long long red[kMaxBlock / 32];
   __shared__ __align__(8) uint64_t full_bar[kMaxSlots];
@@ -1120,31 +978,21 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     // slot / fill number kept incrementally (no 64-bit division per chunk)
     int slot = 0;
     uint32_t j = 0;  // fill number of this slot
-    // This CTA's chunks are c_begin + b + i * grid, i < nk.  Plan order runs
-    // from many small tables (producer-heavy) to hub tables with many tiles
-    // (consumer-heavy); with tu.interleave the CTA alternates between the
-    // front and the back of its list so both sides stay busy.
-    const int64_t mine = c_end - c_begin - (int64_t)blockIdx.x;
-    const int64_t nk = mine > 0 ? (mine + gridDim.x - 1) / gridDim.x : 0;
-    for (int64_t k = 0;; ++k, slot = (slot + 1 == nslots) ? (++j, 0) : slot + 1) {
+    // This CTA's chunks are c_begin + b + k * grid.
+    for (int64_t cix = c_begin + blockIdx.x;; cix += gridDim.x,
+                 slot = (slot + 1 == nslots) ? (++j, 0) : slot + 1) {
       if (j > 0) wait_empty(&empty_bar[slot], (j - 1) & 1, hint);
-      const int64_t i = !tu.interleave ? k : ((k & 1) ? nk - 1 - (k >> 1) : (k >> 1));
-      const int64_t cix = k < nk ? c_begin + blockIdx.x + i * gridDim.x : c_end;
       if (cix >= c_end) {
         if (threadIdx.x == 0) hdr[slot].done = 1;
         mbar_arrive(&full_bar[slot]);
         break;
       }
-      produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], threadIdx.x, PT,
-                 tu.prefetch);
+      produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], threadIdx.x, PT);
       mbar_arrive(&full_bar[slot]);
     }
   } else {
     // ------------------------------------------------------------ consumers
     const int cw = warp - n_prod;
-    int* ring = tu.ring ? reinterpret_cast<int*>(smem + nslots * slot_bytes) +
-                              cw * (kRingDepth * kBatchLong * 32)
-                        : nullptr;
     int slot = 0;
     uint32_t fill = 0;
     for (;; slot = (slot + 1 == nslots) ? (++fill, 0) : slot + 1) {
@@ -1163,7 +1011,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = min((w0 + 7) & ~7, NU);
             w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
           }
-          acc += h.linear ? consume<true>(c, h, w0, w1, pv, ring) : consume<false>(c, h, w0, w1, pv, ring);
+          acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
         } else {  // dynamic: grab `grab` units at a time from the slot's counter
           for (;;) {
             int w0 = 0;
@@ -1171,7 +1019,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = __shfl_sync(0xffffffffu, w0, 0);
             if (w0 >= NU) break;
             const int w1 = min(w0 + grab, NU);
-            acc += h.linear ? consume<true>(c, h, w0, w1, pv, ring) : consume<false>(c, h, w0, w1, pv, ring);
+            acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
           }
         }
       }
@@ -1189,7 +1037,10 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     unsigned long long v = lane < nw ? red[lane] : 0ull;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
-    if (lane == 0 && v) atomicAdd(out, v);
+    if (lane == 0) {
+      if (v) atomicAdd(out, v);
+      if (fuse.own) fused_epilogue(out, fuse);  // f4: the last CTA sums across ranks
+    }
   }
 }
 
@@ -1199,7 +1050,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
 // staging and building latency overlaps the others' probing.
 __global__ void __launch_bounds__(kFlatBlock, kFlatCTAs)
     k_count_flat(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
-                 unsigned long long* __restrict__ out) {
+                 unsigned long long* __restrict__ out, const FuseArgs fuse) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ unsigned long long red[kFlatBlock / 32];
   __shared__ SlotHdr hdr;
@@ -1231,7 +1082,10 @@ __global__ void __launch_bounds__(kFlatBlock, kFlatCTAs)
     unsigned long long v = lane < nw ? red[lane] : 0ull;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
-    if (lane == 0 && v) atomicAdd(out, v);
+    if (lane == 0) {
+      if (v) atomicAdd(out, v);
+      if (fuse.own) fused_epilogue(out, fuse);  // f4: the last CTA sums across ranks
+    }
   }
 }
 
@@ -1308,7 +1162,6 @@ __global__ void k_edge_ends(const int64_t* __restrict__ row_ptr, int64_t n,
   }
 }
 
-bool g_attr_set = false;
 
 int optin_smem() {
   int dev = 0, v = 0;
@@ -1323,15 +1176,44 @@ int static_smem(const void* f) {
   return (int)fa.sharedSizeBytes;
 }
 
-void ensure_attr() {
-  if (g_attr_set) return;
+// cudaFuncSetAttribute applies to the current device's context: the flag is
+// per device (graphs may be built on several devices of one process), and
+// set at most once per device even with concurrent callers.
+constexpr int kMaxDevices = 64;
+std::once_flag g_attr_once[kMaxDevices];
+
+void set_attr() {
   TC_CUDA(cudaFuncSetAttribute(k_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                optin_smem() - static_smem((const void*)k_count)));
   TC_CUDA(cudaFuncSetAttribute(k_count_flat, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                optin_smem() - static_smem((const void*)k_count_flat)));
   TC_CUDA(cudaFuncSetAttribute(k_support, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                optin_smem() - static_smem((const void*)k_support)));
-  g_attr_set = true;
+}
+
+// The device's persisting-L2 set-aside, raised (never lowered) to `bytes`
+// capped at cudaDevAttrMaxPersistingL2CacheSize (Tuning::l2_persist_mb only).
+void ensure_persisting_l2(size_t bytes) {
+  static std::mutex mu;
+  static size_t set[kMaxDevices] = {};
+  int dev = 0, mx = 0;
+  TC_CUDA(cudaGetDevice(&dev));
+  TC_CUDA(cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, dev));
+  bytes = std::min(bytes, (size_t)mx);
+  std::lock_guard<std::mutex> lk(mu);
+  if (dev >= 0 && dev < kMaxDevices && set[dev] >= bytes) return;
+  TC_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes));
+  if (dev >= 0 && dev < kMaxDevices) set[dev] = bytes;
+}
+
+void ensure_attr() {
+  int dev = 0;
+  TC_CUDA(cudaGetDevice(&dev));
+  if (dev < 0 || dev >= kMaxDevices) {  // beyond the table: set it every time (cheap)
+    set_attr();
+    return;
+  }
+  std::call_once(g_attr_once[dev], set_attr);  // a throw leaves the flag unset
 }
 
 int64_t slot_bytes_of(int64_t need) { return (need + 15) & ~int64_t(15); }
@@ -1354,6 +1236,8 @@ PlanView plan_view(const tc_graph* g) {
   pv.short_linear = P.tune.short_linear;
   pv.seg_edge = nullptr;
   pv.sup = nullptr;
+  pv.l2_meta = P.tune.l2_meta;
+  pv.l2_keys = P.tune.l2_keys;
   return pv;
 }
 
@@ -1368,14 +1252,7 @@ int num_sms() {
 
 int max_smem_per_block() { return optin_smem() - static_smem((const void*)k_count); }
 
-// The consumers' cp.async rings (Tuning::ring), sized for all 32 warps.
-int64_t ring_bytes(const Tuning& tu) {
-  return tu.ring ? (int64_t)(kMaxBlock / 32) * kRingDepth * kBatchLong * 32 * 4 : 0;
-}
-
-int max_chunk_smem(const Tuning& tu) {
-  return (int)((max_smem_per_block() - ring_bytes(tu)) / tu.slots) & ~15;
-}
+int max_chunk_smem(const Tuning& tu) { return (max_smem_per_block() / tu.slots) & ~15; }
 
 // One chunk of the flat kernel must leave room for 3 CTAs per SM.
 int max_flat_chunk_smem() {
@@ -1390,7 +1267,7 @@ int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu) {
   ensure_attr();
   int occ = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-      &occ, k_count, block, (size_t)(tu.slots * slot_bytes_of(smem_bytes) + ring_bytes(tu))));
+      &occ, k_count, block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
   return occ;
 }
 
@@ -1402,30 +1279,55 @@ int flat_occupancy(int64_t smem_bytes) {
   return occ;
 }
 
-void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
-                  int64_t e_end, cudaStream_t s, unsigned long long* d_out) {
+int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
+                 int64_t e_end, cudaStream_t s, unsigned long long* d_out, const FuseArgs* fuse) {
   TC_CUDA(cudaMemsetAsync(d_out, 0, sizeof(unsigned long long), s));
   const Plan& P = g->plan;
-  if (c_end <= c_begin || e_end <= e_begin) return;
+  if (c_end <= c_begin || e_end <= e_begin) return 0;
   ensure_attr();
   const PlanView pv = plan_view(g);
-  // long-class chunks [c_begin, min(c_end, nL)): warp-specialised kernel
+  FuseArgs none;
+  memset(&none, 0, sizeof(none));
+  // long-class chunks [c_begin, min(c_end, nL)): warp-specialised kernel;
+  // short-class chunks: flat kernel.  The last launch carries the fused sum.
   const int64_t l0 = c_begin, l1 = std::min(c_end, P.n_long_chunks);
+  const int64_t s0 = std::max(c_begin, P.n_long_chunks), s1 = c_end;
+  // optional L2 access-policy window over the last l2_persist_mb MB of col
+  // (the highest-ranked rows, whose suffixes are re-read most), as a launch
+  // attribute so the caller's stream is left untouched
+  cudaLaunchAttribute attr[1];
+  int nattr = 0;
+  if (P.tune.l2_persist_mb > 0 && g->m > 0) {
+    const size_t want = (size_t)P.tune.l2_persist_mb << 20;
+    const size_t bytes = std::min(want, (size_t)g->m * 4);
+    ensure_persisting_l2(bytes);
+    memset(&attr[0], 0, sizeof(attr[0]));
+    attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+    attr[0].val.accessPolicyWindow.base_ptr =
+        (void*)(g->col.get() + (g->m - (int64_t)(bytes / 4)));
+    attr[0].val.accessPolicyWindow.num_bytes = bytes;
+    attr[0].val.accessPolicyWindow.hitRatio = 1.0f;
+    attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    nattr = 1;
+  }
+  int launched = 0;
   if (l1 > l0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(l1 - l0, P.grid));
     const int64_t sb = slot_bytes_of(P.smem_bytes);
-    k_count<<<grid, P.block, (size_t)(P.tune.slots * sb + ring_bytes(P.tune)), s>>>(
-        pv, l0, l1, e_begin, e_end, sb, P.tune, d_out);
-    TC_LAUNCH();
+    cudaLaunchConfig_t cfg = {dim3(grid), dim3(P.block), (size_t)(P.tune.slots * sb), s, attr, (unsigned)nattr};
+    TC_CUDA(cudaLaunchKernelEx(&cfg, k_count, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out,
+                               (fuse && s1 <= s0) ? *fuse : none));
+    ++launched;
   }
-  // short-class chunks: flat kernel
-  const int64_t s0 = std::max(c_begin, P.n_long_chunks), s1 = c_end;
   if (s1 > s0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(s1 - s0, P.grid_flat));
-    k_count_flat<<<grid, kFlatBlock, (size_t)slot_bytes_of(P.smem_flat), s>>>(pv, s0, s1, e_begin,
-                                                                             e_end, d_out);
-    TC_LAUNCH();
+    cudaLaunchConfig_t cfg = {dim3(grid), dim3(kFlatBlock), (size_t)slot_bytes_of(P.smem_flat), s, attr, (unsigned)nattr};
+    TC_CUDA(cudaLaunchKernelEx(&cfg, k_count_flat, pv, s0, s1, e_begin, e_end, d_out,
+                               fuse ? *fuse : none));
+    ++launched;
   }
+  return launched;
 }
 
 void support_all(const tc_graph* g, cudaStream_t s, unsigned* d_sup) {

@@ -1,82 +1,24 @@
 // tc_fused.cu — SURVEY.md §8(f) row f4: the cross-GPU sum of the partial
 // counts done by the library itself over NVLink peer memory, instead of an
-// NCCL all_reduce.
-//
-// T = sum over ranks of the partial counts of their edge ranges (the
-// per-edge intersections are independent).  After the count kernels of this
-// rank's range (tc_count_range's a7/a8/a9), ONE thread of a finishing kernel
-//   1. zeroes this rank's replica of the OTHER epoch's sum word,
-//   2. adds its partial to the sum word of this epoch on every rank:
-//        multicast: one `multimem.red.add.u64` through the NVLS multicast
-//                   address (the NVSwitch adds it into every replica), or
-//        peers:     one `red.add.u64` per peer replica (P2P over NVLink),
-//   3. bumps the arrival word on every rank the same way, with release
-//      semantics (so the sum add is visible first),
-//   4. spins (acquire) until its own arrival word reaches world * epoch, and
-//   5. reads T from its own replica.
-// Buffer (symmetric: same layout on every rank, zero-initialised):
-//   u64 word[0], word[1] = sum of epochs with parity 0 / 1, word[2] = arrivals.
-// The epoch-parity double buffer is safe: rank r clears its replica of slot
-// (e+1)&1 before it arrives in epoch e, and no rank adds into that slot (in
-// epoch e+1) before it has seen every arrival of epoch e.
+// NCCL all_reduce.  The protocol is fused_sum (tc_fused.cuh); normally the
+// count kernel's last CTA runs it (tc_count.cu, fused_epilogue), so a fused
+// count is the count launches alone.  This file holds the stand-alone
+// finishing kernel for a rank whose range launches no count kernel, and the
+// single-process multicast buffer (tc_mc_buffer_create).
 #include <cuda.h>
 
+#include <cstdlib>
 #include <cstring>
 
+#include "tc_fused.cuh"
 #include "tc_internal.cuh"
 
 namespace tc {
 namespace {
 
-constexpr unsigned long long kArrivalTimeoutNs = 20ull * 1000 * 1000 * 1000;  // 20 s
-
-struct Peers {
-  unsigned long long* p[TC_MAX_PEERS];
-};
-
-__global__ void k_fused_finish(unsigned long long* __restrict__ total, unsigned long long* own,
-                               unsigned long long* mc, Peers peers, int world,
-                               unsigned long long epoch) {
+__global__ void k_fused_finish(unsigned long long* __restrict__ total, FuseArgs f) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
-  const unsigned long long partial = *total;
-  const int slot = (int)(epoch & 1ull);
-  // 1. this rank's replica of the other epoch's sum word
-  asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(own + (slot ^ 1)), "l"(0ull) : "memory");
-  asm volatile("fence.acq_rel.sys;" ::: "memory");
-  // 2. + 3. the partial into every replica, then the arrival (release)
-  if (mc) {
-    asm volatile("multimem.red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(mc + slot), "l"(partial)
-                 : "memory");
-    asm volatile("fence.acq_rel.sys;" ::: "memory");
-    asm volatile("multimem.red.release.sys.global.add.u64 [%0], %1;" ::"l"(mc + 2), "l"(1ull)
-                 : "memory");
-  } else {
-    for (int r = 0; r < world; ++r)
-      asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(peers.p[r] + slot), "l"(partial)
-                   : "memory");
-    asm volatile("fence.acq_rel.sys;" ::: "memory");
-    for (int r = 0; r < world; ++r)
-      asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(peers.p[r] + 2), "l"(1ull)
-                   : "memory");
-  }
-  // 4. every rank's contribution of this epoch has landed in our replica
-  const unsigned long long want = (unsigned long long)world * epoch;
-  unsigned long long seen = 0, t0, now;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
-  for (;;) {
-    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(seen) : "l"(own + 2) : "memory");
-    if (seen >= want) break;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
-    if (now - t0 > kArrivalTimeoutNs) {  // a rank never arrived: report, do not hang
-      *total = ~0ull;
-      return;
-    }
-    __nanosleep(256);
-  }
-  // 5. T
-  unsigned long long t;
-  asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(t) : "l"(own + slot) : "memory");
-  *total = t;
+  fused_sum(total, f);
 }
 
 // ---------------------------------------------------------------- driver API
@@ -102,15 +44,26 @@ void cu_check(CUresult r, const char* what) {
 
 }  // namespace
 
-void fused_finish(unsigned long long* d_total, uint64_t* own, uint64_t* mc,
-                  uint64_t* const* peers, int world, uint64_t epoch, cudaStream_t s) {
-  Peers pp;
-  std::memset(&pp, 0, sizeof(pp));
+FuseArgs fuse_args(uint64_t* own, uint64_t* mc, uint64_t* const* peers, int world,
+                   uint64_t epoch) {
+  FuseArgs f;
+  std::memset(&f, 0, sizeof(f));
+  f.own = reinterpret_cast<unsigned long long*>(own);
+  f.mc = reinterpret_cast<unsigned long long*>(mc);
   if (!mc)
-    for (int r = 0; r < world; ++r) pp.p[r] = reinterpret_cast<unsigned long long*>(peers[r]);
-  k_fused_finish<<<1, 32, 0, s>>>(d_total, reinterpret_cast<unsigned long long*>(own),
-                                  reinterpret_cast<unsigned long long*>(mc), pp, world,
-                                  (unsigned long long)epoch);
+    for (int r = 0; r < world; ++r) f.peers[r] = reinterpret_cast<unsigned long long*>(peers[r]);
+  f.world = world;
+  f.epoch = (unsigned long long)epoch;
+  f.timeout_ns = kArrivalTimeoutNs;
+  if (const char* e = std::getenv("TC_FUSED_TIMEOUT_MS")) {
+    const long long ms = std::atoll(e);
+    if (ms > 0) f.timeout_ns = (unsigned long long)ms * 1000000ull;
+  }
+  return f;
+}
+
+void fused_finish(unsigned long long* d_total, const FuseArgs& f, cudaStream_t s) {
+  k_fused_finish<<<1, 32, 0, s>>>(d_total, f);
   TC_LAUNCH();
 }
 

@@ -10,6 +10,7 @@
 #include <vector>
 
 #include "tc.h"
+#include "tc_fused.cuh"
 
 namespace tc {
 
@@ -111,6 +112,7 @@ struct PlanView {
   int64_t n_long_chunks;
   int probe_mode;
   int short_linear;            // short class always probes linearly (Tuning::short_linear)
+  int l2_meta, l2_keys;        // L2 eviction policy of plan-metadata / key loads (Tuning)
   // support mode only (tc_support; nullptr when counting)
   const int64_t* seg_edge;     // [S] CSR position of segment s's own edge (u,v)
   unsigned* sup;               // [m] per-edge triangle counts (accumulated)
@@ -129,21 +131,32 @@ __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_
 }
 
 // Count-kernel launch tuning (not part of the C-ABI; TC_SLOTS, TC_GRAB_LONG,
-// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_PREFETCH, TC_RING, TC_CS_DIV, TC_SHORT_LINEAR, TC_INTERLEAVE override the defaults for sweeps).
+// TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_CS_DIV, TC_SHORT_LINEAR, TC_L2_META,
+// TC_L2_KEYS, TC_L2_PERSIST_MB override
+// the defaults for sweeps; every setting gives the same count).
 struct Tuning {
   int slots = 3;          // chunk slots in SMEM (2..4)
   int grab_long = 0;      // tiles per consumer grab, long class (0 = static split)
   int grab_short = 0;     // keys per consumer grab, short class (0 = static split)
   int prod_div = 5;       // 1/prod_div of the warps are producers (C3 sweep: 8 -> 57.7 ms, 6 -> 55.0, 5 -> 53.5, 4 -> 54.0)
   int wait_hint_ns = 0;   // mbarrier try_wait suspend hint (0 = none)
-  int prefetch = 0;       // long class: L2 bulk prefetch of each edge's keys at staging
-  int ring = 0;           // long class: key loads as cp.async into per-warp SMEM rings
   int cs_div = 0;         // short-class chunk cost = chunk_cost / cs_div (0: auto, 2 when the live
                           // edges carry < 2 keys on average, e.g. road graphs, else 1)
   int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
-  int interleave = 0;     // long class: each CTA alternates the front and back of its chunk list
+  int l2_meta = 0;        // L2 policy of the producers' plan-metadata loads: 0 normal, 1 evict_first
+  int l2_keys = 0;        // L2 policy of the key loads: 0 normal, 1 evict_first, 2 evict_last
+  int l2_persist_mb = 0;  // > 0: access-policy window marking the hottest (last) MB of col persisting
 };
 Tuning tuning_from_env();
+
+// Bytes of plan metadata a count reads (the method's own bytes, DESIGN.md
+// §6.2): per live edge its key_prefix / seg_start / seg_len / seg_group
+// entries, per (chunk, group) visit the group's ins_prefix / slot_prefix /
+// grp_ibase / grp_code entries, per chunk its two chunk_seg entries and the
+// closing key_prefix / ins_prefix / slot_prefix entries.
+constexpr int64_t kPlanEdgeBytes = 8 + 8 + 4 + 4;
+constexpr int64_t kPlanGroupBytes = 8 + 8 + 8 + 4;
+constexpr int64_t kPlanChunkBytes = 16 + 8 + 16;
 
 struct Plan {
   Options opt;
@@ -153,6 +166,12 @@ struct Plan {
   DevBuf<int64_t> key_prefix, seg_start, ins_prefix, grp_ibase, slot_prefix, chunk_seg;
   DevBuf<int32_t> seg_len, seg_group, grp_code;
   std::vector<int64_t> h_chunk_seg;
+  std::vector<int64_t> h_chunk_cost;  // [n_chunks+1] plan cost prefix at each chunk's first edge
+  int64_t table_words = 0;   // sum over (chunk, group) visits of d+(v): table rows read per count
+  int64_t group_visits = 0;  // (chunk, group) pairs
+  uint64_t method_bytes = 0; // bytes one full count reads as designed (keys + plan + tables)
+  uint64_t method_bytes_long = 0;  // the long class's share (its kernel, k_count)
+  int64_t keys_long = 0;     // trimmed keys of the long class
   int64_t chunk_cost_long = 0, chunk_cost_short = 0;  // after SMEM-driven halving
   int64_t smem_bytes = 0;  // per chunk slot, long class (warp-specialised kernel)
   int64_t smem_flat = 0;   // per chunk, short class (flat kernel)
@@ -199,8 +218,12 @@ void build_from_oriented(const uint64_t* okeys, int64_t m, const int32_t* perm, 
                          int64_t n_input, const Options& opt, cudaStream_t s, tc_graph* g);
 
 // tc_count.cu
-void count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
-                  int64_t e_end, cudaStream_t s, unsigned long long* d_out);
+// Returns the number of count kernels launched.  With `fuse` (f4), the last
+// launch's last CTA adds the partial into the symmetric buffer of every rank
+// and leaves T in *d_out; 0 launches = the caller must run fused_finish.
+int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_begin,
+                 int64_t e_end, cudaStream_t s, unsigned long long* d_out,
+                 const FuseArgs* fuse = nullptr);
 int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu);  // CTAs per SM (0 = cannot launch)
 int max_smem_per_block();
 int max_chunk_smem(const Tuning& tu);  // SMEM one of the kernel's chunk slots may use
@@ -210,9 +233,10 @@ int num_sms();
 void support_all(const tc_graph* g, cudaStream_t s, unsigned* d_sup);   // f1, tc_support
 void edge_ends(const tc_graph* g, cudaStream_t s, int32_t* d_u, int32_t* d_v);
 
-// tc_fused.cu (f4: fused cross-GPU sum over NVLink peer memory)
-void fused_finish(unsigned long long* d_total, uint64_t* own, uint64_t* mc,
-                  uint64_t* const* peers, int world, uint64_t epoch, cudaStream_t s);
+// tc_fused.cu (f4: fused cross-GPU sum over NVLink peer memory, tc_fused.cuh)
+FuseArgs fuse_args(uint64_t* own, uint64_t* mc, uint64_t* const* peers, int world,
+                   uint64_t epoch);
+void fused_finish(unsigned long long* d_total, const FuseArgs& f, cudaStream_t s);
 void* mc_create(size_t bytes, uint64_t** uc, uint64_t** mc);
 void mc_destroy(void* h);
 

@@ -217,12 +217,10 @@ void count_variant(const tc_graph* g, int variant, cudaStream_t s, unsigned long
   k_big_list<<<grid_of(n, kTPB), kTPB, 0, s>>>(g->row_ptr.get(), n, big.get(), n_big.get());
   TC_LAUNCH();
   const size_t smem = sizeof(int) * (kBlockBuckets * kBlockCap + kBlockBuckets);
-  static bool attr = false;
-  if (!attr) {
-    TC_CUDA(cudaFuncSetAttribute(k_trust_block, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)smem));
-    attr = true;
-  }
+  // per launch: the attribute belongs to the current device's context, and
+  // setting it is cheap next to a TRUST count
+  TC_CUDA(cudaFuncSetAttribute(k_trust_block, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               (int)smem));
   k_trust_block<<<num_sms() * 2, kBlockThreads, smem, s>>>(g->row_ptr.get(), g->col.get(),
                                                            big.get(), n_big.get(), bcap, d_out);
   TC_LAUNCH();

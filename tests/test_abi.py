@@ -75,6 +75,11 @@ def test_bad_arguments_rejected_before_device(tc):
     assert L.tc_count(None, None, None) == 1
     assert L.tc_count_range(None, 0, 0, None, None) == 1
     assert L.tc_partition(None, 2, None) == 1
+    assert L.tc_partition_weighted(None, 2, 1.0, 1.0, None) == 1
+    assert L.tc_plan_chunks(None, None, None) == 1
+    d = ctypes.c_double(0)
+    assert L.tc_calibrate(None, None, ctypes.byref(d), ctypes.byref(d)) == 1
+    assert L.tc_count_range_fused(None, 0, 0, None, None, None, 1, 1, None, None) == 1
     assert L.tc_graph_info(None, None) == 1
     assert L.tc_support(None, None, None) == 1
     assert L.tc_edge_list(None, None, None, None) == 1
@@ -113,13 +118,55 @@ def test_struct_layouts_match_header(tc, tmp_path):
     """The ctypes mirrors of tc_options / tc_graph_info_t match the C header."""
     src = tmp_path / "sz.c"
     src.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "tc.h"\n'
-                   'int main(void){printf("%zu %zu %zu %zu\\n", sizeof(tc_options), '
+                   'int main(void){printf("%zu %zu %zu %zu %zu %zu\\n", sizeof(tc_options), '
                    'sizeof(tc_graph_info_t), offsetof(tc_graph_info_t, row_ptr), '
-                   'offsetof(tc_graph_info_t, n_long_chunks));return 0;}\n')
+                   'offsetof(tc_graph_info_t, n_long_chunks), '
+                   'offsetof(tc_graph_info_t, method_bytes), '
+                   'offsetof(tc_graph_info_t, keys_long));return 0;}\n')
     exe = tmp_path / "sz"
     subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
     got = [int(x) for x in subprocess.run([str(exe)], capture_output=True, text=True,
                                           check=True).stdout.split()]
     want = [ctypes.sizeof(tc.Options), ctypes.sizeof(tc.GraphInfo), tc.GraphInfo.row_ptr.offset,
-            tc.GraphInfo.n_long_chunks.offset]
+            tc.GraphInfo.n_long_chunks.offset, tc.GraphInfo.method_bytes.offset,
+            tc.GraphInfo.keys_long.offset]
     assert got == want
+
+
+def _weighted_loads(seg, cost, nL, b, wl, ws):
+    """Weighted cost of each range [b_r, b_{r+1}) (ranges are chunk-aligned)."""
+    W = np.where(np.arange(len(cost)) <= nL, wl * cost,
+                 wl * cost[nL] + ws * (cost - cost[nL])).astype(float)
+    idx = [int(np.searchsorted(seg, x)) for x in b]
+    return [W[idx[r + 1]] - W[idx[r]] for r in range(len(b) - 1)], W
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
+@pytest.mark.parametrize("weights", [(1.0, 1.0), (1.0, 2.2), (3.0, 0.5)])
+def test_partition_chunks_weighted_balance(tc, world, weights):
+    """cuts on the weighted cost prefix; every range within one
+    chunk's weighted cost of the ideal share, chunk-aligned, covering [0, m_live)."""
+    rng = np.random.default_rng(world)
+    nc, nL = 3000, 1800
+    cost = np.concatenate([[0], np.cumsum(rng.integers(1, 400, size=nc))])
+    seg = np.concatenate([[0], np.cumsum(rng.integers(1, 50, size=nc))])
+    b = tc.partition_chunks(seg, cost, nL, world, *weights)
+    assert b[0] == 0 and b[-1] == seg[-1] and all(x <= y for x, y in zip(b, b[1:]))
+    assert set(b) <= set(seg.tolist())
+    loads, W = _weighted_loads(seg, cost, nL, b, *weights)
+    assert abs(sum(loads) - W[-1]) < 1e-6 * W[-1]
+    step = np.diff(W).max()
+    assert max(abs(x - W[-1] / world) for x in loads) <= step
+
+
+def test_partition_chunks_weights_move_the_cut(tc):
+    """Heavier short-class units pull the 2-way cut back into the long class."""
+    seg = np.arange(11, dtype=np.int64) * 10
+    cost = np.arange(11, dtype=np.int64) * 100  # 10 equal chunks, 5 long
+    assert tc.partition_chunks(seg, cost, 5, 2, 1.0, 1.0) == [0, 50, 100]
+    assert tc.partition_chunks(seg, cost, 5, 2, 1.0, 3.0)[1] == 70  # W: 5 + 15 -> cut at 10
+    assert tc.partition_chunks(seg, cost, 5, 2, 3.0, 1.0)[1] == 30
+    with pytest.raises(tc.InvalidArgument):
+        tc.partition_chunks(seg, cost, 5, 2, 0.0, 1.0)
+    with pytest.raises(tc.InvalidArgument):
+        tc.partition_chunks(seg[::-1].copy(), cost, 5, 2)

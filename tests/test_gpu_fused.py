@@ -97,7 +97,7 @@ def test_fused_peers_multi_process(tc, world):
     import torch.multiprocessing as mp
     src, dst, n = tcgen.rmat(15, 16, 5)
     want = oracle.triangles(src, dst)
-    bufs = [torch.zeros(4, dtype=torch.int64, device="cuda") for _ in range(world)]
+    bufs = [torch.zeros(tc.FUSED_WORDS, dtype=torch.int64, device="cuda") for _ in range(world)]
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
@@ -116,3 +116,40 @@ def test_fused_peers_multi_process(tc, world):
         assert err is None, f"rank {rank}: {err}"
         assert res == [want] * 3
     assert int(bufs[0][2].item()) == world * 3  # every rank arrived in every epoch
+
+
+def test_fused_timeout_poisons(tc, monkeypatch):
+    """A peer that never arrives: the last CTA gives up after the arrival bound,
+    sets the buffer's POISON word and yields UINT64_MAX; count_partitioned
+    raises instead of returning it, and the FusedSum refuses further use."""
+    monkeypatch.setenv("TC_FUSED_TIMEOUT_MS", "300")
+    src, dst, n = tcgen.CONFIGS["C1"].generate(1)
+    own = torch.zeros(tc.FUSED_WORDS, dtype=torch.int64, device="cuda")
+    ghost = torch.zeros(tc.FUSED_WORDS, dtype=torch.int64, device="cuda")  # never arrives
+    fs = tc.FusedSum(peers=[own, ghost], own=own)
+    fs.world = 2
+    with tc.build_csr(dev(src), dev(dst), n) as g:
+        out = fs.count_range(g, 0, g.m_live)
+        assert int(out.item()) & (2**64 - 1) == 2**64 - 1
+        assert int(own[3].item()) == 1
+        with pytest.raises(tc.TCError):
+            fs.check(int(out.item()) & (2**64 - 1))
+        assert fs.poisoned
+        with pytest.raises(tc.TCError):
+            fs.count_range(g, 0, g.m_live)
+
+
+def test_fused_is_one_launch_fewer(tc):
+    """The cross-rank sum runs in the count kernel's last CTA: a fused count of a
+    non-empty range launches exactly the count kernels (the ticket word is reset
+    for the next launch), an empty range launches the finishing kernel."""
+    src, dst, n = tcgen.rmat(14, 16, 3)
+    want = oracle.triangles(src, dst)
+    fs = tc.FusedSum(mode="peers")
+    with tc.build_csr(dev(src), dev(dst), n, options={"long_min": 32}) as g:
+        assert g.launches_per_count == 2
+        for _ in range(3):
+            assert tc.count_partitioned(g, fused=fs) == want
+            assert int(fs._keep[0][4].item()) == 0  # grid-completion ticket reset
+        assert int(fs.count_range(g, 0, 0).item()) == 0  # empty range: finishing kernel
+    fs.close()
