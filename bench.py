@@ -392,10 +392,10 @@ def main():
     if a.mode == "support":
         return bench_support(a, tc, g, info, src, dst, n, gen_s, build_wall_ms, world, rank)
 
-    # cost-balanced ranges: at N > 1 every rank calibrates the per-class cost
-    # weights and the ranks agree on their average (one all_reduce)
-    weights = tc.agreed_weights(g) if world > 1 else None
-    bounds = g.partition(world, weights) if weights else g.partition(world)
+    # cost-balanced ranges: at N > 1 every rank measures the plan's time
+    # profile (tc_calibrate) and the ranks agree on its average (one all_reduce)
+    profile = tc.agreed_profile(g) if world > 1 else None
+    bounds = g.partition(world, profile) if profile is not None else g.partition(world)
     e0, e1 = bounds[rank], bounds[rank + 1]
     # the rank's range split at the class boundary: the long class is k_count
     # (a8), the short class k_count_flat (a7); one step = both calls, with an
@@ -463,13 +463,13 @@ def main():
     value = m / (ms_per_step / 1e3)
 
     # ---------------------------------------------------------------- emulated multi-GPU balance
-    # N = 1: the P-rank splits of tc_partition (built-in weights) and of
-    # tc_partition_weighted with this device's calibrated weights, every
-    # range timed alone (L2 flushed, median of 3): max/mean per P
+    # N = 1: the P-rank splits of tc_partition_measured (this device's
+    # 64-slice profile) and of tc_partition (built-in profile), every range
+    # timed alone (L2 flushed, median of 3): max/mean per P
     balance = None
     if world == 1 and not a.variant and not a.no_balance:
-        w = tuple(x if x > 0 else 1.0 for x in g.calibrate())
-        balance = {"weights_ns_per_unit": {"long": w[0], "short": w[1]},
+        w = g.calibrate()
+        balance = {"profile_slices": len(w), "profile_ms_sum": float(w.sum()),
                    "what": "each rank's tc_count_range timed alone on this GPU (CUDA events, "
                            "L2 flushed, median of 3); max/mean over ranks"}
         tmp = torch.zeros(1, dtype=torch.int64, device=dev)
@@ -487,7 +487,7 @@ def main():
             return statistics.median(ts), int(tmp.item())
 
         for P in (2, 4, 8):
-            for label, bb in (("calibrated", g.partition(P, w)), ("builtin", g.partition(P))):
+            for label, bb in (("measured", g.partition(P, w)), ("builtin", g.partition(P))):
                 res = [range_ms(bb[r], bb[r + 1]) for r in range(P)]
                 ms = [x for x, _ in res]
                 balance[f"P{P}_{label}"] = {
@@ -549,7 +549,7 @@ def main():
                                           options=opts or None)
             else:
                 g2 = tc.build_csr_host(ps, pd, n, options=opts or None)
-            b = g2.partition(world, weights) if weights else g2.partition(world)
+            b = g2.partition(world, profile) if profile is not None else g2.partition(world)
             o2 = g2.count_range(b[rank], b[rank + 1])
             if world > 1:
                 dist.all_reduce(o2)

@@ -223,41 +223,57 @@ TC_API tc_status tc_count_variant(const tc_graph* g, int32_t variant, void* stre
  * (per-edge intersections are independent, and edge
  * chunks are the unit of work): h_bounds (host int64[world_size+1])
  * receives 0 = b_0 <= b_1 <= ... <= b_P = m_live, aligned to work chunks.
- * The cut points are binary-searched on the weighted prefix of the plan's
- * per-chunk cost (a6: key lanes + seg_cost per edge + d+(v) and table words
- * per group), long-class cost units weighted w_long and short-class units
- * w_short (any positive doubles, e.g. the ns per unit of tc_calibrate):
- * rank r gets the chunks whose weighted prefix lies in [r/P, (r+1)/P) of the
- * total (rounded to the nearer chunk boundary).  tc_partition uses the
- * plan's built-in weights (TC_PARTITION_W_LONG/SHORT below).  Every rank of a
- * multi-GPU run must pass the same weights.  Host only (no GPU call).
- * Errors: NULL, world_size < 1, non-positive weight -> TC_ERR_INVALID_ARGUMENT.
+ * The cut points are binary-searched on a prefix of the plan's per-chunk
+ * cost (a6: key lanes + seg_cost per edge + d+(v) and table words per group)
+ * weighted by a time profile: the chunk list is cut into n_slices SLICES of
+ * near-equal cost (tc_slice_bounds; for n_slices >= 2 slices never straddle
+ * the class boundary) and slice i's cost units are weighted so that the whole slice
+ * weighs h_ms[i].  Cut r is the chunk boundary nearest to r/P of the total.
+ *   tc_partition          : the built-in profile - two slices (long class,
+ *                           short class), a short-class unit weighing
+ *                           TC_PARTITION_SHORT_RATIO long-class units.
+ *   tc_partition_measured : h_ms from tc_calibrate (every rank must pass the
+ *                           same profile, e.g. the ranks' average).
+ * Host only.  Errors: NULL, world_size < 1, n_slices < 1, a negative or
+ * non-finite h_ms entry -> TC_ERR_INVALID_ARGUMENT.
  */
-#define TC_PARTITION_W_LONG 1.0
-#define TC_PARTITION_W_SHORT 1.0
+#define TC_PARTITION_SHORT_RATIO 2.2 /* short vs long ns per cost unit (C3 2.21, C4 2.09) */
 TC_API tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds);
-TC_API tc_status tc_partition_weighted(const tc_graph* g, int32_t world_size, double w_long,
-                                       double w_short, int64_t* h_bounds);
+TC_API tc_status tc_partition_measured(const tc_graph* g, int32_t world_size, int32_t n_slices,
+                                       const double* h_ms, int64_t* h_bounds);
 
 /*
- * Host-only form of the weighted split (no GPU; CPU-tested): h_seg / h_cost
- * (host int64[n_chunks+1], non-decreasing) are the chunks' first edges and
- * cost prefix as tc_plan_chunks returns them, chunks [0, n_long_chunks) long.
- * Writes h_bounds[0..world_size] as tc_partition_weighted does.
+ * Measure the time profile of the plan on this device: one warm-up count,
+ * then every slice of tc_slice_bounds(n_slices) counted alone (one
+ * tc_count_range call per slice, CUDA events on `stream`).  h_ms (host
+ * double[n_slices]) receives the slices' ms (0 for an empty slice).
+ * Synchronises.  Each slice is ~1/n_slices of a count, so it still fills the
+ * GPU for n_slices up to a few hundred at configs C3/C4.
+ */
+TC_API tc_status tc_calibrate(const tc_graph* g, void* stream, int32_t n_slices, double* h_ms);
+
+/*
+ * Host only: the slices of a profile.  h_first (host int64[n_slices+1])
+ * receives each slice's first CHUNK (h_first[n_slices] = n_chunks).  One
+ * slice is the whole list; otherwise the long
+ * class [0, n_long_chunks) gets round(n_slices * its cost share) slices (at
+ * least 1 if non-empty, at most n_slices - 1 if the short class is
+ * non-empty), the short class the rest; inside a class slice j starts at the
+ * first chunk whose cost prefix reaches j/K of the class's cost.
+ */
+TC_API tc_status tc_slice_bounds(const int64_t* h_cost, int64_t n_chunks, int64_t n_long_chunks,
+                                 int32_t n_slices, int64_t* h_first);
+
+/*
+ * Host-only form of the split (no GPU; CPU-tested): h_seg / h_cost (host
+ * int64[n_chunks+1], non-decreasing) are the chunks' first edges and cost
+ * prefix as tc_plan_chunks returns them, chunks [0, n_long_chunks) long;
+ * h_ms the profile of tc_slice_bounds(n_slices).  Writes h_bounds as
+ * tc_partition_measured does.
  */
 TC_API tc_status tc_partition_chunks(const int64_t* h_seg, const int64_t* h_cost, int64_t n_chunks,
-                                     int64_t n_long_chunks, int32_t world_size, double w_long,
-                                     double w_short, int64_t* h_bounds);
-
-/*
- * Measure the per-class cost weights on this device: one warm-up count, then
- * one timed launch of each class over all its chunks (CUDA events on
- * `stream`).  *h_ns_long / *h_ns_short (host double) receive the ns per plan
- * cost unit of the long / short class (0 if the class is empty).
- * Synchronises.  Feed the ranks' average to tc_partition_weighted.
- */
-TC_API tc_status tc_calibrate(const tc_graph* g, void* stream, double* h_ns_long,
-                              double* h_ns_short);
+                                     int64_t n_long_chunks, int32_t n_slices, const double* h_ms,
+                                     int32_t world_size, int64_t* h_bounds);
 
 /*
  * The plan's work chunks, host copies: h_seg (host int64[n_chunks+1], or
@@ -443,6 +459,15 @@ TC_API void tc_mc_buffer_destroy(void* handle);
 
 /* Release a graph (NULL is a no-op).  Stream-ordered frees on the build stream. */
 TC_API void tc_free(tc_graph* g);
+
+/*
+ * Process-wide diagnostic counters of the count kernels on the current
+ * device: h_counters (host uint64[4]) receives [0] = chunks whose two-choice
+ * (cuckoo) table inserts failed and were rebuilt with linear probing
+ * (reading C-24), [1..3] = 0 (reserved).  reset != 0 zeroes them
+ * after reading.  Synchronises the device.
+ */
+TC_API tc_status tc_counters(uint64_t* h_counters, int32_t reset);
 
 /* Thread-local text for the last non-OK status of this thread. */
 TC_API const char* tc_last_error(void);

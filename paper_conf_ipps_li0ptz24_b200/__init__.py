@@ -36,10 +36,11 @@ EXPORTS = (
     "tc_count_variant", "tc_key_bits", "tc_shard_canon", "tc_shard_histogram", "tc_shard_cuts",
     "tc_shard_bounds", "tc_shard_unique", "tc_shard_degree", "tc_rank_vertices", "tc_shard_orient", "tc_sort_keys",
     "tc_build_from_oriented", "tc_count_range_fused", "tc_mc_buffer_create",
-    "tc_mc_buffer_destroy", "tc_partition_weighted", "tc_calibrate", "tc_plan_chunks",
-    "tc_partition_chunks",
+    "tc_mc_buffer_destroy", "tc_partition_measured", "tc_calibrate", "tc_plan_chunks",
+    "tc_partition_chunks", "tc_slice_bounds", "tc_counters",
 )
 TC_MAX_PEERS = 16
+CALIBRATION_SLICES = 64  # slices of the measured time profile (tc_calibrate)
 FUSED_WORDS = 8  # u64 words of the f4 symmetric buffer (tc_fused.cuh: sums, arrivals, poison, ticket)
 VARIANTS = {"polak": 1, "trust": 2}  # tc_count_variant
 
@@ -111,12 +112,12 @@ def lib():
             "tc_count_range": ([vp, i64, i64, vp, vp], st),
             "tc_partition": ([vp, i32, vp], st),
             "tc_partition_prefix": ([vp, i64, i32, vp], st),
-            "tc_partition_weighted": ([vp, i32, ctypes.c_double, ctypes.c_double, vp], st),
-            "tc_calibrate": ([vp, vp, ctypes.POINTER(ctypes.c_double),
-                              ctypes.POINTER(ctypes.c_double)], st),
+            "tc_partition_measured": ([vp, i32, i32, vp, vp], st),
+            "tc_calibrate": ([vp, vp, i32, vp], st),
             "tc_plan_chunks": ([vp, vp, vp], st),
-            "tc_partition_chunks": ([vp, vp, i64, i64, i32, ctypes.c_double, ctypes.c_double, vp],
-                                    st),
+            "tc_counters": ([vp, i32], st),
+            "tc_partition_chunks": ([vp, vp, i64, i64, i32, vp, i32, vp], st),
+            "tc_slice_bounds": ([vp, i64, i64, i32, vp], st),
             "tc_support": ([vp, vp, vp], st),
             "tc_edge_list": ([vp, vp, vp, vp], st),
             "tc_count_variant": ([vp, i32, vp, vp], st),
@@ -291,25 +292,27 @@ class Graph:
                                   ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(v.data_ptr())))
         return u, v
 
-    def partition(self, world_size: int, weights=None) -> list:
-        """Cost-balanced chunk-aligned cut of [0, m_live) (tc_partition, or
-        tc_partition_weighted with (w_long, w_short), e.g. from calibrate())."""
+    def partition(self, world_size: int, profile=None) -> list:
+        """Cost-balanced chunk-aligned cut of [0, m_live): tc_partition (the
+        built-in profile), or tc_partition_measured with ``profile`` = the
+        per-slice ms of :meth:`calibrate` (the same on every rank)."""
         b = np.zeros(int(world_size) + 1, dtype=np.int64)
-        if weights is None:
+        if profile is None:
             _check(lib().tc_partition(self._h, int(world_size), b.ctypes.data_as(ctypes.c_void_p)))
         else:
-            wl, ws = (float(x) for x in weights)
-            _check(lib().tc_partition_weighted(self._h, int(world_size), wl, ws,
+            ms = np.ascontiguousarray(profile, dtype=np.float64)
+            _check(lib().tc_partition_measured(self._h, int(world_size), int(ms.size),
+                                               ms.ctypes.data_as(ctypes.c_void_p),
                                                b.ctypes.data_as(ctypes.c_void_p)))
         return [int(x) for x in b]
 
-    def calibrate(self, stream=None):
-        """(ns per cost unit of the long class, of the short class) measured on
-        this device (tc_calibrate; 0.0 for an empty class)."""
-        wl, ws = ctypes.c_double(0), ctypes.c_double(0)
-        _check(lib().tc_calibrate(self._h, ctypes.c_void_p(_stream(stream)), ctypes.byref(wl),
-                                  ctypes.byref(ws)))
-        return float(wl.value), float(ws.value)
+    def calibrate(self, n_slices: int = CALIBRATION_SLICES, stream=None) -> np.ndarray:
+        """The plan's time profile on this device: ms of each of ``n_slices``
+        near-equal-cost slices counted alone (tc_calibrate)."""
+        ms = np.zeros(int(n_slices), dtype=np.float64)
+        _check(lib().tc_calibrate(self._h, ctypes.c_void_p(_stream(stream)), int(n_slices),
+                                  ms.ctypes.data_as(ctypes.c_void_p)))
+        return ms
 
     def chunks(self):
         """(first live edge of every chunk, plan cost prefix at it): two int64
@@ -392,19 +395,37 @@ def partition_prefix(prefix: Sequence[int], world_size: int) -> list:
     return [int(x) for x in b]
 
 
-def partition_chunks(seg, cost, n_long_chunks: int, world_size: int, w_long: float = 1.0,
-                     w_short: float = 1.0) -> list:
-    """Host-only weighted chunk split (tc_partition_chunks): seg/cost are the
-    n_chunks+1 first-edge and cost-prefix arrays of Graph.chunks()."""
+def counters(reset: bool = False) -> dict:
+    """Diagnostic counters of the count kernels on the current device (tc_counters)."""
+    h = (ctypes.c_uint64 * 4)()
+    _check(lib().tc_counters(h, 1 if reset else 0))
+    return {"cuckoo_rebuilds": int(h[0])}
+
+
+def slice_bounds(cost, n_long_chunks: int, n_slices: int) -> list:
+    """Host-only slice bounds of a profile (tc_slice_bounds): first chunk of each slice."""
+    cs = np.ascontiguousarray(cost, dtype=np.int64)
+    f = np.zeros(int(n_slices) + 1, dtype=np.int64)
+    _check(lib().tc_slice_bounds(cs.ctypes.data_as(ctypes.c_void_p), cs.size - 1, int(n_long_chunks),
+                                 int(n_slices), f.ctypes.data_as(ctypes.c_void_p)))
+    return [int(x) for x in f]
+
+
+def partition_chunks(seg, cost, n_long_chunks: int, profile, world_size: int) -> list:
+    """Host-only profile-weighted chunk split (tc_partition_chunks): seg/cost are
+    the n_chunks+1 first-edge and cost-prefix arrays of Graph.chunks(), profile
+    the per-slice ms of tc_slice_bounds(len(profile))."""
     sg = np.ascontiguousarray(seg, dtype=np.int64)
     cs = np.ascontiguousarray(cost, dtype=np.int64)
+    ms = np.ascontiguousarray(profile, dtype=np.float64)
     if sg.shape != cs.shape or sg.size < 1:
         raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, "seg/cost must have n_chunks + 1 entries")
     b = np.zeros(int(world_size) + 1, dtype=np.int64)
     _check(lib().tc_partition_chunks(sg.ctypes.data_as(ctypes.c_void_p),
                                      cs.ctypes.data_as(ctypes.c_void_p), sg.size - 1,
-                                     int(n_long_chunks), int(world_size), float(w_long),
-                                     float(w_short), b.ctypes.data_as(ctypes.c_void_p)))
+                                     int(n_long_chunks), int(ms.size),
+                                     ms.ctypes.data_as(ctypes.c_void_p), int(world_size),
+                                     b.ctypes.data_as(ctypes.c_void_p)))
     return [int(x) for x in b]
 
 
@@ -522,30 +543,29 @@ class FusedSum:
             pass
 
 
-def agreed_weights(graph, group=None, stream=None):
-    """Per-class cost weights every rank agrees on: each rank calibrates
-    (tc_calibrate) and the ranks' values are averaged with one all_reduce
-    (the bounds must be identical on every rank).  None when not distributed."""
+def agreed_profile(graph, group=None, stream=None, n_slices: int = CALIBRATION_SLICES):
+    """A time profile every rank agrees on: each rank calibrates (tc_calibrate)
+    and the ranks' profiles are averaged with one all_reduce (the bounds must
+    be identical on every rank).  None when not distributed."""
     import torch
     import torch.distributed as dist
     if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
         return None
-    w = graph.calibrate(stream=stream)
+    ms = graph.calibrate(n_slices, stream=stream)
     dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
-    t = torch.tensor(w, dtype=torch.float64, device=dev)
+    t = torch.as_tensor(ms, dtype=torch.float64).to(dev)
     dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
-    wl, ws = (float(x) / dist.get_world_size(group) for x in t.cpu())
-    return (wl if wl > 0 else 1.0, ws if ws > 0 else 1.0)
+    return (t.cpu().numpy() / dist.get_world_size(group)).astype(np.float64)
 
 
 def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] = None,
-                      weights=None) -> int:
+                      profile=None) -> int:
     """T over a torch.distributed process group.
 
     Every rank holds the same replicated graph; rank r counts the live
     oriented edges [b_r, b_{r+1}) of the cost-balanced split
-    (tc_partition_weighted with ``weights``, the same on every rank — e.g.
-    :func:`agreed_weights` — or tc_partition's built-in weights) and a single
+    (tc_partition_measured with ``profile``, the same on every rank — e.g.
+    :func:`agreed_profile` — or tc_partition's built-in profile) and a single
     all_reduce(SUM) of the 8-byte partials (ProcessGroupNCCL over NVLink on
     the GPU box) gives T on every rank.  Two's-complement int64 addition is
     bit-identical to uint64 addition mod 2^64.  With ``fused`` (a
@@ -556,7 +576,7 @@ def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] 
     on = dist.is_available() and dist.is_initialized()
     world = dist.get_world_size(group) if on else 1
     rank = dist.get_rank(group) if on else 0
-    bounds = graph.partition(world) if weights is None else graph.partition(world, weights)
+    bounds = graph.partition(world) if profile is None else graph.partition(world, profile)
     if fused is not None:  # f4: the library's own sum over NVLink peer memory
         total = fused.count_range(graph, bounds[rank], bounds[rank + 1], stream=stream)
         return fused.check(int(total.item()) & (2**64 - 1))
@@ -569,5 +589,5 @@ def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] 
 from .sharded import build_csr_sharded, shard_cuts  # noqa: E402  (f2)
 
 __all__ = ["FusedSum", "build_csr_sharded", "shard_cuts", "Graph", "Options", "GraphInfo", "build_csr", "build_csr_host", "count_partitioned",
-           "partition_prefix", "partition_chunks", "agreed_weights", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
+           "partition_prefix", "partition_chunks", "slice_bounds", "counters", "agreed_profile", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
            "EXPORTS", "LIB_PATH"]

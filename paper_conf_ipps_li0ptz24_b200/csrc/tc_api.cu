@@ -2,6 +2,7 @@
 // translation (no exception crosses the ABI), the allocator hook, and the
 // host-side range/partition logic.  SURVEY.md §8(b).
 #include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -430,24 +431,86 @@ tc_status tc_partition_prefix(const int64_t* h_prefix, int64_t n_units, int32_t 
   });
 }
 
-tc_status tc_partition_chunks(const int64_t* h_seg, const int64_t* h_cost, int64_t n_chunks,
-                              int64_t n_long_chunks, int32_t world_size, double w_long,
-                              double w_short, int64_t* h_bounds) {
+namespace {
+
+// Slice bounds (chunk indices) of an n_slices profile: tc_slice_bounds.
+void slice_bounds(const int64_t* cost, int64_t nc, int64_t nL, int32_t K, int64_t* first) {
+  if (K == 1) {  // one slice: the whole chunk list
+    first[0] = 0;
+    first[1] = nc;
+    return;
+  }
+  const long double total = (long double)cost[nc], cl = (long double)cost[nL];
+  int KL = 0;
+  if (nL > 0) {
+    KL = total > 0 ? (int)std::llround((long double)K * cl / total) : K;
+    KL = std::max(KL, 1);
+    if (nc > nL) KL = std::min(KL, K - 1);
+    KL = std::min(KL, K);
+  }
+  const int KS = K - KL;
+  auto fill = [&](int64_t c0, int64_t c1, int k, int64_t* out) {
+    // out[j] = first chunk in [c0, c1] whose cost prefix reaches j/k of the class
+    const long double base = (long double)cost[c0], span = (long double)cost[c1] - base;
+    for (int j = 0; j < k; ++j) {
+      const long double t = base + span * j / k;
+      int64_t lo = c0, hi = c1;
+      while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if ((long double)cost[mid] < t) lo = mid + 1; else hi = mid;
+      }
+      out[j] = j == 0 ? c0 : lo;
+    }
+  };
+  if (KL > 0) fill(0, nL, KL, first);
+  if (KS > 0) fill(nL, nc, KS, first + KL);
+  first[K] = nc;
+  for (int j = 1; j <= K; ++j) first[j] = std::max(first[j], first[j - 1]);
+}
+
+}  // namespace
+
+tc_status tc_slice_bounds(const int64_t* h_cost, int64_t n_chunks, int64_t n_long_chunks,
+                          int32_t n_slices, int64_t* h_first) {
   return guarded([&] {
-    require(h_seg && h_cost && h_bounds, "NULL argument");
+    require(h_cost && h_first, "NULL argument");
+    require(n_chunks >= 0 && n_long_chunks >= 0 && n_long_chunks <= n_chunks, "bad chunk counts");
+    require(n_slices >= 1, "n_slices < 1");
+    for (int64_t c = 0; c < n_chunks; ++c) require(h_cost[c] <= h_cost[c + 1], "cost must be non-decreasing");
+    slice_bounds(h_cost, n_chunks, n_long_chunks, n_slices, h_first);
+  });
+}
+
+tc_status tc_partition_chunks(const int64_t* h_seg, const int64_t* h_cost, int64_t n_chunks,
+                              int64_t n_long_chunks, int32_t n_slices, const double* h_ms,
+                              int32_t world_size, int64_t* h_bounds) {
+  return guarded([&] {
+    require(h_seg && h_cost && h_ms && h_bounds, "NULL argument");
     require(n_chunks >= 0 && n_long_chunks >= 0 && n_long_chunks <= n_chunks, "bad chunk counts");
     require(world_size >= 1, "world_size < 1");
-    require(w_long > 0 && w_short > 0, "weights must be > 0");
+    require(n_slices >= 1, "n_slices < 1");
+    for (int32_t i = 0; i < n_slices; ++i)
+      require(std::isfinite(h_ms[i]) && h_ms[i] >= 0, "profile entries must be finite and >= 0");
     for (int64_t c = 0; c < n_chunks; ++c)
       require(h_seg[c] <= h_seg[c + 1] && h_cost[c] <= h_cost[c + 1], "prefixes must be non-decreasing");
-    // Weighted cost prefix over chunks: long chunks [0, nL) come first, so
-    // W(c) = w_long * cost[c] up to nL, then the short class's units at
-    // w_short.  Cut r is the chunk boundary nearest to r/P of W(nc).
-    const int64_t nc = n_chunks, nL = n_long_chunks;
-    const long double CL = (long double)h_cost[nL];
+    const int64_t nc = n_chunks;
+    std::vector<int64_t> first(n_slices + 1);
+    slice_bounds(h_cost, nc, n_long_chunks, n_slices, first.data());
+    // W(c): the profile's time up to chunk boundary c — slice i contributes
+    // h_ms[i] spread over its cost units (a slice without cost weighs its
+    // ms at its first boundary).  Non-decreasing in c.
+    std::vector<long double> Wslice(n_slices + 1, 0);
+    for (int32_t i = 0; i < n_slices; ++i) Wslice[i + 1] = Wslice[i] + (long double)h_ms[i];
+    std::vector<int32_t> slice_of(nc + 1);
+    for (int32_t i = 0; i < n_slices; ++i)
+      for (int64_t c = first[i]; c < first[i + 1]; ++c) slice_of[c] = i;
+    slice_of[nc] = n_slices;
     auto W = [&](int64_t c) -> long double {
-      return c <= nL ? w_long * (long double)h_cost[c]
-                     : w_long * CL + w_short * ((long double)h_cost[c] - CL);
+      const int32_t i = slice_of[c];
+      if (i >= n_slices) return Wslice[n_slices];
+      const long double c0 = (long double)h_cost[first[i]], c1 = (long double)h_cost[first[i + 1]];
+      const long double f = c1 > c0 ? ((long double)h_cost[c] - c0) / (c1 - c0) : 0;
+      return Wslice[i] + f * (long double)h_ms[i];
     };
     const long double total = W(nc);
     h_bounds[0] = h_seg[0];
@@ -467,19 +530,33 @@ tc_status tc_partition_chunks(const int64_t* h_seg, const int64_t* h_cost, int64
   });
 }
 
-tc_status tc_partition_weighted(const tc_graph* g, int32_t world_size, double w_long,
-                                double w_short, int64_t* h_bounds) {
+tc_status tc_partition_measured(const tc_graph* g, int32_t world_size, int32_t n_slices,
+                                const double* h_ms, int64_t* h_bounds) {
   return guarded([&] {
-    require(g && h_bounds, "NULL argument");
+    require(g && h_bounds && h_ms, "NULL argument");
     const tc::Plan& P = g->plan;
     const tc_status st = tc_partition_chunks(P.h_chunk_seg.data(), P.h_chunk_cost.data(), P.n_chunks,
-                                             P.n_long_chunks, world_size, w_long, w_short, h_bounds);
+                                             P.n_long_chunks, n_slices, h_ms, world_size, h_bounds);
     if (st != TC_OK) tc::fail(st, t_last_error);
   });
 }
 
 tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds) {
-  return tc_partition_weighted(g, world_size, TC_PARTITION_W_LONG, TC_PARTITION_W_SHORT, h_bounds);
+  return guarded([&] {
+    require(g && h_bounds, "NULL argument");
+    const tc::Plan& P = g->plan;
+    // the built-in profile: the classes as two slices (one if a class is empty)
+    const int64_t nc = P.n_chunks, nL = P.n_long_chunks;
+    const double cl = (double)P.h_chunk_cost[nL], cs = (double)(P.h_chunk_cost[nc] - P.h_chunk_cost[nL]);
+    double ms[2];
+    int32_t k = 0;
+    if (nL > 0) ms[k++] = cl;
+    if (nc > nL) ms[k++] = TC_PARTITION_SHORT_RATIO * cs;
+    if (k == 0) ms[k++] = 0;
+    const tc_status st = tc_partition_chunks(P.h_chunk_seg.data(), P.h_chunk_cost.data(), nc, nL, k,
+                                             ms, world_size, h_bounds);
+    if (st != TC_OK) tc::fail(st, t_last_error);
+  });
 }
 
 tc_status tc_plan_chunks(const tc_graph* g, int64_t* h_seg, int64_t* h_cost) {
@@ -491,37 +568,39 @@ tc_status tc_plan_chunks(const tc_graph* g, int64_t* h_seg, int64_t* h_cost) {
   });
 }
 
-tc_status tc_calibrate(const tc_graph* g, void* stream, double* h_ns_long, double* h_ns_short) {
+tc_status tc_calibrate(const tc_graph* g, void* stream, int32_t n_slices, double* h_ms) {
   return guarded([&] {
-    require(g && h_ns_long && h_ns_short, "NULL argument");
+    require(g && h_ms, "NULL argument");
+    require(n_slices >= 1, "n_slices < 1");
     const tc::Plan& P = g->plan;
     cudaStream_t s = (cudaStream_t)stream;
-    *h_ns_long = *h_ns_short = 0;
+    for (int32_t i = 0; i < n_slices; ++i) h_ms[i] = 0;
     if (P.n_chunks == 0) return;
-    const int64_t nc = P.n_chunks, nL = P.n_long_chunks;
+    std::vector<int64_t> first(n_slices + 1);
+    slice_bounds(P.h_chunk_cost.data(), P.n_chunks, P.n_long_chunks, n_slices, first.data());
     tc::DevBuf<unsigned long long> d(1, s);
-    cudaEvent_t ev[3] = {};
+    std::vector<cudaEvent_t> ev(n_slices + 1, nullptr);
     struct Guard {
-      cudaEvent_t* e;
+      std::vector<cudaEvent_t>& e;
       ~Guard() {
-        for (int i = 0; i < 3; ++i)
-          if (e[i]) cudaEventDestroy(e[i]);
+        for (auto x : e)
+          if (x) cudaEventDestroy(x);
       }
     } guard{ev};
     for (auto& e : ev) TC_CUDA(cudaEventCreate(&e));
-    tc::count_chunks(g, 0, nc, 0, P.S, s, d.get());  // warm-up
+    tc::count_chunks(g, 0, P.n_chunks, 0, P.S, s, d.get());  // warm-up
     TC_CUDA(cudaEventRecord(ev[0], s));
-    if (nL > 0) tc::count_chunks(g, 0, nL, 0, P.S, s, d.get());
-    TC_CUDA(cudaEventRecord(ev[1], s));
-    if (nc > nL) tc::count_chunks(g, nL, nc, 0, P.S, s, d.get());
-    TC_CUDA(cudaEventRecord(ev[2], s));
-    TC_CUDA(cudaEventSynchronize(ev[2]));
-    float ms_l = 0, ms_s = 0;
-    TC_CUDA(cudaEventElapsedTime(&ms_l, ev[0], ev[1]));
-    TC_CUDA(cudaEventElapsedTime(&ms_s, ev[1], ev[2]));
-    const int64_t cl = P.h_chunk_cost[nL], cs = P.h_chunk_cost[nc] - cl;
-    if (nL > 0 && cl > 0) *h_ns_long = 1e6 * ms_l / (double)cl;
-    if (nc > nL && cs > 0) *h_ns_short = 1e6 * ms_s / (double)cs;
+    for (int32_t i = 0; i < n_slices; ++i) {
+      const int64_t c0 = first[i], c1 = first[i + 1];
+      if (c1 > c0) tc::count_chunks(g, c0, c1, P.h_chunk_seg[c0], P.h_chunk_seg[c1], s, d.get());
+      TC_CUDA(cudaEventRecord(ev[i + 1], s));
+    }
+    TC_CUDA(cudaEventSynchronize(ev[n_slices]));
+    for (int32_t i = 0; i < n_slices; ++i) {
+      float ms = 0;
+      TC_CUDA(cudaEventElapsedTime(&ms, ev[i], ev[i + 1]));
+      h_ms[i] = first[i + 1] > first[i] ? (double)ms : 0.0;
+    }
   });
 }
 
@@ -665,6 +744,13 @@ void tc_free(tc_graph* g) {
   cudaDeviceSynchronize();
   rebind(g, nullptr);
   delete g;
+}
+
+tc_status tc_counters(uint64_t* h_counters, int32_t reset) {
+  return guarded([&] {
+    require(h_counters != nullptr, "NULL argument");
+    tc::read_counters(h_counters, reset != 0);
+  });
 }
 
 const char* tc_last_error(void) { return t_last_error.c_str(); }

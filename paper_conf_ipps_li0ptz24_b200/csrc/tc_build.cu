@@ -1056,6 +1056,7 @@ Tuning tuning_from_env() {
   t.wait_hint_ns = get("TC_WAIT_HINT", t.wait_hint_ns, 0, 10000000);
   t.cs_div = get("TC_CS_DIV", t.cs_div, 0, 64);
   t.short_linear = get("TC_SHORT_LINEAR", t.short_linear, 0, 1);
+  t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
   t.l2_meta = get("TC_L2_META", t.l2_meta, 0, 1);
   t.l2_keys = get("TC_L2_KEYS", t.l2_keys, 0, 2);
   t.l2_persist_mb = get("TC_L2_PERSIST_MB", t.l2_persist_mb, 0, 1 << 16);

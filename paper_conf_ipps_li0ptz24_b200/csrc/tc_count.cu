@@ -60,7 +60,7 @@ constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flig
 #define TC_UNROLL_SHORT 2
 #endif
 constexpr int kUnrollShort = TC_UNROLL_SHORT;  // tiles in flight per consumer warp (short class)
-constexpr int kMaxKicks = 96;    // cuckoo displacement bound before the linear fallback
+constexpr int kMaxKicks = 96;    // cuckoo displacement bound before the linear fallback (Tuning::max_kicks)
 constexpr int kMaxSlots = 4;     // chunk slots in SMEM (runtime count: Tuning::slots)
 
 // ------------------------------------------------------------------ mbarrier (PTX)
@@ -114,6 +114,11 @@ __device__ __forceinline__ int named_sync_or(int id, int nthreads, int pred) {
   return r;
 }
 
+// Diagnostic counters (tc_counters): [0] chunks whose two-choice table
+// inserts failed and were rebuilt with linear probing.  Touched only on that
+// rare path.
+__device__ unsigned long long g_counters[4];
+
 // ------------------------------------------------------------------ L2 policy
 // Cache-policy loads (PTX createpolicy + ld.global.nc.L2::cache_hint; the
 // policy lives in a uniform descriptor, so a hinted load costs no extra
@@ -150,9 +155,10 @@ __device__ __forceinline__ uint32_t hash2(int32_t key, uint32_t n) {
   return __umulhi((uint32_t)key * 0x85EBCA77u + 0x7F4A7C15u, n);
 }
 
-__device__ __forceinline__ bool cuckoo_insert(int* __restrict__ T, uint32_t n, int32_t key) {
+__device__ __forceinline__ bool cuckoo_insert(int* __restrict__ T, uint32_t n, int32_t key,
+                                              int max_kicks) {
   uint32_t pos = hash1(key, n);
-  for (int i = 0; i < kMaxKicks; ++i) {
+  for (int i = 0; i < max_kicks; ++i) {
     const int old = atomicExch(&T[pos], key);
     if (old < 0) return true;
     key = old;  // displaced: move it to its other slot
@@ -174,9 +180,9 @@ __device__ __forceinline__ void linear_insert(int* __restrict__ T, uint32_t n, i
 // Support mode (8-B entries {key, payload}; empty = all ones).  The same
 // two-choice / linear schemes, moving the payload with its key.
 __device__ __forceinline__ bool cuckoo_insert64(unsigned long long* __restrict__ T, uint32_t n,
-                                                int32_t key, unsigned long long e) {
+                                                int32_t key, unsigned long long e, int max_kicks) {
   uint32_t pos = hash1(key, n);
-  for (int i = 0; i < kMaxKicks; ++i) {
+  for (int i = 0; i < max_kicks; ++i) {
     const unsigned long long old = atomicExch(&T[pos], e);
     if ((int)(uint32_t)old < 0) return true;
     e = old;
@@ -895,7 +901,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         unsigned long long* H = reinterpret_cast<unsigned long long*>(c.sHash) + d.x;
         const unsigned long long e = ((unsigned long long)(uint32_t)j << 32) | (uint32_t)key;
         if (lin) linear_insert64(H, (uint32_t)d.y, key, e);
-        else if (!cuckoo_insert64(H, (uint32_t)d.y, key, e)) linear = true;  // flag, below
+        else if (!cuckoo_insert64(H, (uint32_t)d.y, key, e, pv.max_kicks)) linear = true;  // flag, below
       }
     };
     const bool want_linear = linear;
@@ -903,6 +909,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     warp_walk<kInsU>(c.sGP, G, i0, i1, load_row,
                      [&](int g, int k, int32_t key) { ins_sup(g, k, key, want_linear); });
     if (!want_linear && named_sync_or(1, PT, linear)) {  // a cuckoo insert failed
+      if (pt == 0) atomicAdd(&g_counters[0], 1ull);
       for (int i = pt; i < 2 * nslots; i += PT) c.sHash[i] = -1;
       named_sync(1, PT);
       warp_walk<kInsU>(c.sGP, G, i0, i1, load_row,
@@ -925,9 +932,10 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       const int2 d = c.sInfo[g];
       if (d.x < 0) return;
       if (d.y <= 0) bitmap_insert(c.sHash + d.x, d.y, key);
-      else if (!cuckoo_insert(c.sHash + d.x, (uint32_t)d.y, key)) ok = false;
+      else if (!cuckoo_insert(c.sHash + d.x, (uint32_t)d.y, key, pv.max_kicks)) ok = false;
     });
     if (named_sync_or(1, PT, !ok)) {  // uniform over producers: rebuild with linear probing
+      if (pt == 0) atomicAdd(&g_counters[0], 1ull);
       linear = true;
       for (int i = pt; i < nslots; i += PT) c.sHash[i] = -1;
       named_sync(1, PT);
@@ -1236,12 +1244,21 @@ PlanView plan_view(const tc_graph* g) {
   pv.short_linear = P.tune.short_linear;
   pv.seg_edge = nullptr;
   pv.sup = nullptr;
+  pv.max_kicks = P.tune.max_kicks;
   pv.l2_meta = P.tune.l2_meta;
   pv.l2_keys = P.tune.l2_keys;
   return pv;
 }
 
 }  // namespace
+
+void read_counters(uint64_t* h, bool reset) {
+  TC_CUDA(cudaMemcpyFromSymbol(h, g_counters, sizeof(unsigned long long) * 4));
+  if (reset) {
+    const unsigned long long z[4] = {0, 0, 0, 0};
+    TC_CUDA(cudaMemcpyToSymbol(g_counters, z, sizeof(z)));
+  }
+}
 
 int num_sms() {
   int dev = 0, v = 0;

@@ -113,6 +113,7 @@ struct PlanView {
   int probe_mode;
   int short_linear;            // short class always probes linearly (Tuning::short_linear)
   int l2_meta, l2_keys;        // L2 eviction policy of plan-metadata / key loads (Tuning)
+  int max_kicks;               // cuckoo displacement bound (Tuning::max_kicks)
   // support mode only (tc_support; nullptr when counting)
   const int64_t* seg_edge;     // [S] CSR position of segment s's own edge (u,v)
   unsigned* sup;               // [m] per-edge triangle counts (accumulated)
@@ -143,6 +144,8 @@ struct Tuning {
   int cs_div = 0;         // short-class chunk cost = chunk_cost / cs_div (0: auto, 2 when the live
                           // edges carry < 2 keys on average, e.g. road graphs, else 1)
   int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
+  int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
+                          // 0 forces the rebuild of every chunk with a hash table: tests)
   int l2_meta = 0;        // L2 policy of the producers' plan-metadata loads: 0 normal, 1 evict_first
   int l2_keys = 0;        // L2 policy of the key loads: 0 normal, 1 evict_first, 2 evict_last
   int l2_persist_mb = 0;  // > 0: access-policy window marking the hottest (last) MB of col persisting
@@ -232,6 +235,7 @@ int flat_occupancy(int64_t smem_bytes);
 int num_sms();
 void support_all(const tc_graph* g, cudaStream_t s, unsigned* d_sup);   // f1, tc_support
 void edge_ends(const tc_graph* g, cudaStream_t s, int32_t* d_u, int32_t* d_v);
+void read_counters(uint64_t* h, bool reset);  // tc_counters
 
 // tc_fused.cu (f4: fused cross-GPU sum over NVLink peer memory, tc_fused.cuh)
 FuseArgs fuse_args(uint64_t* own, uint64_t* mc, uint64_t* const* peers, int world,

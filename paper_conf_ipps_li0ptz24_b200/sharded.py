@@ -217,7 +217,9 @@ def build_csr_sharded(src, dst, num_vertices: int, group=None, keep_isolated: bo
     bound (required: all ranks must key the same way).  Returns a
     :class:`Graph` equal, byte for byte in its CSR, to ``build_csr`` of the
     concatenated pairs.  ``timings`` (optional dict) receives host wall ms
-    per phase (after a stream sync at each phase end).
+    per phase (after a stream sync at each phase end).  ``stream``: the
+    CUDA stream of every step; it is made torch's current stream for the
+    duration, so the collectives are ordered after the native steps.
     """
     import time
     import torch
@@ -226,6 +228,13 @@ def build_csr_sharded(src, dst, num_vertices: int, group=None, keep_isolated: bo
         raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, "build_csr_sharded needs num_vertices >= 0")
     if src.shape != dst.shape or src.dim() != 1:
         raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, "src/dst must be 1-D of equal length")
+    if stream is not None and steps is None:
+        # the collectives order after torch's CURRENT stream: make the given
+        # stream current for the whole build so the native steps (enqueued on
+        # it) and the collectives are ordered with each other
+        with torch.cuda.stream(stream):
+            return build_csr_sharded(src, dst, num_vertices, group, keep_isolated, options,
+                                     None, None, timings)
     n = int(num_vertices)
     steps = steps or NativeSteps(stream)
     comm = _Comm(group)

@@ -52,11 +52,11 @@ def main():
     T = g.count()
     w = None
     if a.calibrate:
-        w = tuple(x if x > 0 else 1.0 for x in g.calibrate())
-        print(json.dumps({"calibration_ns_per_unit": w}), flush=True)
+        w = g.calibrate()
+        print(json.dumps({"profile_ms": w.round(3).tolist()}), flush=True)
     full, _ = time_range(g, 0, g.m_live, flush, a.reps, out)
     for P in [int(x) for x in a.worlds.split(",")]:
-        b = g.partition(P, w) if w else g.partition(P)
+        b = g.partition(P, w) if w is not None else g.partition(P)
         ms, parts = [], []
         for r in range(P):
             t, p = time_range(g, b[r], b[r + 1], flush, a.reps, out)
@@ -65,7 +65,7 @@ def main():
         mean = sum(ms) / P
         print(json.dumps({"config": a.config, "P": P, "full_ms": full, "range_ms": ms,
                           "max_over_mean": max(ms) / mean, "sum_ms": sum(ms),
-                          "weights": w, "bounds": b, "sum_ok": (sum(parts) & (2**64 - 1)) == T}), flush=True)
+                          "bounds": b, "sum_ok": (sum(parts) & (2**64 - 1)) == T}), flush=True)
     g.close()
 
 

@@ -75,10 +75,10 @@ def test_bad_arguments_rejected_before_device(tc):
     assert L.tc_count(None, None, None) == 1
     assert L.tc_count_range(None, 0, 0, None, None) == 1
     assert L.tc_partition(None, 2, None) == 1
-    assert L.tc_partition_weighted(None, 2, 1.0, 1.0, None) == 1
+    assert L.tc_partition_measured(None, 2, 1, None, None) == 1
     assert L.tc_plan_chunks(None, None, None) == 1
-    d = ctypes.c_double(0)
-    assert L.tc_calibrate(None, None, ctypes.byref(d), ctypes.byref(d)) == 1
+    assert L.tc_calibrate(None, None, 4, None) == 1
+    assert L.tc_slice_bounds(None, 0, 0, 1, None) == 1
     assert L.tc_count_range_fused(None, 0, 0, None, None, None, 1, 1, None, None) == 1
     assert L.tc_graph_info(None, None) == 1
     assert L.tc_support(None, None, None) == 1
@@ -133,40 +133,70 @@ def test_struct_layouts_match_header(tc, tmp_path):
     assert got == want
 
 
-def _weighted_loads(seg, cost, nL, b, wl, ws):
-    """Weighted cost of each range [b_r, b_{r+1}) (ranges are chunk-aligned)."""
-    W = np.where(np.arange(len(cost)) <= nL, wl * cost,
-                 wl * cost[nL] + ws * (cost - cost[nL])).astype(float)
-    idx = [int(np.searchsorted(seg, x)) for x in b]
-    return [W[idx[r + 1]] - W[idx[r]] for r in range(len(b) - 1)], W
+def _profile_W(seg, cost, nL, first, ms):
+    """The profile's time at every chunk boundary (tc_partition_chunks' W)."""
+    W = np.zeros(len(cost))
+    acc = 0.0
+    for i in range(len(ms)):
+        c0, c1 = first[i], first[i + 1]
+        span = cost[c1] - cost[c0]
+        for c in range(c0, c1):
+            W[c] = acc + (ms[i] * (cost[c] - cost[c0]) / span if span > 0 else 0.0)
+        acc += ms[i]
+    W[-1] = acc
+    return W
+
+
+@pytest.mark.parametrize("K", [1, 2, 7, 64])
+def test_slice_bounds(tc, K):
+    """Slices cover the chunks in order, never straddle the class boundary and
+    split each class at near-equal cost."""
+    rng = np.random.default_rng(K)
+    nc, nL = 3000, 1800
+    cost = np.concatenate([[0], np.cumsum(rng.integers(1, 400, size=nc))])
+    f = tc.slice_bounds(cost, nL, K)
+    assert f[0] == 0 and f[-1] == nc and all(a <= b for a, b in zip(f, f[1:]))
+    if K >= 2:
+        assert nL in f  # the class boundary is a slice boundary
+    step = np.diff(cost).max()
+    for cls0, cls1 in ((0, nL), (nL, nc)):
+        inner = [i for i in range(K) if cls0 <= f[i] and f[i + 1] <= cls1 and f[i + 1] > f[i]]
+        if len(inner) > 1:
+            sizes = [cost[f[i + 1]] - cost[f[i]] for i in inner]
+            assert max(sizes) - min(sizes) <= 2 * step
+    assert tc.slice_bounds(cost, 0, 4)[-1] == nc and tc.slice_bounds(cost, nc, 4)[-1] == nc
 
 
 @pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
-@pytest.mark.parametrize("weights", [(1.0, 1.0), (1.0, 2.2), (3.0, 0.5)])
-def test_partition_chunks_weighted_balance(tc, world, weights):
-    """cuts on the weighted cost prefix; every range within one
-    chunk's weighted cost of the ideal share, chunk-aligned, covering [0, m_live)."""
-    rng = np.random.default_rng(world)
+@pytest.mark.parametrize("K", [2, 16, 64])
+def test_partition_chunks_profile_balance(tc, world, K):
+    """cuts on the profile-weighted cost prefix; every range
+    within one chunk's weight of the ideal share, chunk-aligned, covering
+    [0, m_live); a non-uniform profile moves the cuts."""
+    rng = np.random.default_rng(world * 100 + K)
     nc, nL = 3000, 1800
     cost = np.concatenate([[0], np.cumsum(rng.integers(1, 400, size=nc))])
     seg = np.concatenate([[0], np.cumsum(rng.integers(1, 50, size=nc))])
-    b = tc.partition_chunks(seg, cost, nL, world, *weights)
+    ms = rng.uniform(0.5, 3.0, size=K)
+    b = tc.partition_chunks(seg, cost, nL, ms, world)
     assert b[0] == 0 and b[-1] == seg[-1] and all(x <= y for x, y in zip(b, b[1:]))
     assert set(b) <= set(seg.tolist())
-    loads, W = _weighted_loads(seg, cost, nL, b, *weights)
-    assert abs(sum(loads) - W[-1]) < 1e-6 * W[-1]
-    step = np.diff(W).max()
-    assert max(abs(x - W[-1] / world) for x in loads) <= step
+    W = _profile_W(seg, cost, nL, tc.slice_bounds(cost, nL, K), ms)
+    assert abs(W[-1] - ms.sum()) < 1e-9 * ms.sum()
+    idx = [int(np.searchsorted(seg, x)) for x in b]
+    loads = [W[idx[r + 1]] - W[idx[r]] for r in range(world)]
+    assert max(abs(x - W[-1] / world) for x in loads) <= np.diff(W).max() + 1e-12
 
 
-def test_partition_chunks_weights_move_the_cut(tc):
-    """Heavier short-class units pull the 2-way cut back into the long class."""
+def test_partition_chunks_profile_moves_the_cut(tc):
+    """A slower long class pulls the 2-way cut toward the front."""
     seg = np.arange(11, dtype=np.int64) * 10
     cost = np.arange(11, dtype=np.int64) * 100  # 10 equal chunks, 5 long
-    assert tc.partition_chunks(seg, cost, 5, 2, 1.0, 1.0) == [0, 50, 100]
-    assert tc.partition_chunks(seg, cost, 5, 2, 1.0, 3.0)[1] == 70  # W: 5 + 15 -> cut at 10
-    assert tc.partition_chunks(seg, cost, 5, 2, 3.0, 1.0)[1] == 30
+    assert tc.slice_bounds(cost, 5, 2) == [0, 5, 10]
+    assert tc.partition_chunks(seg, cost, 5, [1.0, 1.0], 2) == [0, 50, 100]
+    assert tc.partition_chunks(seg, cost, 5, [1.0, 3.0], 2)[1] == 70  # W: 1 + 3 -> cut at 2
+    assert tc.partition_chunks(seg, cost, 5, [3.0, 1.0], 2)[1] == 30
     with pytest.raises(tc.InvalidArgument):
-        tc.partition_chunks(seg, cost, 5, 2, 0.0, 1.0)
+        tc.partition_chunks(seg, cost, 5, [-1.0, 1.0], 2)
     with pytest.raises(tc.InvalidArgument):
-        tc.partition_chunks(seg[::-1].copy(), cost, 5, 2)
+        tc.partition_chunks(seg[::-1].copy(), cost, 5, [1.0, 1.0], 2)

@@ -1,9 +1,9 @@
 """Measured balance of the multi-GPU edge ranges, emulated
-on one B200: every rank's tc_count_range of the tc_partition_weighted split
-(weights = this device's tc_calibrate ns per cost unit) is timed alone with
-CUDA events, L2 flushed before each; the slowest range may exceed the mean
-by at most 5 %, and the partials sum to the oracle's stored T (the
-per-edge intersections are independent, so any cut is exact)."""
+on one B200: every rank's tc_count_range of the tc_partition_measured split
+(profile = this device's tc_calibrate, 64 slices) is timed alone with CUDA
+events, L2 flushed before each; the slowest range may exceed the mean by at
+most 5 %, and the partials sum to the oracle's stored T (the per-edge
+intersections are independent, so any cut is exact)."""
 import json
 import os
 import statistics
@@ -52,7 +52,7 @@ def test_partition_balance_measured(tc, cfg):
     with tc.build_csr(ds, dd, n) as g:
         del ds, dd
         w = g.calibrate()
-        assert w[0] > 0 and w[1] > 0
+        assert (w >= 0).all() and w.sum() > 0
         flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
         out = torch.zeros(1, dtype=torch.int64, device="cuda")
         report = {}
@@ -63,6 +63,6 @@ def test_partition_balance_measured(tc, cfg):
             assert sum(p for _, p in res) & (2**64 - 1) == stored["triangles"]
             report[P] = (max(ms) / (sum(ms) / P), [round(t, 3) for t in ms])
         del flush
-        print(cfg, "weights ns/unit", w, report)
+        print(cfg, "profile ms", np.round(w, 3).tolist(), report)
         for P, (ratio, ms) in report.items():
-            assert ratio <= BALANCE_MAX, f"{cfg} P={P}: max/mean {ratio:.3f} {ms} (weights {w})"
+            assert ratio <= BALANCE_MAX, f"{cfg} P={P}: max/mean {ratio:.3f} {ms}"
