@@ -119,31 +119,6 @@ __device__ __forceinline__ int named_sync_or(int id, int nthreads, int pred) {
 // rare path.
 __device__ unsigned long long g_counters[4];
 
-// ------------------------------------------------------------------ L2 policy
-// Cache-policy loads (PTX createpolicy + ld.global.nc.L2::cache_hint; the
-// policy lives in a uniform descriptor, so a hinted load costs no extra
-// instruction).  kind: 0 evict_normal, 1 evict_first, 2 evict_last.
-__device__ __forceinline__ uint64_t l2_policy(int kind) {
-  uint64_t p;
-  if (kind == 1)
-    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-  else if (kind == 2)
-    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-  else
-    asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
-  return p;
-}
-__device__ __forceinline__ int32_t ldp(const int32_t* a, uint64_t pol) {
-  int32_t v;
-  asm("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
-  return v;
-}
-__device__ __forceinline__ int64_t ldp(const int64_t* a, uint64_t pol) {
-  int64_t v;
-  asm("ld.global.nc.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(v) : "l"(a), "l"(pol));
-  return v;
-}
-
 // ------------------------------------------------------------------ hashing
 // A table is (off, n): n slots starting at sHash[off].  The slot of a key is
 // a multiplicative hash mapped onto [0, n) by a 32x32 -> high-32 multiply
@@ -400,7 +375,7 @@ __device__ __forceinline__ unsigned probe_tile(const ChunkSmem& c, int z, int zw
 // measured slower: 4-tile batches 66 ms, 8-tile batches spill, vs 62.5 ms.)
 template <int kB>
 __device__ __forceinline__ void load_batch(const ChunkSmem& c, const int32_t* colL, int t,
-                                           int32_t (&key)[kB], uint64_t pk) {
+                                           int32_t (&key)[kB]) {
   int x[kB];
 #pragma unroll
   for (int q = 0; q < kB; q += 4)
@@ -409,7 +384,7 @@ __device__ __forceinline__ void load_batch(const ChunkSmem& c, const int32_t* co
   // ONE IMAD.WIDE.U32 x * 4 + colL (left to itself, nvcc re-associates it into
   // a 64-bit add-with-carry + LEA pair, 4 instructions per key)
 #pragma unroll
-  for (int u = 0; u < kB; ++u) key[u] = ldp(colL + (uint32_t)x[u], pk);
+  for (int u = 0; u < kB; ++u) key[u] = __ldg(colL + (uint32_t)x[u]);
 }
 
 // col + lane in a register the compiler cannot see through.
@@ -427,11 +402,10 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   unsigned cnt = 0;
   const int lane = threadIdx.x & 31;
   const int32_t* colL = lane_base(pv.col, lane);
-  const uint64_t pk = l2_policy(pv.l2_keys);
   int t = t0;
   for (; t + kB <= t1; t += kB) {
     int32_t key[kB];
-    load_batch<kB>(c, colL, t, key, pk);
+    load_batch<kB>(c, colL, t, key);
     int z[kB], zw[kB];
 #pragma unroll
     for (int q = 0; q < kB; q += 4) {
@@ -463,7 +437,7 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
     int z[8], zw[8];
     int32_t key[8];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) key[u] = ldp(colL + (uint32_t)c.sT0[min(t + u, t1 - 1)], pk);
+    for (int u = 0; u < 8; ++u) key[u] = __ldg(colL + (uint32_t)c.sT0[min(t + u, t1 - 1)]);
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const int tt = min(t + u, t1 - 1);
@@ -479,6 +453,136 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   return cnt;
 }
 
+// ------------------------------------------------------------------ bulk-staged keys
+// LONG class with the keys staged in shared memory by the bulk-copy engine
+// (cp.async.bulk global -> shared, completion counted in bytes on an
+// mbarrier), instead of loaded into registers: each consumer warp owns a ring
+// of kR stages of one 8-tile batch each, and keeps kR - 1 batches in flight
+// while it probes the current one, so the keys in flight are bounded by
+// shared memory rather than by the 64 registers of a 1024-thread CTA (the
+// long-scoreboard wait on the key load is the top stall of walk_long).
+// A batch's 8 tiles are grouped into RUNS of chained windows (x_u within
+// [x_{u-1}, x_{u-1} + 32]: consecutive tiles of one suffix); each run is one
+// copy of its 16-B aligned superset [x_head & ~3, (x_last + 35) & ~3), so a
+// stage holds at most 8 x 144 B.  Tile u's keys start at int offs[u] of the
+// stage; lane l reads offs[u] + l (one conflict-free LDS).
+constexpr int kStageInts = 8 * 36;  // 8 tiles x 144 B
+
+struct KeyRing {
+  int* data;      // [kR][kStageInts]
+  int* offs;      // [kR][8]
+  uint64_t* bar;  // [kR], count 1 (lane 0's arrive.expect_tx)
+};
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(
+                   smem_u32(b)),
+               "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// Issue the copies of tiles [t, t + 8) (clamped to t1 - 1) into stage st.
+__device__ __forceinline__ void ring_issue(const ChunkSmem& c, const int32_t* col, int t, int t1,
+                                           const KeyRing& kr, int st, int lane) {
+  constexpr unsigned FULL = 0xffffffffu;
+  const int u = min(lane, 7);
+  const int x = c.sT0[min(t + u, t1 - 1)];
+  const int xp = __shfl_up_sync(FULL, x, 1);
+  const bool head = lane < 8 && (lane == 0 || x < xp || x > xp + 32);
+  const unsigned H = __ballot_sync(FULL, head);
+  const unsigned above = H & ~((2u << u) - 1u);          // heads after tile u
+  const int last = above ? __ffs(above) - 2 : 7;         // last tile of u's run (heads only)
+  const int hl = 31 - __clz(H & ((2u << u) - 1u));        // u's run head
+  const int xl = __shfl_sync(FULL, x, last);
+  uint32_t a = 0, bytes = 0;
+  if (head) {
+    a = (uint32_t)x & ~3u;
+    bytes = 4u * ((((uint32_t)xl + 35u) & ~3u) - a);
+  }
+  uint32_t incl = bytes;
+#pragma unroll
+  for (int o = 1; o < 8; o <<= 1) {
+    const uint32_t v = __shfl_up_sync(FULL, incl, o);
+    if (lane >= o) incl += v;
+  }
+  const uint32_t excl = incl - bytes, total = __shfl_sync(FULL, incl, 7);
+  const uint32_t hd = __shfl_sync(FULL, excl, hl), ha = __shfl_sync(FULL, a, hl);
+  if (lane < 8) kr.offs[st * 8 + lane] = (int)(hd / 4u + ((uint32_t)x - ha));
+  if (lane == 0) mbar_expect_tx(kr.bar + st, total);
+  __syncwarp();
+  if (head) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // WAR vs the stage's last LDS reads
+    bulk_g2s(kr.data + st * kStageInts + excl / 4u, col + a, bytes, kr.bar + st);
+  }
+}
+
+template <bool kLinear, bool kHuge, int kR>
+__device__ __forceinline__ unsigned walk_long_staged(const ChunkSmem& c, int t0, int t1,
+                                                     const PlanView& pv, int64_t ga,
+                                                     const KeyRing& kr, uint32_t& phase) {
+  unsigned cnt = 0;
+  const int lane = threadIdx.x & 31;
+  const int nb = (t1 - t0 + 7) >> 3;
+#pragma unroll
+  for (int j = 0; j < kR - 1; ++j)
+    if (j < nb) ring_issue(c, pv.col, t0 + 8 * j, t1, kr, j, lane);
+  int st = 0;  // stage of batch b
+  for (int b = 0; b < nb; ++b) {
+    if (b + kR - 1 < nb) ring_issue(c, pv.col, t0 + 8 * (b + kR - 1), t1, kr, (st + kR - 1) % kR, lane);
+    const int t = t0 + 8 * b;
+    mbar_wait(kr.bar + st, (phase >> st) & 1u, 0);
+    phase ^= 1u << st;
+    int o[8], z[8], zw[8];
+    *reinterpret_cast<int4*>(o) = *reinterpret_cast<const int4*>(kr.offs + st * 8);
+    *reinterpret_cast<int4*>(o + 4) = *reinterpret_cast<const int4*>(kr.offs + st * 8 + 4);
+    const int* sd = kr.data + st * kStageInts + lane;
+    int32_t key[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) key[u] = sd[o[u]];
+    if (t + 8 <= t1) {
+#pragma unroll
+      for (int q = 0; q < 8; q += 4) {
+        *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
+        *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
+      }
+    } else {  // last, partial batch: tiles past t1 repeat the last one, every lane masked
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int tt = min(t + u, t1 - 1);
+        z[u] = c.sT1[tt];
+        zw[u] = c.sT2[tt] | (t + u < t1 ? 0 : 32);
+      }
+    }
+    int zw_or = 0;
+#pragma unroll
+    for (int u = 0; u < 8; ++u) zw_or |= zw[u];
+    if ((zw_or >> 6) == 0) {
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const unsigned word = (unsigned)c.sT0[(key[u] >> 5) + z[u]];
+        const unsigned hit = (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
+        if (lane >= (zw[u] & 63)) cnt += hit;
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const unsigned hit = probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
+        if (lane >= (zw[u] & 63)) cnt += hit;
+      }
+    }
+    st = (st + 1 == kR) ? 0 : st + 1;
+  }
+  return cnt;
+}
+
 // SHORT class: the warp owns the flat keys [k0w, k1w) of the chunk.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0w, int k1w,
@@ -487,7 +591,6 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
   if (k0w >= k1w) return cnt;
   const int lane = threadIdx.x & 31;
   const unsigned below = (1u << lane) - 1u;
-  const uint64_t pk = l2_policy(pv.l2_keys);
   int s = seg_of(c.sA, S, k0w);
   for (int k0 = k0w; k0 < k1w; k0 += 32 * kUnrollShort) {
     int seg[kUnrollShort];
@@ -512,7 +615,7 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
         // col index sB + k < m < 2^32: a 32-bit add on the low word of sB
         // (two's complement wraps correctly) and one IMAD.WIDE
         const uint32_t lo = reinterpret_cast<const uint32_t*>(c.sB)[2 * seg[u]];
-        key[u] = ldp(pv.col + (lo + (uint32_t)k), pk);
+        key[u] = __ldg(pv.col + (lo + (uint32_t)k));
         gl[u] = c.sD[seg[u]];
       }
     }
@@ -537,9 +640,15 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
   return cnt;
 }
 
-template <bool kLinear>
+template <bool kLinear, int kR = 0>
 __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
-                                            const PlanView& pv) {
+                                            const PlanView& pv, const KeyRing* kr = nullptr,
+                                            uint32_t* phase = nullptr) {
+  if constexpr (kR > 0) {
+    if (h.is_long)
+      return h.huge ? walk_long_staged<kLinear, true, kR>(c, w0, w1, pv, h.ga, *kr, *phase)
+                    : walk_long_staged<kLinear, false, kR>(c, w0, w1, pv, h.ga, *kr, *phase);
+  }
   if (h.is_long)
     return h.huge ? walk_long<kLinear, true>(c, w0, w1, pv, h.ga)
                   : walk_long<kLinear, false>(c, w0, w1, pv, h.ga);
@@ -746,8 +855,7 @@ template <int kB, bool kSup = false>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
                                         int pt, int PT) {
-  const uint64_t pm = l2_policy(pv.l2_meta);  // plan metadata: read once per count
-  const int64_t sa = max(ldp(pv.chunk_seg + (cix), pm), e_begin), sb = min(ldp(pv.chunk_seg + (cix + 1), pm), e_end);
+  const int64_t sa = max(__ldg(pv.chunk_seg + (cix)), e_begin), sb = min(__ldg(pv.chunk_seg + (cix + 1)), e_end);
   if (sa >= sb) {  // empty after clipping to the range
     if (pt == 0) {
       hdr.S = 0;
@@ -757,12 +865,12 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   }
   const bool is_long = cix < pv.n_long_chunks;
   const int S = (int)(sb - sa);
-  const int64_t ga = ldp(pv.seg_group + (sa), pm), gb = (int64_t)ldp(pv.seg_group + (sb - 1), pm) + 1;
+  const int64_t ga = __ldg(pv.seg_group + (sa)), gb = (int64_t)__ldg(pv.seg_group + (sb - 1)) + 1;
   const int G = (int)(gb - ga);
-  const int64_t slot0 = ldp(pv.slot_prefix + (ga), pm);
-  const int nslots = (int)(ldp(pv.slot_prefix + (gb), pm) - slot0);
-  const int64_t kp0 = ldp(pv.key_prefix + (sa), pm);
-  const int T = is_long ? (int)((ldp(pv.key_prefix + (sb), pm) - kp0) >> 5) : 0;
+  const int64_t slot0 = __ldg(pv.slot_prefix + (ga));
+  const int nslots = (int)(__ldg(pv.slot_prefix + (gb)) - slot0);
+  const int64_t kp0 = __ldg(pv.key_prefix + (sa));
+  const int T = is_long ? (int)((__ldg(pv.key_prefix + (sb)) - kp0) >> 5) : 0;
   ChunkSmem c = kSup ? slot_view_sup(region, S, G, T, nslots) : slot_view(region, S, G, T);
 
   // 1. stage edges and groups; empty slots.  Each producer thread handles
@@ -777,11 +885,11 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       kp[r] = 0;
       st[r] = 0;
       ln[r] = gr[r] = 0;
-      if (i <= S) kp[r] = ldp(pv.key_prefix + (sa + i), pm);
+      if (i <= S) kp[r] = __ldg(pv.key_prefix + (sa + i));
       if (i < S) {
-        st[r] = ldp(pv.seg_start + (sa + i), pm);
-        ln[r] = ldp(pv.seg_len + (sa + i), pm);
-        gr[r] = ldp(pv.seg_group + (sa + i), pm);
+        st[r] = __ldg(pv.seg_start + (sa + i));
+        ln[r] = __ldg(pv.seg_len + (sa + i));
+        gr[r] = __ldg(pv.seg_group + (sa + i));
       }
     }
 #pragma unroll
@@ -797,8 +905,8 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     }
   }
   if (kSup)
-    for (int i = pt; i < S; i += PT) c.sE[i] = ldp(pv.seg_edge + (sa + i), pm);
-  const int64_t ip0 = ldp(pv.ins_prefix + (ga), pm);
+    for (int i = pt; i < S; i += PT) c.sE[i] = __ldg(pv.seg_edge + (sa + i));
+  const int64_t ip0 = __ldg(pv.ins_prefix + (ga));
   int huge = 0;
   for (int base = pt; base <= G; base += PT * kB) {
     int64_t ip[kB], sp[kB], sp1[kB], ib[kB];
@@ -808,12 +916,12 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       const int i = base + r * PT;
       ip[r] = sp[r] = sp1[r] = ib[r] = 0;
       cd[r] = 0;
-      if (i <= G) ip[r] = ldp(pv.ins_prefix + (ga + i), pm);
+      if (i <= G) ip[r] = __ldg(pv.ins_prefix + (ga + i));
       if (i < G) {
-        sp[r] = ldp(pv.slot_prefix + (ga + i), pm);
-        sp1[r] = ldp(pv.slot_prefix + (ga + i + 1), pm);
-        ib[r] = ldp(pv.grp_ibase + (ga + i), pm);
-        cd[r] = ldp(pv.grp_code + (ga + i), pm);
+        sp[r] = __ldg(pv.slot_prefix + (ga + i));
+        sp1[r] = __ldg(pv.slot_prefix + (ga + i + 1));
+        ib[r] = __ldg(pv.grp_ibase + (ga + i));
+        cd[r] = __ldg(pv.grp_code + (ga + i));
       }
     }
 #pragma unroll
@@ -958,6 +1066,12 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   }
 }
 
+// Bytes of one consumer warp's key ring (kR stages; see walk_long_staged).
+__host__ __device__ constexpr int ring_warp_bytes(int kR) {
+  return kR > 0 ? ((kR * (kStageInts * 4 + 8 * 4 + 8)) + 15) & ~15 : 0;
+}
+
+template <int kR>
 __global__ void __launch_bounds__(kMaxBlock, 1)
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
             int64_t slot_bytes, Tuning tu, unsigned long long* __restrict__ out,
@@ -976,6 +1090,18 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     for (int i = 0; i < nslots; ++i) {
       mbar_init(&full_bar[i], PT);       // every producer thread arrives
       mbar_init(&empty_bar[i], n_cons);  // one lane per consumer warp
+    }
+  }
+  // consumer warp cw's key ring (kR > 0): after the slots
+  KeyRing kr{nullptr, nullptr, nullptr};
+  if constexpr (kR > 0) {
+    if (warp >= n_prod) {
+      unsigned char* base = smem + nslots * slot_bytes + (warp - n_prod) * ring_warp_bytes(kR);
+      kr.data = reinterpret_cast<int*>(base);
+      kr.offs = kr.data + kR * kStageInts;
+      kr.bar = reinterpret_cast<uint64_t*>(kr.offs + kR * 8);
+      if (lane == 0)
+        for (int i = 0; i < kR; ++i) mbar_init(kr.bar + i, 1);
     }
   }
   __syncthreads();
@@ -1003,6 +1129,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     const int cw = warp - n_prod;
     int slot = 0;
     uint32_t fill = 0;
+    uint32_t phase = 0;  // parity of each key-ring stage (kR > 0)
     for (;; slot = (slot + 1 == nslots) ? (++fill, 0) : slot + 1) {
       wait_full(&full_bar[slot], fill & 1u, hint);
       const SlotHdr h = hdr[slot];
@@ -1019,7 +1146,8 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = min((w0 + 7) & ~7, NU);
             w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
           }
-          acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+          acc += h.linear ? consume<true, kR>(c, h, w0, w1, pv, &kr, &phase)
+                          : consume<false, kR>(c, h, w0, w1, pv, &kr, &phase);
         } else {  // dynamic: grab `grab` units at a time from the slot's counter
           for (;;) {
             int w0 = 0;
@@ -1027,7 +1155,8 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = __shfl_sync(0xffffffffu, w0, 0);
             if (w0 >= NU) break;
             const int w1 = min(w0 + grab, NU);
-            acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+            acc += h.linear ? consume<true, kR>(c, h, w0, w1, pv, &kr, &phase)
+                            : consume<false, kR>(c, h, w0, w1, pv, &kr, &phase);
           }
         }
       }
@@ -1191,27 +1320,14 @@ constexpr int kMaxDevices = 64;
 std::once_flag g_attr_once[kMaxDevices];
 
 void set_attr() {
-  TC_CUDA(cudaFuncSetAttribute(k_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               optin_smem() - static_smem((const void*)k_count)));
+  for (const void* f : {(const void*)k_count<0>, (const void*)k_count<2>, (const void*)k_count<3>,
+                        (const void*)k_count<4>})
+    TC_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 optin_smem() - static_smem(f)));
   TC_CUDA(cudaFuncSetAttribute(k_count_flat, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                optin_smem() - static_smem((const void*)k_count_flat)));
   TC_CUDA(cudaFuncSetAttribute(k_support, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                optin_smem() - static_smem((const void*)k_support)));
-}
-
-// The device's persisting-L2 set-aside, raised (never lowered) to `bytes`
-// capped at cudaDevAttrMaxPersistingL2CacheSize (Tuning::l2_persist_mb only).
-void ensure_persisting_l2(size_t bytes) {
-  static std::mutex mu;
-  static size_t set[kMaxDevices] = {};
-  int dev = 0, mx = 0;
-  TC_CUDA(cudaGetDevice(&dev));
-  TC_CUDA(cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, dev));
-  bytes = std::min(bytes, (size_t)mx);
-  std::lock_guard<std::mutex> lk(mu);
-  if (dev >= 0 && dev < kMaxDevices && set[dev] >= bytes) return;
-  TC_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes));
-  if (dev >= 0 && dev < kMaxDevices) set[dev] = bytes;
 }
 
 void ensure_attr() {
@@ -1245,8 +1361,6 @@ PlanView plan_view(const tc_graph* g) {
   pv.seg_edge = nullptr;
   pv.sup = nullptr;
   pv.max_kicks = P.tune.max_kicks;
-  pv.l2_meta = P.tune.l2_meta;
-  pv.l2_keys = P.tune.l2_keys;
   return pv;
 }
 
@@ -1267,9 +1381,27 @@ int num_sms() {
   return v;
 }
 
-int max_smem_per_block() { return optin_smem() - static_smem((const void*)k_count); }
+int max_smem_per_block() { return optin_smem() - static_smem((const void*)k_count<0>); }
 
-int max_chunk_smem(const Tuning& tu) { return (max_smem_per_block() / tu.slots) & ~15; }
+// The consumers' key rings (Tuning::key_stages), one per consumer warp.
+int64_t ring_bytes(const Tuning& tu, int block) {
+  if (tu.key_stages <= 0) return 0;
+  const int nw = block / 32, n_prod = std::max(1, std::min(nw - 1, nw / tu.prod_div));
+  return (int64_t)(nw - n_prod) * ring_warp_bytes(tu.key_stages);
+}
+
+const void* count_kernel(int key_stages) {
+  switch (key_stages) {
+    case 2: return (const void*)k_count<2>;
+    case 3: return (const void*)k_count<3>;
+    case 4: return (const void*)k_count<4>;
+    default: return (const void*)k_count<0>;
+  }
+}
+
+int max_chunk_smem(const Tuning& tu, int block) {
+  return (int)((max_smem_per_block() - ring_bytes(tu, block)) / tu.slots) & ~15;
+}
 
 // One chunk of the flat kernel must leave room for 3 CTAs per SM.
 int max_flat_chunk_smem() {
@@ -1284,7 +1416,8 @@ int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu) {
   ensure_attr();
   int occ = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-      &occ, k_count, block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
+      &occ, count_kernel(tu.key_stages), block,
+      (size_t)(tu.slots * slot_bytes_of(smem_bytes) + ring_bytes(tu, block))));
   return occ;
 }
 
@@ -1309,32 +1442,22 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
   // short-class chunks: flat kernel.  The last launch carries the fused sum.
   const int64_t l0 = c_begin, l1 = std::min(c_end, P.n_long_chunks);
   const int64_t s0 = std::max(c_begin, P.n_long_chunks), s1 = c_end;
-  // optional L2 access-policy window over the last l2_persist_mb MB of col
-  // (the highest-ranked rows, whose suffixes are re-read most), as a launch
-  // attribute so the caller's stream is left untouched
-  cudaLaunchAttribute attr[1];
-  int nattr = 0;
-  if (P.tune.l2_persist_mb > 0 && g->m > 0) {
-    const size_t want = (size_t)P.tune.l2_persist_mb << 20;
-    const size_t bytes = std::min(want, (size_t)g->m * 4);
-    ensure_persisting_l2(bytes);
-    memset(&attr[0], 0, sizeof(attr[0]));
-    attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
-    attr[0].val.accessPolicyWindow.base_ptr =
-        (void*)(g->col.get() + (g->m - (int64_t)(bytes / 4)));
-    attr[0].val.accessPolicyWindow.num_bytes = bytes;
-    attr[0].val.accessPolicyWindow.hitRatio = 1.0f;
-    attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-    nattr = 1;
-  }
+  cudaLaunchAttribute* attr = nullptr;
+  const int nattr = 0;
   int launched = 0;
   if (l1 > l0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(l1 - l0, P.grid));
     const int64_t sb = slot_bytes_of(P.smem_bytes);
-    cudaLaunchConfig_t cfg = {dim3(grid), dim3(P.block), (size_t)(P.tune.slots * sb), s, attr, (unsigned)nattr};
-    TC_CUDA(cudaLaunchKernelEx(&cfg, k_count, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out,
-                               (fuse && s1 <= s0) ? *fuse : none));
+    cudaLaunchConfig_t cfg = {dim3(grid), dim3(P.block),
+                              (size_t)(P.tune.slots * sb + ring_bytes(P.tune, P.block)), s, attr,
+                              (unsigned)nattr};
+    const FuseArgs& fa = (fuse && s1 <= s0) ? *fuse : none;
+    switch (P.tune.key_stages) {
+      case 2: TC_CUDA(cudaLaunchKernelEx(&cfg, k_count<2>, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, fa)); break;
+      case 3: TC_CUDA(cudaLaunchKernelEx(&cfg, k_count<3>, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, fa)); break;
+      case 4: TC_CUDA(cudaLaunchKernelEx(&cfg, k_count<4>, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, fa)); break;
+      default: TC_CUDA(cudaLaunchKernelEx(&cfg, k_count<0>, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, fa));
+    }
     ++launched;
   }
   if (s1 > s0) {
