@@ -559,13 +559,14 @@ def agreed_profile(graph, group=None, stream=None, n_slices: int = CALIBRATION_S
 
 
 def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] = None,
-                      profile=None) -> int:
+                      profile="auto") -> int:
     """T over a torch.distributed process group.
 
     Every rank holds the same replicated graph; rank r counts the live
     oriented edges [b_r, b_{r+1}) of the cost-balanced split
-    (tc_partition_measured with ``profile``, the same on every rank — e.g.
-    :func:`agreed_profile` — or tc_partition's built-in profile) and a single
+    (tc_partition_measured with ``profile``, the same on every rank; the
+    default "auto" measures it once per graph with :func:`agreed_profile` when
+    there is more than one rank; None = tc_partition's built-in profile) and a single
     all_reduce(SUM) of the 8-byte partials (ProcessGroupNCCL over NVLink on
     the GPU box) gives T on every rank.  Two's-complement int64 addition is
     bit-identical to uint64 addition mod 2^64.  With ``fused`` (a
@@ -576,6 +577,13 @@ def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] 
     on = dist.is_available() and dist.is_initialized()
     world = dist.get_world_size(group) if on else 1
     rank = dist.get_rank(group) if on else 0
+    if isinstance(profile, str):
+        if profile != "auto":
+            raise InvalidArgument(TC_ERR_INVALID_ARGUMENT, f"unknown profile {profile!r}")
+        profile = getattr(graph, "_agreed_profile", None)
+        if profile is None and world > 1:  # collective: every rank measures once per graph
+            profile = agreed_profile(graph, group, stream)
+            graph._agreed_profile = profile
     bounds = graph.partition(world) if profile is None else graph.partition(world, profile)
     if fused is not None:  # f4: the library's own sum over NVLink peer memory
         total = fused.count_range(graph, bounds[rank], bounds[rank + 1], stream=stream)

@@ -461,16 +461,12 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
 // while it probes the current one, so the keys in flight are bounded by
 // shared memory rather than by the 64 registers of a 1024-thread CTA (the
 // long-scoreboard wait on the key load is the top stall of walk_long).
-// A batch's 8 tiles are grouped into RUNS of chained windows (x_u within
-// [x_{u-1}, x_{u-1} + 32]: consecutive tiles of one suffix); each run is one
-// copy of its 16-B aligned superset [x_head & ~3, (x_last + 35) & ~3), so a
-// stage holds at most 8 x 144 B.  Tile u's keys start at int offs[u] of the
-// stage; lane l reads offs[u] + l (one conflict-free LDS).
+// Each tile is one copy of its 16-B aligned superset (see ring_issue); lane
+// l reads its key with one conflict-free LDS.
 constexpr int kStageInts = 8 * 36;  // 8 tiles x 144 B
 
 struct KeyRing {
   int* data;      // [kR][kStageInts]
-  int* offs;      // [kR][8]
   uint64_t* bar;  // [kR], count 1 (lane 0's arrive.expect_tx)
 };
 
@@ -489,38 +485,22 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 
-// Issue the copies of tiles [t, t + 8) (clamped to t1 - 1) into stage st.
+// Issue the copies of tiles [t, t + 8) (clamped to t1 - 1) into stage st:
+// lane u < 8 copies tile u's 16-B aligned superset [x & ~3, (x + 35) & ~3)
+// (128 or 144 B) to stage int u * 36; its key l is then at u * 36 + (x & 3) + l.
 __device__ __forceinline__ void ring_issue(const ChunkSmem& c, const int32_t* col, int t, int t1,
                                            const KeyRing& kr, int st, int lane) {
-  constexpr unsigned FULL = 0xffffffffu;
-  const int u = min(lane, 7);
-  const int x = c.sT0[min(t + u, t1 - 1)];
-  const int xp = __shfl_up_sync(FULL, x, 1);
-  const bool head = lane < 8 && (lane == 0 || x < xp || x > xp + 32);
-  const unsigned H = __ballot_sync(FULL, head);
-  const unsigned above = H & ~((2u << u) - 1u);          // heads after tile u
-  const int last = above ? __ffs(above) - 2 : 7;         // last tile of u's run (heads only)
-  const int hl = 31 - __clz(H & ((2u << u) - 1u));        // u's run head
-  const int xl = __shfl_sync(FULL, x, last);
   uint32_t a = 0, bytes = 0;
-  if (head) {
-    a = (uint32_t)x & ~3u;
-    bytes = 4u * ((((uint32_t)xl + 35u) & ~3u) - a);
+  if (lane < 8) {
+    const uint32_t x = (uint32_t)c.sT0[min(t + lane, t1 - 1)];
+    a = x & ~3u;
+    bytes = 4u * (((x + 35u) & ~3u) - a);
   }
-  uint32_t incl = bytes;
-#pragma unroll
-  for (int o = 1; o < 8; o <<= 1) {
-    const uint32_t v = __shfl_up_sync(FULL, incl, o);
-    if (lane >= o) incl += v;
-  }
-  const uint32_t excl = incl - bytes, total = __shfl_sync(FULL, incl, 7);
-  const uint32_t hd = __shfl_sync(FULL, excl, hl), ha = __shfl_sync(FULL, a, hl);
-  if (lane < 8) kr.offs[st * 8 + lane] = (int)(hd / 4u + ((uint32_t)x - ha));
+  const uint32_t total = __reduce_add_sync(0xffffffffu, bytes);
   if (lane == 0) mbar_expect_tx(kr.bar + st, total);
-  __syncwarp();
-  if (head) {
+  if (lane < 8) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // WAR vs the stage's last LDS reads
-    bulk_g2s(kr.data + st * kStageInts + excl / 4u, col + a, bytes, kr.bar + st);
+    bulk_g2s(kr.data + st * kStageInts + lane * 36, col + a, bytes, kr.bar + st);
   }
 }
 
@@ -540,13 +520,13 @@ __device__ __forceinline__ unsigned walk_long_staged(const ChunkSmem& c, int t0,
     const int t = t0 + 8 * b;
     mbar_wait(kr.bar + st, (phase >> st) & 1u, 0);
     phase ^= 1u << st;
-    int o[8], z[8], zw[8];
-    *reinterpret_cast<int4*>(o) = *reinterpret_cast<const int4*>(kr.offs + st * 8);
-    *reinterpret_cast<int4*>(o + 4) = *reinterpret_cast<const int4*>(kr.offs + st * 8 + 4);
+    int x[8], z[8], zw[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) x[u] = c.sT0[min(t + u, t1 - 1)];
     const int* sd = kr.data + st * kStageInts + lane;
     int32_t key[8];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) key[u] = sd[o[u]];
+    for (int u = 0; u < 8; ++u) key[u] = sd[u * 36 + (x[u] & 3)];
     if (t + 8 <= t1) {
 #pragma unroll
       for (int q = 0; q < 8; q += 4) {
@@ -1068,7 +1048,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
 
 // Bytes of one consumer warp's key ring (kR stages; see walk_long_staged).
 __host__ __device__ constexpr int ring_warp_bytes(int kR) {
-  return kR > 0 ? ((kR * (kStageInts * 4 + 8 * 4 + 8)) + 15) & ~15 : 0;
+  return kR > 0 ? ((kR * (kStageInts * 4 + 8)) + 15) & ~15 : 0;
 }
 
 template <int kR>
@@ -1093,13 +1073,12 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     }
   }
   // consumer warp cw's key ring (kR > 0): after the slots
-  KeyRing kr{nullptr, nullptr, nullptr};
+  KeyRing kr{nullptr, nullptr};
   if constexpr (kR > 0) {
     if (warp >= n_prod) {
       unsigned char* base = smem + nslots * slot_bytes + (warp - n_prod) * ring_warp_bytes(kR);
       kr.data = reinterpret_cast<int*>(base);
-      kr.offs = kr.data + kR * kStageInts;
-      kr.bar = reinterpret_cast<uint64_t*>(kr.offs + kR * 8);
+      kr.bar = reinterpret_cast<uint64_t*>(kr.data + kR * kStageInts);
       if (lane == 0)
         for (int i = 0; i < kR; ++i) mbar_init(kr.bar + i, 1);
     }

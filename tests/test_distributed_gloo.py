@@ -17,16 +17,29 @@ import torch.multiprocessing as mp
 
 
 class FakeGraph:
-    """Per-edge counts c_e; partition/count_range mimic the C-ABI contract."""
+    """Per-edge counts c_e in chunks of 7 edges (the first 60% "long");
+    partition/calibrate/count_range mimic the C-ABI contract.  calibrate()
+    returns a rank-dependent profile, so only an agreed (averaged) profile
+    gives every rank the same bounds."""
 
     def __init__(self, per_edge):
         self.c = np.asarray(per_edge, dtype=np.uint64)
         self.m_live = len(self.c)
+        self.seg = np.concatenate([np.arange(0, self.m_live, 7), [self.m_live]]).astype(np.int64)
+        self.cost = self.seg * 3  # cost units: 3 per edge
+        self.n_long = (len(self.seg) - 1) * 6 // 10
 
-    def partition(self, world):
+    def calibrate(self, n_slices=64, stream=None):
+        import torch.distributed as dist
+        rng = np.random.default_rng(dist.get_rank() if dist.is_initialized() else 0)
+        return rng.uniform(0.5, 2.0, size=n_slices)
+
+    def partition(self, world, profile=None):
         import paper_conf_ipps_li0ptz24_b200 as tc
-        prefix = np.concatenate([[0], np.cumsum(self.c.astype(np.int64) + 1)])
-        return tc.partition_prefix(prefix, world)
+        if profile is None:
+            prefix = np.concatenate([[0], np.cumsum(self.c.astype(np.int64) + 1)])
+            return tc.partition_prefix(prefix, world)
+        return tc.partition_chunks(self.seg, self.cost, self.n_long, profile, world)
 
     def count_range(self, b, e, stream=None):
         s = int(self.c[b:e].sum(dtype=np.uint64))
@@ -46,7 +59,8 @@ def _worker(rank, world, port, per_edge, q):
     try:
         import paper_conf_ipps_li0ptz24_b200 as tc
         g = FakeGraph(per_edge)
-        q.put((rank, tc.count_partitioned(g), g.partition(world)))
+        t = tc.count_partitioned(g)  # "auto": one agreed (all_reduce-averaged) profile
+        q.put((rank, t, g.partition(world, g._agreed_profile)))
     finally:
         dist.destroy_process_group()
 
@@ -72,7 +86,8 @@ def test_count_partitioned_two_ranks():
     total = int(per_edge.sum())
     assert [r[1] for r in out] == [total, total]
     b = out[0][2]
-    assert b[0] == 0 and b[-1] == len(per_edge) and b == out[1][2]
+    assert b[0] == 0 and b[-1] == len(per_edge) and b == out[1][2]  # same bounds on both ranks
+    assert set(b) <= set(FakeGraph(per_edge).seg.tolist())  # chunk-aligned
 
 
 def test_count_partitioned_exceeds_63_bits():
