@@ -371,7 +371,8 @@ def main():
         opts["chunk_cost"] = a.chunk_cost
     if a.block:
         opts["block_threads"] = a.block
-    for kv in a.opt:
+    # plan options: --opt k=v (repeatable) and BENCH_OPT="k=v,k=v" (for A/B drivers)
+    for kv in a.opt + [x for x in os.environ.get("BENCH_OPT", "").split(",") if x]:
         k, v = kv.split("=")
         opts[k] = int(v)
 

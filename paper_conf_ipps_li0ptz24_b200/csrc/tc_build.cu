@@ -1057,8 +1057,6 @@ Tuning tuning_from_env() {
   t.cs_div = get("TC_CS_DIV", t.cs_div, 0, 64);
   t.short_linear = get("TC_SHORT_LINEAR", t.short_linear, 0, 1);
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
-  t.key_stages = get("TC_KEY_STAGES", t.key_stages, 0, 4);
-  if (t.key_stages == 1) t.key_stages = 2;
   return t;
 }
 
@@ -1145,7 +1143,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P.tune = tuning_from_env();
   // SMEM of one chunk slot of the count kernel; a table may use at most half
   // of it (bigger tables are "huge": probed in global memory)
-  const int64_t slot_limit = max_chunk_smem(P.tune, P.block);
+  const int64_t slot_limit = max_chunk_smem(P.tune);
   const int64_t flat_limit = max_flat_chunk_smem();
   const int64_t max_slots_long = slot_limit / 8, max_slots_short = flat_limit / 8;  // half a slot
   P.seg_start = DevBuf<int64_t>(S, s, true);

@@ -453,116 +453,6 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   return cnt;
 }
 
-// ------------------------------------------------------------------ bulk-staged keys
-// LONG class with the keys staged in shared memory by the bulk-copy engine
-// (cp.async.bulk global -> shared, completion counted in bytes on an
-// mbarrier), instead of loaded into registers: each consumer warp owns a ring
-// of kR stages of one 8-tile batch each, and keeps kR - 1 batches in flight
-// while it probes the current one, so the keys in flight are bounded by
-// shared memory rather than by the 64 registers of a 1024-thread CTA (the
-// long-scoreboard wait on the key load is the top stall of walk_long).
-// Each tile is one copy of its 16-B aligned superset (see ring_issue); lane
-// l reads its key with one conflict-free LDS.
-constexpr int kStageInts = 8 * 36;  // 8 tiles x 144 B
-
-struct KeyRing {
-  int* data;      // [kR][kStageInts]
-  uint64_t* bar;  // [kR], count 1 (lane 0's arrive.expect_tx)
-};
-
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
-  asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(
-                   smem_u32(b)),
-               "r"(bytes)
-               : "memory");
-}
-
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          smem_u32(dst)),
-      "l"(src), "r"(bytes), "r"(smem_u32(bar))
-      : "memory");
-}
-
-// Issue the copies of tiles [t, t + 8) (clamped to t1 - 1) into stage st:
-// lane u < 8 copies tile u's 16-B aligned superset [x & ~3, (x + 35) & ~3)
-// (128 or 144 B) to stage int u * 36; its key l is then at u * 36 + (x & 3) + l.
-__device__ __forceinline__ void ring_issue(const ChunkSmem& c, const int32_t* col, int t, int t1,
-                                           const KeyRing& kr, int st, int lane) {
-  uint32_t a = 0, bytes = 0;
-  if (lane < 8) {
-    const uint32_t x = (uint32_t)c.sT0[min(t + lane, t1 - 1)];
-    a = x & ~3u;
-    bytes = 4u * (((x + 35u) & ~3u) - a);
-  }
-  const uint32_t total = __reduce_add_sync(0xffffffffu, bytes);
-  if (lane == 0) mbar_expect_tx(kr.bar + st, total);
-  if (lane < 8) {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // WAR vs the stage's last LDS reads
-    bulk_g2s(kr.data + st * kStageInts + lane * 36, col + a, bytes, kr.bar + st);
-  }
-}
-
-template <bool kLinear, bool kHuge, int kR>
-__device__ __forceinline__ unsigned walk_long_staged(const ChunkSmem& c, int t0, int t1,
-                                                     const PlanView& pv, int64_t ga,
-                                                     const KeyRing& kr, uint32_t& phase) {
-  unsigned cnt = 0;
-  const int lane = threadIdx.x & 31;
-  const int nb = (t1 - t0 + 7) >> 3;
-#pragma unroll
-  for (int j = 0; j < kR - 1; ++j)
-    if (j < nb) ring_issue(c, pv.col, t0 + 8 * j, t1, kr, j, lane);
-  int st = 0;  // stage of batch b
-  for (int b = 0; b < nb; ++b) {
-    if (b + kR - 1 < nb) ring_issue(c, pv.col, t0 + 8 * (b + kR - 1), t1, kr, (st + kR - 1) % kR, lane);
-    const int t = t0 + 8 * b;
-    mbar_wait(kr.bar + st, (phase >> st) & 1u, 0);
-    phase ^= 1u << st;
-    int x[8], z[8], zw[8];
-#pragma unroll
-    for (int u = 0; u < 8; ++u) x[u] = c.sT0[min(t + u, t1 - 1)];
-    const int* sd = kr.data + st * kStageInts + lane;
-    int32_t key[8];
-#pragma unroll
-    for (int u = 0; u < 8; ++u) key[u] = sd[u * 36 + (x[u] & 3)];
-    if (t + 8 <= t1) {
-#pragma unroll
-      for (int q = 0; q < 8; q += 4) {
-        *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
-        *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
-      }
-    } else {  // last, partial batch: tiles past t1 repeat the last one, every lane masked
-#pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        const int tt = min(t + u, t1 - 1);
-        z[u] = c.sT1[tt];
-        zw[u] = c.sT2[tt] | (t + u < t1 ? 0 : 32);
-      }
-    }
-    int zw_or = 0;
-#pragma unroll
-    for (int u = 0; u < 8; ++u) zw_or |= zw[u];
-    if ((zw_or >> 6) == 0) {
-#pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        const unsigned word = (unsigned)c.sT0[(key[u] >> 5) + z[u]];
-        const unsigned hit = (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
-        if (lane >= (zw[u] & 63)) cnt += hit;
-      }
-    } else {
-#pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        const unsigned hit = probe_tile<kLinear, kHuge>(c, z[u], zw[u], key[u], lane, pv, ga);
-        if (lane >= (zw[u] & 63)) cnt += hit;
-      }
-    }
-    st = (st + 1 == kR) ? 0 : st + 1;
-  }
-  return cnt;
-}
-
 // SHORT class: the warp owns the flat keys [k0w, k1w) of the chunk.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0w, int k1w,
@@ -620,15 +510,9 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
   return cnt;
 }
 
-template <bool kLinear, int kR = 0>
+template <bool kLinear>
 __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
-                                            const PlanView& pv, const KeyRing* kr = nullptr,
-                                            uint32_t* phase = nullptr) {
-  if constexpr (kR > 0) {
-    if (h.is_long)
-      return h.huge ? walk_long_staged<kLinear, true, kR>(c, w0, w1, pv, h.ga, *kr, *phase)
-                    : walk_long_staged<kLinear, false, kR>(c, w0, w1, pv, h.ga, *kr, *phase);
-  }
+                                            const PlanView& pv) {
   if (h.is_long)
     return h.huge ? walk_long<kLinear, true>(c, w0, w1, pv, h.ga)
                   : walk_long<kLinear, false>(c, w0, w1, pv, h.ga);
@@ -1046,12 +930,6 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   }
 }
 
-// Bytes of one consumer warp's key ring (kR stages; see walk_long_staged).
-__host__ __device__ constexpr int ring_warp_bytes(int kR) {
-  return kR > 0 ? ((kR * (kStageInts * 4 + 8)) + 15) & ~15 : 0;
-}
-
-template <int kR>
 __global__ void __launch_bounds__(kMaxBlock, 1)
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
             int64_t slot_bytes, Tuning tu, unsigned long long* __restrict__ out,
@@ -1070,17 +948,6 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     for (int i = 0; i < nslots; ++i) {
       mbar_init(&full_bar[i], PT);       // every producer thread arrives
       mbar_init(&empty_bar[i], n_cons);  // one lane per consumer warp
-    }
-  }
-  // consumer warp cw's key ring (kR > 0): after the slots
-  KeyRing kr{nullptr, nullptr};
-  if constexpr (kR > 0) {
-    if (warp >= n_prod) {
-      unsigned char* base = smem + nslots * slot_bytes + (warp - n_prod) * ring_warp_bytes(kR);
-      kr.data = reinterpret_cast<int*>(base);
-      kr.bar = reinterpret_cast<uint64_t*>(kr.data + kR * kStageInts);
-      if (lane == 0)
-        for (int i = 0; i < kR; ++i) mbar_init(kr.bar + i, 1);
     }
   }
   __syncthreads();
@@ -1108,7 +975,6 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
     const int cw = warp - n_prod;
     int slot = 0;
     uint32_t fill = 0;
-    uint32_t phase = 0;  // parity of each key-ring stage (kR > 0)
     for (;; slot = (slot + 1 == nslots) ? (++fill, 0) : slot + 1) {
       wait_full(&full_bar[slot], fill & 1u, hint);
       const SlotHdr h = hdr[slot];
@@ -1125,8 +991,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = min((w0 + 7) & ~7, NU);
             w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
           }
-          acc += h.linear ? consume<true, kR>(c, h, w0, w1, pv, &kr, &phase)
-                          : consume<false, kR>(c, h, w0, w1, pv, &kr, &phase);
+          acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
         } else {  // dynamic: grab `grab` units at a time from the slot's counter
           for (;;) {
             int w0 = 0;
@@ -1134,8 +999,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = __shfl_sync(0xffffffffu, w0, 0);
             if (w0 >= NU) break;
             const int w1 = min(w0 + grab, NU);
-            acc += h.linear ? consume<true, kR>(c, h, w0, w1, pv, &kr, &phase)
-                            : consume<false, kR>(c, h, w0, w1, pv, &kr, &phase);
+            acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
           }
         }
       }
@@ -1299,10 +1163,8 @@ constexpr int kMaxDevices = 64;
 std::once_flag g_attr_once[kMaxDevices];
 
 void set_attr() {
-  for (const void* f : {(const void*)k_count<0>, (const void*)k_count<2>, (const void*)k_count<3>,
-                        (const void*)k_count<4>})
-    TC_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 optin_smem() - static_smem(f)));
+  TC_CUDA(cudaFuncSetAttribute(k_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               optin_smem() - static_smem((const void*)k_count)));
   TC_CUDA(cudaFuncSetAttribute(k_count_flat, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                optin_smem() - static_smem((const void*)k_count_flat)));
   TC_CUDA(cudaFuncSetAttribute(k_support, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1360,27 +1222,9 @@ int num_sms() {
   return v;
 }
 
-int max_smem_per_block() { return optin_smem() - static_smem((const void*)k_count<0>); }
+int max_smem_per_block() { return optin_smem() - static_smem((const void*)k_count); }
 
-// The consumers' key rings (Tuning::key_stages), one per consumer warp.
-int64_t ring_bytes(const Tuning& tu, int block) {
-  if (tu.key_stages <= 0) return 0;
-  const int nw = block / 32, n_prod = std::max(1, std::min(nw - 1, nw / tu.prod_div));
-  return (int64_t)(nw - n_prod) * ring_warp_bytes(tu.key_stages);
-}
-
-const void* count_kernel(int key_stages) {
-  switch (key_stages) {
-    case 2: return (const void*)k_count<2>;
-    case 3: return (const void*)k_count<3>;
-    case 4: return (const void*)k_count<4>;
-    default: return (const void*)k_count<0>;
-  }
-}
-
-int max_chunk_smem(const Tuning& tu, int block) {
-  return (int)((max_smem_per_block() - ring_bytes(tu, block)) / tu.slots) & ~15;
-}
+int max_chunk_smem(const Tuning& tu) { return (max_smem_per_block() / tu.slots) & ~15; }
 
 // One chunk of the flat kernel must leave room for 3 CTAs per SM.
 int max_flat_chunk_smem() {
@@ -1395,8 +1239,7 @@ int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu) {
   ensure_attr();
   int occ = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-      &occ, count_kernel(tu.key_stages), block,
-      (size_t)(tu.slots * slot_bytes_of(smem_bytes) + ring_bytes(tu, block))));
+      &occ, k_count, block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
   return occ;
 }
 
@@ -1421,29 +1264,20 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
   // short-class chunks: flat kernel.  The last launch carries the fused sum.
   const int64_t l0 = c_begin, l1 = std::min(c_end, P.n_long_chunks);
   const int64_t s0 = std::max(c_begin, P.n_long_chunks), s1 = c_end;
-  cudaLaunchAttribute* attr = nullptr;
-  const int nattr = 0;
   int launched = 0;
   if (l1 > l0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(l1 - l0, P.grid));
     const int64_t sb = slot_bytes_of(P.smem_bytes);
-    cudaLaunchConfig_t cfg = {dim3(grid), dim3(P.block),
-                              (size_t)(P.tune.slots * sb + ring_bytes(P.tune, P.block)), s, attr,
-                              (unsigned)nattr};
-    const FuseArgs& fa = (fuse && s1 <= s0) ? *fuse : none;
-    switch (P.tune.key_stages) {
-      case 2: TC_CUDA(cudaLaunchKernelEx(&cfg, k_count<2>, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, fa)); break;
-      case 3: TC_CUDA(cudaLaunchKernelEx(&cfg, k_count<3>, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, fa)); break;
-      case 4: TC_CUDA(cudaLaunchKernelEx(&cfg, k_count<4>, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, fa)); break;
-      default: TC_CUDA(cudaLaunchKernelEx(&cfg, k_count<0>, pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, fa));
-    }
+    k_count<<<grid, P.block, (size_t)(P.tune.slots * sb), s>>>(
+        pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, (fuse && s1 <= s0) ? *fuse : none);
+    TC_LAUNCH();
     ++launched;
   }
   if (s1 > s0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(s1 - s0, P.grid_flat));
-    cudaLaunchConfig_t cfg = {dim3(grid), dim3(kFlatBlock), (size_t)slot_bytes_of(P.smem_flat), s, attr, (unsigned)nattr};
-    TC_CUDA(cudaLaunchKernelEx(&cfg, k_count_flat, pv, s0, s1, e_begin, e_end, d_out,
-                               fuse ? *fuse : none));
+    k_count_flat<<<grid, kFlatBlock, (size_t)slot_bytes_of(P.smem_flat), s>>>(
+        pv, s0, s1, e_begin, e_end, d_out, fuse ? *fuse : none);
+    TC_LAUNCH();
     ++launched;
   }
   return launched;

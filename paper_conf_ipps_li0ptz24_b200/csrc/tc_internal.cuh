@@ -132,7 +132,7 @@ __host__ __device__ inline int64_t chunk_smem_bytes(int64_t S, int64_t G, int64_
 
 // Count-kernel launch tuning (not part of the C-ABI; TC_SLOTS, TC_GRAB_LONG,
 // TC_GRAB_SHORT, TC_PROD_DIV, TC_WAIT_HINT, TC_CS_DIV, TC_SHORT_LINEAR,
-// TC_CUCKOO_KICKS, TC_KEY_STAGES override
+// TC_CUCKOO_KICKS override
 // the defaults for sweeps; every setting gives the same count).
 struct Tuning {
   int slots = 3;          // chunk slots in SMEM (2..4)
@@ -145,8 +145,6 @@ struct Tuning {
   int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
-  int key_stages = 0;     // long class: 0 = keys loaded into registers (walk_long); 2..4 = keys
-                          // staged by bulk copies into a per-warp ring of that many batches
 };
 Tuning tuning_from_env();
 
@@ -227,7 +225,7 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
                  const FuseArgs* fuse = nullptr);
 int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu);  // CTAs per SM (0 = cannot launch)
 int max_smem_per_block();
-int max_chunk_smem(const Tuning& tu, int block);  // SMEM one of the kernel's chunk slots may use
+int max_chunk_smem(const Tuning& tu);  // SMEM one of the kernel's chunk slots may use
 int max_flat_chunk_smem();      // SMEM one short-class chunk may use (3 CTAs per SM)
 int flat_occupancy(int64_t smem_bytes);
 int num_sms();
