@@ -220,6 +220,12 @@ __global__ void k_csr(const uint64_t* __restrict__ okey, int64_t m, int64_t n, i
   }
 }
 
+__global__ void k_narrow_u32(const int64_t* __restrict__ in, int64_t n, uint32_t* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = (uint32_t)(uint64_t)in[i];
+}
+
 __global__ void k_fill_i64(int64_t* p, int64_t n, int64_t v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
@@ -331,7 +337,7 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint64_t* __r
                            int huge_degree, int table_factor, int bitmap_factor,
                            int64_t max_slots_long, int64_t max_slots_short,
                            const int32_t* __restrict__ col,
-                           int32_t* __restrict__ grp_code, int64_t* __restrict__ seg_start,
+                           int32_t* __restrict__ grp_code, uint32_t* __restrict__ seg_start,
                            int32_t* __restrict__ seg_len, int32_t* __restrict__ seg_group,
                            int64_t* __restrict__ units, int64_t* __restrict__ grp_row,
                            int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots) {
@@ -342,7 +348,7 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint64_t* __r
     const int32_t g = gincl[s] - 1;
     const int32_t len = (int32_t)(x & 0xFFFFFFu);
     seg_group[s] = g;
-    seg_start[s] = (int64_t)(x >> 24);
+    seg_start[s] = (uint32_t)(x >> 24);  // < m < 2^32
     seg_len[s] = len;
     units[s] = s < S_long ? (int64_t)((len + 31) & ~31) : (int64_t)len;
     if (s == 0 || key[s] != key[s - 1]) {
@@ -448,7 +454,7 @@ __global__ void k_chunk_bounds(const int64_t* __restrict__ cost_prefix, int64_t 
 __global__ void k_split(const int64_t* __restrict__ chunk_seg, int64_t n_chunks, int64_t nL,
                         const int32_t* __restrict__ seg_group,
                         const int64_t* __restrict__ slot_prefix,
-                        const int64_t* __restrict__ key_prefix, int64_t limit_long,
+                        const uint32_t* __restrict__ key_prefix, int64_t limit_long,
                         int64_t limit_short, int64_t* __restrict__ pieces,
                         const int64_t* __restrict__ off, int64_t* __restrict__ bounds,
                         unsigned long long* need_max) {  // need_max[0] long, [1] short
@@ -468,7 +474,8 @@ __global__ void k_split(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
       // fast path: the whole chunk fits one slot (all but the outliers) —
       // its layout follows from the prefixes in O(1), no walk over its edges
       const int64_t ga = seg_group[sa], gb = seg_group[sb - 1];
-      const int64_t tiles = is_long ? (key_prefix[sb] - key_prefix[sa]) >> 5 : 0;
+      // key_prefix is mod 2^32; a chunk's units are < 2^32
+      const int64_t tiles = is_long ? (int64_t)((key_prefix[sb] - key_prefix[sa]) >> 5) : 0;
       const int64_t need = chunk_smem_bytes(sb - sa, gb - ga + 1, slot_prefix[gb + 1] - slot_prefix[ga], tiles);
       if (need <= limit) {
         if (bounds) bounds[o] = sa;
@@ -482,7 +489,7 @@ __global__ void k_split(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
     int64_t p0 = sa, g0 = seg_group[sa], ok_need = 0;
     for (int64_t s = sa; s < sb; ++s) {
       const int64_t g = seg_group[s];
-      const int64_t tiles = is_long ? (key_prefix[s + 1] - key_prefix[p0]) >> 5 : 0;
+      const int64_t tiles = is_long ? (int64_t)((key_prefix[s + 1] - key_prefix[p0]) >> 5) : 0;
       int64_t need = chunk_smem_bytes(s + 1 - p0, g - g0 + 1, slot_prefix[g + 1] - slot_prefix[g0], tiles);
       if (need > limit && s > p0) {  // close the piece [p0, s), start a new one at s
         if (bounds) bounds[o + cnt] = p0;
@@ -490,7 +497,7 @@ __global__ void k_split(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
         ++cnt;
         p0 = s;
         g0 = g;
-        const int64_t t1 = is_long ? (key_prefix[s + 1] - key_prefix[s]) >> 5 : 0;
+        const int64_t t1 = is_long ? (int64_t)((key_prefix[s + 1] - key_prefix[s]) >> 5) : 0;
         need = chunk_smem_bytes(1, 1, slot_prefix[g + 1] - slot_prefix[g], t1);
       }
       ok_need = need;
@@ -1057,6 +1064,7 @@ Tuning tuning_from_env() {
   t.cs_div = get("TC_CS_DIV", t.cs_div, 0, 64);
   t.short_linear = get("TC_SHORT_LINEAR", t.short_linear, 0, 1);
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
+  t.batch = get("TC_BATCH", t.batch, 0, 64);
   return t;
 }
 
@@ -1107,8 +1115,8 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   const int64_t S = (int64_t)h_stats[2], S_long = (int64_t)h_stats[3];
   P.S = S;
   P.S_long = S_long;
-  P.key_prefix = DevBuf<int64_t>(S + 1, s, true);
-  TC_CUDA(cudaMemsetAsync(P.key_prefix.get(), 0, sizeof(int64_t), s));
+  P.key_prefix = DevBuf<uint32_t>(S + 1, s, true);
+  TC_CUDA(cudaMemsetAsync(P.key_prefix.get(), 0, sizeof(uint32_t), s));
   if (S == 0) {
     P.chunk_seg = DevBuf<int64_t>(1, s, true);
     TC_CUDA(cudaMemsetAsync(P.chunk_seg.get(), 0, sizeof(int64_t), s));
@@ -1146,10 +1154,11 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   const int64_t slot_limit = max_chunk_smem(P.tune);
   const int64_t flat_limit = max_flat_chunk_smem();
   const int64_t max_slots_long = slot_limit / 8, max_slots_short = flat_limit / 8;  // half a slot
-  P.seg_start = DevBuf<int64_t>(S, s, true);
+  P.seg_start = DevBuf<uint32_t>(S, s, true);
   P.seg_len = DevBuf<int32_t>(S, s, true);
   P.seg_group = DevBuf<int32_t>(S, s, true);
   DevBuf<int64_t> units(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
+  int64_t units_total = 0;  // host copy (read after the next sync)
   P.grp_code = DevBuf<int32_t>(G, s, true);
   k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted, val_sorted, gincl.get(), S, S_long,
                                          g->bits, row_ptr,
@@ -1164,7 +1173,13 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   skey2.reset();
   sval.reset();
   sval2.reset();
-  exclusive_prefix(units.get(), S, P.key_prefix.get(), s);
+  {  // the unit prefix in 64 bits, kept mod 2^32 in the plan (chunk-relative use only)
+    DevBuf<int64_t> kp64(S + 1, s);
+    exclusive_prefix(units.get(), S, kp64.get(), s);
+    k_narrow_u32<<<grid_for(S + 1), TPB, 0, s>>>(kp64.get(), S + 1, P.key_prefix.get());
+    TC_LAUNCH();
+    TC_CUDA(cudaMemcpyAsync(&units_total, kp64.get() + S, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  }
   P.ins_prefix = DevBuf<int64_t>(G + 1, s, true);
   P.slot_prefix = DevBuf<int64_t>(G + 1, s, true);
   exclusive_prefix(grp_d.get(), G, P.ins_prefix.get(), s);
@@ -1182,17 +1197,15 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   grp_row.reset();
   grp_d.reset();
   grp_slots.reset();
-  int64_t h_cp[3];
+  int64_t h_cp[2];
   TC_CUDA(cudaMemcpyAsync(&h_cp[0], cost_prefix.get() + S_long, sizeof(int64_t),
                           cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaMemcpyAsync(&h_cp[1], cost_prefix.get() + S, sizeof(int64_t), cudaMemcpyDeviceToHost,
                           s));
-  TC_CUDA(cudaMemcpyAsync(&h_cp[2], P.key_prefix.get() + S, sizeof(int64_t),
-                          cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));
   const int64_t cost_long = h_cp[0], cost_short = h_cp[1] - h_cp[0];
   tr("groups + prefixes + costs");
-  P.units_total = h_cp[2];
+  P.units_total = units_total;
 
   // Chunking, per class: cost chunks (long class 4x larger: its edges carry
   // ~150 keys each), then every chunk is split where its SMEM layout would

@@ -394,10 +394,9 @@ __device__ __forceinline__ const int32_t* lane_base(const int32_t* col, int lane
   return p;
 }
 
-template <bool kLinear, bool kHuge>
+template <bool kLinear, bool kHuge, int kB = kBatchLong>
 __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1,
                                               const PlanView& pv, int64_t ga) {
-  constexpr int kB = kBatchLong;
   static_assert(kB % 4 == 0, "batches of whole int4 reads");
   unsigned cnt = 0;
   const int lane = threadIdx.x & 31;
@@ -510,12 +509,12 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
   return cnt;
 }
 
-template <bool kLinear>
+template <bool kLinear, int kB = kBatchLong>
 __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
                                             const PlanView& pv) {
   if (h.is_long)
-    return h.huge ? walk_long<kLinear, true>(c, w0, w1, pv, h.ga)
-                  : walk_long<kLinear, false>(c, w0, w1, pv, h.ga);
+    return h.huge ? walk_long<kLinear, true, kB>(c, w0, w1, pv, h.ga)
+                  : walk_long<kLinear, false, kB>(c, w0, w1, pv, h.ga);
   return h.huge ? walk_short<kLinear, true>(c, h.S, w0, w1, pv, h.ga)
                 : walk_short<kLinear, false>(c, h.S, w0, w1, pv, h.ga);
 }
@@ -733,7 +732,8 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   const int G = (int)(gb - ga);
   const int64_t slot0 = __ldg(pv.slot_prefix + (ga));
   const int nslots = (int)(__ldg(pv.slot_prefix + (gb)) - slot0);
-  const int64_t kp0 = __ldg(pv.key_prefix + (sa));
+  // key_prefix is mod 2^32: chunk-relative differences are exact (< 2^32)
+  const uint32_t kp0 = __ldg(pv.key_prefix + (sa));
   const int T = is_long ? (int)((__ldg(pv.key_prefix + (sb)) - kp0) >> 5) : 0;
   ChunkSmem c = kSup ? slot_view_sup(region, S, G, T, nslots) : slot_view(region, S, G, T);
 
@@ -741,7 +741,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   //    kB items per batch with all their global loads issued before any
   //    store, so a batch costs one memory latency.
   for (int base = pt; base <= S; base += PT * kB) {
-    int64_t kp[kB], st[kB];
+    uint32_t kp[kB], st[kB];
     int ln[kB], gr[kB];
 #pragma unroll
     for (int r = 0; r < kB; ++r) {
@@ -759,10 +759,10 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
 #pragma unroll
     for (int r = 0; r < kB; ++r) {
       const int i = base + r * PT;
-      const int rel = (int)(kp[r] - kp0);
+      const int rel = (int)(kp[r] - kp0);  // u32 arithmetic
       if (i <= S) c.sA[i] = is_long ? (rel >> 5) : rel;
       if (i < S) {
-        c.sB[i] = is_long ? st[r] : st[r] - rel;
+        c.sB[i] = is_long ? (int64_t)st[r] : (int64_t)st[r] - rel;
         c.sC[i] = ln[r];
         c.sD[i] = gr[r] - (int)ga;
       }
@@ -930,7 +930,11 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
   }
 }
 
-__global__ void __launch_bounds__(kMaxBlock, 1)
+// kBlock: the launch bound (1024 threads cap a thread at 64 registers, which
+// bounds the key loads in flight to kB = 8 tiles per lane; smaller CTAs buy
+// registers for deeper batches: Tuning::batch, block_threads).
+template <int kBlock, int kB>
+__global__ void __launch_bounds__(kBlock, 1)
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
             int64_t slot_bytes, Tuning tu, unsigned long long* __restrict__ out,
             const FuseArgs fuse) {
@@ -991,7 +995,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = min((w0 + 7) & ~7, NU);
             w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
           }
-          acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+          acc += h.linear ? consume<true, kB>(c, h, w0, w1, pv) : consume<false, kB>(c, h, w0, w1, pv);
         } else {  // dynamic: grab `grab` units at a time from the slot's counter
           for (;;) {
             int w0 = 0;
@@ -999,7 +1003,7 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
             w0 = __shfl_sync(0xffffffffu, w0, 0);
             if (w0 >= NU) break;
             const int w1 = min(w0 + grab, NU);
-            acc += h.linear ? consume<true>(c, h, w0, w1, pv) : consume<false>(c, h, w0, w1, pv);
+            acc += h.linear ? consume<true, kB>(c, h, w0, w1, pv) : consume<false, kB>(c, h, w0, w1, pv);
           }
         }
       }
@@ -1022,6 +1026,19 @@ __global__ void __launch_bounds__(kMaxBlock, 1)
       if (fuse.own) fused_epilogue(out, fuse);  // f4: the last CTA sums across ranks
     }
   }
+}
+
+// The long-class kernel's instances: (launch bound, tiles per batch).
+const void* const kCountKernels[] = {
+    (const void*)k_count<1024, 8>, (const void*)k_count<768, 8>, (const void*)k_count<768, 12>,
+    (const void*)k_count<768, 16>, (const void*)k_count<512, 16>, (const void*)k_count<512, 24>};
+
+// The instance for a block size and batch (Tuning::batch; 0 = the default 8):
+// block > 768 or an unknown pair runs the 1024-bound, 8-tile instance.
+const void* count_kernel(int block, int batch) {
+  if (block <= 512) return batch >= 24 ? kCountKernels[5] : kCountKernels[4];
+  if (block <= 768) return batch >= 16 ? kCountKernels[3] : batch >= 12 ? kCountKernels[2] : kCountKernels[1];
+  return kCountKernels[0];
 }
 
 // SHORT-class chunks: every warp stages, builds and probes (no producer /
@@ -1111,14 +1128,14 @@ __device__ __forceinline__ int64_t last_le(const int64_t* __restrict__ a, int64_
 // its suffix, v = the head whose row starts at grp_ibase + ins_prefix, and
 // (u,v) = the position of v in N+(u), which precedes the suffix.
 __global__ void k_seg_edge(const int64_t* __restrict__ row_ptr, int64_t n,
-                           const int32_t* __restrict__ col, const int64_t* __restrict__ seg_start,
+                           const int32_t* __restrict__ col, const uint32_t* __restrict__ seg_start,
                            const int32_t* __restrict__ seg_group,
                            const int64_t* __restrict__ grp_ibase,
                            const int64_t* __restrict__ ins_prefix, int64_t S,
                            int64_t* __restrict__ seg_edge) {
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
        s += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t st = seg_start[s];
+    const int64_t st = (int64_t)seg_start[s];
     const int g = seg_group[s];
     const int64_t u = last_le(row_ptr, n + 1, st);
     const int32_t v = (int32_t)last_le(row_ptr, n + 1, grp_ibase[g] + ins_prefix[g]);
@@ -1163,8 +1180,9 @@ constexpr int kMaxDevices = 64;
 std::once_flag g_attr_once[kMaxDevices];
 
 void set_attr() {
-  TC_CUDA(cudaFuncSetAttribute(k_count, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               optin_smem() - static_smem((const void*)k_count)));
+  for (const void* f : kCountKernels)
+    TC_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 optin_smem() - static_smem(f)));
   TC_CUDA(cudaFuncSetAttribute(k_count_flat, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                optin_smem() - static_smem((const void*)k_count_flat)));
   TC_CUDA(cudaFuncSetAttribute(k_support, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1222,7 +1240,7 @@ int num_sms() {
   return v;
 }
 
-int max_smem_per_block() { return optin_smem() - static_smem((const void*)k_count); }
+int max_smem_per_block() { return optin_smem() - static_smem(kCountKernels[0]); }
 
 int max_chunk_smem(const Tuning& tu) { return (max_smem_per_block() / tu.slots) & ~15; }
 
@@ -1239,7 +1257,7 @@ int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu) {
   ensure_attr();
   int occ = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-      &occ, k_count, block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
+      &occ, count_kernel(block, tu.batch), block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
   return occ;
 }
 
@@ -1268,9 +1286,11 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
   if (l1 > l0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(l1 - l0, P.grid));
     const int64_t sb = slot_bytes_of(P.smem_bytes);
-    k_count<<<grid, P.block, (size_t)(P.tune.slots * sb), s>>>(
-        pv, l0, l1, e_begin, e_end, sb, P.tune, d_out, (fuse && s1 <= s0) ? *fuse : none);
-    TC_LAUNCH();
+    const FuseArgs& fa = (fuse && s1 <= s0) ? *fuse : none;
+    void* args[] = {(void*)&pv, (void*)&l0, (void*)&l1, (void*)&e_begin, (void*)&e_end,
+                    (void*)&sb, (void*)&P.tune, (void*)&d_out, (void*)&fa};
+    TC_CUDA(cudaLaunchKernel(count_kernel(P.block, P.tune.batch), dim3(grid), dim3(P.block), args,
+                             (size_t)(P.tune.slots * sb), s));
     ++launched;
   }
   if (s1 > s0) {

@@ -100,8 +100,8 @@ Options resolve_options(const tc_options* o);
 //                near-equal cost; chunks [0, n_long_chunks) are long.
 struct PlanView {
   const int32_t* col;
-  const int64_t* key_prefix;   // [S+1] work-unit prefix
-  const int64_t* seg_start;    // [S]
+  const uint32_t* key_prefix;  // [S+1] work-unit prefix mod 2^32 (chunk-relative differences < 2^32)
+  const uint32_t* seg_start;   // [S] (col index; m < 2^32)
   const int32_t* seg_len;      // [S]
   const int32_t* seg_group;    // [S]
   const int64_t* ins_prefix;   // [G+1] prefix of d+(v)
@@ -143,6 +143,7 @@ struct Tuning {
   int cs_div = 0;         // short-class chunk cost = chunk_cost / cs_div (0: auto, 2 when the live
                           // edges carry < 2 keys on average, e.g. road graphs, else 1)
   int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
+  int batch = 0;          // long-class tiles per batch for block_threads <= 768 (TC_BATCH; see count_kernel)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
 };
@@ -153,16 +154,17 @@ Tuning tuning_from_env();
 // entries, per (chunk, group) visit the group's ins_prefix / slot_prefix /
 // grp_ibase / grp_code entries, per chunk its two chunk_seg entries and the
 // closing key_prefix / ins_prefix / slot_prefix entries.
-constexpr int64_t kPlanEdgeBytes = 8 + 8 + 4 + 4;
+constexpr int64_t kPlanEdgeBytes = 4 + 4 + 4 + 4;
 constexpr int64_t kPlanGroupBytes = 8 + 8 + 8 + 4;
-constexpr int64_t kPlanChunkBytes = 16 + 8 + 16;
+constexpr int64_t kPlanChunkBytes = 16 + 4 + 16;
 
 struct Plan {
   Options opt;
   Tuning tune;
   int64_t S = 0, S_long = 0, G = 0, n_chunks = 0, n_long_chunks = 0, keys_total = 0;
   int64_t units_total = 0;
-  DevBuf<int64_t> key_prefix, seg_start, ins_prefix, grp_ibase, slot_prefix, chunk_seg;
+  DevBuf<uint32_t> key_prefix, seg_start;  // 32-bit: see PlanView
+  DevBuf<int64_t> ins_prefix, grp_ibase, slot_prefix, chunk_seg;
   DevBuf<int32_t> seg_len, seg_group, grp_code;
   std::vector<int64_t> h_chunk_seg;
   std::vector<int64_t> h_chunk_cost;  // [n_chunks+1] plan cost prefix at each chunk's first edge

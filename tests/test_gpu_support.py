@@ -121,24 +121,80 @@ def test_c5_lattice_full(tc):
     check_full(tc, src, dst, n)
 
 
+def stratified_positions(g, n_random=20000, n_hubs=64, per_hub=50, n_heads=2000, min_head_degree=0,
+                         seed=5):
+    """CSR positions to check one by one: edges of the n_hubs highest-degree
+    vertices (up to per_hub each, in- and out-edges), one in-edge (a member of
+    its group) and one out-edge (a table entry) of each of the n_heads heads v
+    with the largest d+(v) (every head with d+(v) > min_head_degree when that
+    is given: the global-probe "huge" groups of a low huge_degree), and
+    n_random uniform positions."""
+    rp, col, _ = g.csr()
+    m = g.m
+    gen = torch.Generator(device="cuda").manual_seed(seed)
+    dplus = rp[1:] - rp[:-1]
+    dminus = torch.bincount(col.long(), minlength=g.n)
+    deg = dplus + dminus
+    picks = [torch.randint(0, m, (n_random,), device="cuda", generator=gen)]
+    hubs = torch.topk(deg, min(n_hubs, g.n)).indices
+    heads = (torch.nonzero(dplus > min_head_degree).flatten() if min_head_degree
+             else torch.topk(dplus, min(n_heads, g.n)).indices)
+    # in-edges (u, x) of x in hubs / heads: positions where col == x
+    for verts, cap in ((hubs, per_hub), (heads, 1)):
+        mark = torch.zeros(g.n, dtype=torch.bool, device="cuda")
+        mark[verts] = True
+        pos = torch.nonzero(mark[col.long()]).flatten()
+        if pos.numel():
+            key = col.long()[pos] * (m + 1) + torch.randint(0, m, (pos.numel(),), device="cuda",
+                                                          generator=gen)
+            pos = pos[torch.argsort(key)]
+            c = col.long()[pos]
+            first = torch.ones_like(c, dtype=torch.bool)
+            first[1:] = c[1:] != c[:-1]
+            start = torch.nonzero(first).flatten()
+            rank_in = torch.arange(pos.numel(), device="cuda") - start[torch.cumsum(first.long(), 0) - 1]
+            picks.append(pos[rank_in < cap])
+        # out-edges of x: positions rp[x] .. rp[x] + min(d+, cap)
+        lo, d = rp[verts], dplus[verts]
+        k = torch.arange(cap, device="cuda")
+        outp = (lo[:, None] + k[None, :])[(k[None, :] < d[:, None])]
+        picks.append(outp)
+    return torch.unique(torch.cat(picks))
+
+
+def check_positions(g, sup, idx, src, dst, n):
+    u, v = g.edge_list()
+    su, sv, ss = (x[idx].cpu().numpy() for x in (u, v, sup))
+    og = oracle.SupportGraph(src, dst, n)
+    want = og.pairs(su, sv)
+    og.close()
+    assert (want >= 0).all()  # every GPU edge is an edge of the cleaned input
+    bad = np.nonzero(ss.view(np.uint32).astype(np.int64) != want)[0]
+    assert bad.size == 0, f"{bad.size} of {len(idx)} edges differ, e.g. {su[bad[:5]]}-{sv[bad[:5]]}"
+
+
 @pytest.mark.parametrize("cfg", ["C2", "C3"])
-def test_full_size_sampled(tc, cfg):
-    """C2 / C3 at BASELINE size with the bench's launch configuration: 20,000
-    sampled edges against the oracle one by one, and sum = 3T (stored oracle T)."""
+def test_full_size_stratified(tc, cfg):
+    """C2 / C3 at BASELINE size with the bench's launch configuration: sum = 3T
+    (the oracle's stored T), and against the oracle one by one the edges of the
+    64 highest-degree vertices, an in- and an out-edge of the 2,000 heads with
+    the largest tables, and 20,000 uniform edges.  Then the same graph with
+    huge_degree = 256, so every head with d+(v) > 256 is probed in global
+    memory (32 at C2, whose max d+ is ~100): one in- and one out-edge of each.""" 
     import json, os
     src, dst, n = tcgen.CONFIGS[cfg].generate(1)
     stored = json.load(open(os.path.join(os.path.dirname(__file__), "golden",
                                          "config_counts.json")))[f"{cfg}/seed1"]
     with tc.build_csr(dev(src), dev(dst), n) as g:
-        sup = g.support()
-        total = int(sup.to(torch.int64).sum().item())  # values < 2^31: int32 view is exact
-        idx = torch.randint(0, g.m, (20000,), generator=torch.Generator().manual_seed(5)).cuda()
-        u, v = g.edge_list()
-        su, sv, ss = (x[idx].cpu().numpy() for x in (u, v, sup))
         assert g.m == stored["m"]
-    assert total == 3 * stored["triangles"]
-    og = oracle.SupportGraph(src, dst, n)
-    want = og.pairs(su, sv)
-    og.close()
-    assert (want >= 0).all()  # every GPU edge is an edge of the cleaned input
-    assert np.array_equal(ss.view(np.uint32).astype(np.int64), want)
+        sup = g.support()
+        assert int(sup.to(torch.int64).sum().item()) == 3 * stored["triangles"]
+        idx = stratified_positions(g)
+        check_positions(g, sup, idx, src, dst, n)
+    hd = {"C2": 32, "C3": 256}[cfg]
+    with tc.build_csr(dev(src), dev(dst), n, options={"huge_degree": hd}) as g:
+        sup = g.support()
+        assert int(sup.to(torch.int64).sum().item()) == 3 * stored["triangles"]
+        idx = stratified_positions(g, n_random=2000, n_hubs=16, per_hub=8, min_head_degree=hd)
+        assert idx.numel() > 4000
+        check_positions(g, sup, idx, src, dst, n)
