@@ -596,13 +596,24 @@ def main():
         share = float(cost[c1] - cost[c0]) / float(cost[nl])
     long_s = long_total_ms / a.steps / 1e3
     kern_s = kern_total_ms / a.steps / 1e3
-    if split:
+    short_s = kern_s - long_s
+    if split and long_s >= short_s:
         b_launch = float(info.method_bytes_long) * share
         kname, kdesc = "k_count", "k_count (long class, a8), timed alone between its events"
+        k_s = long_s
+    elif split:  # the short class dominates (C2, C5): k_count_flat
+        sshare = 1.0
+        if world > 1 and cost[-1] > cost[nl]:
+            c0, c1 = (int(np.searchsorted(seg, x, side="left")) for x in (s0, s1))
+            sshare = float(cost[max(c1, nl)] - cost[max(c0, nl)]) / float(cost[-1] - cost[nl])
+        b_launch = float(info.method_bytes - info.method_bytes_long) * sshare
+        kname, kdesc = "k_count_flat", "k_count_flat (short class, a7), timed alone between its events"
+        k_s = short_s
     else:  # variant / fused: one call, whole-step bytes
         b_launch = float(info.method_bytes) * (share if world > 1 else 1.0)
         kname, kdesc = "k_count", "whole count step (variant or fused: one call)"
-    achieved = b_launch / long_s / 1e9
+        k_s = kern_s
+    achieved = b_launch / k_s / 1e9
     frac = achieved / hbm
     prof, why = profile_kernel(a.config, kname) if world == 1 and not a.variant else (None, "N>1 or variant")
     step_bytes = float(info.method_bytes) * (1.0 if world == 1 else (e1 - e0) / max(1, info.m_live))
@@ -611,10 +622,11 @@ def main():
             "traffic": None if prof is None else prof["dram_bytes"] * share,
             "traffic_source": (f"ncu --set full, capture {why}, same sources (src_hash {src_hash()})"
                                if prof is not None else f"none: {why}"),
-            "bytes_per_launch": b_launch, "kernel_ms": long_s * 1e3,
-            "bytes_def": "method bytes = 4*keys + 24 B plan entries per live edge + "
-                         "(4*d+(v) + 28 B) per (chunk, group) + 40 B per chunk, long class "
-                         "(info.method_bytes_long); x this rank's cost share for N>1",
+            "bytes_per_launch": b_launch, "kernel_ms": k_s * 1e3,
+            "bytes_def": "method bytes of the kernel's class = 4*keys + 16 B plan entries per "
+                         "live edge + (4*d+(v) + 28 B) per (chunk, group) + 36 B per chunk "
+                         "(info.method_bytes_long, or method_bytes - method_bytes_long for the "
+                         "short class); x this rank's cost share for N>1",
             "peak_source": peak_src,
             "step": {"bytes": step_bytes, "ms": kern_s * 1e3,
                      "frac": step_bytes / kern_s / 1e9 / hbm,

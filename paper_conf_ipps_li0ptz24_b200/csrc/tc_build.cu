@@ -150,14 +150,21 @@ __global__ void k_uniq_tail(const int* err, const int64_t* nsel, const uint64_t*
 }
 
 // ------------------------------------------------------------------ a3
+// The first endpoints of sorted keys come in runs: lanes holding the same
+// one add their count with one atomic (__match_any_sync); the second
+// endpoint takes one atomic per key.  Exact for any key order.
 __global__ void k_degree(const uint64_t* __restrict__ key, int64_t m, int bits,
                          int32_t* __restrict__ deg) {
   const uint64_t mask = (uint64_t(1) << bits) - 1;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    uint64_t k = key[i];
-    atomicAdd(&deg[k >> bits], 1);
-    atomicAdd(&deg[k & mask], 1);
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t m_round = (m + 31) & ~int64_t(31);  // whole warps stay converged
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m_round; i += stride) {
+    const bool in = i < m;
+    const uint64_t k = in ? key[i] : ~0ull;
+    const unsigned a = in ? (unsigned)(k >> bits) : 0xffffffffu;
+    const unsigned same = __match_any_sync(0xffffffffu, a);
+    if (in && (threadIdx.x & 31) == __ffs(same) - 1) atomicAdd(&deg[a], __popc(same));
+    if (in) atomicAdd(&deg[k & mask], 1);
   }
 }
 
@@ -205,14 +212,18 @@ __global__ void k_orient(const uint64_t* __restrict__ key, int64_t m, int bits,
   }
 }
 
+// CSR of sorted oriented keys; also the row of every position (rowid, the
+// plan's first input: one write here instead of a separate pass over rows).
 __global__ void k_csr(const uint64_t* __restrict__ okey, int64_t m, int64_t n, int bits2,
-                      int32_t* __restrict__ col, int64_t* __restrict__ row_ptr) {
+                      int32_t* __restrict__ col, int64_t* __restrict__ row_ptr,
+                      int32_t* __restrict__ rowid) {
   const uint64_t mask = (uint64_t(1) << bits2) - 1;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
        i += (int64_t)gridDim.x * blockDim.x) {
     uint64_t k = okey[i];
     int64_t u = (int64_t)(k >> bits2);
     col[i] = (int32_t)(k & mask);
+    rowid[i] = (int32_t)u;
     int64_t prev = i ? (int64_t)(okey[i - 1] >> bits2) : -1;
     for (int64_t x = prev + 1; x <= u; ++x) row_ptr[x] = i;
     if (i == m - 1)
@@ -252,6 +263,16 @@ __global__ void k_rowid(const int64_t* __restrict__ row_ptr, int64_t n,
     for (int64_t p = row_ptr[u], e = row_ptr[u + 1]; p < e; ++p) rowid[p] = (int32_t)u;
 }
 
+// Per row v: {min N+(v), max N+(v)} (rows are sorted), {INT_MAX, -1} if empty.
+__global__ void k_vmm(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
+                      int64_t n, int2* __restrict__ vmm) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+       v += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = row_ptr[v], b = row_ptr[v + 1];
+    vmm[v] = b > a ? make_int2(col[a], col[b - 1]) : make_int2(0x7fffffff, -1);
+  }
+}
+
 __device__ __forceinline__ int64_t lower_bound_i32(const int32_t* __restrict__ a, int64_t lo,
                                                    int64_t hi, int32_t x) {
   while (lo < hi) {
@@ -279,7 +300,8 @@ __device__ __forceinline__ int64_t upper_bound_i32(const int32_t* __restrict__ a
 // (untrimmed), [1] trimmed keys, [2] live, [3] live long,
 // [4] trimmed keys of the long class.
 __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                            const int32_t* __restrict__ rowid, int64_t m, int long_min, int bits,
+                            const int32_t* __restrict__ rowid, const int2* __restrict__ vmm,
+                            int64_t m, int long_min, int bits,
                             uint32_t dead, uint32_t* __restrict__ skey, uint64_t* __restrict__ sval,
                             unsigned long long* stats) {
   typedef cub::BlockReduce<unsigned long long, TPB> BR;
@@ -293,8 +315,9 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
     b += 4ull * (unsigned long long)(suf + dv) + 12ull;
     int64_t lo = p + 1, len = 0;
     if (suf > 0 && dv > 0) {
-      lo = lower_bound_i32(col, p + 1, rend, col[rv]);
-      len = upper_bound_i32(col, lo, rend, col[rv + dv - 1]) - lo;
+      const int2 w = vmm[v];  // [min N+(v), max N+(v)]: one 8-B read instead of two in col
+      lo = lower_bound_i32(col, p + 1, rend, w.x);
+      len = upper_bound_i32(col, lo, rend, w.y) - lo;
     }
     const uint32_t cls = len < long_min ? 1u : 0u;
     skey[p] = len > 0 ? ((cls << bits) | (uint32_t)v) : dead;
@@ -715,7 +738,9 @@ void csr_from_sorted(const uint64_t* okey, int64_t m, int64_t n_act, cudaStream_
   g->row_ptr = DevBuf<int64_t>(n_act + 1, s, true);
   g->col = DevBuf<int32_t>(std::max<int64_t>(m, 1), s, true);
   if (m > 0) {
-    k_csr<<<grid_for(m), TPB, 0, s>>>(okey, m, n_act, bits2, g->col.get(), g->row_ptr.get());
+    g->rowid = DevBuf<int32_t>(m, s);  // scratch for the plan (build_plan frees it)
+    k_csr<<<grid_for(m), TPB, 0, s>>>(okey, m, n_act, bits2, g->col.get(), g->row_ptr.get(),
+                                      g->rowid.get());
     TC_LAUNCH();
   } else {
     k_fill_i64<<<grid_for(n_act + 1), TPB, 0, s>>>(g->row_ptr.get(), n_act + 1, 0);
@@ -1086,11 +1111,19 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   const int kbits = g->bits + 1;
   const uint32_t dead = kbits < 32 ? (1u << kbits) : 0xFFFFFFFFu;
   const int end_bit = kbits < 32 ? kbits + 1 : 32;
-  DevBuf<int32_t> rowid(std::max<int64_t>(m, 1), s);
+  // the row of every position: left by the CSR build (k_csr), else one pass over rows
+  DevBuf<int32_t> rowid;
+  rowid.swap(g->rowid);
   DevBuf<uint32_t> skey(std::max<int64_t>(m, 1), s), skey2(std::max<int64_t>(m, 1), s);
   DevBuf<uint64_t> sval(std::max<int64_t>(m, 1), s), sval2(std::max<int64_t>(m, 1), s);
   if (m > 0) {
-    k_rowid<<<grid_for(n), TPB, 0, s>>>(row_ptr, n, rowid.get());
+    if (!rowid.get()) {
+      rowid = DevBuf<int32_t>(m, s);
+      k_rowid<<<grid_for(n), TPB, 0, s>>>(row_ptr, n, rowid.get());
+      TC_LAUNCH();
+    }
+    DevBuf<int2> vmm(std::max<int64_t>(n, 1), s);
+    k_vmm<<<grid_for(n), TPB, 0, s>>>(row_ptr, col, n, vmm.get());
     TC_LAUNCH();
     // a long-class tile always holds 32 keys of its own edge (walk_long shifts
     // a partial last tile back onto the edge), so long_min < 32 acts as 32
@@ -1100,8 +1133,8 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     // long_min keeps the split.
     constexpr int64_t kSmallGraph = int64_t(1) << 20;
     const int long_min = (opt.long_min_auto && m < kSmallGraph) ? (1 << 30) : std::max(opt.long_min, 32);
-    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), m, long_min, g->bits,
-                                            dead, skey.get(), sval.get(), stats.get());
+    k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), vmm.get(), m, long_min,
+                                            g->bits, dead, skey.get(), sval.get(), stats.get());
     TC_LAUNCH();
   }
   rowid.reset();

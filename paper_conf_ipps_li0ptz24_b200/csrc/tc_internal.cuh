@@ -186,6 +186,7 @@ struct tc_graph {
   int bits = 1;  // bits of a vertex id in [0, n)
   tc::DevBuf<int64_t> row_ptr;
   tc::DevBuf<int32_t> col, perm;
+  tc::DevBuf<int32_t> rowid;  // build scratch: row of every CSR position (a5 -> a6), then freed
   tc::Plan plan;
   uint64_t b_itc = 0;
   float ms[6] = {0, 0, 0, 0, 0, 0};
