@@ -138,11 +138,15 @@ struct Tuning {
   int slots = 3;          // chunk slots in SMEM (2..4)
   int grab_long = 0;      // tiles per consumer grab, long class (0 = static split)
   int grab_short = 0;     // keys per consumer grab, short class (0 = static split)
-  int prod_div = 5;       // 1/prod_div of the warps are producers (C3 sweep: 8 -> 57.7 ms, 6 -> 55.0, 5 -> 53.5, 4 -> 54.0)
+  int prod_div = 4;       // 1/prod_div of the warps are producers (r2h, C3 k_count: 5 -> 44.9 ms, 4 -> 42.9,
+                          // 3 -> 44.3; C4: 629 / 583 / 576 ms)
   int wait_hint_ns = 0;   // mbarrier try_wait suspend hint (0 = none)
   int cs_div = 0;         // short-class chunk cost = chunk_cost / cs_div (0: auto, 2 when the live
                           // edges carry < 2 keys on average, e.g. road graphs, else 1)
   int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
+  int head_permille = 0;  // > 0: the first head_permille/1000 of the long class's cost is a separate
+                          // launch with 1/head_prod_div producer warps (TC_HEAD_PERMILLE)
+  int head_prod_div = 2;  // (TC_HEAD_PROD_DIV)
   int batch = 0;          // long-class tiles per batch for block_threads <= 768 (TC_BATCH; see count_kernel)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
