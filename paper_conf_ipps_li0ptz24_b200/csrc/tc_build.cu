@@ -1090,8 +1090,6 @@ Tuning tuning_from_env() {
   t.short_linear = get("TC_SHORT_LINEAR", t.short_linear, 0, 1);
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
   t.batch = get("TC_BATCH", t.batch, 0, 64);
-  t.head_permille = get("TC_HEAD_PERMILLE", t.head_permille, 0, 1000);
-  t.head_prod_div = get("TC_HEAD_PROD_DIV", t.head_prod_div, 2, 32);
   return t;
 }
 

@@ -1283,27 +1283,12 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
   const int64_t l0 = c_begin, l1 = std::min(c_end, P.n_long_chunks);
   const int64_t s0 = std::max(c_begin, P.n_long_chunks), s1 = c_end;
   int launched = 0;
-  // the long class's producer-heavy head (many small tables: the first
-  // chunks, lowest-ranked heads) may run as its own launch with more
-  // producer warps (Tuning::head_permille / head_prod_div)
-  int64_t lsplit = l0;
-  if (P.tune.head_permille > 0 && P.n_long_chunks > 0) {
-    const auto& cc = P.h_chunk_cost;
-    const int64_t target = cc[P.n_long_chunks] / 1000 * P.tune.head_permille;
-    lsplit = std::lower_bound(cc.begin(), cc.begin() + P.n_long_chunks + 1, target) - cc.begin();
-    lsplit = std::min(std::max(lsplit, l0), l1);
-  }
-  for (int part = 0; part < 2; ++part) {
-    const int64_t a = part == 0 ? l0 : lsplit, b = part == 0 ? lsplit : l1;
-    if (b <= a) continue;
-    Tuning tu = P.tune;
-    if (part == 0) tu.prod_div = P.tune.head_prod_div;
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(b - a, P.grid));
+  if (l1 > l0) {
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(l1 - l0, P.grid));
     const int64_t sb = slot_bytes_of(P.smem_bytes);
-    const bool last = s1 <= s0 && (part == 1 || l1 <= lsplit);  // no later launch follows
-    const FuseArgs& fa = (fuse && last) ? *fuse : none;
-    void* args[] = {(void*)&pv, (void*)&a, (void*)&b, (void*)&e_begin, (void*)&e_end,
-                    (void*)&sb, (void*)&tu, (void*)&d_out, (void*)&fa};
+    const FuseArgs& fa = (fuse && s1 <= s0) ? *fuse : none;  // no later launch follows
+    void* args[] = {(void*)&pv, (void*)&l0, (void*)&l1, (void*)&e_begin, (void*)&e_end,
+                    (void*)&sb, (void*)&P.tune, (void*)&d_out, (void*)&fa};
     TC_CUDA(cudaLaunchKernel(count_kernel(P.block, P.tune.batch), dim3(grid), dim3(P.block), args,
                              (size_t)(P.tune.slots * sb), s));
     ++launched;

@@ -144,9 +144,6 @@ struct Tuning {
   int cs_div = 0;         // short-class chunk cost = chunk_cost / cs_div (0: auto, 2 when the live
                           // edges carry < 2 keys on average, e.g. road graphs, else 1)
   int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
-  int head_permille = 0;  // > 0: the first head_permille/1000 of the long class's cost is a separate
-                          // launch with 1/head_prod_div producer warps (TC_HEAD_PERMILLE)
-  int head_prod_div = 2;  // (TC_HEAD_PROD_DIV)
   int batch = 0;          // long-class tiles per batch for block_threads <= 768 (TC_BATCH; see count_kernel)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
