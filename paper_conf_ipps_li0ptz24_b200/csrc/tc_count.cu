@@ -452,6 +452,75 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   return cnt;
 }
 
+// walk_long software-pipelined: batch b + 1's kB key loads are issued before
+// batch b is probed, so a warp has loads in flight while it probes (kB = 4:
+// 4 to 8 loads in flight per lane instead of 8 then 0; Tuning::pipe).
+// The general (hash / huge) probe of a 4-tile batch, out of line so that the
+// pipelined walk keeps its registers for the keys in flight.
+template <bool kLinear, bool kHuge>
+__device__ __noinline__ unsigned probe4_general(const ChunkSmem& c, int t, int32_t k0, int32_t k1,
+                                                int32_t k2, int32_t k3, int lane,
+                                                const PlanView& pv, int64_t ga) {
+  const int32_t key[4] = {k0, k1, k2, k3};
+  unsigned cnt = 0;
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const int z = c.sT1[t + u], zw = c.sT2[t + u];
+    const unsigned hit = probe_tile<kLinear, kHuge>(c, z, zw, key[u], lane, pv, ga);
+    if (lane >= (zw & 63)) cnt += hit;
+  }
+  return cnt;
+}
+
+template <bool kLinear, bool kHuge, int kB>
+__device__ __forceinline__ unsigned probe_batch(const ChunkSmem& c, int t, const int32_t (&key)[kB],
+                                                int lane, const PlanView& pv, int64_t ga) {
+  unsigned cnt = 0;
+  int z[kB], zw[kB];
+#pragma unroll
+  for (int q = 0; q < kB; q += 4) {
+    *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
+    *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
+  }
+  int zw_or = 0;
+#pragma unroll
+  for (int u = 0; u < kB; ++u) zw_or |= zw[u];
+  if ((zw_or >> 6) == 0) {
+#pragma unroll
+    for (int u = 0; u < kB; ++u) {
+      const unsigned word = (unsigned)c.sT0[(key[u] >> 5) + z[u]];
+      const unsigned hit = (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
+      if (lane >= zw[u]) cnt += hit;
+    }
+  } else {
+    static_assert(kB == 4, "the out-of-line general path takes 4 keys");
+    cnt += probe4_general<kLinear, kHuge>(c, t, key[0], key[1], key[2], key[3], lane, pv, ga);
+  }
+  return cnt;
+}
+
+template <bool kLinear, bool kHuge, int kB>
+__device__ __forceinline__ unsigned walk_long_pipe(const ChunkSmem& c, int t0, int t1,
+                                                   const PlanView& pv, int64_t ga) {
+  unsigned cnt = 0;
+  const int lane = threadIdx.x & 31;
+  const int32_t* colL = lane_base(pv.col, lane);
+  int t = t0;
+  int32_t ka[kB], kb[kB];
+  if (t + kB <= t1) load_batch<kB>(c, colL, t, ka);
+  for (; t + 2 * kB <= t1; t += 2 * kB) {  // two batches per trip: the buffers swap roles
+    load_batch<kB>(c, colL, t + kB, kb);
+    cnt += probe_batch<kLinear, kHuge, kB>(c, t, ka, lane, pv, ga);
+    if (t + 3 * kB <= t1) load_batch<kB>(c, colL, t + 2 * kB, ka);
+    cnt += probe_batch<kLinear, kHuge, kB>(c, t + kB, kb, lane, pv, ga);
+  }
+  if (t + kB <= t1) {  // one loaded batch left
+    cnt += probe_batch<kLinear, kHuge, kB>(c, t, ka, lane, pv, ga);
+    t += kB;
+  }
+  return cnt + walk_long<kLinear, kHuge, 8>(c, t, t1, pv, ga);  // < kB tiles: its tail loop
+}
+
 // SHORT class: the warp owns the flat keys [k0w, k1w) of the chunk.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0w, int k1w,
@@ -509,9 +578,14 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
   return cnt;
 }
 
-template <bool kLinear, int kB = kBatchLong>
+template <bool kLinear, int kB = kBatchLong, bool kPipe = false>
 __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
                                             const PlanView& pv) {
+  if constexpr (kPipe) {
+    if (h.is_long)
+      return h.huge ? walk_long_pipe<kLinear, true, kB>(c, w0, w1, pv, h.ga)
+                    : walk_long_pipe<kLinear, false, kB>(c, w0, w1, pv, h.ga);
+  }
   if (h.is_long)
     return h.huge ? walk_long<kLinear, true, kB>(c, w0, w1, pv, h.ga)
                   : walk_long<kLinear, false, kB>(c, w0, w1, pv, h.ga);
@@ -717,7 +791,7 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
 template <int kB, bool kSup = false>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
-                                        int pt, int PT) {
+                                        int pt, int PT, int bar = 1) {
   const int64_t sa = max(__ldg(pv.chunk_seg + (cix)), e_begin), sb = min(__ldg(pv.chunk_seg + (cix + 1)), e_end);
   if (sa >= sb) {  // empty after clipping to the range
     if (pt == 0) {
@@ -807,7 +881,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     for (int i = pt; i < (nwords >> 2); i += PT) h4[i] = make_int4(-1, -1, -1, -1);
     for (int i = (nwords & ~3) + pt; i < nwords; i += PT) c.sHash[i] = -1;
   }
-  const int any_huge = named_sync_or(1, PT, huge);
+  const int any_huge = named_sync_or(bar, PT, huge);
 
   // 2. long class: one descriptor per 32-key tile (producer thread per edge)
   if (is_long) {
@@ -880,10 +954,10 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
     linear = false;
     warp_walk<kInsU>(c.sGP, G, i0, i1, load_row,
                      [&](int g, int k, int32_t key) { ins_sup(g, k, key, want_linear); });
-    if (!want_linear && named_sync_or(1, PT, linear)) {  // a cuckoo insert failed
+    if (!want_linear && named_sync_or(bar, PT, linear)) {  // a cuckoo insert failed
       if (pt == 0) atomicAdd(&g_counters[0], 1ull);
       for (int i = pt; i < 2 * nslots; i += PT) c.sHash[i] = -1;
-      named_sync(1, PT);
+      named_sync(bar, PT);
       warp_walk<kInsU>(c.sGP, G, i0, i1, load_row,
                        [&](int g, int k, int32_t key) { ins_sup(g, k, key, true); });
       linear = true;
@@ -906,11 +980,11 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
       if (d.y <= 0) bitmap_insert(c.sHash + d.x, d.y, key);
       else if (!cuckoo_insert(c.sHash + d.x, (uint32_t)d.y, key, pv.max_kicks)) ok = false;
     });
-    if (named_sync_or(1, PT, !ok)) {  // uniform over producers: rebuild with linear probing
+    if (named_sync_or(bar, PT, !ok)) {  // uniform over producers: rebuild with linear probing
       if (pt == 0) atomicAdd(&g_counters[0], 1ull);
       linear = true;
       for (int i = pt; i < nslots; i += PT) c.sHash[i] = -1;
-      named_sync(1, PT);
+      named_sync(bar, PT);
       warp_walk<kInsU>(c.sGP, G, i0, i1, load_row, insert_linear);
     }
   }
@@ -933,7 +1007,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
 // kBlock: the launch bound (1024 threads cap a thread at 64 registers, which
 // bounds the key loads in flight to kB = 8 tiles per lane; smaller CTAs buy
 // registers for deeper batches: Tuning::batch, block_threads).
-template <int kBlock, int kB>
+template <int kBlock, int kB, bool kPipe = false>
 __global__ void __launch_bounds__(kBlock, 1)
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
             int64_t slot_bytes, Tuning tu, unsigned long long* __restrict__ out,
@@ -948,9 +1022,15 @@ __global__ void __launch_bounds__(kBlock, 1)
   const int PT = n_prod * 32;
   const int nslots = tu.slots;
   const uint32_t hint = (uint32_t)tu.wait_hint_ns;
+  // producer groups (Tuning::prod_groups): group g fills the CTA's chunks
+  // k = g, g + ng, ... into slot k mod nslots, on its own named barrier, so
+  // ng chunks are in production at once (a chunk's staging and table build
+  // are latency-bound where its tables are many and small)
+  const int ng = max(1, min(tu.prod_groups, n_prod));
+  const int gsz = n_prod / ng, PTg = gsz * 32;
   if (threadIdx.x == 0) {
     for (int i = 0; i < nslots; ++i) {
-      mbar_init(&full_bar[i], PT);       // every producer thread arrives
+      mbar_init(&full_bar[i], PTg);      // every thread of the filling group arrives
       mbar_init(&empty_bar[i], n_cons);  // one lane per consumer warp
     }
   }
@@ -959,20 +1039,29 @@ __global__ void __launch_bounds__(kBlock, 1)
   unsigned long long acc = 0;
   if (warp < n_prod) {
     // ------------------------------------------------------------ producers
-    // slot / fill number kept incrementally (no 64-bit division per chunk)
-    int slot = 0;
-    uint32_t j = 0;  // fill number of this slot
-    // This CTA's chunks are c_begin + b + k * grid.
-    for (int64_t cix = c_begin + blockIdx.x;; cix += gridDim.x,
-                 slot = (slot + 1 == nslots) ? (++j, 0) : slot + 1) {
-      if (j > 0) wait_empty(&empty_bar[slot], (j - 1) & 1, hint);
-      if (cix >= c_end) {
-        if (threadIdx.x == 0) hdr[slot].done = 1;
+    const int g = warp / gsz;
+    if (warp < ng * gsz) {  // (warps beyond ng * gsz, if n_prod is odd, idle)
+      const int pt = threadIdx.x - g * PTg;
+      // slot / fill number kept incrementally (no 64-bit division per chunk)
+      int slot = g;
+      uint32_t j = 0;  // fill number of this slot
+      // This CTA's chunks are c_begin + b + k * grid; this group's k = g + i * ng.
+      for (int64_t cix = c_begin + blockIdx.x + (int64_t)g * gridDim.x;;
+           cix += (int64_t)ng * gridDim.x) {
+        if (j > 0) wait_empty(&empty_bar[slot], (j - 1) & 1, hint);
+        if (cix >= c_end) {
+          if (pt == 0) hdr[slot].done = 1;
+          mbar_arrive(&full_bar[slot]);
+          break;
+        }
+        produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], pt, PTg, 1 + g);
         mbar_arrive(&full_bar[slot]);
-        break;
+        slot += ng;
+        if (slot >= nslots) {
+          slot -= nslots;
+          ++j;
+        }
       }
-      produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], threadIdx.x, PT);
-      mbar_arrive(&full_bar[slot]);
     }
   } else {
     // ------------------------------------------------------------ consumers
@@ -995,7 +1084,8 @@ __global__ void __launch_bounds__(kBlock, 1)
             w0 = min((w0 + 7) & ~7, NU);
             w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
           }
-          acc += h.linear ? consume<true, kB>(c, h, w0, w1, pv) : consume<false, kB>(c, h, w0, w1, pv);
+          acc += h.linear ? consume<true, kB, kPipe>(c, h, w0, w1, pv)
+                          : consume<false, kB, kPipe>(c, h, w0, w1, pv);
         } else {  // dynamic: grab `grab` units at a time from the slot's counter
           for (;;) {
             int w0 = 0;
@@ -1003,7 +1093,8 @@ __global__ void __launch_bounds__(kBlock, 1)
             w0 = __shfl_sync(0xffffffffu, w0, 0);
             if (w0 >= NU) break;
             const int w1 = min(w0 + grab, NU);
-            acc += h.linear ? consume<true, kB>(c, h, w0, w1, pv) : consume<false, kB>(c, h, w0, w1, pv);
+            acc += h.linear ? consume<true, kB, kPipe>(c, h, w0, w1, pv)
+                            : consume<false, kB, kPipe>(c, h, w0, w1, pv);
           }
         }
       }
@@ -1031,11 +1122,14 @@ __global__ void __launch_bounds__(kBlock, 1)
 // The long-class kernel's instances: (launch bound, tiles per batch).
 const void* const kCountKernels[] = {
     (const void*)k_count<1024, 8>, (const void*)k_count<768, 8>, (const void*)k_count<768, 12>,
-    (const void*)k_count<768, 16>, (const void*)k_count<512, 16>, (const void*)k_count<512, 24>};
+    (const void*)k_count<768, 16>, (const void*)k_count<512, 16>, (const void*)k_count<512, 24>,
+    (const void*)k_count<1024, 4, true>, (const void*)k_count<768, 4, true>};
 
-// The instance for a block size and batch (Tuning::batch; 0 = the default 8):
-// block > 768 or an unknown pair runs the 1024-bound, 8-tile instance.
-const void* count_kernel(int block, int batch) {
+// The instance for a block size and batch (Tuning::batch; 0 = the default 8)
+// and Tuning::pipe: block > 768 or an unknown pair runs the 1024-bound,
+// 8-tile instance.
+const void* count_kernel(int block, int batch, int pipe) {
+  if (pipe) return block <= 768 ? kCountKernels[7] : kCountKernels[6];
   if (block <= 512) return batch >= 24 ? kCountKernels[5] : kCountKernels[4];
   if (block <= 768) return batch >= 16 ? kCountKernels[3] : batch >= 12 ? kCountKernels[2] : kCountKernels[1];
   return kCountKernels[0];
@@ -1257,7 +1351,7 @@ int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu) {
   ensure_attr();
   int occ = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-      &occ, count_kernel(block, tu.batch), block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
+      &occ, count_kernel(block, tu.batch, tu.pipe), block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
   return occ;
 }
 
@@ -1289,7 +1383,7 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
     const FuseArgs& fa = (fuse && s1 <= s0) ? *fuse : none;  // no later launch follows
     void* args[] = {(void*)&pv, (void*)&l0, (void*)&l1, (void*)&e_begin, (void*)&e_end,
                     (void*)&sb, (void*)&P.tune, (void*)&d_out, (void*)&fa};
-    TC_CUDA(cudaLaunchKernel(count_kernel(P.block, P.tune.batch), dim3(grid), dim3(P.block), args,
+    TC_CUDA(cudaLaunchKernel(count_kernel(P.block, P.tune.batch, P.tune.pipe), dim3(grid), dim3(P.block), args,
                              (size_t)(P.tune.slots * sb), s));
     ++launched;
   }
