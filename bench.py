@@ -567,6 +567,7 @@ def main():
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
         e2e_ms = float(et[0]) / max(1, len(ts))
         e2e = {"value": m / (e2e_ms / 1e3), "unit": UNIT, "ms_per_step": e2e_ms,
+               "step_ms": [round(x, 3) for x in ts],
                "h2d_bytes_per_step": int(src.nbytes + dst.nbytes) * (hi - lo) // max(1, len(src)),
                "d2h_bytes_per_step": 8 + 8 * (n_chunks + 1) + 96,
                "what": ("tc_build_csr_host (H2D of the raw pinned edge list + a1..a6)" if world == 1

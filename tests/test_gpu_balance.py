@@ -1,7 +1,7 @@
 """Measured balance of the multi-GPU edge ranges, emulated
 on one B200: every rank's tc_count_range of the tc_partition_measured split
 (profile = this device's tc_calibrate, 64 slices) is timed alone with CUDA
-events, L2 flushed before each; the slowest range may exceed the mean by at
+events, L2 flushed before each (median of 5); the slowest range may exceed the mean by at
 most 5 %, and the partials sum to the oracle's stored T (the per-edge
 intersections are independent, so any cut is exact)."""
 import json
@@ -28,7 +28,7 @@ def tc():
     return tc
 
 
-def _range_ms(g, b, e, flush, out, reps=3):
+def _range_ms(g, b, e, flush, out, reps=5):
     s = torch.cuda.current_stream()
     ts = []
     for i in range(reps):
