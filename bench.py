@@ -463,38 +463,6 @@ def main():
     ms_per_step = total_ms / a.steps
     value = m / (ms_per_step / 1e3)
 
-    # ---------------------------------------------------------------- emulated multi-GPU balance
-    # N = 1: the P-rank splits of tc_partition_measured (this device's
-    # 64-slice profile) and of tc_partition (built-in profile), every range
-    # timed alone (L2 flushed, median of 3): max/mean per P
-    balance = None
-    if world == 1 and not a.variant and not a.no_balance:
-        w = g.calibrate()
-        balance = {"profile_slices": len(w), "profile_ms_sum": float(w.sum()),
-                   "what": "each rank's tc_count_range timed alone on this GPU (CUDA events, "
-                           "L2 flushed, median of 3); max/mean over ranks"}
-        tmp = torch.zeros(1, dtype=torch.int64, device=dev)
-
-        def range_ms(b, e):
-            ts = []
-            for r in range(3):
-                flush.fill_(r)
-                y0, y1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                y0.record(stream)
-                g.count_range(b, e, out=tmp)
-                y1.record(stream)
-                torch.cuda.synchronize()
-                ts.append(y0.elapsed_time(y1))
-            return statistics.median(ts), int(tmp.item())
-
-        for P in (2, 4, 8):
-            for label, bb in (("measured", g.partition(P, w)), ("builtin", g.partition(P))):
-                res = [range_ms(bb[r], bb[r + 1]) for r in range(P)]
-                ms = [x for x, _ in res]
-                balance[f"P{P}_{label}"] = {
-                    "max_over_mean": max(ms) / (sum(ms) / P), "range_ms": [round(x, 3) for x in ms],
-                    "partials_sum_to_T": (sum(p for _, p in res) & (2**64 - 1)) == T}
-
     # ---------------------------------------------------------------- sharded build (f2)
     # Every rank holds the contiguous 1/world slice of the raw pairs and the
     # ranks build the identical replicated graph (tc_shard_* + NCCL
@@ -573,6 +541,40 @@ def main():
                "what": ("tc_build_csr_host (H2D of the raw pinned edge list + a1..a6)" if world == 1
                         else "H2D of this rank's 1/N pinned slice + build_csr_sharded (f2)")
                        + " + tc_count_range + all_reduce + 8-B D2H of T"}
+
+    # ---------------------------------------------------------------- emulated multi-GPU balance
+    # (after the e2e leg: its many short launches perturbed the e2e timing
+    # that followed them, 13.6 -> 37 ms at C5)
+    # N = 1: the P-rank splits of tc_partition_measured (this device's
+    # 64-slice profile) and of tc_partition (built-in profile), every range
+    # timed alone (L2 flushed, median of 3): max/mean per P
+    balance = None
+    if world == 1 and not a.variant and not a.no_balance:
+        w = g.calibrate()
+        balance = {"profile_slices": len(w), "profile_ms_sum": float(w.sum()),
+                   "what": "each rank's tc_count_range timed alone on this GPU (CUDA events, "
+                           "L2 flushed, median of 3); max/mean over ranks"}
+        tmp = torch.zeros(1, dtype=torch.int64, device=dev)
+
+        def range_ms(b, e):
+            ts = []
+            for r in range(3):
+                flush.fill_(r)
+                y0, y1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                y0.record(stream)
+                g.count_range(b, e, out=tmp)
+                y1.record(stream)
+                torch.cuda.synchronize()
+                ts.append(y0.elapsed_time(y1))
+            return statistics.median(ts), int(tmp.item())
+
+        for P in (2, 4, 8):
+            for label, bb in (("measured", g.partition(P, w)), ("builtin", g.partition(P))):
+                res = [range_ms(bb[r], bb[r + 1]) for r in range(P)]
+                ms = [x for x, _ in res]
+                balance[f"P{P}_{label}"] = {
+                    "max_over_mean": max(ms) / (sum(ms) / P), "range_ms": [round(x, 3) for x in ms],
+                    "partials_sum_to_T": (sum(p for _, p in res) & (2**64 - 1)) == T}
 
     if rank != 0:
         if world > 1:

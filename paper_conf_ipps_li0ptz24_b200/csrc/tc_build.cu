@@ -1090,8 +1090,7 @@ Tuning tuning_from_env() {
   t.short_linear = get("TC_SHORT_LINEAR", t.short_linear, 0, 1);
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
   t.batch = get("TC_BATCH", t.batch, 0, 64);
-  t.pipe = get("TC_PIPE", t.pipe, 0, 1);
-  t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 2);
+  t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 3);
   return t;
 }
 

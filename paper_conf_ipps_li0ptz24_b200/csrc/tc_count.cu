@@ -452,75 +452,6 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   return cnt;
 }
 
-// walk_long software-pipelined: batch b + 1's kB key loads are issued before
-// batch b is probed, so a warp has loads in flight while it probes (kB = 4:
-// 4 to 8 loads in flight per lane instead of 8 then 0; Tuning::pipe).
-// The general (hash / huge) probe of a 4-tile batch, out of line so that the
-// pipelined walk keeps its registers for the keys in flight.
-template <bool kLinear, bool kHuge>
-__device__ __noinline__ unsigned probe4_general(const ChunkSmem& c, int t, int32_t k0, int32_t k1,
-                                                int32_t k2, int32_t k3, int lane,
-                                                const PlanView& pv, int64_t ga) {
-  const int32_t key[4] = {k0, k1, k2, k3};
-  unsigned cnt = 0;
-#pragma unroll
-  for (int u = 0; u < 4; ++u) {
-    const int z = c.sT1[t + u], zw = c.sT2[t + u];
-    const unsigned hit = probe_tile<kLinear, kHuge>(c, z, zw, key[u], lane, pv, ga);
-    if (lane >= (zw & 63)) cnt += hit;
-  }
-  return cnt;
-}
-
-template <bool kLinear, bool kHuge, int kB>
-__device__ __forceinline__ unsigned probe_batch(const ChunkSmem& c, int t, const int32_t (&key)[kB],
-                                                int lane, const PlanView& pv, int64_t ga) {
-  unsigned cnt = 0;
-  int z[kB], zw[kB];
-#pragma unroll
-  for (int q = 0; q < kB; q += 4) {
-    *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
-    *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
-  }
-  int zw_or = 0;
-#pragma unroll
-  for (int u = 0; u < kB; ++u) zw_or |= zw[u];
-  if ((zw_or >> 6) == 0) {
-#pragma unroll
-    for (int u = 0; u < kB; ++u) {
-      const unsigned word = (unsigned)c.sT0[(key[u] >> 5) + z[u]];
-      const unsigned hit = (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
-      if (lane >= zw[u]) cnt += hit;
-    }
-  } else {
-    static_assert(kB == 4, "the out-of-line general path takes 4 keys");
-    cnt += probe4_general<kLinear, kHuge>(c, t, key[0], key[1], key[2], key[3], lane, pv, ga);
-  }
-  return cnt;
-}
-
-template <bool kLinear, bool kHuge, int kB>
-__device__ __forceinline__ unsigned walk_long_pipe(const ChunkSmem& c, int t0, int t1,
-                                                   const PlanView& pv, int64_t ga) {
-  unsigned cnt = 0;
-  const int lane = threadIdx.x & 31;
-  const int32_t* colL = lane_base(pv.col, lane);
-  int t = t0;
-  int32_t ka[kB], kb[kB];
-  if (t + kB <= t1) load_batch<kB>(c, colL, t, ka);
-  for (; t + 2 * kB <= t1; t += 2 * kB) {  // two batches per trip: the buffers swap roles
-    load_batch<kB>(c, colL, t + kB, kb);
-    cnt += probe_batch<kLinear, kHuge, kB>(c, t, ka, lane, pv, ga);
-    if (t + 3 * kB <= t1) load_batch<kB>(c, colL, t + 2 * kB, ka);
-    cnt += probe_batch<kLinear, kHuge, kB>(c, t + kB, kb, lane, pv, ga);
-  }
-  if (t + kB <= t1) {  // one loaded batch left
-    cnt += probe_batch<kLinear, kHuge, kB>(c, t, ka, lane, pv, ga);
-    t += kB;
-  }
-  return cnt + walk_long<kLinear, kHuge, 8>(c, t, t1, pv, ga);  // < kB tiles: its tail loop
-}
-
 // SHORT class: the warp owns the flat keys [k0w, k1w) of the chunk.
 template <bool kLinear, bool kHuge>
 __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0w, int k1w,
@@ -578,14 +509,9 @@ __device__ __forceinline__ unsigned walk_short(const ChunkSmem& c, int S, int k0
   return cnt;
 }
 
-template <bool kLinear, int kB = kBatchLong, bool kPipe = false>
+template <bool kLinear, int kB = kBatchLong>
 __device__ __forceinline__ unsigned consume(const ChunkSmem& c, const SlotHdr& h, int w0, int w1,
                                             const PlanView& pv) {
-  if constexpr (kPipe) {
-    if (h.is_long)
-      return h.huge ? walk_long_pipe<kLinear, true, kB>(c, w0, w1, pv, h.ga)
-                    : walk_long_pipe<kLinear, false, kB>(c, w0, w1, pv, h.ga);
-  }
   if (h.is_long)
     return h.huge ? walk_long<kLinear, true, kB>(c, w0, w1, pv, h.ga)
                   : walk_long<kLinear, false, kB>(c, w0, w1, pv, h.ga);
@@ -1007,7 +933,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
 // kBlock: the launch bound (1024 threads cap a thread at 64 registers, which
 // bounds the key loads in flight to kB = 8 tiles per lane; smaller CTAs buy
 // registers for deeper batches: Tuning::batch, block_threads).
-template <int kBlock, int kB, bool kPipe = false>
+template <int kBlock, int kB>
 __global__ void __launch_bounds__(kBlock, 1)
     k_count(PlanView pv, int64_t c_begin, int64_t c_end, int64_t e_begin, int64_t e_end,
             int64_t slot_bytes, Tuning tu, unsigned long long* __restrict__ out,
@@ -1084,8 +1010,7 @@ __global__ void __launch_bounds__(kBlock, 1)
             w0 = min((w0 + 7) & ~7, NU);
             w1 = cw + 1 == n_cons ? NU : min((w1 + 7) & ~7, NU);
           }
-          acc += h.linear ? consume<true, kB, kPipe>(c, h, w0, w1, pv)
-                          : consume<false, kB, kPipe>(c, h, w0, w1, pv);
+          acc += h.linear ? consume<true, kB>(c, h, w0, w1, pv) : consume<false, kB>(c, h, w0, w1, pv);
         } else {  // dynamic: grab `grab` units at a time from the slot's counter
           for (;;) {
             int w0 = 0;
@@ -1093,8 +1018,7 @@ __global__ void __launch_bounds__(kBlock, 1)
             w0 = __shfl_sync(0xffffffffu, w0, 0);
             if (w0 >= NU) break;
             const int w1 = min(w0 + grab, NU);
-            acc += h.linear ? consume<true, kB, kPipe>(c, h, w0, w1, pv)
-                            : consume<false, kB, kPipe>(c, h, w0, w1, pv);
+            acc += h.linear ? consume<true, kB>(c, h, w0, w1, pv) : consume<false, kB>(c, h, w0, w1, pv);
           }
         }
       }
@@ -1122,14 +1046,11 @@ __global__ void __launch_bounds__(kBlock, 1)
 // The long-class kernel's instances: (launch bound, tiles per batch).
 const void* const kCountKernels[] = {
     (const void*)k_count<1024, 8>, (const void*)k_count<768, 8>, (const void*)k_count<768, 12>,
-    (const void*)k_count<768, 16>, (const void*)k_count<512, 16>, (const void*)k_count<512, 24>,
-    (const void*)k_count<1024, 4, true>, (const void*)k_count<768, 4, true>};
+    (const void*)k_count<768, 16>, (const void*)k_count<512, 16>, (const void*)k_count<512, 24>};
 
-// The instance for a block size and batch (Tuning::batch; 0 = the default 8)
-// and Tuning::pipe: block > 768 or an unknown pair runs the 1024-bound,
-// 8-tile instance.
-const void* count_kernel(int block, int batch, int pipe) {
-  if (pipe) return block <= 768 ? kCountKernels[7] : kCountKernels[6];
+// The instance for a block size and batch (Tuning::batch; 0 = the default 8):
+// block > 768 or an unknown pair runs the 1024-bound, 8-tile instance.
+const void* count_kernel(int block, int batch) {
   if (block <= 512) return batch >= 24 ? kCountKernels[5] : kCountKernels[4];
   if (block <= 768) return batch >= 16 ? kCountKernels[3] : batch >= 12 ? kCountKernels[2] : kCountKernels[1];
   return kCountKernels[0];
@@ -1351,7 +1272,7 @@ int count_occupancy(int block, int64_t smem_bytes, const Tuning& tu) {
   ensure_attr();
   int occ = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-      &occ, count_kernel(block, tu.batch, tu.pipe), block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
+      &occ, count_kernel(block, tu.batch), block, (size_t)(tu.slots * slot_bytes_of(smem_bytes))));
   return occ;
 }
 
@@ -1383,7 +1304,7 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
     const FuseArgs& fa = (fuse && s1 <= s0) ? *fuse : none;  // no later launch follows
     void* args[] = {(void*)&pv, (void*)&l0, (void*)&l1, (void*)&e_begin, (void*)&e_end,
                     (void*)&sb, (void*)&P.tune, (void*)&d_out, (void*)&fa};
-    TC_CUDA(cudaLaunchKernel(count_kernel(P.block, P.tune.batch, P.tune.pipe), dim3(grid), dim3(P.block), args,
+    TC_CUDA(cudaLaunchKernel(count_kernel(P.block, P.tune.batch), dim3(grid), dim3(P.block), args,
                              (size_t)(P.tune.slots * sb), s));
     ++launched;
   }
