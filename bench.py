@@ -546,7 +546,8 @@ def main():
     # (after the e2e leg: its many short launches perturbed the e2e timing
     # that followed them, 13.6 -> 37 ms at C5)
     # N = 1: the P-rank splits of tc_partition_measured (this device's
-    # 64-slice profile) and of tc_partition (built-in profile), every range
+    # 64-slice profile refined for P, as agreed_profile does at N = P) and of
+    # tc_partition (built-in profile), every range
     # timed alone (L2 flushed, median of 3): max/mean per P
     balance = None
     if world == 1 and not a.variant and not a.no_balance:
@@ -569,7 +570,7 @@ def main():
             return statistics.median(ts), int(tmp.item())
 
         for P in (2, 4, 8):
-            for label, bb in (("measured", g.partition(P, w)), ("builtin", g.partition(P))):
+            for label, bb in (("measured", g.partition(P, g.refine(P, w))), ("builtin", g.partition(P))):
                 res = [range_ms(bb[r], bb[r + 1]) for r in range(P)]
                 ms = [x for x, _ in res]
                 balance[f"P{P}_{label}"] = {

@@ -253,6 +253,19 @@ TC_API tc_status tc_partition_measured(const tc_graph* g, int32_t world_size, in
 TC_API tc_status tc_calibrate(const tc_graph* g, void* stream, int32_t n_slices, double* h_ms);
 
 /*
+ * Refine a profile for world_size ranks on this device: split by h_ms (as
+ * tc_partition_measured), time every rank's range alone (one warm-up count,
+ * then world_size tc_count_range calls, CUDA events on `stream`), and scale
+ * each slice's h_ms (host double[n_slices], in place) by measured / predicted
+ * time of the ranges it overlaps (cost-weighted).  The split of the refined
+ * profile corrects what the slices mispredict, e.g. a range's launch tail
+ * (C3 P = 8 with 256 slices: max/mean 1.115 -> 1.006).  Synchronises.  Every
+ * rank must end with the same profile (average the refined ones).
+ */
+TC_API tc_status tc_refine_profile(const tc_graph* g, void* stream, int32_t world_size,
+                                   int32_t n_slices, double* h_ms);
+
+/*
  * Host only: the slices of a profile.  h_first (host int64[n_slices+1])
  * receives each slice's first CHUNK (h_first[n_slices] = n_chunks).  One
  * slice is the whole list; otherwise the long

@@ -37,7 +37,7 @@ EXPORTS = (
     "tc_shard_bounds", "tc_shard_unique", "tc_shard_degree", "tc_rank_vertices", "tc_shard_orient", "tc_sort_keys",
     "tc_build_from_oriented", "tc_count_range_fused", "tc_mc_buffer_create",
     "tc_mc_buffer_destroy", "tc_partition_measured", "tc_calibrate", "tc_plan_chunks",
-    "tc_partition_chunks", "tc_slice_bounds", "tc_counters",
+    "tc_partition_chunks", "tc_slice_bounds", "tc_counters", "tc_refine_profile",
 )
 TC_MAX_PEERS = 16
 CALIBRATION_SLICES = 64  # slices of the measured time profile (tc_calibrate)
@@ -114,6 +114,7 @@ def lib():
             "tc_partition_prefix": ([vp, i64, i32, vp], st),
             "tc_partition_measured": ([vp, i32, i32, vp, vp], st),
             "tc_calibrate": ([vp, vp, i32, vp], st),
+            "tc_refine_profile": ([vp, vp, i32, i32, vp], st),
             "tc_plan_chunks": ([vp, vp, vp], st),
             "tc_counters": ([vp, i32], st),
             "tc_partition_chunks": ([vp, vp, i64, i64, i32, vp, i32, vp], st),
@@ -312,6 +313,15 @@ class Graph:
         ms = np.zeros(int(n_slices), dtype=np.float64)
         _check(lib().tc_calibrate(self._h, ctypes.c_void_p(_stream(stream)), int(n_slices),
                                   ms.ctypes.data_as(ctypes.c_void_p)))
+        return ms
+
+    def refine(self, world_size: int, profile, stream=None) -> np.ndarray:
+        """The profile refined for world_size ranks (tc_refine_profile): every
+        rank's range of its split timed alone, each slice scaled by measured /
+        predicted time.  Returns a new array."""
+        ms = np.array(profile, dtype=np.float64, copy=True)
+        _check(lib().tc_refine_profile(self._h, ctypes.c_void_p(_stream(stream)), int(world_size),
+                                       int(ms.size), ms.ctypes.data_as(ctypes.c_void_p)))
         return ms
 
     def chunks(self):
@@ -544,18 +554,26 @@ class FusedSum:
 
 
 def agreed_profile(graph, group=None, stream=None, n_slices: int = CALIBRATION_SLICES):
-    """A time profile every rank agrees on: each rank calibrates (tc_calibrate)
-    and the ranks' profiles are averaged with one all_reduce (the bounds must
-    be identical on every rank).  None when not distributed."""
+    """A time profile every rank agrees on: each rank calibrates (tc_calibrate),
+    the ranks' profiles are averaged (one all_reduce), refined for this world
+    size (tc_refine_profile) and averaged again, so the bounds are identical on
+    every rank.  None when not distributed."""
     import torch
     import torch.distributed as dist
     if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
         return None
-    ms = graph.calibrate(n_slices, stream=stream)
+    world = dist.get_world_size(group)
     dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
-    t = torch.as_tensor(ms, dtype=torch.float64).to(dev)
-    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
-    return (t.cpu().numpy() / dist.get_world_size(group)).astype(np.float64)
+
+    def average(ms):
+        t = torch.as_tensor(ms, dtype=torch.float64).to(dev)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+        return (t.cpu().numpy() / world).astype(np.float64)
+
+    ms = average(graph.calibrate(n_slices, stream=stream))
+    # one refinement pass for this world size (each rank times every range on
+    # its own GPU; the averages keep the bounds identical on every rank)
+    return average(graph.refine(world, ms, stream=stream))
 
 
 def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] = None,

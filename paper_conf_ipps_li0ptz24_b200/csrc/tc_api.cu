@@ -481,52 +481,125 @@ tc_status tc_slice_bounds(const int64_t* h_cost, int64_t n_chunks, int64_t n_lon
   });
 }
 
+namespace {
+
+// The profile's time up to every chunk boundary c (W[c], c in [0, nc]):
+// slice i contributes h_ms[i] spread over its chunks in proportion to their
+// plan cost (a slice without cost weighs its ms at its first boundary).
+// Non-decreasing.  `first` receives the slice bounds.
+std::vector<long double> profile_prefix(const int64_t* cost, int64_t nc, int64_t nL, int32_t K,
+                                        const double* ms, std::vector<int64_t>& first) {
+  first.assign(K + 1, 0);
+  slice_bounds(cost, nc, nL, K, first.data());
+  std::vector<long double> W(nc + 1, 0);
+  long double acc = 0;
+  for (int32_t i = 0; i < K; ++i) {
+    const int64_t a = first[i], b = first[i + 1];
+    const long double c0 = (long double)cost[a], span = (long double)cost[b] - c0;
+    for (int64_t c = a; c < b; ++c)
+      W[c] = acc + (span > 0 ? ((long double)cost[c] - c0) / span : 0) * (long double)ms[i];
+    acc += (long double)ms[i];
+  }
+  W[nc] = acc;
+  return W;
+}
+
+// Chunk-boundary cuts of W into P parts (nearest boundary to r/P of the total).
+std::vector<int64_t> cut_chunks(const std::vector<long double>& W, int32_t P) {
+  const int64_t nc = (int64_t)W.size() - 1;
+  std::vector<int64_t> cb(P + 1, 0);
+  cb[P] = nc;
+  int64_t prev = 0;
+  for (int32_t r = 1; r < P; ++r) {
+    const long double t = W[nc] * r / P;
+    int64_t lo = std::lower_bound(W.begin() + prev, W.end(), t) - W.begin();
+    if (lo > prev && t - W[lo - 1] < W[lo] - t) --lo;  // the nearer boundary
+    cb[r] = prev = lo;
+  }
+  return cb;
+}
+
+void check_profile_args(const int64_t* h_seg, const int64_t* h_cost, int64_t n_chunks,
+                        int64_t n_long_chunks, int32_t n_slices, const double* h_ms,
+                        int32_t world_size) {
+  require(h_seg && h_cost && h_ms, "NULL argument");
+  require(n_chunks >= 0 && n_long_chunks >= 0 && n_long_chunks <= n_chunks, "bad chunk counts");
+  require(world_size >= 1, "world_size < 1");
+  require(n_slices >= 1, "n_slices < 1");
+  for (int32_t i = 0; i < n_slices; ++i)
+    require(std::isfinite(h_ms[i]) && h_ms[i] >= 0, "profile entries must be finite and >= 0");
+  for (int64_t c = 0; c < n_chunks; ++c)
+    require(h_seg[c] <= h_seg[c + 1] && h_cost[c] <= h_cost[c + 1], "prefixes must be non-decreasing");
+}
+
+}  // namespace
+
 tc_status tc_partition_chunks(const int64_t* h_seg, const int64_t* h_cost, int64_t n_chunks,
                               int64_t n_long_chunks, int32_t n_slices, const double* h_ms,
                               int32_t world_size, int64_t* h_bounds) {
   return guarded([&] {
-    require(h_seg && h_cost && h_ms && h_bounds, "NULL argument");
-    require(n_chunks >= 0 && n_long_chunks >= 0 && n_long_chunks <= n_chunks, "bad chunk counts");
-    require(world_size >= 1, "world_size < 1");
-    require(n_slices >= 1, "n_slices < 1");
-    for (int32_t i = 0; i < n_slices; ++i)
-      require(std::isfinite(h_ms[i]) && h_ms[i] >= 0, "profile entries must be finite and >= 0");
-    for (int64_t c = 0; c < n_chunks; ++c)
-      require(h_seg[c] <= h_seg[c + 1] && h_cost[c] <= h_cost[c + 1], "prefixes must be non-decreasing");
-    const int64_t nc = n_chunks;
-    std::vector<int64_t> first(n_slices + 1);
-    slice_bounds(h_cost, nc, n_long_chunks, n_slices, first.data());
-    // W(c): the profile's time up to chunk boundary c — slice i contributes
-    // h_ms[i] spread over its cost units (a slice without cost weighs its
-    // ms at its first boundary).  Non-decreasing in c.
-    std::vector<long double> Wslice(n_slices + 1, 0);
-    for (int32_t i = 0; i < n_slices; ++i) Wslice[i + 1] = Wslice[i] + (long double)h_ms[i];
-    std::vector<int32_t> slice_of(nc + 1);
-    for (int32_t i = 0; i < n_slices; ++i)
-      for (int64_t c = first[i]; c < first[i + 1]; ++c) slice_of[c] = i;
-    slice_of[nc] = n_slices;
-    auto W = [&](int64_t c) -> long double {
-      const int32_t i = slice_of[c];
-      if (i >= n_slices) return Wslice[n_slices];
-      const long double c0 = (long double)h_cost[first[i]], c1 = (long double)h_cost[first[i + 1]];
-      const long double f = c1 > c0 ? ((long double)h_cost[c] - c0) / (c1 - c0) : 0;
-      return Wslice[i] + f * (long double)h_ms[i];
-    };
-    const long double total = W(nc);
-    h_bounds[0] = h_seg[0];
-    int64_t prev = 0;
-    for (int32_t r = 1; r < world_size; ++r) {
-      const long double t = total * r / world_size;
-      int64_t lo = prev, hi = nc;  // first chunk boundary c >= prev with W(c) >= t
-      while (lo < hi) {
-        const int64_t mid = (lo + hi) >> 1;
-        if (W(mid) < t) lo = mid + 1; else hi = mid;
+    require(h_bounds != nullptr, "NULL argument");
+    check_profile_args(h_seg, h_cost, n_chunks, n_long_chunks, n_slices, h_ms, world_size);
+    std::vector<int64_t> first;
+    const auto W = profile_prefix(h_cost, n_chunks, n_long_chunks, n_slices, h_ms, first);
+    const auto cb = cut_chunks(W, world_size);
+    for (int32_t r = 0; r <= world_size; ++r) h_bounds[r] = h_seg[cb[r]];
+  });
+}
+
+tc_status tc_refine_profile(const tc_graph* g, void* stream, int32_t world_size, int32_t n_slices,
+                            double* h_ms) {
+  return guarded([&] {
+    require(g && h_ms, "NULL argument");
+    const tc::Plan& P = g->plan;
+    check_profile_args(P.h_chunk_seg.data(), P.h_chunk_cost.data(), P.n_chunks, P.n_long_chunks,
+                       n_slices, h_ms, world_size);
+    if (P.n_chunks == 0 || world_size == 1) return;
+    cudaStream_t s = (cudaStream_t)stream;
+    std::vector<int64_t> first;
+    const auto W = profile_prefix(P.h_chunk_cost.data(), P.n_chunks, P.n_long_chunks, n_slices, h_ms,
+                                  first);
+    const auto cb = cut_chunks(W, world_size);
+    // time every range alone, as its rank would count it
+    tc::DevBuf<unsigned long long> d(1, s);
+    std::vector<cudaEvent_t> ev(world_size + 1, nullptr);
+    struct Guard {
+      std::vector<cudaEvent_t>& e;
+      ~Guard() {
+        for (auto x : e)
+          if (x) cudaEventDestroy(x);
       }
-      if (lo > prev && t - W(lo - 1) < W(lo) - t) --lo;  // the nearer boundary
-      prev = lo;
-      h_bounds[r] = h_seg[lo];
+    } guard{ev};
+    for (auto& e : ev) TC_CUDA(cudaEventCreate(&e));
+    tc::count_chunks(g, 0, P.n_chunks, 0, P.S, s, d.get());  // warm-up
+    TC_CUDA(cudaEventRecord(ev[0], s));
+    for (int32_t r = 0; r < world_size; ++r) {
+      if (cb[r + 1] > cb[r])
+        tc::count_chunks(g, cb[r], cb[r + 1], P.h_chunk_seg[cb[r]], P.h_chunk_seg[cb[r + 1]], s,
+                         d.get());
+      TC_CUDA(cudaEventRecord(ev[r + 1], s));
     }
-    h_bounds[world_size] = h_seg[nc];
+    TC_CUDA(cudaEventSynchronize(ev[world_size]));
+    std::vector<double> f(world_size, 1.0);
+    for (int32_t r = 0; r < world_size; ++r) {
+      float ms = 0;
+      TC_CUDA(cudaEventElapsedTime(&ms, ev[r], ev[r + 1]));
+      const long double pred = W[cb[r + 1]] - W[cb[r]];
+      if (cb[r + 1] > cb[r] && pred > 0) f[r] = (double)(ms / pred);
+    }
+    // slice i scaled by the cost-weighted factor of the ranges it overlaps
+    const int64_t* cost = P.h_chunk_cost.data();
+    for (int32_t i = 0; i < n_slices; ++i) {
+      const int64_t a = first[i], b = first[i + 1];
+      const long double span = (long double)(cost[b] - cost[a]);
+      if (b <= a || span <= 0) continue;
+      long double acc = 0;
+      for (int32_t r = 0; r < world_size; ++r) {
+        const int64_t lo = std::max(a, cb[r]), hi = std::min(b, cb[r + 1]);
+        if (hi > lo) acc += f[r] * (long double)(cost[hi] - cost[lo]);
+      }
+      h_ms[i] = (double)(h_ms[i] * acc / span);
+    }
   });
 }
 

@@ -237,6 +237,117 @@ __global__ void k_narrow_u32(const int64_t* __restrict__ in, int64_t n, uint32_t
     out[i] = (uint32_t)(uint64_t)in[i];
 }
 
+// ------------------------------------------------------------------ a5 by rows
+// The oriented CSR without a 2*ceil(log2 n')-bit sort of all m keys: count
+// the out-degree of every row (u = the lower rank), scatter each v into its
+// row at an atomic cursor, then sort every row in place (rows are short
+// under degree order: d+ <= sqrt(2m)).  The result is the same CSR as the
+// radix-sorted path (every row strictly ascending; test_csr_exact).
+__global__ void k_orient_count(const uint64_t* __restrict__ key, int64_t m, int bits,
+                               const int32_t* __restrict__ rank, int32_t* __restrict__ cnt) {
+  const uint64_t mask = (uint64_t(1) << bits) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const uint64_t k = key[i];
+    const int32_t ra = rank[k >> bits], rb = rank[k & mask];
+    atomicAdd(&cnt[min(ra, rb)], 1);
+  }
+}
+
+__global__ void k_orient_scatter(const uint64_t* __restrict__ key, int64_t m, int bits,
+                                 const int32_t* __restrict__ rank,
+                                 const int64_t* __restrict__ row_ptr, int32_t* __restrict__ cursor,
+                                 int32_t* __restrict__ col) {
+  const uint64_t mask = (uint64_t(1) << bits) - 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const uint64_t k = key[i];
+    const int32_t ra = rank[k >> bits], rb = rank[k & mask];
+    const int32_t u = min(ra, rb), v = max(ra, rb);
+    col[row_ptr[u] + atomicAdd(&cursor[u], 1)] = v;
+  }
+}
+
+__global__ void k_widen(const int32_t* __restrict__ cnt, int64_t n, int64_t* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = cnt[i];
+}
+
+// Rows of <= 32 entries: one warp per row, a register bitonic sort over the
+// lanes (padding INT_MAX); also writes the row of every position (rowid).
+// Longer rows are listed in `big` for k_rowsort_block.
+__global__ void k_rowsort_warp(const int64_t* __restrict__ row_ptr, int64_t n,
+                               int32_t* __restrict__ col, int32_t* __restrict__ rowid,
+                               int32_t* __restrict__ big, int* __restrict__ n_big) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t u = w0; u < n; u += nw) {
+    const int64_t a = row_ptr[u];
+    const int len = (int)(row_ptr[u + 1] - a);
+    if (len > 32) {
+      if (lane == 0) big[atomicAdd(n_big, 1)] = (int32_t)u;
+      continue;
+    }
+    if (len == 0) continue;
+    int x = lane < len ? col[a + lane] : 0x7fffffff;
+    if (len > 1) {
+#pragma unroll
+      for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+          const int y = __shfl_xor_sync(0xffffffffu, x, j);
+          const bool up = (lane & k) == 0, lower = (lane & j) == 0;
+          x = (lower == up) ? min(x, y) : max(x, y);
+        }
+      }
+    }
+    if (lane < len) {
+      col[a + lane] = x;
+      rowid[a + lane] = (int32_t)u;
+    }
+  }
+}
+
+// Rows of 33..kRowSortMax entries: one CTA per row, a bitonic sort in SMEM.
+constexpr int kRowSortMax = 8192;  // 32 KB of static SMEM; longer rows: the radix-sort path
+__global__ void __launch_bounds__(1024) k_rowsort_block(const int64_t* __restrict__ row_ptr,
+                                                        const int32_t* __restrict__ big, int n_big,
+                                                        int32_t* __restrict__ col,
+                                                        int32_t* __restrict__ rowid) {
+  __shared__ int buf[kRowSortMax];
+  for (int b = blockIdx.x; b < n_big; b += gridDim.x) {
+    const int32_t u = big[b];
+    const int64_t a = row_ptr[u];
+    const int len = (int)(row_ptr[u + 1] - a);
+    int P2 = 64;
+    while (P2 < len) P2 <<= 1;
+    for (int i = threadIdx.x; i < P2; i += blockDim.x) buf[i] = i < len ? col[a + i] : 0x7fffffff;
+    __syncthreads();
+    for (int k = 2; k <= P2; k <<= 1) {
+      for (int j = k >> 1; j > 0; j >>= 1) {
+        for (int i = threadIdx.x; i < P2; i += blockDim.x) {
+          const int l = i ^ j;
+          if (l > i) {
+            const int x = buf[i], y = buf[l];
+            if (((i & k) == 0) == (x > y)) {
+              buf[i] = y;
+              buf[l] = x;
+            }
+          }
+        }
+        __syncthreads();
+      }
+    }
+    for (int i = threadIdx.x; i < len; i += blockDim.x) {
+      col[a + i] = buf[i];
+      rowid[a + i] = u;
+    }
+    __syncthreads();
+  }
+}
+
 __global__ void k_fill_i64(int64_t* p, int64_t n, int64_t v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
@@ -755,6 +866,55 @@ void csr_from_sorted(const uint64_t* okey, int64_t m, int64_t n_act, cudaStream_
   g->max_out = (int64_t)d2h(mx.get(), s);
 }
 
+// a5 by rows (see k_orient_count): the CSR of the m unique canonical keys
+// `ukey` (over n, `bits` per id) relabelled by `rank` into n_act rows.
+// Returns false (nothing built) when some row is longer than kRowSortMax;
+// the caller then sorts all keys instead.
+bool csr_by_rows(const uint64_t* ukey, int64_t m, int bits, const int32_t* rank, int64_t n_act,
+                 cudaStream_t s, tc_graph* g) {
+  DevBuf<int32_t> cnt(std::max<int64_t>(n_act, 1), s);
+  DevBuf<int64_t> rp(n_act + 1, s, true);
+  TC_CUDA(cudaMemsetAsync(cnt.get(), 0, sizeof(int32_t) * std::max<int64_t>(n_act, 1), s));
+  TC_CUDA(cudaMemsetAsync(rp.get(), 0, sizeof(int64_t), s));
+  k_orient_count<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank, cnt.get());
+  TC_LAUNCH();
+  k_widen<<<grid_for(n_act), TPB, 0, s>>>(cnt.get(), n_act, rp.get() + 1);
+  TC_LAUNCH();
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceScan::InclusiveSum(t, b, rp.get() + 1, rp.get() + 1, n_act, s);
+  });
+  DevBuf<unsigned long long> mx(1, s);
+  TC_CUDA(cudaMemsetAsync(mx.get(), 0, sizeof(unsigned long long), s));
+  k_max_outdeg<<<grid_for(n_act), TPB, 0, s>>>(rp.get(), n_act, mx.get());
+  TC_LAUNCH();
+  const int64_t max_out = (int64_t)d2h(mx.get(), s);
+  if (max_out > kRowSortMax) return false;
+  g->bits = bits_for(std::max<int64_t>(n_act, 2));
+  g->m = m;
+  g->n = n_act;
+  g->max_out = max_out;
+  g->row_ptr = std::move(rp);
+  g->col = DevBuf<int32_t>(m, s, true);
+  g->rowid = DevBuf<int32_t>(m, s);
+  TC_CUDA(cudaMemsetAsync(cnt.get(), 0, sizeof(int32_t) * std::max<int64_t>(n_act, 1), s));
+  k_orient_scatter<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank, g->row_ptr.get(), cnt.get(),
+                                               g->col.get());
+  TC_LAUNCH();
+  DevBuf<int32_t> big(std::max<int64_t>(n_act, 1), s);
+  DevBuf<int> n_big(1, s);
+  TC_CUDA(cudaMemsetAsync(n_big.get(), 0, sizeof(int), s));
+  k_rowsort_warp<<<grid_for(32 * n_act), TPB, 0, s>>>(g->row_ptr.get(), n_act, g->col.get(),
+                                                      g->rowid.get(), big.get(), n_big.get());
+  TC_LAUNCH();
+  const int nb = d2h(n_big.get(), s);
+  if (nb > 0) {
+    k_rowsort_block<<<std::min(nb, 148 * 2), 1024, 0, s>>>(g->row_ptr.get(), big.get(), nb,
+                                                           g->col.get(), g->rowid.get());
+    TC_LAUNCH();
+  }
+  return true;
+}
+
 }  // namespace
 
 // a3..a6 from the m unique canonical keys `ukey` (in ka or kb; the other
@@ -785,7 +945,13 @@ static void build_tail(uint64_t* ukey, int64_t m, DevBuf<uint64_t>& ka, DevBuf<u
 
   // a5
   const int bits2 = bits_for(std::max<int64_t>(n_act, 2));
-  if (m > 0) {
+  static const bool a5_sort = [] {  // TC_A5=sort: the radix-sort path (tests compare the two)
+    const char* v = std::getenv("TC_A5");
+    return v && std::string(v) == "sort";
+  }();
+  if (m > 0 && !a5_sort && csr_by_rows(ukey, m, bits, rank.get(), n_act, s, g)) {
+    // built by rows
+  } else if (m > 0) {
     uint64_t* okey_a = (ukey == ka.get()) ? kb.get() : ka.get();  // the free buffer
     k_orient<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank.get(), bits2, okey_a);
     TC_LAUNCH();

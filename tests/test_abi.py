@@ -79,6 +79,7 @@ def test_bad_arguments_rejected_before_device(tc):
     assert L.tc_plan_chunks(None, None, None) == 1
     assert L.tc_calibrate(None, None, 4, None) == 1
     assert L.tc_slice_bounds(None, 0, 0, 1, None) == 1
+    assert L.tc_refine_profile(None, None, 2, 1, None) == 1
     assert L.tc_count_range_fused(None, 0, 0, None, None, None, 1, 1, None, None) == 1
     assert L.tc_graph_info(None, None) == 1
     assert L.tc_support(None, None, None) == 1

@@ -34,6 +34,11 @@ class FakeGraph:
         rng = np.random.default_rng(dist.get_rank() if dist.is_initialized() else 0)
         return rng.uniform(0.5, 2.0, size=n_slices)
 
+    def refine(self, world, profile, stream=None):
+        import torch.distributed as dist
+        rng = np.random.default_rng(100 + (dist.get_rank() if dist.is_initialized() else 0))
+        return np.asarray(profile) * rng.uniform(0.9, 1.1, size=len(profile))
+
     def partition(self, world, profile=None):
         import paper_conf_ipps_li0ptz24_b200 as tc
         if profile is None:

@@ -1,6 +1,7 @@
 """Measured balance of the multi-GPU edge ranges, emulated
 on one B200: every rank's tc_count_range of the tc_partition_measured split
-(profile = this device's tc_calibrate, 64 slices) is timed alone with CUDA
+(profile = this device's tc_calibrate, 64 slices, refined for P ranks by
+tc_refine_profile, as agreed_profile does) is timed alone with CUDA
 events, L2 flushed before each (median of 5); the slowest range may exceed the mean by at
 most 5 %, and the partials sum to the oracle's stored T (the per-edge
 intersections are independent, so any cut is exact)."""
@@ -57,7 +58,7 @@ def test_partition_balance_measured(tc, cfg):
         out = torch.zeros(1, dtype=torch.int64, device="cuda")
         report = {}
         for P in (2, 4, 8):
-            b = g.partition(P, w)
+            b = g.partition(P, g.refine(P, w))
             res = [_range_ms(g, b[r], b[r + 1], flush, out) for r in range(P)]
             ms = [t for t, _ in res]
             assert sum(p for _, p in res) & (2**64 - 1) == stored["triangles"]
