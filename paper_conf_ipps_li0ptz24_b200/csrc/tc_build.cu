@@ -275,42 +275,75 @@ __global__ void k_widen(const int32_t* __restrict__ cnt, int64_t n, int64_t* __r
 }
 
 // Rows of <= 32 entries: one warp per row, a register bitonic sort over the
-// lanes (padding INT_MAX); also writes the row of every position (rowid).
-// Longer rows are listed in `big` for k_rowsort_block.
-__global__ void k_rowsort_warp(const int64_t* __restrict__ row_ptr, int64_t n,
-                               int32_t* __restrict__ col, int32_t* __restrict__ rowid,
-                               int32_t* __restrict__ big, int* __restrict__ n_big) {
+// lanes (padding INT_MAX); rows of 33..kRowWarpMax entries: one warp per row,
+// a bitonic sort in the warp's own shared-memory buffer (__syncwarp between
+// stages).  Also writes the row of every position (rowid).  Longer rows are
+// listed in `big` for k_rowsort_block.
+constexpr int kRowWarpMax = 1024;
+constexpr int kRowSortThreads = 256;
+__global__ void __launch_bounds__(kRowSortThreads) k_rowsort_warp(
+    const int64_t* __restrict__ row_ptr, int64_t n, int32_t* __restrict__ col,
+    int32_t* __restrict__ rowid, int32_t* __restrict__ big, int* __restrict__ n_big) {
+  __shared__ int sbuf[kRowSortThreads / 32][kRowWarpMax];
   const int lane = threadIdx.x & 31;
+  int* buf = sbuf[threadIdx.x >> 5];
   const int64_t w0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t u = w0; u < n; u += nw) {
     const int64_t a = row_ptr[u];
     const int len = (int)(row_ptr[u + 1] - a);
-    if (len > 32) {
+    if (len == 0) continue;
+    if (len > kRowWarpMax) {
       if (lane == 0) big[atomicAdd(n_big, 1)] = (int32_t)u;
       continue;
     }
-    if (len == 0) continue;
-    int x = lane < len ? col[a + lane] : 0x7fffffff;
-    if (len > 1) {
+    if (len <= 32) {
+      int x = lane < len ? col[a + lane] : 0x7fffffff;
+      if (len > 1) {
 #pragma unroll
-      for (int k = 2; k <= 32; k <<= 1) {
+        for (int k = 2; k <= 32; k <<= 1) {
 #pragma unroll
-        for (int j = k >> 1; j > 0; j >>= 1) {
-          const int y = __shfl_xor_sync(0xffffffffu, x, j);
-          const bool up = (lane & k) == 0, lower = (lane & j) == 0;
-          x = (lower == up) ? min(x, y) : max(x, y);
+          for (int j = k >> 1; j > 0; j >>= 1) {
+            const int y = __shfl_xor_sync(0xffffffffu, x, j);
+            const bool up = (lane & k) == 0, lower = (lane & j) == 0;
+            x = (lower == up) ? min(x, y) : max(x, y);
+          }
         }
       }
+      if (lane < len) {
+        col[a + lane] = x;
+        rowid[a + lane] = (int32_t)u;
+      }
+      continue;
     }
-    if (lane < len) {
-      col[a + lane] = x;
-      rowid[a + lane] = (int32_t)u;
+    int P2 = 64;
+    while (P2 < len) P2 <<= 1;
+    for (int i = lane; i < P2; i += 32) buf[i] = i < len ? col[a + i] : 0x7fffffff;
+    __syncwarp();
+    for (int k = 2; k <= P2; k <<= 1) {
+      for (int j = k >> 1; j > 0; j >>= 1) {
+        for (int i = lane; i < P2; i += 32) {
+          const int l = i ^ j;
+          if (l > i) {
+            const int x = buf[i], y = buf[l];
+            if (((i & k) == 0) == (x > y)) {
+              buf[i] = y;
+              buf[l] = x;
+            }
+          }
+        }
+        __syncwarp();
+      }
     }
+    for (int i = lane; i < len; i += 32) {
+      col[a + i] = buf[i];
+      rowid[a + i] = (int32_t)u;
+    }
+    __syncwarp();
   }
 }
 
-// Rows of 33..kRowSortMax entries: one CTA per row, a bitonic sort in SMEM.
+// Rows of kRowWarpMax+1..kRowSortMax entries: one CTA per row, a bitonic sort in SMEM.
 constexpr int kRowSortMax = 8192;  // 32 KB of static SMEM; longer rows: the radix-sort path
 __global__ void __launch_bounds__(1024) k_rowsort_block(const int64_t* __restrict__ row_ptr,
                                                         const int32_t* __restrict__ big, int n_big,
@@ -903,8 +936,12 @@ bool csr_by_rows(const uint64_t* ukey, int64_t m, int bits, const int32_t* rank,
   DevBuf<int32_t> big(std::max<int64_t>(n_act, 1), s);
   DevBuf<int> n_big(1, s);
   TC_CUDA(cudaMemsetAsync(n_big.get(), 0, sizeof(int), s));
-  k_rowsort_warp<<<grid_for(32 * n_act), TPB, 0, s>>>(g->row_ptr.get(), n_act, g->col.get(),
-                                                      g->rowid.get(), big.get(), n_big.get());
+  {
+    const int64_t blocks = (32 * n_act + kRowSortThreads - 1) / kRowSortThreads;
+    k_rowsort_warp<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16)),
+                     kRowSortThreads, 0, s>>>(g->row_ptr.get(), n_act, g->col.get(),
+                                              g->rowid.get(), big.get(), n_big.get());
+  }
   TC_LAUNCH();
   const int nb = d2h(n_big.get(), s);
   if (nb > 0) {

@@ -460,3 +460,28 @@ def test_table_cap_fallbacks(tc, n, opts):
     the count is unchanged (K_n: C(n, 3), > 2^32 at n = 3000)."""
     (src, dst, nn), t = graphs.complete(n)
     assert gpu_count(tc, src, dst, nn, options=opts) == t
+
+
+def test_more_than_2_31_edges(tc):
+    """m in [2^31, 2^32): every col index of the plan and the count kernel's
+    32-bit tile descriptors passes 2^31 (the guard only rejects m >= 2^32).
+    A disjoint union of c copies of K_64 with m = c * C(64, 2) > 2^31 unique
+    edges, generated on the device; T = c * C(64, 3) in closed form (C-16)."""
+    free, _ = torch.cuda.mem_get_info()
+    if free < (170 << 30):
+        pytest.skip(f"needs ~170 GB of device memory, {free >> 30} GB free")
+    k = 64
+    iu = torch.triu_indices(k, k, offset=1, device="cuda").to(torch.int32)  # C(64, 2) pairs
+    c = (2**31) // iu.shape[1] + 4096
+    m = c * iu.shape[1]
+    assert 2**31 < m < 2**32
+    off = (torch.arange(c, device="cuda", dtype=torch.int32) * k)[:, None]
+    src = (off + iu[0][None, :]).reshape(-1)
+    dst = (off + iu[1][None, :]).reshape(-1)
+    del off
+    with tc.build_csr(src, dst, c * k) as g:
+        del src, dst
+        assert g.m == m and g.n == c * k and g.info.max_out_degree == k - 1
+        assert g.count() == c * comb(k, 3)
+        b = g.partition(3)
+        assert sum(int(g.count_range(b[r], b[r + 1]).item()) for r in range(3)) == c * comb(k, 3)
