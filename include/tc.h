@@ -482,6 +482,14 @@ TC_API void tc_free(tc_graph* g);
  */
 TC_API tc_status tc_counters(uint64_t* h_counters, int32_t reset);
 
+/*
+ * Return the device memory the library keeps cached for reuse (its
+ * stream-ordered pools keep freed blocks mapped so repeated builds do not
+ * re-map memory) to the driver, for the current device.  Live graphs are
+ * untouched.  Synchronises the device.
+ */
+TC_API tc_status tc_release_memory(void);
+
 /* Thread-local text for the last non-OK status of this thread. */
 TC_API const char* tc_last_error(void);
 

@@ -38,6 +38,7 @@ EXPORTS = (
     "tc_build_from_oriented", "tc_count_range_fused", "tc_mc_buffer_create",
     "tc_mc_buffer_destroy", "tc_partition_measured", "tc_calibrate", "tc_plan_chunks",
     "tc_partition_chunks", "tc_slice_bounds", "tc_counters", "tc_refine_profile",
+    "tc_release_memory",
 )
 TC_MAX_PEERS = 16
 CALIBRATION_SLICES = 64  # slices of the measured time profile (tc_calibrate)
@@ -117,6 +118,7 @@ def lib():
             "tc_refine_profile": ([vp, vp, i32, i32, vp], st),
             "tc_plan_chunks": ([vp, vp, vp], st),
             "tc_counters": ([vp, i32], st),
+            "tc_release_memory": ([], st),
             "tc_partition_chunks": ([vp, vp, i64, i64, i32, vp, i32, vp], st),
             "tc_slice_bounds": ([vp, i64, i64, i32, vp], st),
             "tc_support": ([vp, vp, vp], st),
@@ -405,6 +407,11 @@ def partition_prefix(prefix: Sequence[int], world_size: int) -> list:
     return [int(x) for x in b]
 
 
+def release_memory():
+    """Give the library's cached device memory back to the driver (tc_release_memory)."""
+    _check(lib().tc_release_memory())
+
+
 def counters(reset: bool = False) -> dict:
     """Diagnostic counters of the count kernels on the current device (tc_counters)."""
     h = (ctypes.c_uint64 * 4)()
@@ -615,5 +622,5 @@ def count_partitioned(graph, group=None, stream=None, fused: Optional[FusedSum] 
 from .sharded import build_csr_sharded, shard_cuts  # noqa: E402  (f2)
 
 __all__ = ["FusedSum", "build_csr_sharded", "shard_cuts", "Graph", "Options", "GraphInfo", "build_csr", "build_csr_host", "count_partitioned",
-           "partition_prefix", "partition_chunks", "slice_bounds", "counters", "agreed_profile", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
+           "partition_prefix", "partition_chunks", "slice_bounds", "counters", "release_memory", "agreed_profile", "version", "lib", "TCError", "InvalidArgument", "OutOfMemory",
            "EXPORTS", "LIB_PATH"]

@@ -142,6 +142,16 @@ void reserve_pool(size_t bytes, cudaStream_t s) {
   cudaGetLastError();
 }
 
+// Give the pools' cached (freed but still mapped) memory of the current
+// device back to the driver: tc_release_memory.
+void trim_pools() {
+  TC_CUDA(cudaDeviceSynchronize());
+  for (bool persistent : {false, true}) {
+    cudaMemPool_t pool = pool_of(persistent);
+    if (pool) TC_CUDA(cudaMemPoolTrimTo(pool, 0));
+  }
+}
+
 void dev_free(void* p, size_t bytes, cudaStream_t s) {
   if (!p) return;
   if (g_free) {
@@ -824,6 +834,10 @@ tc_status tc_counters(uint64_t* h_counters, int32_t reset) {
     require(h_counters != nullptr, "NULL argument");
     tc::read_counters(h_counters, reset != 0);
   });
+}
+
+tc_status tc_release_memory(void) {
+  return guarded([&] { tc::trim_pools(); });
 }
 
 const char* tc_last_error(void) { return t_last_error.c_str(); }

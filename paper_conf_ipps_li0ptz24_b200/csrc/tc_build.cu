@@ -231,155 +231,6 @@ __global__ void k_csr(const uint64_t* __restrict__ okey, int64_t m, int64_t n, i
   }
 }
 
-__global__ void k_narrow_u32(const int64_t* __restrict__ in, int64_t n, uint32_t* __restrict__ out) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
-       i += (int64_t)gridDim.x * blockDim.x)
-    out[i] = (uint32_t)(uint64_t)in[i];
-}
-
-// ------------------------------------------------------------------ a5 by rows
-// The oriented CSR without a 2*ceil(log2 n')-bit sort of all m keys: count
-// the out-degree of every row (u = the lower rank), scatter each v into its
-// row at an atomic cursor, then sort every row in place (rows are short
-// under degree order: d+ <= sqrt(2m)).  The result is the same CSR as the
-// radix-sorted path (every row strictly ascending; test_csr_exact).
-__global__ void k_orient_count(const uint64_t* __restrict__ key, int64_t m, int bits,
-                               const int32_t* __restrict__ rank, int32_t* __restrict__ cnt) {
-  const uint64_t mask = (uint64_t(1) << bits) - 1;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    const uint64_t k = key[i];
-    const int32_t ra = rank[k >> bits], rb = rank[k & mask];
-    atomicAdd(&cnt[min(ra, rb)], 1);
-  }
-}
-
-__global__ void k_orient_scatter(const uint64_t* __restrict__ key, int64_t m, int bits,
-                                 const int32_t* __restrict__ rank,
-                                 const int64_t* __restrict__ row_ptr, int32_t* __restrict__ cursor,
-                                 int32_t* __restrict__ col) {
-  const uint64_t mask = (uint64_t(1) << bits) - 1;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    const uint64_t k = key[i];
-    const int32_t ra = rank[k >> bits], rb = rank[k & mask];
-    const int32_t u = min(ra, rb), v = max(ra, rb);
-    col[row_ptr[u] + atomicAdd(&cursor[u], 1)] = v;
-  }
-}
-
-__global__ void k_widen(const int32_t* __restrict__ cnt, int64_t n, int64_t* __restrict__ out) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
-       i += (int64_t)gridDim.x * blockDim.x)
-    out[i] = cnt[i];
-}
-
-// Rows of <= 32 entries: one warp per row, a register bitonic sort over the
-// lanes (padding INT_MAX); rows of 33..kRowWarpMax entries: one warp per row,
-// a bitonic sort in the warp's own shared-memory buffer (__syncwarp between
-// stages).  Also writes the row of every position (rowid).  Longer rows are
-// listed in `big` for k_rowsort_block.
-constexpr int kRowWarpMax = 1024;
-constexpr int kRowSortThreads = 256;
-__global__ void __launch_bounds__(kRowSortThreads) k_rowsort_warp(
-    const int64_t* __restrict__ row_ptr, int64_t n, int32_t* __restrict__ col,
-    int32_t* __restrict__ rowid, int32_t* __restrict__ big, int* __restrict__ n_big) {
-  __shared__ int sbuf[kRowSortThreads / 32][kRowWarpMax];
-  const int lane = threadIdx.x & 31;
-  int* buf = sbuf[threadIdx.x >> 5];
-  const int64_t w0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t u = w0; u < n; u += nw) {
-    const int64_t a = row_ptr[u];
-    const int len = (int)(row_ptr[u + 1] - a);
-    if (len == 0) continue;
-    if (len > kRowWarpMax) {
-      if (lane == 0) big[atomicAdd(n_big, 1)] = (int32_t)u;
-      continue;
-    }
-    if (len <= 32) {
-      int x = lane < len ? col[a + lane] : 0x7fffffff;
-      if (len > 1) {
-#pragma unroll
-        for (int k = 2; k <= 32; k <<= 1) {
-#pragma unroll
-          for (int j = k >> 1; j > 0; j >>= 1) {
-            const int y = __shfl_xor_sync(0xffffffffu, x, j);
-            const bool up = (lane & k) == 0, lower = (lane & j) == 0;
-            x = (lower == up) ? min(x, y) : max(x, y);
-          }
-        }
-      }
-      if (lane < len) {
-        col[a + lane] = x;
-        rowid[a + lane] = (int32_t)u;
-      }
-      continue;
-    }
-    int P2 = 64;
-    while (P2 < len) P2 <<= 1;
-    for (int i = lane; i < P2; i += 32) buf[i] = i < len ? col[a + i] : 0x7fffffff;
-    __syncwarp();
-    for (int k = 2; k <= P2; k <<= 1) {
-      for (int j = k >> 1; j > 0; j >>= 1) {
-        for (int i = lane; i < P2; i += 32) {
-          const int l = i ^ j;
-          if (l > i) {
-            const int x = buf[i], y = buf[l];
-            if (((i & k) == 0) == (x > y)) {
-              buf[i] = y;
-              buf[l] = x;
-            }
-          }
-        }
-        __syncwarp();
-      }
-    }
-    for (int i = lane; i < len; i += 32) {
-      col[a + i] = buf[i];
-      rowid[a + i] = (int32_t)u;
-    }
-    __syncwarp();
-  }
-}
-
-// Rows of kRowWarpMax+1..kRowSortMax entries: one CTA per row, a bitonic sort in SMEM.
-constexpr int kRowSortMax = 8192;  // 32 KB of static SMEM; longer rows: the radix-sort path
-__global__ void __launch_bounds__(1024) k_rowsort_block(const int64_t* __restrict__ row_ptr,
-                                                        const int32_t* __restrict__ big, int n_big,
-                                                        int32_t* __restrict__ col,
-                                                        int32_t* __restrict__ rowid) {
-  __shared__ int buf[kRowSortMax];
-  for (int b = blockIdx.x; b < n_big; b += gridDim.x) {
-    const int32_t u = big[b];
-    const int64_t a = row_ptr[u];
-    const int len = (int)(row_ptr[u + 1] - a);
-    int P2 = 64;
-    while (P2 < len) P2 <<= 1;
-    for (int i = threadIdx.x; i < P2; i += blockDim.x) buf[i] = i < len ? col[a + i] : 0x7fffffff;
-    __syncthreads();
-    for (int k = 2; k <= P2; k <<= 1) {
-      for (int j = k >> 1; j > 0; j >>= 1) {
-        for (int i = threadIdx.x; i < P2; i += blockDim.x) {
-          const int l = i ^ j;
-          if (l > i) {
-            const int x = buf[i], y = buf[l];
-            if (((i & k) == 0) == (x > y)) {
-              buf[i] = y;
-              buf[l] = x;
-            }
-          }
-        }
-        __syncthreads();
-      }
-    }
-    for (int i = threadIdx.x; i < len; i += blockDim.x) {
-      col[a + i] = buf[i];
-      rowid[a + i] = u;
-    }
-    __syncthreads();
-  }
-}
 
 __global__ void k_fill_i64(int64_t* p, int64_t n, int64_t v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
@@ -446,7 +297,8 @@ __device__ __forceinline__ int64_t upper_bound_i32(const int32_t* __restrict__ a
 __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
                             const int32_t* __restrict__ rowid, const int2* __restrict__ vmm,
                             int64_t m, int long_min, int bits,
-                            uint32_t dead, uint32_t* __restrict__ skey, uint64_t* __restrict__ sval,
+                            uint32_t dead, uint32_t* __restrict__ skey, uint32_t* __restrict__ sidx,
+                            uint64_t* __restrict__ sval,
                             unsigned long long* stats) {
   typedef cub::BlockReduce<unsigned long long, TPB> BR;
   __shared__ typename BR::TempStorage tmp;
@@ -465,6 +317,7 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
     }
     const uint32_t cls = len < long_min ? 1u : 0u;
     skey[p] = len > 0 ? ((cls << bits) | (uint32_t)v) : dead;
+    sidx[p] = (uint32_t)p;  // m < 2^32
     sval[p] = ((uint64_t)lo << 24) | (uint64_t)len;  // len <= d+(u) < 2^24
     keys += (unsigned long long)len;
     nl += len > 0;
@@ -498,7 +351,8 @@ __global__ void k_group_mark(const uint32_t* __restrict__ key, int64_t S,
 
 // Per segment (sorted live edge): start, length, group, work units; per
 // group (at its first segment): row start, d+(v) and its table.
-__global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val,
+__global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint32_t* __restrict__ idx,
+                           const uint64_t* __restrict__ val,
                            const int32_t* __restrict__ gincl, int64_t S, int64_t S_long,
                            int bits, const int64_t* __restrict__ row_ptr,
                            int huge_degree, int table_factor, int bitmap_factor,
@@ -506,18 +360,28 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint64_t* __r
                            const int32_t* __restrict__ col,
                            int32_t* __restrict__ grp_code, uint32_t* __restrict__ seg_start,
                            int32_t* __restrict__ seg_len, int32_t* __restrict__ seg_group,
-                           int64_t* __restrict__ units, int64_t* __restrict__ grp_row,
-                           int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots) {
+                           uint32_t* __restrict__ units, int64_t* __restrict__ grp_row,
+                           int64_t* __restrict__ grp_d, int64_t* __restrict__ grp_slots,
+                           int seg_cost, int64_t* __restrict__ cost,
+                           unsigned long long* __restrict__ units_total) {
+  typedef cub::BlockReduce<unsigned long long, TPB> BR;
+  __shared__ typename BR::TempStorage tmp;
   const uint32_t mask = (uint32_t)((1ull << bits) - 1);
+  unsigned long long usum = 0;
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
        s += (int64_t)gridDim.x * blockDim.x) {
-    const uint64_t x = val[s];
+    const uint64_t x = val[idx[s]];
     const int32_t g = gincl[s] - 1;
     const int32_t len = (int32_t)(x & 0xFFFFFFu);
     seg_group[s] = g;
     seg_start[s] = (uint32_t)(x >> 24);  // < m < 2^32
     seg_len[s] = len;
-    units[s] = s < S_long ? (int64_t)((len + 31) & ~31) : (int64_t)len;
+    const uint32_t u = s < S_long ? (uint32_t)((len + 31) & ~31) : (uint32_t)len;
+    units[s] = u;
+    usum += u;
+    // the segment's plan cost (k_chunk_bounds): seg_cost + its units, plus
+    // its group's d+(v) and table words at the group's first segment
+    int64_t c = seg_cost + (int64_t)u;
     if (s == 0 || key[s] != key[s - 1]) {
       const int64_t v = key[s] & mask;
       const int64_t rs = row_ptr[v], d = row_ptr[v + 1] - rs;
@@ -558,22 +422,14 @@ __global__ void k_seg_fill(const uint32_t* __restrict__ key, const uint64_t* __r
       }
       grp_code[g] = code;
       grp_slots[g] = slots;
+      c += d + slots;
     }
-  }
-}
-
-__global__ void k_seg_cost(const int64_t* __restrict__ units, const int32_t* __restrict__ seg_group,
-                           const int64_t* __restrict__ grp_d,
-                           const int64_t* __restrict__ grp_slots, int64_t S, int seg_cost,
-                           int64_t* __restrict__ cost) {
-  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
-       s += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t g = seg_group[s];
-    int64_t c = seg_cost + units[s];
-    if (s == 0 || seg_group[s - 1] != g) c += grp_d[g] + grp_slots[g];
     cost[s] = c;
   }
+  const unsigned long long r = BR(tmp).Sum(usum);
+  if (threadIdx.x == 0) atomicAdd(units_total, r);
 }
+
 
 __global__ void k_grp_ibase(const int64_t* __restrict__ grp_row,
                             const int64_t* __restrict__ ins_prefix, int64_t G,
@@ -653,22 +509,30 @@ __global__ void k_split(const int64_t* __restrict__ chunk_seg, int64_t n_chunks,
         continue;
       }
     }
-    int64_t p0 = sa, g0 = seg_group[sa], ok_need = 0;
-    for (int64_t s = sa; s < sb; ++s) {
-      const int64_t g = seg_group[s];
-      const int64_t tiles = is_long ? (int64_t)((key_prefix[s + 1] - key_prefix[p0]) >> 5) : 0;
-      int64_t need = chunk_smem_bytes(s + 1 - p0, g - g0 + 1, slot_prefix[g + 1] - slot_prefix[g0], tiles);
-      if (need > limit && s > p0) {  // close the piece [p0, s), start a new one at s
-        if (bounds) bounds[o + cnt] = p0;
-        else atomicMax(nm, (unsigned long long)ok_need);
-        ++cnt;
-        p0 = s;
-        g0 = g;
-        const int64_t t1 = is_long ? (int64_t)((key_prefix[s + 1] - key_prefix[s]) >> 5) : 0;
-        need = chunk_smem_bytes(1, 1, slot_prefix[g + 1] - slot_prefix[g], t1);
+    // outlier: cut it into pieces, each the longest run [p0, e) whose layout
+    // fits `limit` (at least one edge).  The layout size grows with e, so e is
+    // binary-searched (the pieces a walk edge by edge would cut).
+    auto need_of = [&](int64_t a, int64_t e) {
+      const int64_t g0 = seg_group[a], g1 = seg_group[e - 1];
+      const int64_t tiles = is_long ? (int64_t)((key_prefix[e] - key_prefix[a]) >> 5) : 0;
+      return chunk_smem_bytes(e - a, g1 - g0 + 1, slot_prefix[g1 + 1] - slot_prefix[g0], tiles);
+    };
+    int64_t p0 = sa;
+    for (;;) {
+      int64_t lo = p0 + 1, hi = sb;
+      if (need_of(p0, lo) <= limit) {
+        while (lo < hi) {  // largest e in [p0 + 1, sb] with need <= limit
+          const int64_t mid = (lo + hi + 1) >> 1;
+          if (need_of(p0, mid) <= limit) lo = mid; else hi = mid - 1;
+        }
       }
-      ok_need = need;
+      if (lo >= sb) break;  // [p0, sb) is the last piece
+      if (bounds) bounds[o + cnt] = p0;
+      else atomicMax(nm, (unsigned long long)need_of(p0, lo));
+      ++cnt;
+      p0 = lo;
     }
+    const int64_t ok_need = need_of(p0, sb);
     if (bounds) bounds[o + cnt] = p0;
     else {
       atomicMax(nm, (unsigned long long)ok_need);
@@ -899,59 +763,6 @@ void csr_from_sorted(const uint64_t* okey, int64_t m, int64_t n_act, cudaStream_
   g->max_out = (int64_t)d2h(mx.get(), s);
 }
 
-// a5 by rows (see k_orient_count): the CSR of the m unique canonical keys
-// `ukey` (over n, `bits` per id) relabelled by `rank` into n_act rows.
-// Returns false (nothing built) when some row is longer than kRowSortMax;
-// the caller then sorts all keys instead.
-bool csr_by_rows(const uint64_t* ukey, int64_t m, int bits, const int32_t* rank, int64_t n_act,
-                 cudaStream_t s, tc_graph* g) {
-  DevBuf<int32_t> cnt(std::max<int64_t>(n_act, 1), s);
-  DevBuf<int64_t> rp(n_act + 1, s, true);
-  TC_CUDA(cudaMemsetAsync(cnt.get(), 0, sizeof(int32_t) * std::max<int64_t>(n_act, 1), s));
-  TC_CUDA(cudaMemsetAsync(rp.get(), 0, sizeof(int64_t), s));
-  k_orient_count<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank, cnt.get());
-  TC_LAUNCH();
-  k_widen<<<grid_for(n_act), TPB, 0, s>>>(cnt.get(), n_act, rp.get() + 1);
-  TC_LAUNCH();
-  cub_run(s, [&](void* t, size_t& b) {
-    return cub::DeviceScan::InclusiveSum(t, b, rp.get() + 1, rp.get() + 1, n_act, s);
-  });
-  DevBuf<unsigned long long> mx(1, s);
-  TC_CUDA(cudaMemsetAsync(mx.get(), 0, sizeof(unsigned long long), s));
-  k_max_outdeg<<<grid_for(n_act), TPB, 0, s>>>(rp.get(), n_act, mx.get());
-  TC_LAUNCH();
-  const int64_t max_out = (int64_t)d2h(mx.get(), s);
-  if (max_out > kRowSortMax) return false;
-  g->bits = bits_for(std::max<int64_t>(n_act, 2));
-  g->m = m;
-  g->n = n_act;
-  g->max_out = max_out;
-  g->row_ptr = std::move(rp);
-  g->col = DevBuf<int32_t>(m, s, true);
-  g->rowid = DevBuf<int32_t>(m, s);
-  TC_CUDA(cudaMemsetAsync(cnt.get(), 0, sizeof(int32_t) * std::max<int64_t>(n_act, 1), s));
-  k_orient_scatter<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank, g->row_ptr.get(), cnt.get(),
-                                               g->col.get());
-  TC_LAUNCH();
-  DevBuf<int32_t> big(std::max<int64_t>(n_act, 1), s);
-  DevBuf<int> n_big(1, s);
-  TC_CUDA(cudaMemsetAsync(n_big.get(), 0, sizeof(int), s));
-  {
-    const int64_t blocks = (32 * n_act + kRowSortThreads - 1) / kRowSortThreads;
-    k_rowsort_warp<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16)),
-                     kRowSortThreads, 0, s>>>(g->row_ptr.get(), n_act, g->col.get(),
-                                              g->rowid.get(), big.get(), n_big.get());
-  }
-  TC_LAUNCH();
-  const int nb = d2h(n_big.get(), s);
-  if (nb > 0) {
-    k_rowsort_block<<<std::min(nb, 148 * 2), 1024, 0, s>>>(g->row_ptr.get(), big.get(), nb,
-                                                           g->col.get(), g->rowid.get());
-    TC_LAUNCH();
-  }
-  return true;
-}
-
 }  // namespace
 
 // a3..a6 from the m unique canonical keys `ukey` (in ka or kb; the other
@@ -982,13 +793,7 @@ static void build_tail(uint64_t* ukey, int64_t m, DevBuf<uint64_t>& ka, DevBuf<u
 
   // a5
   const int bits2 = bits_for(std::max<int64_t>(n_act, 2));
-  static const bool a5_sort = [] {  // TC_A5=sort: the radix-sort path (tests compare the two)
-    const char* v = std::getenv("TC_A5");
-    return v && std::string(v) == "sort";
-  }();
-  if (m > 0 && !a5_sort && csr_by_rows(ukey, m, bits, rank.get(), n_act, s, g)) {
-    // built by rows
-  } else if (m > 0) {
+  if (m > 0) {
     uint64_t* okey_a = (ukey == ka.get()) ? kb.get() : ka.get();  // the free buffer
     k_orient<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank.get(), bits2, okey_a);
     TC_LAUNCH();
@@ -1319,7 +1124,10 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   DevBuf<int32_t> rowid;
   rowid.swap(g->rowid);
   DevBuf<uint32_t> skey(std::max<int64_t>(m, 1), s), skey2(std::max<int64_t>(m, 1), s);
-  DevBuf<uint64_t> sval(std::max<int64_t>(m, 1), s), sval2(std::max<int64_t>(m, 1), s);
+  // the sort moves 4-B edge indices; the packed (start, length) stays put and
+  // is gathered by index afterwards (12 -> 8 B per element per sort pass)
+  DevBuf<uint32_t> sidx(std::max<int64_t>(m, 1), s), sidx2(std::max<int64_t>(m, 1), s);
+  DevBuf<uint64_t> sval(std::max<int64_t>(m, 1), s);
   if (m > 0) {
     if (!rowid.get()) {
       rowid = DevBuf<int32_t>(m, s);
@@ -1338,7 +1146,8 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     constexpr int64_t kSmallGraph = int64_t(1) << 20;
     const int long_min = (opt.long_min_auto && m < kSmallGraph) ? (1 << 30) : std::max(opt.long_min, 32);
     k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), vmm.get(), m, long_min,
-                                            g->bits, dead, skey.get(), sval.get(), stats.get());
+                                            g->bits, dead, skey.get(), sidx.get(), sval.get(),
+                                            stats.get());
     TC_LAUNCH();
   }
   rowid.reset();
@@ -1366,12 +1175,12 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   // live edges ordered by (class, head v, position): the radix sort is stable
   // and the edges arrive in position order; dead edges sort past S
   cub::DoubleBuffer<uint32_t> dk(skey.get(), skey2.get());
-  cub::DoubleBuffer<uint64_t> dv(sval.get(), sval2.get());
+  cub::DoubleBuffer<uint32_t> dv(sidx.get(), sidx2.get());
   cub_run(s, [&](void* t, size_t& b) {
     return cub::DeviceRadixSort::SortPairs(t, b, dk, dv, m, 0, end_bit, s);
   });
   const uint32_t* key_sorted = dk.Current();
-  const uint64_t* val_sorted = dv.Current();
+  const uint32_t* idx_sorted = dv.Current();
   tr("select + class sort");
 
   DevBuf<int32_t> gincl(S, s);
@@ -1394,39 +1203,40 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P.seg_start = DevBuf<uint32_t>(S, s, true);
   P.seg_len = DevBuf<int32_t>(S, s, true);
   P.seg_group = DevBuf<int32_t>(S, s, true);
-  DevBuf<int64_t> units(S, s), grp_row(G, s), grp_d(G, s), grp_slots(G, s);
-  int64_t units_total = 0;  // host copy (read after the next sync)
+  DevBuf<uint32_t> units(S, s);
+  DevBuf<int64_t> grp_row(G, s), grp_d(G, s), grp_slots(G, s), cost(S, s), cost_prefix(S + 1, s);
+  DevBuf<unsigned long long> d_units_total(1, s);
+  TC_CUDA(cudaMemsetAsync(d_units_total.get(), 0, sizeof(unsigned long long), s));
+  unsigned long long units_total = 0;  // host copy (read after the next sync)
   P.grp_code = DevBuf<int32_t>(G, s, true);
-  k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted, val_sorted, gincl.get(), S, S_long,
+  k_seg_fill<<<grid_for(S), TPB, 0, s>>>(key_sorted, idx_sorted, sval.get(), gincl.get(), S, S_long,
                                          g->bits, row_ptr,
                                          opt.huge_degree, opt.table_factor, opt.bitmap_factor,
                                          max_slots_long, max_slots_short, col, P.grp_code.get(),
                                          P.seg_start.get(),
                                          P.seg_len.get(), P.seg_group.get(), units.get(),
-                                         grp_row.get(), grp_d.get(), grp_slots.get());
+                                         grp_row.get(), grp_d.get(), grp_slots.get(), opt.seg_cost,
+                                         cost.get(), d_units_total.get());
   TC_LAUNCH();
   gincl.reset();
   skey.reset();
   skey2.reset();
   sval.reset();
-  sval2.reset();
-  {  // the unit prefix in 64 bits, kept mod 2^32 in the plan (chunk-relative use only)
-    DevBuf<int64_t> kp64(S + 1, s);
-    exclusive_prefix(units.get(), S, kp64.get(), s);
-    k_narrow_u32<<<grid_for(S + 1), TPB, 0, s>>>(kp64.get(), S + 1, P.key_prefix.get());
-    TC_LAUNCH();
-    TC_CUDA(cudaMemcpyAsync(&units_total, kp64.get() + S, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-  }
+  sidx.reset();
+  sidx2.reset();
+  // the unit prefix mod 2^32 (uint32 arithmetic wraps exactly; only
+  // chunk-relative differences are used), key_prefix[0] = 0 (memset above)
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceScan::InclusiveSum(t, b, units.get(), P.key_prefix.get() + 1, S, s);
+  });
+  TC_CUDA(cudaMemcpyAsync(&units_total, d_units_total.get(), sizeof(units_total),
+                          cudaMemcpyDeviceToHost, s));
   P.ins_prefix = DevBuf<int64_t>(G + 1, s, true);
   P.slot_prefix = DevBuf<int64_t>(G + 1, s, true);
   exclusive_prefix(grp_d.get(), G, P.ins_prefix.get(), s);
   exclusive_prefix(grp_slots.get(), G, P.slot_prefix.get(), s);
   P.grp_ibase = DevBuf<int64_t>(G, s, true);
   k_grp_ibase<<<grid_for(G), TPB, 0, s>>>(grp_row.get(), P.ins_prefix.get(), G, P.grp_ibase.get());
-  TC_LAUNCH();
-  DevBuf<int64_t> cost(S, s), cost_prefix(S + 1, s);
-  k_seg_cost<<<grid_for(S), TPB, 0, s>>>(units.get(), P.seg_group.get(), grp_d.get(),
-                                         grp_slots.get(), S, opt.seg_cost, cost.get());
   TC_LAUNCH();
   exclusive_prefix(cost.get(), S, cost_prefix.get(), s);
   cost.reset();
@@ -1442,7 +1252,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   TC_CUDA(cudaStreamSynchronize(s));
   const int64_t cost_long = h_cp[0], cost_short = h_cp[1] - h_cp[0];
   tr("groups + prefixes + costs");
-  P.units_total = units_total;
+  P.units_total = (int64_t)units_total;
 
   // Chunking, per class: cost chunks (long class 4x larger: its edges carry
   // ~150 keys each), then every chunk is split where its SMEM layout would

@@ -35,6 +35,7 @@ void check_cuda(cudaError_t e, const char* what, const char* file, int line);
 void* dev_alloc(size_t bytes, cudaStream_t s, bool persistent);  // throws TC_ERR_OUT_OF_MEMORY
 void dev_free(void* p, size_t bytes, cudaStream_t s);
 void reserve_pool(size_t bytes, cudaStream_t s);  // grow the scratch pool once, up front
+void trim_pools();  // tc_release_memory
 
 // Owning device buffer (stream-ordered free on the stream it was made on).
 template <class T>

@@ -404,36 +404,6 @@ def test_dedup_paths_agree(tc):
     assert int(out["sort"][1]) == oracle.triangles(src, dst)
 
 
-@pytest.mark.parametrize("gen", ["rmat16", "skewed", "complete"])
-def test_a5_paths_agree(tc, gen):
-    """a5 by rows (counting scatter + per-row warp / CTA sorts, the default) and
-    by one radix sort of all oriented keys (TC_A5=sort, in a child process)
-    build byte-identical CSRs (row_ptr, col, perm) and the same count; the
-    complete graph has rows longer than 32 (the CTA sort) and skewed RMAT hubs."""
-    import subprocess
-    import sys
-    make = {"rmat16": "tcgen.rmat(16, 16, 9)", "skewed": "tcgen.rmat(15, 24, 7, abc=(0.65, 0.15, 0.15))",
-            "complete": "graphs.complete(700)[0]"}[gen]
-    code = ("import sys, hashlib, numpy as np, torch; sys.path.insert(0, %r); import tcgen;"
-            "from tests import graphs;"
-            "import paper_conf_ipps_li0ptz24_b200 as tc;"
-            "s, d, n = %s;"
-            "g = tc.build_csr(torch.as_tensor(np.ascontiguousarray(s, np.int32)).cuda(),"
-            " torch.as_tensor(np.ascontiguousarray(d, np.int32)).cuda(), n);"
-            "h = hashlib.sha256(); [h.update(x.cpu().numpy().tobytes()) for x in g.csr()];"
-            "print(h.hexdigest(), g.count(), g.info.max_out_degree)") % (ROOT, make)
-    out = {}
-    for mode in ("rows", "sort"):
-        env = dict(os.environ, TC_A5=mode)
-        r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
-                           timeout=300, cwd=ROOT)
-        assert r.returncode == 0, r.stderr[-2000:]
-        out[mode] = r.stdout.split()[-3:]
-    assert out["rows"] == out["sort"]
-    if gen == "complete":
-        assert int(out["rows"][2]) > 32  # the CTA row sort ran
-
-
 def test_host_pipelined_build_equals_device(tc):
     """Above 2^25 pairs tc_build_csr_host overlaps the H2D copy of piece i+1
     with the sort of piece i and merges the sorted runs: the graph must be
@@ -467,6 +437,8 @@ def test_more_than_2_31_edges(tc):
     32-bit tile descriptors passes 2^31 (the guard only rejects m >= 2^32).
     A disjoint union of c copies of K_64 with m = c * C(64, 2) > 2^31 unique
     edges, generated on the device; T = c * C(64, 3) in closed form (C-16)."""
+    torch.cuda.empty_cache()
+    tc.release_memory()  # the earlier tests' cached pool memory
     free, _ = torch.cuda.mem_get_info()
     if free < (170 << 30):
         pytest.skip(f"needs ~170 GB of device memory, {free >> 30} GB free")
