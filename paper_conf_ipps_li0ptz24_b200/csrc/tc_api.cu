@@ -152,6 +152,20 @@ void trim_pools() {
   }
 }
 
+const Plan& host_plan(const tc_graph* g) {
+  const Plan& P = g->plan;
+  std::call_once(*P.host_once, [&] {
+    std::vector<int64_t> seg(P.n_chunks + 1), cost(P.n_chunks + 1);
+    TC_CUDA(cudaMemcpy(seg.data(), P.chunk_seg.get(), sizeof(int64_t) * seg.size(),
+                       cudaMemcpyDeviceToHost));
+    TC_CUDA(cudaMemcpy(cost.data(), P.chunk_cost.get(), sizeof(int64_t) * cost.size(),
+                       cudaMemcpyDeviceToHost));
+    P.h_chunk_seg.swap(seg);
+    P.h_chunk_cost.swap(cost);
+  });
+  return P;
+}
+
 void dev_free(void* p, size_t bytes, cudaStream_t s) {
   if (!p) return;
   if (g_free) {
@@ -195,8 +209,8 @@ namespace {
 void rebind(tc_graph* g, cudaStream_t s) {
   g->row_ptr.s = g->col.s = g->perm.s = s;
   tc::Plan& P = g->plan;
-  P.key_prefix.s = P.seg_start.s = P.ins_prefix.s = P.grp_ibase.s = P.slot_prefix.s =
-      P.chunk_seg.s = s;
+  P.key_prefix.s = P.seg_start.s = s;
+  P.ins_prefix.s = P.grp_ibase.s = P.slot_prefix.s = P.chunk_seg.s = P.chunk_cost.s = s;
   P.seg_len.s = P.seg_group.s = P.grp_code.s = s;
 }
 
@@ -204,10 +218,14 @@ void rebind(tc_graph* g, cudaStream_t s) {
 // > e_begin up to the last whose start is < e_end.
 void chunk_range(const tc_graph* g, int64_t e_begin, int64_t e_end, int64_t* c_begin,
                  int64_t* c_end) {
-  const tc::Plan& P = g->plan;
-  const auto& cs = P.h_chunk_seg;
   *c_begin = *c_end = 0;
   if (e_end <= e_begin) return;
+  if (e_begin == 0 && e_end == g->plan.S) {  // the whole graph: no host chunk arrays needed
+    *c_end = g->plan.n_chunks;
+    return;
+  }
+  const tc::Plan& P = tc::host_plan(g);
+  const auto& cs = P.h_chunk_seg;
   *c_begin = std::max<int64_t>(std::upper_bound(cs.begin(), cs.end(), e_begin) - cs.begin() - 1, 0);
   *c_end = std::min<int64_t>(std::lower_bound(cs.begin(), cs.end(), e_end) - cs.begin(), P.n_chunks);
 }
@@ -561,7 +579,7 @@ tc_status tc_refine_profile(const tc_graph* g, void* stream, int32_t world_size,
                             double* h_ms) {
   return guarded([&] {
     require(g && h_ms, "NULL argument");
-    const tc::Plan& P = g->plan;
+    const tc::Plan& P = tc::host_plan(g);
     check_profile_args(P.h_chunk_seg.data(), P.h_chunk_cost.data(), P.n_chunks, P.n_long_chunks,
                        n_slices, h_ms, world_size);
     if (P.n_chunks == 0 || world_size == 1) return;
@@ -617,7 +635,7 @@ tc_status tc_partition_measured(const tc_graph* g, int32_t world_size, int32_t n
                                 const double* h_ms, int64_t* h_bounds) {
   return guarded([&] {
     require(g && h_bounds && h_ms, "NULL argument");
-    const tc::Plan& P = g->plan;
+    const tc::Plan& P = tc::host_plan(g);
     const tc_status st = tc_partition_chunks(P.h_chunk_seg.data(), P.h_chunk_cost.data(), P.n_chunks,
                                              P.n_long_chunks, n_slices, h_ms, world_size, h_bounds);
     if (st != TC_OK) tc::fail(st, t_last_error);
@@ -627,7 +645,13 @@ tc_status tc_partition_measured(const tc_graph* g, int32_t world_size, int32_t n
 tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds) {
   return guarded([&] {
     require(g && h_bounds, "NULL argument");
-    const tc::Plan& P = g->plan;
+    require(world_size >= 1, "world_size < 1");
+    if (world_size == 1) {  // one rank: the whole range (no host chunk arrays needed)
+      h_bounds[0] = 0;
+      h_bounds[1] = g->plan.S;
+      return;
+    }
+    const tc::Plan& P = tc::host_plan(g);
     // the built-in profile: the classes as two slices (one if a class is empty)
     const int64_t nc = P.n_chunks, nL = P.n_long_chunks;
     const double cl = (double)P.h_chunk_cost[nL], cs = (double)(P.h_chunk_cost[nc] - P.h_chunk_cost[nL]);
@@ -645,7 +669,7 @@ tc_status tc_partition(const tc_graph* g, int32_t world_size, int64_t* h_bounds)
 tc_status tc_plan_chunks(const tc_graph* g, int64_t* h_seg, int64_t* h_cost) {
   return guarded([&] {
     require(g != nullptr, "graph is NULL");
-    const tc::Plan& P = g->plan;
+    const tc::Plan& P = tc::host_plan(g);
     if (h_seg) std::copy(P.h_chunk_seg.begin(), P.h_chunk_seg.end(), h_seg);
     if (h_cost) std::copy(P.h_chunk_cost.begin(), P.h_chunk_cost.end(), h_cost);
   });
@@ -655,7 +679,7 @@ tc_status tc_calibrate(const tc_graph* g, void* stream, int32_t n_slices, double
   return guarded([&] {
     require(g && h_ms, "NULL argument");
     require(n_slices >= 1, "n_slices < 1");
-    const tc::Plan& P = g->plan;
+    const tc::Plan& P = tc::host_plan(g);
     cudaStream_t s = (cudaStream_t)stream;
     for (int32_t i = 0; i < n_slices; ++i) h_ms[i] = 0;
     if (P.n_chunks == 0) return;

@@ -1162,8 +1162,8 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   if (S == 0) {
     P.chunk_seg = DevBuf<int64_t>(1, s, true);
     TC_CUDA(cudaMemsetAsync(P.chunk_seg.get(), 0, sizeof(int64_t), s));
-    P.h_chunk_seg.assign(1, 0);
-    P.h_chunk_cost.assign(1, 0);
+    P.chunk_cost = DevBuf<int64_t>(1, s, true);
+    TC_CUDA(cudaMemsetAsync(P.chunk_cost.get(), 0, sizeof(int64_t), s));
     TC_CUDA(cudaStreamSynchronize(s));
     return;
   }
@@ -1299,21 +1299,16 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P.chunk_cost_short = CS;
   tr("chunking");
   {
-    DevBuf<int64_t> ccost(P.n_chunks + 1, s);
+    P.chunk_cost = DevBuf<int64_t>(P.n_chunks + 1, s, true);
     DevBuf<unsigned long long> st2(4, s);
     TC_CUDA(cudaMemsetAsync(st2.get(), 0, 4 * sizeof(unsigned long long), s));
     k_chunk_meta<<<grid_for(P.n_chunks + 1), TPB, 0, s>>>(P.chunk_seg.get(), P.n_chunks,
                                                           P.n_long_chunks,
                                                           P.seg_group.get(), P.ins_prefix.get(),
-                                                          cost_prefix.get(), ccost.get(), st2.get());
+                                                          cost_prefix.get(), P.chunk_cost.get(),
+                                                          st2.get());
     TC_LAUNCH();
-    P.h_chunk_seg.resize(P.n_chunks + 1);
-    P.h_chunk_cost.resize(P.n_chunks + 1);
     unsigned long long h_st2[4];
-    TC_CUDA(cudaMemcpyAsync(P.h_chunk_seg.data(), P.chunk_seg.get(),
-                            sizeof(int64_t) * (P.n_chunks + 1), cudaMemcpyDeviceToHost, s));
-    TC_CUDA(cudaMemcpyAsync(P.h_chunk_cost.data(), ccost.get(), sizeof(int64_t) * (P.n_chunks + 1),
-                            cudaMemcpyDeviceToHost, s));
     TC_CUDA(cudaMemcpyAsync(h_st2, st2.get(), sizeof(h_st2), cudaMemcpyDeviceToHost, s));
     TC_CUDA(cudaStreamSynchronize(s));
     P.table_words = (int64_t)h_st2[0];

@@ -5,6 +5,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <memory>
+#include <mutex>
 #include <string>
 #include <utility>
 #include <vector>
@@ -171,8 +173,11 @@ struct Plan {
   DevBuf<uint32_t> key_prefix, seg_start;  // 32-bit: see PlanView
   DevBuf<int64_t> ins_prefix, grp_ibase, slot_prefix, chunk_seg;
   DevBuf<int32_t> seg_len, seg_group, grp_code;
-  std::vector<int64_t> h_chunk_seg;
-  std::vector<int64_t> h_chunk_cost;  // [n_chunks+1] plan cost prefix at each chunk's first edge
+  DevBuf<int64_t> chunk_cost;  // [n_chunks+1] plan cost prefix at each chunk's first edge
+  // Host copies of chunk_seg / chunk_cost, made on first use (host_plan):
+  // a count of the whole graph and a 1-rank partition never need them.
+  mutable std::vector<int64_t> h_chunk_seg, h_chunk_cost;
+  mutable std::shared_ptr<std::once_flag> host_once = std::make_shared<std::once_flag>();
   int64_t table_words = 0;   // sum over (chunk, group) visits of d+(v): table rows read per count
   int64_t group_visits = 0;  // (chunk, group) pairs
   uint64_t method_bytes = 0; // bytes one full count reads as designed (keys + plan + tables)
@@ -198,6 +203,10 @@ struct tc_graph {
 };
 
 namespace tc {
+
+// The plan with its host chunk arrays present (copied from the device on
+// first use; the graph's build has completed).  tc_api.cu.
+const Plan& host_plan(const tc_graph* g);
 
 // tc_build.cu
 void build_graph(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen, int64_t n,
