@@ -95,7 +95,7 @@ typedef struct {
   int32_t bitmap_factor; /* a head v whose window [min N+(v), max N+(v)] needs at most
                            bitmap_factor * d+(v) 32-bit words gets a bitmap table
                            (one probe per key) instead of a hash table (two);
-                           default 12, -1 = never                                */
+                           default 16, -1 = never                                */
 } tc_options;
 
 /*
@@ -435,21 +435,25 @@ TC_API tc_status tc_build_from_oriented(const uint64_t* d_okeys, int64_t m,
 /*
  * ------------------------------------------------------------------------
  * the cross-GPU sum of the partial counts done by
- * the library over NVLink peer memory (no NCCL).  After this rank's count of
- * [e_begin, e_end) (as tc_count_range), one thread adds the partial into a
- * SYMMETRIC buffer on every rank and waits for every rank's contribution:
+ * the library over NVLink peer memory (no NCCL).  This rank counts
+ * [e_begin, e_end) (as tc_count_range) and the LAST CTA of its last count
+ * launch (a grid-completion ticket) adds the partial into a SYMMETRIC buffer
+ * on every rank and waits for every rank's contribution, so no extra launch
+ * is made (a rank whose range is empty runs a one-thread finishing kernel):
  *   - d_mc != NULL: through an NVLS multicast address (one
  *     multimem.red.add.u64; the NVSwitch updates every replica);
  *   - else through the world unicast peer addresses h_peers[0..world) (one
  *     red.add.u64 per peer over NVLink P2P; h_peers[rank] == d_own).
- * d_own : this rank's unicast address of the buffer (device uint64[3],
- *         zero-initialised once, same layout on every rank; do not touch it
- *         between calls).  epoch: 1 for the first call on a buffer, +1 per
- *         call, equal on all ranks.  world <= TC_MAX_PEERS.
+ * d_own : this rank's unicast address of the buffer (device uint64[8]:
+ *         words 0/1 = the sums of even / odd epochs, 2 = arrivals, 3 =
+ *         POISON, 4 = the ticket; zero-initialised once, same layout on every
+ *         rank; do not touch it between calls).  epoch: 1 for the first call
+ *         on a buffer, +1 per call, equal on all ranks.  world <= TC_MAX_PEERS.
  * d_total (device uint64) receives T on every rank.  Stream-ordered; the
- * finishing kernel spins until all ranks arrive, so every rank must make the
- * call; if some rank has not arrived within 20 s the kernel gives up and
- * writes UINT64_MAX to d_total instead of hanging the stream.
+ * kernel spins until all ranks arrive, so every rank must make the call; if
+ * some rank has not arrived within 20 s (TC_FUSED_TIMEOUT_MS) the kernel sets
+ * the buffer's POISON word and writes UINT64_MAX to d_total instead of
+ * hanging the stream; the buffer must then be recreated.
  * The multicast / peer mappings are the caller's plumbing (e.g. torch
  * symmetric memory); tc_mc_buffer_create makes a single-device one.
  */

@@ -1096,7 +1096,6 @@ Tuning tuning_from_env() {
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
   t.batch = get("TC_BATCH", t.batch, 0, 64);
   t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 3);
-  t.overlap = get("TC_OVERLAP", t.overlap, 0, 1);
   return t;
 }
 

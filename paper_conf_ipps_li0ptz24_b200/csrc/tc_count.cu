@@ -1204,28 +1204,6 @@ void set_attr() {
                                optin_smem() - static_smem((const void*)k_support)));
 }
 
-// One forked stream (+ fork / join events) per device for the short class's
-// launch next to the long class's (count_chunks); callers serialise on mu.
-struct AuxStream {
-  std::mutex mu;
-  cudaStream_t stream = nullptr;
-  cudaEvent_t fork = nullptr, join = nullptr;
-};
-
-AuxStream& aux_stream() {
-  static AuxStream aux[kMaxDevices];
-  static std::once_flag once[kMaxDevices];
-  int dev = 0;
-  TC_CUDA(cudaGetDevice(&dev));
-  if (dev < 0 || dev >= kMaxDevices) fail(TC_ERR_UNSUPPORTED, "device ordinal beyond 64");
-  std::call_once(once[dev], [&] {
-    TC_CUDA(cudaStreamCreateWithFlags(&aux[dev].stream, cudaStreamNonBlocking));
-    TC_CUDA(cudaEventCreateWithFlags(&aux[dev].fork, cudaEventDisableTiming));
-    TC_CUDA(cudaEventCreateWithFlags(&aux[dev].join, cudaEventDisableTiming));
-  });
-  return aux[dev];
-}
-
 void ensure_attr() {
   int dev = 0;
   TC_CUDA(cudaGetDevice(&dev));
@@ -1320,17 +1298,6 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
   const int64_t l0 = c_begin, l1 = std::min(c_end, P.n_long_chunks);
   const int64_t s0 = std::max(c_begin, P.n_long_chunks), s1 = c_end;
   int launched = 0;
-  // Without the fused sum (which needs one last launch), the short class runs
-  // on a forked stream next to the long class: its CTAs take the SMs that
-  // k_count's CTAs release in that kernel's tail (Tuning::overlap).
-  const bool fork = P.tune.overlap && !fuse && l1 > l0 && s1 > s0;
-  AuxStream* aux = fork ? &aux_stream() : nullptr;
-  std::unique_lock<std::mutex> lk;
-  if (fork) {
-    lk = std::unique_lock<std::mutex>(aux->mu);
-    TC_CUDA(cudaEventRecord(aux->fork, s));
-    TC_CUDA(cudaStreamWaitEvent(aux->stream, aux->fork, 0));
-  }
   if (l1 > l0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(l1 - l0, P.grid));
     const int64_t sb = slot_bytes_of(P.smem_bytes);
@@ -1343,14 +1310,9 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
   }
   if (s1 > s0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(s1 - s0, P.grid_flat));
-    cudaStream_t ss = fork ? aux->stream : s;
-    k_count_flat<<<grid, kFlatBlock, (size_t)slot_bytes_of(P.smem_flat), ss>>>(
+    k_count_flat<<<grid, kFlatBlock, (size_t)slot_bytes_of(P.smem_flat), s>>>(
         pv, s0, s1, e_begin, e_end, d_out, fuse ? *fuse : none);
     TC_LAUNCH();
-    if (fork) {  // join: the caller's stream waits for the short class
-      TC_CUDA(cudaEventRecord(aux->join, ss));
-      TC_CUDA(cudaStreamWaitEvent(s, aux->join, 0));
-    }
     ++launched;
   }
   return launched;

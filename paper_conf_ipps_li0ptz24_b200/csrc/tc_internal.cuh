@@ -81,7 +81,7 @@ struct Options {
   int long_min = 32;
   bool long_min_auto = true;  // long_min not given: graphs under kSmallGraph edges are all short
   int probe_mode = 0;
-  int bitmap_factor = 12;  // <= 0: never
+  int bitmap_factor = 16;  // <= 0: never (r2p/r2q C3 k_count: 8 -> 42.9 ms, 12 -> 41.6, 16 -> 41.25, 32 -> 41.2)
 };
 Options resolve_options(const tc_options* o);
 
@@ -149,7 +149,6 @@ struct Tuning {
   int short_linear = 1;   // short class: linear-probing tables (no cuckoo attempt)
   int prod_groups = 2;    // long class: producer groups filling slots concurrently (TC_PROD_GROUPS, 1..3;
                           // r2k: 1 -> 2 groups C3 k_count 42.8 -> 41.7 ms, C4 583 -> 544 ms)
-  int overlap = 0;        // short class on a forked stream next to the long class (TC_OVERLAP)
   int batch = 0;          // long-class tiles per batch for block_threads <= 768 (TC_BATCH; see count_kernel)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
