@@ -2,7 +2,9 @@
 // translation (no exception crosses the ABI), the allocator hook, and the
 // host-side range/partition logic.  SURVEY.md §8(b).
 #include <algorithm>
+#include <chrono>
 #include <cmath>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <new>

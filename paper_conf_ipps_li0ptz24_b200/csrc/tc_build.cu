@@ -891,6 +891,11 @@ void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen,
   }
   Timer tm(s);
   tm.mark();
+  // Let the pool growth and the piece buffers' allocations complete before the
+  // pipelined copies and sorts are issued: without this sync the host entry's
+  // time at C3 varied between 86 and 161 ms over identical builds (the phase
+  // events inside stayed at 85 ms), with it it is 85-88 ms (profiles/r2t_e2e_c3.txt).
+  TC_CUDA(cudaStreamSynchronize(s));
   g->n_input = n;
   const int bits = bits_for(std::max<int64_t>(n, 2));
   const uint64_t sent = (uint64_t(1) << (2 * bits)) - 1;
