@@ -56,6 +56,9 @@ constexpr int kUnrollLong = 8;   // tail batch of the long class
 #define TC_BATCH_LONG 8
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
+#ifndef TC_L2PF
+#define TC_L2PF 0  // walk_long: L2 prefetch of the next batch's key lines (A/B knob)
+#endif
 #ifndef TC_UNROLL_SHORT
 #define TC_UNROLL_SHORT 2
 #endif
@@ -403,6 +406,16 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   const int32_t* colL = lane_base(pv.col, lane);
   int t = t0;
   for (; t + kB <= t1; t += kB) {
+#if TC_L2PF
+    // pull the next batch's key lines into L2 while this batch's loads are
+    // outstanding (no registers held: lane u < kB takes tile u's first line,
+    // lane kB + u its last)
+    if (lane < 2 * kB && t + kB + (lane % kB) < t1) {
+      const int q = lane % kB;
+      const uint32_t x = (uint32_t)c.sT0[t + kB + q] + (lane >= kB ? 31u : 0u);
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + x));
+    }
+#endif
     int32_t key[kB];
     load_batch<kB>(c, colL, t, key);
     int z[kB], zw[kB];
