@@ -66,6 +66,11 @@ def parse():
     ap.add_argument("--reduce", default="nccl", choices=["nccl", "fused"],
                     help="cross-GPU sum of the partial counts: NCCL all_reduce, or the library's "
                          "own over NVLink peer memory (tc_count_range_fused, SURVEY.md §8(f) f4)")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for N > 1 (gloo: test mode only)")
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="test mode: all ranks on cuda:0 with --backend gloo (exercises the N > 1 "
+                         "code path on a one-GPU box; its timings are not scaling numbers)")
     ap.add_argument("--no-balance", action="store_true",
                     help="skip the N = 1 emulated multi-GPU balance measurement")
     ap.add_argument("--no-sharded", action="store_true",
@@ -356,9 +361,14 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != a.gpus and rank == 0:
         print(f"warning: --gpus {a.gpus} but WORLD_SIZE {world}", file=sys.stderr)
+    if a.share_gpu:  # test mode: every rank on cuda:0 (gloo), to exercise the N > 1 path on one GPU
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if a.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(a.backend)
     dev = torch.device("cuda", local)
 
     cfg = tcgen.CONFIGS[a.config]
