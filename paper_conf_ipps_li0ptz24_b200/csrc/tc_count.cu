@@ -57,8 +57,8 @@ constexpr int kUnrollLong = 8;   // tail batch of the long class
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
 #ifndef TC_L2PF
-#define TC_L2PF 0  // walk_long: L2 prefetch of the next batch's key lines (A/B knob)
-#endif
+#define TC_L2PF 1  // walk_long: L2 prefetch of the key lines TC_L2PF batches ahead (0: off;
+#endif             // r2v C3 k_count 42.2 -> 38.9 ms, C4 564 -> 545 ms with 1)
 #ifndef TC_UNROLL_SHORT
 #define TC_UNROLL_SHORT 2
 #endif
@@ -407,12 +407,13 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   int t = t0;
   for (; t + kB <= t1; t += kB) {
 #if TC_L2PF
-    // pull the next batch's key lines into L2 while this batch's loads are
-    // outstanding (no registers held: lane u < kB takes tile u's first line,
-    // lane kB + u its last)
-    if (lane < 2 * kB && t + kB + (lane % kB) < t1) {
+    // pull the key lines of the batch TC_L2PF batches ahead into L2 while this
+    // batch's loads are outstanding: the loads in flight per lane are bounded
+    // by registers, a prefetch holds none (lane u < kB takes tile u's first
+    // line, lane kB + u its last)
+    if (lane < 2 * kB && t + TC_L2PF * kB + (lane % kB) < t1) {
       const int q = lane % kB;
-      const uint32_t x = (uint32_t)c.sT0[t + kB + q] + (lane >= kB ? 31u : 0u);
+      const uint32_t x = (uint32_t)c.sT0[t + TC_L2PF * kB + q] + (lane >= kB ? 31u : 0u);
       asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + x));
     }
 #endif
