@@ -56,6 +56,9 @@ constexpr int kUnrollLong = 8;   // tail batch of the long class
 #define TC_BATCH_LONG 8
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
+#ifndef TC_PF_SHORT
+#define TC_PF_SHORT 0  // produce: L2 prefetch of every short-class edge's keys at staging (A/B knob)
+#endif
 #ifndef TC_PF_NEXT
 #define TC_PF_NEXT 0  // k_count producers: L2 prefetch of the next chunk's plan rows (A/B knob)
 #endif
@@ -809,6 +812,16 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         c.sB[i] = is_long ? (int64_t)st[r] : (int64_t)st[r] - rel;
         c.sC[i] = ln[r];
         c.sD[i] = gr[r] - (int)ga;
+#if TC_PF_SHORT
+        // short class: pull the edge's keys (< 32, at most two lines) into L2
+        // now; the walk reads them after the tables are built
+        if (!is_long && !kSup) {
+          const int32_t* k0 = pv.col + st[r];
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(k0));
+          if (((uintptr_t)k0 & 127) + 4 * (uintptr_t)ln[r] > 128)
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(k0 + ln[r] - 1));
+        }
+#endif
       }
     }
   }
