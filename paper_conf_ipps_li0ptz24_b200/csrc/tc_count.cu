@@ -59,9 +59,6 @@ constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flig
 #ifndef TC_PF_SHORT
 #define TC_PF_SHORT 0  // produce: L2 prefetch of every short-class edge's keys at staging (A/B knob)
 #endif
-#ifndef TC_PF_NEXT
-#define TC_PF_NEXT 0  // k_count producers: L2 prefetch of the next chunk's plan rows (A/B knob)
-#endif
 #ifndef TC_L2PF
 #define TC_L2PF 1  // walk_long: L2 prefetch of the key lines TC_L2PF batches ahead (0: off;
 #endif             // r2v C3 k_count 42.2 -> 38.9 ms, C4 564 -> 545 ms with 1)
@@ -734,37 +731,10 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
 // in [0, PT); the PT producer threads synchronise on named barrier 1.  The
 // header is written by producer 0 before its own mbarrier arrive, so the
 // consumers see it once every producer has arrived.
-// L2 prefetch of the plan rows of chunk cix (its edges' and groups' entries),
-// spread over the PT producer threads: the producers of the chunk after the
-// one they are staging find these rows in L2 (TC_PF_NEXT).
-__device__ __forceinline__ void prefetch_line_range(const void* base, int64_t bytes, int pt, int PT) {
-  const char* p = static_cast<const char*>(base);
-  for (int64_t off = (int64_t)pt * 128; off < bytes; off += (int64_t)PT * 128)
-    asm volatile("prefetch.global.L2 [%0];" ::"l"(p + off));
-}
-
-__device__ __forceinline__ void prefetch_chunk_plan(const PlanView& pv, int64_t cix, int pt, int PT) {
-  const int64_t sa = __ldg(pv.chunk_seg + cix), sb = __ldg(pv.chunk_seg + cix + 1);
-  if (sa >= sb) return;
-  const int64_t ga = __ldg(pv.seg_group + sa), gb = (int64_t)__ldg(pv.seg_group + (sb - 1)) + 1;
-  const int64_t S = sb - sa, G = gb - ga;
-  prefetch_line_range(pv.key_prefix + sa, 4 * (S + 1), pt, PT);
-  prefetch_line_range(pv.seg_start + sa, 4 * S, pt, PT);
-  prefetch_line_range(pv.seg_len + sa, 4 * S, pt, PT);
-  prefetch_line_range(pv.seg_group + sa, 4 * S, pt, PT);
-  prefetch_line_range(pv.ins_prefix + ga, 8 * (G + 1), pt, PT);
-  prefetch_line_range(pv.slot_prefix + ga, 8 * (G + 1), pt, PT);
-  prefetch_line_range(pv.grp_ibase + ga, 8 * G, pt, PT);
-  prefetch_line_range(pv.grp_code + ga, 4 * G, pt, PT);
-}
-
 template <int kB, bool kSup = false>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
-                                        int pt, int PT, int bar = 1, int64_t next_cix = -1) {
-#if TC_PF_NEXT
-  if (next_cix >= 0) prefetch_chunk_plan(pv, next_cix, pt, PT);
-#endif
+                                        int pt, int PT, int bar = 1) {
   const int64_t sa = max(__ldg(pv.chunk_seg + (cix)), e_begin), sb = min(__ldg(pv.chunk_seg + (cix + 1)), e_end);
   if (sa >= sb) {  // empty after clipping to the range
     if (pt == 0) {
@@ -1037,9 +1007,7 @@ __global__ void __launch_bounds__(kBlock, 1)
           mbar_arrive(&full_bar[slot]);
           break;
         }
-        const int64_t nxt = cix + (int64_t)ng * gridDim.x;  // this group's next chunk
-        produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], pt, PTg, 1 + g,
-                   nxt < c_end ? nxt : -1);
+        produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], pt, PTg, 1 + g);
         mbar_arrive(&full_bar[slot]);
         slot += ng;
         if (slot >= nslots) {
