@@ -56,6 +56,9 @@ constexpr int kUnrollLong = 8;   // tail batch of the long class
 #define TC_BATCH_LONG 8
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
+#ifndef TC_PF_ROWS
+#define TC_PF_ROWS 0  // produce: L2 prefetch of each group's N+(v) head at staging (A/B knob)
+#endif
 #ifndef TC_PF_SHORT
 #define TC_PF_SHORT 0  // produce: L2 prefetch of every short-class edge's keys at staging (A/B knob)
 #endif
@@ -824,6 +827,15 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         c.sInfo[i] = ns > 0 ? make_int2((int)(sp[r] - slot0), cd[r]) : make_int2(-1, 0);
         huge |= ns == 0;
         c.sGB[i] = ib[r] + ip0;  // row start - chunk-relative insert prefix
+#if TC_PF_ROWS
+        // pull the head of N+(v) (the table's keys, inserted after the tables
+        // are initialised) toward L2: its first two lines
+        if (ns > 0) {
+          const int32_t* row = pv.col + (ib[r] + ip[r]);
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(row));
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(row + 32));
+        }
+#endif
       }
     }
   }
