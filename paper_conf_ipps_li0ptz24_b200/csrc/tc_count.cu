@@ -831,9 +831,9 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         // pull the head of N+(v) (the table's keys, inserted after the tables
         // are initialised) toward L2: its first two lines
         if (ns > 0) {
-          const int32_t* row = pv.col + (ib[r] + ip[r]);
-          asm volatile("prefetch.global.L2 [%0];" ::"l"(row));
-          asm volatile("prefetch.global.L2 [%0];" ::"l"(row + 32));
+          const int64_t rs = ib[r] + ip[r];
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + rs));
+          if (rs + 32 < pv.m) asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + rs + 32));
         }
 #endif
       }
@@ -1274,6 +1274,7 @@ PlanView plan_view(const tc_graph* g) {
   pv.seg_edge = nullptr;
   pv.sup = nullptr;
   pv.max_kicks = P.tune.max_kicks;
+  pv.m = g->m;
   return pv;
 }
 

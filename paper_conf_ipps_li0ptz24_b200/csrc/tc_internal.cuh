@@ -116,6 +116,7 @@ struct PlanView {
   int probe_mode;
   int short_linear;            // short class always probes linearly (Tuning::short_linear)
   int max_kicks;               // cuckoo displacement bound (Tuning::max_kicks)
+  int64_t m;                   // entries of col
   // support mode only (tc_support; nullptr when counting)
   const int64_t* seg_edge;     // [S] CSR position of segment s's own edge (u,v)
   unsigned* sup;               // [m] per-edge triangle counts (accumulated)
