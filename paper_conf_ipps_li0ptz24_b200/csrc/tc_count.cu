@@ -56,6 +56,9 @@ constexpr int kUnrollLong = 8;   // tail batch of the long class
 #define TC_BATCH_LONG 8
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
+#ifndef TC_PF_FIRST
+#define TC_PF_FIRST 0  // produce: L2 prefetch of each consumer warp's first batch (A/B knob)
+#endif
 #ifndef TC_PF_ROWS
 #define TC_PF_ROWS 0  // produce: L2 prefetch of each group's N+(v) head at staging (A/B knob)
 #endif
@@ -737,7 +740,7 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
 template <int kB, bool kSup = false>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
-                                        int pt, int PT, int bar = 1) {
+                                        int pt, int PT, int bar = 1, int n_cons = 0) {
   const int64_t sa = max(__ldg(pv.chunk_seg + (cix)), e_begin), sb = min(__ldg(pv.chunk_seg + (cix + 1)), e_end);
   if (sa >= sb) {  // empty after clipping to the range
     if (pt == 0) {
@@ -873,6 +876,16 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
           c.sT0[t] = (int)(uint32_t)(p - (32 - lanes));
           c.sT1[t] = d.x < 0 ? toff : (int)(c.sHash - c.sT0) + (d.y <= 0 ? d.x + d.y : d.x);
           c.sT2[t] = ((d.x < 0 ? -1 : (d.y <= 0 ? 0 : d.y)) * 64) | (32 - lanes);
+#if TC_PF_FIRST
+          // the first batch of every consumer warp's share (the walk's own
+          // prefetch covers the batches after it): tiles within 8 of a raw
+          // boundary T * w / n_cons, pulled toward L2 now
+          if (n_cons > 0 && (int)(((unsigned)t * (unsigned)n_cons) % (unsigned)T) < 8 * n_cons) {
+            const int32_t* k0 = pv.col + (p - (32 - lanes));
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(k0));
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(k0 + 31));
+          }
+#endif
         }
       }
     }
@@ -1019,7 +1032,8 @@ __global__ void __launch_bounds__(kBlock, 1)
           mbar_arrive(&full_bar[slot]);
           break;
         }
-        produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], pt, PTg, 1 + g);
+        produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], pt, PTg, 1 + g,
+                   n_cons);
         mbar_arrive(&full_bar[slot]);
         slot += ng;
         if (slot >= nslots) {
