@@ -63,7 +63,7 @@ constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flig
 #define TC_PF_ROWS 0  // produce: L2 prefetch of each group's N+(v) head at staging (A/B knob)
 #endif
 #ifndef TC_PF_SHORT
-#define TC_PF_SHORT 0  // produce: L2 prefetch of every short-class edge's keys at staging (A/B knob)
+#define TC_PF_SHORT 1  // produce: L2 prefetch of every short-class edge's keys at staging (r2y: C2 -1.6%)
 #endif
 #ifndef TC_L2PF
 #define TC_L2PF 1  // walk_long: L2 prefetch of the key lines TC_L2PF batches ahead (0: off;
