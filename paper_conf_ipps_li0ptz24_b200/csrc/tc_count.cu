@@ -59,12 +59,6 @@ constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flig
 #ifndef TC_SUP_L2PF
 #define TC_SUP_L2PF 0  // walk_long_sup: L2 prefetch of the next batch's key lines (A/B knob)
 #endif
-#ifndef TC_PF_FIRST
-#define TC_PF_FIRST 0  // produce: L2 prefetch of each consumer warp's first batch (A/B knob)
-#endif
-#ifndef TC_PF_ROWS
-#define TC_PF_ROWS 0  // produce: L2 prefetch of each group's N+(v) head at staging (A/B knob)
-#endif
 #ifndef TC_PF_SHORT
 #define TC_PF_SHORT 1  // produce: L2 prefetch of every short-class edge's keys at staging (r2y: C2 -1.6%)
 #endif
@@ -754,7 +748,7 @@ __device__ __forceinline__ void walk_short_sup(const ChunkSmem& c, int S, int k0
 template <int kB, bool kSup = false>
 __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t e_begin,
                                         int64_t e_end, unsigned char* region, SlotHdr& hdr,
-                                        int pt, int PT, int bar = 1, int n_cons = 0) {
+                                        int pt, int PT, int bar = 1) {
   const int64_t sa = max(__ldg(pv.chunk_seg + (cix)), e_begin), sb = min(__ldg(pv.chunk_seg + (cix + 1)), e_end);
   if (sa >= sb) {  // empty after clipping to the range
     if (pt == 0) {
@@ -844,15 +838,6 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
         c.sInfo[i] = ns > 0 ? make_int2((int)(sp[r] - slot0), cd[r]) : make_int2(-1, 0);
         huge |= ns == 0;
         c.sGB[i] = ib[r] + ip0;  // row start - chunk-relative insert prefix
-#if TC_PF_ROWS
-        // pull the head of N+(v) (the table's keys, inserted after the tables
-        // are initialised) toward L2: its first two lines
-        if (ns > 0) {
-          const int64_t rs = ib[r] + ip[r];
-          asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + rs));
-          if (rs + 32 < pv.m) asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + rs + 32));
-        }
-#endif
       }
     }
   }
@@ -890,16 +875,6 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
           c.sT0[t] = (int)(uint32_t)(p - (32 - lanes));
           c.sT1[t] = d.x < 0 ? toff : (int)(c.sHash - c.sT0) + (d.y <= 0 ? d.x + d.y : d.x);
           c.sT2[t] = ((d.x < 0 ? -1 : (d.y <= 0 ? 0 : d.y)) * 64) | (32 - lanes);
-#if TC_PF_FIRST
-          // the first batch of every consumer warp's share (the walk's own
-          // prefetch covers the batches after it): tiles within 8 of a raw
-          // boundary T * w / n_cons, pulled toward L2 now
-          if (n_cons > 0 && (int)(((unsigned)t * (unsigned)n_cons) % (unsigned)T) < 8 * n_cons) {
-            const int32_t* k0 = pv.col + (p - (32 - lanes));
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(k0));
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(k0 + 31));
-          }
-#endif
         }
       }
     }
@@ -1046,8 +1021,7 @@ __global__ void __launch_bounds__(kBlock, 1)
           mbar_arrive(&full_bar[slot]);
           break;
         }
-        produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], pt, PTg, 1 + g,
-                   n_cons);
+        produce<4>(pv, cix, e_begin, e_end, smem + slot * slot_bytes, hdr[slot], pt, PTg, 1 + g);
         mbar_arrive(&full_bar[slot]);
         slot += ng;
         if (slot >= nslots) {
