@@ -314,7 +314,9 @@ def bench_support(a, tc, g, info, src, dst, n, gen_s, build_wall_ms, world, rank
     else:
         cpu = None
     hbm, peak_src = peaks()
-    b = int(info.b_itc) + 4 * m + 24 * T
+    # the count's method bytes + the zeroed output + a 4-B read-modify-write for
+    # each of the 3 edges of every triangle (random u32 atomics in L2: 3T of them)
+    b = int(info.method_bytes) + 4 * m + 24 * T
     achieved = b / (ms / 1e3) / 1e9
     line = {
         "metric": METRIC + " (per-edge support)", "value": m / (ms / 1e3), "unit": UNIT,
@@ -327,8 +329,13 @@ def bench_support(a, tc, g, info, src, dst, n, gen_s, build_wall_ms, world, rank
         "triangles": str(T), "parity_vs_oracle": parity,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                      "frac": achieved / hbm, "traffic": None, "bytes_per_launch": b,
-                     "bytes_def": "B_ITC + 4m (zero-init) + 24T (3 u32 read-modify-writes "
-                                  "per triangle)", "peak_source": peak_src},
+                     "kernel": "k_support (both classes)", "kernel_ms": ms,
+                     "bytes_def": "method bytes (tc_graph_info.method_bytes) + 4m (zero-init) + "
+                                  "24T (3 u32 read-modify-writes per triangle)",
+                     "atomics_per_s": 3 * T / (ms / 1e3),
+                     "note": "bound by the L2's random u32 atomics (3 per triangle, the (u,v) ones "
+                             "aggregated per tile run in the long class)",
+                     "peak_source": peak_src},
         "gpu_launches": a.steps * 2,
         "build_ms": {"wall": build_wall_ms, "total_events": info.ms_total},
         "clocks": clocks, "gen_s": round(gen_s, 2), "step_ms": step_ms,

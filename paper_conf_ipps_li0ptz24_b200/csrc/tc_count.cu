@@ -56,9 +56,6 @@ constexpr int kUnrollLong = 8;   // tail batch of the long class
 #define TC_BATCH_LONG 8
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
-#ifndef TC_SUP_L2PF
-#define TC_SUP_L2PF 0  // walk_long_sup: L2 prefetch of the next batch's key lines (A/B knob)
-#endif
 #ifndef TC_PF_SHORT
 #define TC_PF_SHORT 1  // produce: L2 prefetch of every short-class edge's keys at staging (r2y: C2 -1.6%)
 #endif
@@ -644,17 +641,6 @@ __device__ __forceinline__ void walk_long_sup(const ChunkSmem& c, int t0, int t1
   uint32_t cur = 0u;
 #endif
   for (int t = t0; t < t1; t += kUnrollSup) {
-#if TC_SUP_L2PF
-    // the next batch's key lines toward L2 (as walk_long): lane u < kUnrollSup
-    // tile u's first line, lane 16 + u its last
-    {
-      const int q = lane & 15;
-      if (q < kUnrollSup && t + kUnrollSup + q < t1) {
-        const uint32_t x = (uint32_t)c.sT0[t + kUnrollSup + q] + (lane >= 16 ? 31u : 0u);
-        if (lane < 16 || x < (uint32_t)pv.m) asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + x));
-      }
-    }
-#endif
     int32_t key[kUnrollSup];
     uint32_t p[kUnrollSup], vr[kUnrollSup], own[kUnrollSup];
     int g6[kUnrollSup];
