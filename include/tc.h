@@ -82,8 +82,8 @@ typedef struct {
   int32_t huge_degree;  /* d+(v) above which N+(v) is probed in global memory by
                            binary search instead of an SMEM hash (default 8192)    */
   int32_t block_threads;/* threads per CTA of the long-class count kernel,
-                           64..1024; 1/5 of the warps build tables, the rest probe
-                           (default 1024)                                          */
+                           64..1024; 1/4 of the warps (TC_PROD_DIV) build tables in
+                           two groups, the rest probe (default 1024)                                          */
   int32_t table_factor; /* hash slots = table_factor * d+(v) (rounded up to a
                            multiple of 4), 2..16 (default 6, i.e. load <= 1/6)     */
   int32_t long_min;     /* trimmed suffixes with >= long_min keys go to the

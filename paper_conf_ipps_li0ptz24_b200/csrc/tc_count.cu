@@ -11,8 +11,9 @@
 // cost, covering a run of groups.  Two kernels, one per class:
 //   k_count (LONG class, suffix >= long_min keys): one persistent 1024-thread
 //   CTA per SM, warp-specialised, with three chunk slots in shared memory.
-//   PRODUCER warps (1/5 of the CTA) stage the CTA's next chunk into a free
-//     slot: its edges, its per-32-key tile descriptors, and one table per
+//   PRODUCER warps (1/4 of the CTA, in two groups that fill alternate
+//     chunks concurrently) stage the CTA's next chunks into free
+//     slots: each chunk's edges, its per-32-key tile descriptors, and one table per
 //     group built from N+(v) (the GroupTC idea of a table shared by a block
 //     of edges): a bitmap of N+(v)'s rank window (one probe per key)
 //     or a two-choice (cuckoo) hash, as in TRUST, instead of the
