@@ -1101,6 +1101,8 @@ Tuning tuning_from_env() {
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
   t.batch = get("TC_BATCH", t.batch, 0, 64);
   t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 3);
+  t.short_ws = get("TC_SHORT_WS", t.short_ws, 0, 1);
+  t.prod_div_short = get("TC_PROD_DIV_SHORT", t.prod_div_short, 2, 32);
   return t;
 }
 

@@ -153,6 +153,8 @@ struct Tuning {
   int batch = 0;          // long-class tiles per batch for block_threads <= 768 (TC_BATCH; see count_kernel)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
+  int short_ws = 0;       // short class on the warp-specialised kernel instead of k_count_flat (TC_SHORT_WS)
+  int prod_div_short = 2; // ... with 1/prod_div_short of its warps producing (TC_PROD_DIV_SHORT)
 };
 Tuning tuning_from_env();
 

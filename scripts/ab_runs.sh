@@ -184,6 +184,13 @@ r3b)
     -o $O/r3b_c3_count python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e --no-sharded --no-balance > $O/r3b_ncu.log 2>&1
   python -c "import bench; print(bench.src_hash())" > $O/r3b_src_hash.txt
   ;;
+r4b)
+  # short class on the warp-specialised kernel (TC_SHORT_WS) vs k_count_flat
+  TC_SHORT_WS=1 timeout 900 python -m pytest -q -x tests/test_gpu_parity.py -k "closed_forms or c1_rmat10 or rmat_medium or options or karate or golden or c2_chung or c5_lattice or chung_lu_small or partition or ranges or huge or cap" > $O/r4b_pytest_short_ws.txt 2>&1; echo "rc=$?" >> $O/r4b_pytest_short_ws.txt
+  for c in C2 C5 C3; do
+    bash scripts/gpu_ab.sh r4b_$c $c 10 "" "TC_SHORT_WS=1" "TC_SHORT_WS=1 TC_PROD_DIV_SHORT=3" "TC_SHORT_WS=1 TC_PROD_DIV_SHORT=4" "TC_SHORT_WS=1 TC_PROD_DIV_SHORT=2 TC_PROD_GROUPS=3" ""
+  done
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
