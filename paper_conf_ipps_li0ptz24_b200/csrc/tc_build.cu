@@ -65,6 +65,36 @@ struct Trace {
   }
 };
 
+// The build's large sorts: tc_sort.cu's radix sort (TC_SORT=cub: CUB's onesweep,
+// the only choice at or above 2^32 keys or below 2^20, where launch count matters).
+bool own_sort(int64_t n) {
+  static const bool cub_only = [] {
+    const char* v = std::getenv("TC_SORT");
+    return v && std::string(v) == "cub";
+  }();
+  return !cub_only && n >= (int64_t(1) << 20) && n < (int64_t(1) << 32);
+}
+
+void sort_keys_u64(cub::DoubleBuffer<uint64_t>& db, int64_t n, int end_bit, cudaStream_t s) {
+  if (own_sort(n)) {
+    if (radix_sort_keys(db.Current(), db.Alternate(), n, 0, end_bit, s)) db.selector ^= 1;
+    return;
+  }
+  cub_run(s, [&](void* t, size_t& b) { return cub::DeviceRadixSort::SortKeys(t, b, db, n, 0, end_bit, s); });
+}
+
+void sort_pairs_u32_u64(cub::DoubleBuffer<uint32_t>& dk, cub::DoubleBuffer<uint64_t>& dv, int64_t n,
+                        int end_bit, cudaStream_t s) {
+  if (own_sort(n)) {
+    if (radix_sort_pairs(dk.Current(), dk.Alternate(), dv.Current(), dv.Alternate(), n, 0, end_bit, s)) {
+      dk.selector ^= 1;
+      dv.selector ^= 1;
+    }
+    return;
+  }
+  cub_run(s, [&](void* t, size_t& b) { return cub::DeviceRadixSort::SortPairs(t, b, dk, dv, n, 0, end_bit, s); });
+}
+
 template <class T>
 T d2h(const T* d, cudaStream_t s) {
   T h;
@@ -258,13 +288,15 @@ __global__ void k_rowid(const int64_t* __restrict__ row_ptr, int64_t n,
     for (int64_t p = row_ptr[u], e = row_ptr[u + 1]; p < e; ++p) rowid[p] = (int32_t)u;
 }
 
-// Per row v: {min N+(v), max N+(v)} (rows are sorted), {INT_MAX, -1} if empty.
+// Per row v: {min N+(v), max N+(v), d+(v), 0} (rows are sorted), {INT_MAX,
+// -1, 0, 0} if empty: the one 16-B record k_edge_trim reads at random per edge
+// (instead of row_ptr[v], row_ptr[v+1] and the two ends in col).
 __global__ void k_vmm(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                      int64_t n, int2* __restrict__ vmm) {
+                      int64_t n, int4* __restrict__ vmm) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
        v += (int64_t)gridDim.x * blockDim.x) {
     const int64_t a = row_ptr[v], b = row_ptr[v + 1];
-    vmm[v] = b > a ? make_int2(col[a], col[b - 1]) : make_int2(0x7fffffff, -1);
+    vmm[v] = b > a ? make_int4(col[a], col[b - 1], (int)(b - a), 0) : make_int4(0x7fffffff, -1, 0, 0);
   }
 }
 
@@ -295,7 +327,7 @@ __device__ __forceinline__ int64_t upper_bound_i32(const int32_t* __restrict__ a
 // (untrimmed), [1] trimmed keys, [2] live, [3] live long,
 // [4] trimmed keys of the long class.
 __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                            const int32_t* __restrict__ rowid, const int2* __restrict__ vmm,
+                            const int32_t* __restrict__ rowid, const int4* __restrict__ vmm,
                             int64_t m, int long_min, int bits,
                             uint32_t dead, uint32_t* __restrict__ skey, uint64_t* __restrict__ sval,
                             unsigned long long* stats) {
@@ -306,11 +338,10 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
        p += (int64_t)gridDim.x * blockDim.x) {
     const int32_t u = rowid[p], v = col[p];
     const int64_t rend = row_ptr[u + 1], suf = rend - p - 1;
-    const int64_t rv = row_ptr[v], dv = row_ptr[v + 1] - rv;
-    b += 4ull * (unsigned long long)(suf + dv) + 12ull;
+    const int4 w = vmm[v];  // {min N+(v), max N+(v), d+(v)}
+    b += 4ull * (unsigned long long)(suf + w.z) + 12ull;
     int64_t lo = p + 1, len = 0;
-    if (suf > 0 && dv > 0) {
-      const int2 w = vmm[v];  // [min N+(v), max N+(v)]: one 8-B read instead of two in col
+    if (suf > 0 && w.z > 0) {
       lo = lower_bound_i32(col, p + 1, rend, w.x);
       len = upper_bound_i32(col, lo, rend, w.y) - lo;
     }
@@ -655,9 +686,7 @@ uint64_t* canon_unique(const int32_t* d_src, const int32_t* d_dst, int64_t m_gen
   uint64_t* ukey = ka;
   if (m_gen > 0) {
     cub::DoubleBuffer<uint64_t> db(ka, kb);
-    cub_run(s, [&](void* t, size_t& b) {
-      return cub::DeviceRadixSort::SortKeys(t, b, db, m_gen, 0, 2 * bits, s);
-    });
+    sort_keys_u64(db, m_gen, 2 * bits, s);
     uint64_t* sorted = db.Current();
     uint64_t* other = sorted == ka ? kb : ka;
     cub_run(s, [&](void* t, size_t& b) {
@@ -795,9 +824,7 @@ static void build_tail(uint64_t* ukey, int64_t m, DevBuf<uint64_t>& ka, DevBuf<u
     k_orient<<<grid_for(m), TPB, 0, s>>>(ukey, m, bits, rank.get(), bits2, okey_a);
     TC_LAUNCH();
     cub::DoubleBuffer<uint64_t> db(okey_a, ukey);
-    cub_run(s, [&](void* t, size_t& b) {
-      return cub::DeviceRadixSort::SortKeys(t, b, db, m, 0, 2 * bits2, s);
-    });
+    sort_keys_u64(db, m, 2 * bits2, s);
     csr_from_sorted(db.Current(), m, n_act, s, g);
   } else {
     csr_from_sorted(nullptr, 0, n_act, s, g);
@@ -940,9 +967,7 @@ void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen,
                                         ka.get() + lo[i], err.get());
     TC_LAUNCH();
     cub::DoubleBuffer<uint64_t> db(ka.get() + lo[i], kb.get() + lo[i]);
-    cub_run(s, [&](void* t, size_t& b) {
-      return cub::DeviceRadixSort::SortKeys(t, b, db, c, 0, 2 * bits, s);
-    });
+    sort_keys_u64(db, c, 2 * bits, s);
     if (db.Current() != ka.get() + lo[i])
       TC_CUDA(cudaMemcpyAsync(ka.get() + lo[i], db.Current(), sizeof(uint64_t) * c,
                               cudaMemcpyDeviceToDevice, s));
@@ -1013,9 +1038,7 @@ void sort_keys(uint64_t* keys, int64_t cnt, int64_t n, cudaStream_t s) {
   if (cnt <= 1) return;
   DevBuf<uint64_t> kb(cnt, s);
   cub::DoubleBuffer<uint64_t> db(keys, kb.get());
-  cub_run(s, [&](void* t, size_t& b) {
-    return cub::DeviceRadixSort::SortKeys(t, b, db, cnt, 0, 2 * key_bits(n), s);
-  });
+  sort_keys_u64(db, cnt, 2 * key_bits(n), s);
   if (db.Current() != keys)
     TC_CUDA(cudaMemcpyAsync(keys, db.Current(), sizeof(uint64_t) * cnt, cudaMemcpyDeviceToDevice, s));
 }
@@ -1026,9 +1049,7 @@ int64_t shard_unique(uint64_t* keys, int64_t cnt, int64_t n, cudaStream_t s, int
   DevBuf<uint64_t> kb(cnt, s);
   DevBuf<int64_t> nsel(1, s);
   cub::DoubleBuffer<uint64_t> db(keys, kb.get());
-  cub_run(s, [&](void* t, size_t& b) {
-    return cub::DeviceRadixSort::SortKeys(t, b, db, cnt, 0, 2 * bits, s);
-  });
+  sort_keys_u64(db, cnt, 2 * bits, s);
   uint64_t* sorted = db.Current();
   uint64_t* other = sorted == keys ? kb.get() : keys;
   cub_run(s, [&](void* t, size_t& b) {
@@ -1101,8 +1122,6 @@ Tuning tuning_from_env() {
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
   t.batch = get("TC_BATCH", t.batch, 0, 64);
   t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 3);
-  t.short_ws = get("TC_SHORT_WS", t.short_ws, 0, 1);
-  t.prod_div_short = get("TC_PROD_DIV_SHORT", t.prod_div_short, 2, 32);
   return t;
 }
 
@@ -1137,7 +1156,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
       k_rowid<<<grid_for(n), TPB, 0, s>>>(row_ptr, n, rowid.get());
       TC_LAUNCH();
     }
-    DevBuf<int2> vmm(std::max<int64_t>(n, 1), s);
+    DevBuf<int4> vmm(std::max<int64_t>(n, 1), s);
     k_vmm<<<grid_for(n), TPB, 0, s>>>(row_ptr, col, n, vmm.get());
     TC_LAUNCH();
     // a long-class tile always holds 32 keys of its own edge (walk_long shifts
@@ -1178,9 +1197,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   // and the edges arrive in position order; dead edges sort past S
   cub::DoubleBuffer<uint32_t> dk(skey.get(), skey2.get());
   cub::DoubleBuffer<uint64_t> dv(sval.get(), sval2.get());
-  cub_run(s, [&](void* t, size_t& b) {
-    return cub::DeviceRadixSort::SortPairs(t, b, dk, dv, m, 0, end_bit, s);
-  });
+  sort_pairs_u32_u64(dk, dv, m, end_bit, s);
   const uint32_t* key_sorted = dk.Current();
   const uint64_t* val_sorted = dv.Current();
   tr("select + class sort");

@@ -1337,19 +1337,7 @@ int count_chunks(const tc_graph* g, int64_t c_begin, int64_t c_end, int64_t e_be
                              (size_t)(P.tune.slots * sb), s));
     ++launched;
   }
-  if (s1 > s0 && P.tune.short_ws) {
-    // short class on the warp-specialised kernel (consume() takes walk_short)
-    Tuning tu = P.tune;
-    tu.prod_div = tu.prod_div_short;
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(s1 - s0, (int64_t)num_sms()));
-    const int64_t sb = slot_bytes_of(std::max(P.smem_bytes, P.smem_flat));
-    const FuseArgs& fa = fuse ? *fuse : none;
-    void* args[] = {(void*)&pv, (void*)&s0, (void*)&s1, (void*)&e_begin, (void*)&e_end,
-                    (void*)&sb, (void*)&tu, (void*)&d_out, (void*)&fa};
-    TC_CUDA(cudaLaunchKernel(count_kernel(P.block, tu.batch), dim3(grid), dim3(P.block), args,
-                             (size_t)(tu.slots * sb), s));
-    ++launched;
-  } else if (s1 > s0) {
+  if (s1 > s0) {
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(s1 - s0, P.grid_flat));
     k_count_flat<<<grid, kFlatBlock, (size_t)slot_bytes_of(P.smem_flat), s>>>(
         pv, s0, s1, e_begin, e_end, d_out, fuse ? *fuse : none);

@@ -71,6 +71,14 @@ struct DevBuf {
   T* get() const { return p; }
 };
 
+// ---------------------------------------------------------------- sort
+// tc_sort.cu: stable LSD radix sort (8-bit digits, reduce-then-scan) of n <
+// 2^32 keys on bits [begin_bit, end_bit); ping-pongs between the two buffers
+// and returns true when the result is in the second one.
+bool radix_sort_keys(uint64_t* k0, uint64_t* k1, int64_t n, int begin_bit, int end_bit, cudaStream_t s);
+bool radix_sort_pairs(uint32_t* k0, uint32_t* k1, uint64_t* v0, uint64_t* v1, int64_t n, int begin_bit,
+                      int end_bit, cudaStream_t s);
+
 // ---------------------------------------------------------------- options
 struct Options {
   int chunk_cost = 16384;
@@ -153,8 +161,6 @@ struct Tuning {
   int batch = 0;          // long-class tiles per batch for block_threads <= 768 (TC_BATCH; see count_kernel)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
-  int short_ws = 0;       // short class on the warp-specialised kernel instead of k_count_flat (TC_SHORT_WS)
-  int prod_div_short = 2; // ... with 1/prod_div_short of its warps producing (TC_PROD_DIV_SHORT)
 };
 Tuning tuning_from_env();
 

@@ -191,6 +191,23 @@ r4b)
     bash scripts/gpu_ab.sh r4b_$c $c 10 "" "TC_SHORT_WS=1" "TC_SHORT_WS=1 TC_PROD_DIV_SHORT=3" "TC_SHORT_WS=1 TC_PROD_DIV_SHORT=4" "TC_SHORT_WS=1 TC_PROD_DIV_SHORT=2 TC_PROD_GROUPS=3" ""
   done
   ;;
+r4c)
+  # flat-kernel shape and next-chunk plan prefetch (compile-time); packed 16-B trim record in the build
+  timeout 900 python -m pytest -q -x tests/test_gpu_parity.py -k "csr_exact or host or dedup or options or c2_chung or c5_lattice or full_size" > $O/r4c_pytest.txt 2>&1; echo "rc=$?" >> $O/r4c_pytest.txt
+  timeout 600 python bench.py --steps 10 --warmup 3 --no-sharded --no-balance --out $O/r4c_bench_c3.json > $O/r4c_bench_c3.log 2>&1
+  for c in C2 C5 C3; do
+    bash scripts/gpu_abbuild.sh r4c_$c $c 10 "" "-DTC_FLAT_PF=1" "-DTC_FLAT_BLOCK=256 -DTC_FLAT_CTAS=6" "-DTC_FLAT_BLOCK=192 -DTC_FLAT_CTAS=8" "-DTC_FLAT_BLOCK=512 -DTC_FLAT_CTAS=3" "-DTC_FLAT_PF=1 -DTC_FLAT_BLOCK=256 -DTC_FLAT_CTAS=6" ""
+  done
+  ;;
+r4d)
+  # tc_sort.cu radix sort vs CUB onesweep: microbenchmark, parity, build / e2e A/B at C3
+  timeout 600 build/sort_bench > $O/r4d_sort_bench.txt 2>&1; echo "rc=$?" >> $O/r4d_sort_bench.txt
+  timeout 1500 python -m pytest -q -x tests/test_gpu_parity.py tests/test_gpu_sharded.py > $O/r4d_pytest.txt 2>&1; echo "rc=$?" >> $O/r4d_pytest.txt
+  i=0; for kv in "" "TC_SORT=cub" ""; do
+    i=$((i+1)); tag=${i}_$(echo "${kv:-own}" | tr ' =' '__')
+    env $kv timeout 900 python bench.py --steps 10 --warmup 3 --no-balance --out $O/r4d_bench_c3_$tag.json > $O/r4d_bench_c3_$tag.log 2>&1
+  done
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt

@@ -1,0 +1,263 @@
+// Radix-sort policy sweep for the build's three big sorts (a2/a5: 64-bit keys
+// with 2*24 significant bits; a6: 32-bit key of 26 bits with a 64-bit value).
+// Dev tool, not part of the product:
+//   nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -o build/sort_bench scripts/sort_bench.cu
+//   build/sort_bench [n_keys]
+// Times each policy with CUDA events (median of 5 after a warm-up) and checks
+// its output against the default policy's.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <stdexcept>
+
+// the product's sort (tc_sort.cu) with minimal stand-ins for libtc's allocator / error hooks
+#include "../paper_conf_ipps_li0ptz24_b200/csrc/tc_sort.cu"
+namespace tc {
+void* dev_alloc(size_t bytes, cudaStream_t, bool) {
+  void* p = nullptr;
+  if (cudaMalloc(&p, bytes) != cudaSuccess) throw std::runtime_error("oom");
+  return p;
+}
+void dev_free(void* p, size_t, cudaStream_t) { cudaFree(p); }
+void check_cuda(cudaError_t e, const char* what, const char* file, int line) {
+  if (e != cudaSuccess) {
+    printf("CUDA %s: %s at %s:%d\n", cudaGetErrorString(e), what, file, line);
+    exit(1);
+  }
+}
+[[noreturn]] void fail(tc_status, const std::string& m) { throw std::runtime_error(m); }
+}  // namespace tc
+#include <cstdio>
+#include <vector>
+
+#define CK(x)                                                                 \
+  do {                                                                        \
+    cudaError_t e_ = (x);                                                     \
+    if (e_ != cudaSuccess) {                                                  \
+      printf("CUDA %s at %s:%d\n", cudaGetErrorString(e_), __FILE__, __LINE__); \
+      exit(1);                                                                \
+    }                                                                         \
+  } while (0)
+
+__global__ void k_fill64(uint64_t* k, int64_t n, int bits, uint64_t seed) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t z = (uint64_t)i * 0x9E3779B97F4A7C15ull + seed;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    k[i] = z & ((1ull << bits) - 1);
+  }
+}
+__global__ void k_fill32(uint32_t* k, uint64_t* v, int64_t n, int bits, uint64_t seed) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t z = (uint64_t)i * 0x9E3779B97F4A7C15ull + seed;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    k[i] = (uint32_t)(z & ((1ull << bits) - 1));
+    v[i] = (uint64_t)i;
+  }
+}
+
+using OffsetT = unsigned long long;
+
+template <class K, class V, bool kOnesweep, int kThreads, int kItems, int kBits>
+struct Hub {
+  using Base = typename cub::detail::radix::policy_hub<K, V, OffsetT>::Policy1000;
+  using DominantT = ::cuda::std::_If<(sizeof(V) > sizeof(K)), V, K>;
+  struct P : cub::ChainedPolicy<1000, P, P> {
+    static constexpr bool ONESWEEP = kOnesweep;
+    static constexpr int ONESWEEP_RADIX_BITS = kBits;
+    using HistogramPolicy = cub::AgentRadixSortHistogramPolicy<128, 16, 1, K, kBits>;
+    using ExclusiveSumPolicy = cub::AgentRadixSortExclusiveSumPolicy<256, kBits>;
+    using OnesweepPolicy =
+        cub::AgentRadixSortOnesweepPolicy<kThreads, kItems, DominantT, 1, cub::RADIX_RANK_MATCH_EARLY_COUNTS_ANY,
+                                          cub::BLOCK_SCAN_RAKING_MEMOIZE, cub::RADIX_SORT_STORE_DIRECT, kBits>;
+    using ScanPolicy = typename Base::ScanPolicy;
+    using DownsweepPolicy =
+        cub::AgentRadixSortDownsweepPolicy<kThreads, kItems, DominantT, cub::BLOCK_LOAD_TRANSPOSE, cub::LOAD_DEFAULT,
+                                           cub::RADIX_RANK_MATCH, cub::BLOCK_SCAN_WARP_SCANS, kBits>;
+    using AltDownsweepPolicy = DownsweepPolicy;
+    using UpsweepPolicy = cub::AgentRadixSortUpsweepPolicy<kThreads, kItems, DominantT, cub::LOAD_DEFAULT, kBits>;
+    using AltUpsweepPolicy = UpsweepPolicy;
+    using SingleTilePolicy = typename Base::SingleTilePolicy;
+    using SegmentedPolicy = typename Base::SegmentedPolicy;
+    using AltSegmentedPolicy = typename Base::AltSegmentedPolicy;
+  };
+  using MaxPolicy = P;
+};
+
+template <class K, class V, class H>
+float run(cub::DoubleBuffer<K>& dk, cub::DoubleBuffer<V>& dv, int64_t n, int end_bit, void* tmp, size_t& tb,
+          cudaStream_t s) {
+  using D = cub::DispatchRadixSort<false, K, V, OffsetT, H>;
+  size_t need = 0;
+  CK(D::Dispatch(nullptr, need, dk, dv, (OffsetT)n, 0, end_bit, true, s));
+  if (need > tb) {
+    printf("temp %zu > %zu\n", need, tb);
+    return -1;
+  }
+  cudaEvent_t a, b;
+  CK(cudaEventCreate(&a));
+  CK(cudaEventCreate(&b));
+  CK(cudaEventRecord(a, s));
+  CK(D::Dispatch(tmp, need, dk, dv, (OffsetT)n, 0, end_bit, true, s));
+  CK(cudaEventRecord(b, s));
+  CK(cudaEventSynchronize(b));
+  float ms = 0;
+  CK(cudaEventElapsedTime(&ms, a, b));
+  return ms;
+}
+
+template <class K, class V, class H>
+void bench(const char* name, K* k0, K* k1, V* v0, V* v1, const K* src_k, const V* src_v, const K* ref, int64_t n,
+           int end_bit, void* tmp, size_t tb, cudaStream_t s) {
+  std::vector<float> t;
+  const K* out = nullptr;
+  for (int r = 0; r < 6; ++r) {
+    CK(cudaMemcpyAsync(k0, src_k, sizeof(K) * n, cudaMemcpyDeviceToDevice, s));
+    if (v0) CK(cudaMemcpyAsync(v0, src_v, sizeof(V) * n, cudaMemcpyDeviceToDevice, s));
+    cub::DoubleBuffer<K> dk(k0, k1);
+    cub::DoubleBuffer<V> dv(v0, v1);
+    float ms = run<K, V, H>(dk, dv, n, end_bit, tmp, tb, s);
+    if (ms < 0) return;
+    if (r) t.push_back(ms);
+    out = dk.Current();
+  }
+  std::sort(t.begin(), t.end());
+  bool ok = true;
+  if (ref) {
+    std::vector<K> a(1 << 20), b(1 << 20);
+    for (int64_t off : {int64_t(0), n / 2, n - (1 << 20)}) {
+      CK(cudaMemcpy(a.data(), out + off, sizeof(K) << 20, cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(b.data(), ref + off, sizeof(K) << 20, cudaMemcpyDeviceToHost));
+      ok = ok && a == b;
+    }
+  }
+  const double bytes = 2.0 * (sizeof(K) + (v0 ? sizeof(V) : 0)) * n;
+  printf("%-44s median %8.3f ms  (%.2f TB/s per %d-bit pass equivalent)  %s\n", name, t[t.size() / 2],
+         bytes * ((end_bit + 7) / 8) / (t[t.size() / 2] * 1e9), 8, ref ? (ok ? "same" : "DIFFERENT") : "ref");
+}
+
+template <class K, class V>
+void bench_own(const char* name, K* k0, K* k1, V* v0, V* v1, const K* src_k, const V* src_v, const K* ref,
+               const V* ref_v, int64_t n, int end_bit, cudaStream_t s) {
+  std::vector<float> t;
+  const K* out = nullptr;
+  const V* outv = nullptr;
+  cudaEvent_t a, b;
+  CK(cudaEventCreate(&a));
+  CK(cudaEventCreate(&b));
+  for (int r = 0; r < 6; ++r) {
+    CK(cudaMemcpyAsync(k0, src_k, sizeof(K) * n, cudaMemcpyDeviceToDevice, s));
+    if (v0) CK(cudaMemcpyAsync(v0, src_v, sizeof(V) * n, cudaMemcpyDeviceToDevice, s));
+    CK(cudaEventRecord(a, s));
+    bool alt;
+    if constexpr (sizeof(K) == 8) alt = tc::radix_sort_keys((uint64_t*)k0, (uint64_t*)k1, n, 0, end_bit, s);
+    else alt = tc::radix_sort_pairs((uint32_t*)k0, (uint32_t*)k1, (uint64_t*)v0, (uint64_t*)v1, n, 0, end_bit, s);
+    CK(cudaEventRecord(b, s));
+    CK(cudaEventSynchronize(b));
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, a, b));
+    if (r) t.push_back(ms);
+    out = alt ? k1 : k0;
+    outv = alt ? v1 : v0;
+  }
+  std::sort(t.begin(), t.end());
+  bool ok = true;
+  std::vector<K> x(1 << 20), y(1 << 20);
+  for (int64_t off : {int64_t(0), n / 3, n / 2, n - (1 << 20)}) {
+    CK(cudaMemcpy(x.data(), out + off, sizeof(K) << 20, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(y.data(), ref + off, sizeof(K) << 20, cudaMemcpyDeviceToHost));
+    ok = ok && x == y;
+    if (ref_v && v0) {
+      std::vector<V> xv(1 << 20), yv(1 << 20);
+      CK(cudaMemcpy(xv.data(), outv + off, sizeof(V) << 20, cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(yv.data(), ref_v + off, sizeof(V) << 20, cudaMemcpyDeviceToHost));
+      ok = ok && xv == yv;
+    }
+  }
+  printf("%-44s median %8.3f ms  %s\n", name, t[t.size() / 2], ok ? "same" : "DIFFERENT");
+}
+
+int main(int argc, char** argv) {
+  const int64_t n = argc > 1 ? atoll(argv[1]) : 268435456ll;
+  cudaStream_t s;
+  CK(cudaStreamCreate(&s));
+  size_t tb = (size_t)3 << 30;
+  void* tmp;
+  CK(cudaMalloc(&tmp, tb));
+  {  // a2 / a5: 64-bit keys, 48 significant bits
+    uint64_t *src, *k0, *k1, *ref;
+    CK(cudaMalloc(&src, 8 * n));
+    CK(cudaMalloc(&k0, 8 * n));
+    CK(cudaMalloc(&k1, 8 * n));
+    CK(cudaMalloc(&ref, 8 * n));
+    k_fill64<<<148 * 16, 256, 0, s>>>(src, n, 48, 1);
+    using N = cub::NullType;
+    N* nv = nullptr;
+    bench<uint64_t, N, typename cub::detail::radix::policy_hub<uint64_t, N, OffsetT>>(
+        "u64 keys 48b: default", k0, k1, nv, nv, src, nv, nullptr, n, 48, tmp, tb, s);
+    {
+      cub::DoubleBuffer<uint64_t> dk(k0, k1);
+      cub::DoubleBuffer<N> dv(nv, nv);
+      CK(cudaMemcpyAsync(k0, src, 8 * n, cudaMemcpyDeviceToDevice, s));
+      run<uint64_t, N, typename cub::detail::radix::policy_hub<uint64_t, N, OffsetT>>(dk, dv, n, 48, tmp, tb, s);
+      CK(cudaMemcpyAsync(ref, dk.Current(), 8 * n, cudaMemcpyDeviceToDevice, s));
+    }
+#define B64(OS, T, I, BITS) \
+  bench<uint64_t, N, Hub<uint64_t, N, OS, T, I, BITS>>("u64 keys 48b: " #OS " " #T "x" #I " " #BITS "b", k0, k1, nv, nv, src, nv, ref, n, 48, tmp, tb, s)
+    bench_own<uint64_t, N>("u64 keys 48b: tc_sort", k0, k1, nv, nv, src, nv, ref, nullptr, n, 48, s);
+    B64(true, 384, 30, 8);
+    B64(true, 512, 22, 8);
+    B64(true, 256, 44, 8);
+    B64(true, 384, 30, 6);
+    B64(true, 384, 30, 7);
+    B64(false, 256, 23, 7);
+    B64(false, 256, 23, 6);
+    CK(cudaFree(src));
+    CK(cudaFree(k0));
+    CK(cudaFree(k1));
+    CK(cudaFree(ref));
+  }
+  {  // a6: 32-bit key (26 bits) + 64-bit value
+    uint32_t *src, *k0, *k1, *ref;
+    uint64_t *vs, *v0, *v1;
+    CK(cudaMalloc(&src, 4 * n));
+    CK(cudaMalloc(&k0, 4 * n));
+    CK(cudaMalloc(&k1, 4 * n));
+    CK(cudaMalloc(&ref, 4 * n));
+    CK(cudaMalloc(&vs, 8 * n));
+    CK(cudaMalloc(&v0, 8 * n));
+    CK(cudaMalloc(&v1, 8 * n));
+    k_fill32<<<148 * 16, 256, 0, s>>>(src, vs, n, 26, 2);
+    bench<uint32_t, uint64_t, typename cub::detail::radix::policy_hub<uint32_t, uint64_t, OffsetT>>(
+        "u32 key 26b + u64 value: default", k0, k1, v0, v1, src, vs, nullptr, n, 26, tmp, tb, s);
+    {
+      cub::DoubleBuffer<uint32_t> dk(k0, k1);
+      cub::DoubleBuffer<uint64_t> dv(v0, v1);
+      CK(cudaMemcpyAsync(k0, src, 4 * n, cudaMemcpyDeviceToDevice, s));
+      CK(cudaMemcpyAsync(v0, vs, 8 * n, cudaMemcpyDeviceToDevice, s));
+      run<uint32_t, uint64_t, typename cub::detail::radix::policy_hub<uint32_t, uint64_t, OffsetT>>(dk, dv, n, 26, tmp, tb, s);
+      CK(cudaMemcpyAsync(ref, dk.Current(), 4 * n, cudaMemcpyDeviceToDevice, s));
+      CK(cudaMemcpyAsync(vs, dv.Current(), 8 * n, cudaMemcpyDeviceToDevice, s));  // sorted values (ref)
+      k_fill32<<<148 * 16, 256, 0, s>>>(src, v1, n, 26, 2);                       // v1 = unsorted values
+      CK(cudaMemcpyAsync(v0, v1, 8 * n, cudaMemcpyDeviceToDevice, s));
+    }
+    uint64_t* refv = nullptr;
+    CK(cudaMalloc(&refv, 8 * n));
+    CK(cudaMemcpyAsync(refv, vs, 8 * n, cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(vs, v1, 8 * n, cudaMemcpyDeviceToDevice, s));  // vs = unsorted values again
+    bench_own<uint32_t, uint64_t>("u32k+u64v 26b: tc_sort", k0, k1, v0, v1, src, vs, ref, refv, n, 26, s);
+#define B32(OS, T, I, BITS)                                                                                     \
+  bench<uint32_t, uint64_t, Hub<uint32_t, uint64_t, OS, T, I, BITS>>("u32k+u64v 26b: " #OS " " #T "x" #I " " #BITS "b", \
+                                                                     k0, k1, v0, v1, src, vs, ref, n, 26, tmp, tb, s)
+    B32(true, 384, 24, 8);
+    B32(true, 384, 28, 8);
+    B32(true, 512, 18, 8);
+    B32(true, 384, 24, 7);
+    B32(true, 384, 24, 9);
+    B32(false, 256, 23, 7);
+  }
+  return 0;
+}

@@ -404,6 +404,34 @@ def test_dedup_paths_agree(tc):
     assert int(out["sort"][1]) == oracle.triangles(src, dst)
 
 
+@pytest.mark.parametrize("scale,ef,seed", [(18, 16, 3), (20, 8, 4)])
+def test_sort_paths_agree(tc, scale, ef, seed):
+    """The build's radix sort (tc_sort.cu: a2, a5, a6 above 2^20 keys) and
+    CUB's onesweep (forced with TC_SORT=cub in a child process) build the same
+    CSR, B_ITC and count.  Scale 18 sorts 36-bit keys in 5 passes (the result
+    lands in the second buffer), scale 20 in 5 / 6."""
+    import subprocess
+    import sys
+    src, dst, n = tcgen.rmat(scale, ef, seed)
+    assert len(src) >= (1 << 20)
+    code = ("import sys, hashlib, numpy as np, torch; sys.path.insert(0, %r); import tcgen;"
+            "import paper_conf_ipps_li0ptz24_b200 as tc;"
+            "s, d, n = tcgen.rmat(%d, %d, %d);"
+            "g = tc.build_csr(torch.from_numpy(s).cuda(), torch.from_numpy(d).cuda(), n);"
+            "h = hashlib.sha256(); [h.update(x.cpu().numpy().tobytes()) for x in g.csr()];"
+            "print(h.hexdigest(), g.info.b_itc, g.info.keys_total, g.count())") % (ROOT, scale, ef, seed)
+    out = {}
+    for mode, env_kv in (("own", {}), ("cub", {"TC_SORT": "cub"})):
+        env = dict(os.environ, **env_kv)
+        env.pop("TC_SORT", None) if mode == "own" else None
+        r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                           timeout=300)
+        assert r.returncode == 0, r.stderr[-2000:]
+        out[mode] = r.stdout.split()[-4:]
+    assert out["own"] == out["cub"]
+    assert int(out["own"][3]) == oracle.triangles(src, dst)
+
+
 def test_host_pipelined_build_equals_device(tc):
     """Above 2^25 pairs tc_build_csr_host overlaps the H2D copy of piece i+1
     with the sort of piece i and merges the sorted runs: the graph must be
