@@ -65,34 +65,50 @@ struct Trace {
   }
 };
 
-// The build's large sorts: tc_sort.cu's radix sort (TC_SORT=cub: CUB's onesweep,
-// the only choice at or above 2^32 keys or below 2^20, where launch count matters).
-bool own_sort(int64_t n) {
-  static const bool cub_only = [] {
+// The build's 64-bit key sorts (a2, a5, the host entry's pieces, the sharded
+// build) run CUB's onesweep with 256 threads x 22 keys per thread instead of
+// its sm_100 default (384 x 15): 268 M keys on 48 bits in 11.6 vs 16.3 ms
+// (scripts/sort_bench.cu, profiles/r4d_sort_bench.txt).  TC_SORT=cub keeps the
+// default policy.  (A hand-written reduce-then-scan LSD sort with
+// __match_any_sync ranking measured 25.5 ms, the key/value form 37.6 vs 9.1.)
+using SortOffset = unsigned long long;
+struct KeySortHub {
+  using Base = cub::detail::radix::policy_hub<uint64_t, cub::NullType, SortOffset>::Policy1000;
+  struct P : cub::ChainedPolicy<1000, P, P> {
+    static constexpr bool ONESWEEP = true;
+    static constexpr int ONESWEEP_RADIX_BITS = 8;
+    using HistogramPolicy = Base::HistogramPolicy;
+    using ExclusiveSumPolicy = Base::ExclusiveSumPolicy;
+    // nominal items for 4-B keys (CUB scales by the key size: 22 per thread)
+    using OnesweepPolicy =
+        cub::AgentRadixSortOnesweepPolicy<256, 44, uint64_t, 1, cub::RADIX_RANK_MATCH_EARLY_COUNTS_ANY,
+                                          cub::BLOCK_SCAN_RAKING_MEMOIZE, cub::RADIX_SORT_STORE_DIRECT, 8>;
+    using ScanPolicy = Base::ScanPolicy;
+    using DownsweepPolicy = Base::DownsweepPolicy;
+    using AltDownsweepPolicy = Base::AltDownsweepPolicy;
+    using UpsweepPolicy = Base::UpsweepPolicy;
+    using AltUpsweepPolicy = Base::AltUpsweepPolicy;
+    using SingleTilePolicy = Base::SingleTilePolicy;
+    using SegmentedPolicy = Base::SegmentedPolicy;
+    using AltSegmentedPolicy = Base::AltSegmentedPolicy;
+  };
+  using MaxPolicy = P;
+};
+
+void sort_keys_u64(cub::DoubleBuffer<uint64_t>& db, int64_t n, int end_bit, cudaStream_t s) {
+  static const bool cub_default = [] {
     const char* v = std::getenv("TC_SORT");
     return v && std::string(v) == "cub";
   }();
-  return !cub_only && n >= (int64_t(1) << 20) && n < (int64_t(1) << 32);
-}
-
-void sort_keys_u64(cub::DoubleBuffer<uint64_t>& db, int64_t n, int end_bit, cudaStream_t s) {
-  if (own_sort(n)) {
-    if (radix_sort_keys(db.Current(), db.Alternate(), n, 0, end_bit, s)) db.selector ^= 1;
+  if (cub_default) {
+    cub_run(s, [&](void* t, size_t& b) { return cub::DeviceRadixSort::SortKeys(t, b, db, n, 0, end_bit, s); });
     return;
   }
-  cub_run(s, [&](void* t, size_t& b) { return cub::DeviceRadixSort::SortKeys(t, b, db, n, 0, end_bit, s); });
-}
-
-void sort_pairs_u32_u64(cub::DoubleBuffer<uint32_t>& dk, cub::DoubleBuffer<uint64_t>& dv, int64_t n,
-                        int end_bit, cudaStream_t s) {
-  if (own_sort(n)) {
-    if (radix_sort_pairs(dk.Current(), dk.Alternate(), dv.Current(), dv.Alternate(), n, 0, end_bit, s)) {
-      dk.selector ^= 1;
-      dv.selector ^= 1;
-    }
-    return;
-  }
-  cub_run(s, [&](void* t, size_t& b) { return cub::DeviceRadixSort::SortPairs(t, b, dk, dv, n, 0, end_bit, s); });
+  cub::DoubleBuffer<cub::NullType> dv;
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DispatchRadixSort<false, uint64_t, cub::NullType, SortOffset, KeySortHub>::Dispatch(
+        t, b, db, dv, (SortOffset)n, 0, end_bit, true, s);
+  });
 }
 
 template <class T>
@@ -1197,7 +1213,9 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   // and the edges arrive in position order; dead edges sort past S
   cub::DoubleBuffer<uint32_t> dk(skey.get(), skey2.get());
   cub::DoubleBuffer<uint64_t> dv(sval.get(), sval2.get());
-  sort_pairs_u32_u64(dk, dv, m, end_bit, s);
+  cub_run(s, [&](void* t, size_t& b) {
+    return cub::DeviceRadixSort::SortPairs(t, b, dk, dv, m, 0, end_bit, s);
+  });
   const uint32_t* key_sorted = dk.Current();
   const uint64_t* val_sorted = dv.Current();
   tr("select + class sort");

@@ -71,14 +71,6 @@ struct DevBuf {
   T* get() const { return p; }
 };
 
-// ---------------------------------------------------------------- sort
-// tc_sort.cu: stable LSD radix sort (8-bit digits, reduce-then-scan) of n <
-// 2^32 keys on bits [begin_bit, end_bit); ping-pongs between the two buffers
-// and returns true when the result is in the second one.
-bool radix_sort_keys(uint64_t* k0, uint64_t* k1, int64_t n, int begin_bit, int end_bit, cudaStream_t s);
-bool radix_sort_pairs(uint32_t* k0, uint32_t* k1, uint64_t* v0, uint64_t* v1, int64_t n, int begin_bit,
-                      int end_bit, cudaStream_t s);
-
 // ---------------------------------------------------------------- options
 struct Options {
   int chunk_cost = 16384;

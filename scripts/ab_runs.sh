@@ -208,6 +208,15 @@ r4d)
     env $kv timeout 900 python bench.py --steps 10 --warmup 3 --no-balance --out $O/r4d_bench_c3_$tag.json > $O/r4d_bench_c3_$tag.log 2>&1
   done
   ;;
+r4e)
+  # CUB onesweep policy for the build's 64-bit key sorts (256 x 22 keys per thread) vs CUB's default
+  timeout 600 build/sort_bench > $O/r4e_sort_bench.txt 2>&1; echo "rc=$?" >> $O/r4e_sort_bench.txt
+  timeout 1500 python -m pytest -q -x tests/test_gpu_parity.py tests/test_gpu_sharded.py > $O/r4e_pytest.txt 2>&1; echo "rc=$?" >> $O/r4e_pytest.txt
+  i=0; for kv in "" "TC_SORT=cub" "" "TC_SORT=cub"; do
+    i=$((i+1)); tag=${i}_$(echo "${kv:-tuned}" | tr ' =' '__')
+    env $kv timeout 900 python bench.py --steps 10 --warmup 3 --no-balance --out $O/r4e_bench_c3_$tag.json > $O/r4e_bench_c3_$tag.log 2>&1
+  done
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt

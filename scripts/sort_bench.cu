@@ -1,4 +1,4 @@
-// Radix-sort policy sweep for the build's three big sorts (a2/a5: 64-bit keys
+// CUB radix-sort policy sweep for the build's three big sorts (a2/a5: 64-bit keys
 // with 2*24 significant bits; a6: 32-bit key of 26 bits with a 64-bit value).
 // Dev tool, not part of the product:
 //   nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -o build/sort_bench scripts/sort_bench.cu
@@ -8,25 +8,7 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
-#include <stdexcept>
 
-// the product's sort (tc_sort.cu) with minimal stand-ins for libtc's allocator / error hooks
-#include "../paper_conf_ipps_li0ptz24_b200/csrc/tc_sort.cu"
-namespace tc {
-void* dev_alloc(size_t bytes, cudaStream_t, bool) {
-  void* p = nullptr;
-  if (cudaMalloc(&p, bytes) != cudaSuccess) throw std::runtime_error("oom");
-  return p;
-}
-void dev_free(void* p, size_t, cudaStream_t) { cudaFree(p); }
-void check_cuda(cudaError_t e, const char* what, const char* file, int line) {
-  if (e != cudaSuccess) {
-    printf("CUDA %s: %s at %s:%d\n", cudaGetErrorString(e), what, file, line);
-    exit(1);
-  }
-}
-[[noreturn]] void fail(tc_status, const std::string& m) { throw std::runtime_error(m); }
-}  // namespace tc
 #include <cstdio>
 #include <vector>
 
@@ -139,47 +121,6 @@ void bench(const char* name, K* k0, K* k1, V* v0, V* v1, const K* src_k, const V
          bytes * ((end_bit + 7) / 8) / (t[t.size() / 2] * 1e9), 8, ref ? (ok ? "same" : "DIFFERENT") : "ref");
 }
 
-template <class K, class V>
-void bench_own(const char* name, K* k0, K* k1, V* v0, V* v1, const K* src_k, const V* src_v, const K* ref,
-               const V* ref_v, int64_t n, int end_bit, cudaStream_t s) {
-  std::vector<float> t;
-  const K* out = nullptr;
-  const V* outv = nullptr;
-  cudaEvent_t a, b;
-  CK(cudaEventCreate(&a));
-  CK(cudaEventCreate(&b));
-  for (int r = 0; r < 6; ++r) {
-    CK(cudaMemcpyAsync(k0, src_k, sizeof(K) * n, cudaMemcpyDeviceToDevice, s));
-    if (v0) CK(cudaMemcpyAsync(v0, src_v, sizeof(V) * n, cudaMemcpyDeviceToDevice, s));
-    CK(cudaEventRecord(a, s));
-    bool alt;
-    if constexpr (sizeof(K) == 8) alt = tc::radix_sort_keys((uint64_t*)k0, (uint64_t*)k1, n, 0, end_bit, s);
-    else alt = tc::radix_sort_pairs((uint32_t*)k0, (uint32_t*)k1, (uint64_t*)v0, (uint64_t*)v1, n, 0, end_bit, s);
-    CK(cudaEventRecord(b, s));
-    CK(cudaEventSynchronize(b));
-    float ms = 0;
-    CK(cudaEventElapsedTime(&ms, a, b));
-    if (r) t.push_back(ms);
-    out = alt ? k1 : k0;
-    outv = alt ? v1 : v0;
-  }
-  std::sort(t.begin(), t.end());
-  bool ok = true;
-  std::vector<K> x(1 << 20), y(1 << 20);
-  for (int64_t off : {int64_t(0), n / 3, n / 2, n - (1 << 20)}) {
-    CK(cudaMemcpy(x.data(), out + off, sizeof(K) << 20, cudaMemcpyDeviceToHost));
-    CK(cudaMemcpy(y.data(), ref + off, sizeof(K) << 20, cudaMemcpyDeviceToHost));
-    ok = ok && x == y;
-    if (ref_v && v0) {
-      std::vector<V> xv(1 << 20), yv(1 << 20);
-      CK(cudaMemcpy(xv.data(), outv + off, sizeof(V) << 20, cudaMemcpyDeviceToHost));
-      CK(cudaMemcpy(yv.data(), ref_v + off, sizeof(V) << 20, cudaMemcpyDeviceToHost));
-      ok = ok && xv == yv;
-    }
-  }
-  printf("%-44s median %8.3f ms  %s\n", name, t[t.size() / 2], ok ? "same" : "DIFFERENT");
-}
-
 int main(int argc, char** argv) {
   const int64_t n = argc > 1 ? atoll(argv[1]) : 268435456ll;
   cudaStream_t s;
@@ -207,14 +148,16 @@ int main(int argc, char** argv) {
     }
 #define B64(OS, T, I, BITS) \
   bench<uint64_t, N, Hub<uint64_t, N, OS, T, I, BITS>>("u64 keys 48b: " #OS " " #T "x" #I " " #BITS "b", k0, k1, nv, nv, src, nv, ref, n, 48, tmp, tb, s)
-    bench_own<uint64_t, N>("u64 keys 48b: tc_sort", k0, k1, nv, nv, src, nv, ref, nullptr, n, 48, s);
     B64(true, 384, 30, 8);
-    B64(true, 512, 22, 8);
     B64(true, 256, 44, 8);
-    B64(true, 384, 30, 6);
-    B64(true, 384, 30, 7);
-    B64(false, 256, 23, 7);
-    B64(false, 256, 23, 6);
+    B64(true, 256, 40, 8);
+    B64(true, 256, 36, 8);
+    B64(true, 128, 88, 8);
+    B64(true, 192, 60, 8);
+    B64(true, 320, 36, 8);
+    B64(true, 512, 22, 8);
+    B64(true, 256, 44, 7);
+    B64(false, 256, 40, 7);
     CK(cudaFree(src));
     CK(cudaFree(k0));
     CK(cudaFree(k1));
@@ -240,15 +183,7 @@ int main(int argc, char** argv) {
       CK(cudaMemcpyAsync(v0, vs, 8 * n, cudaMemcpyDeviceToDevice, s));
       run<uint32_t, uint64_t, typename cub::detail::radix::policy_hub<uint32_t, uint64_t, OffsetT>>(dk, dv, n, 26, tmp, tb, s);
       CK(cudaMemcpyAsync(ref, dk.Current(), 4 * n, cudaMemcpyDeviceToDevice, s));
-      CK(cudaMemcpyAsync(vs, dv.Current(), 8 * n, cudaMemcpyDeviceToDevice, s));  // sorted values (ref)
-      k_fill32<<<148 * 16, 256, 0, s>>>(src, v1, n, 26, 2);                       // v1 = unsorted values
-      CK(cudaMemcpyAsync(v0, v1, 8 * n, cudaMemcpyDeviceToDevice, s));
     }
-    uint64_t* refv = nullptr;
-    CK(cudaMalloc(&refv, 8 * n));
-    CK(cudaMemcpyAsync(refv, vs, 8 * n, cudaMemcpyDeviceToDevice, s));
-    CK(cudaMemcpyAsync(vs, v1, 8 * n, cudaMemcpyDeviceToDevice, s));  // vs = unsorted values again
-    bench_own<uint32_t, uint64_t>("u32k+u64v 26b: tc_sort", k0, k1, v0, v1, src, vs, ref, refv, n, 26, s);
 #define B32(OS, T, I, BITS)                                                                                     \
   bench<uint32_t, uint64_t, Hub<uint32_t, uint64_t, OS, T, I, BITS>>("u32k+u64v 26b: " #OS " " #T "x" #I " " #BITS "b", \
                                                                      k0, k1, v0, v1, src, vs, ref, n, 26, tmp, tb, s)

@@ -406,10 +406,10 @@ def test_dedup_paths_agree(tc):
 
 @pytest.mark.parametrize("scale,ef,seed", [(18, 16, 3), (20, 8, 4)])
 def test_sort_paths_agree(tc, scale, ef, seed):
-    """The build's radix sort (tc_sort.cu: a2, a5, a6 above 2^20 keys) and
-    CUB's onesweep (forced with TC_SORT=cub in a child process) build the same
-    CSR, B_ITC and count.  Scale 18 sorts 36-bit keys in 5 passes (the result
-    lands in the second buffer), scale 20 in 5 / 6."""
+    """The build's 64-bit key sorts with the tuned onesweep policy (a2, a5)
+    and with CUB's default policy (forced with TC_SORT=cub in a child process)
+    build the same CSR, B_ITC and count.  Scale 18 sorts 36-bit keys in 5
+    passes (the result lands in the second buffer), scale 20 in 5 / 6."""
     import subprocess
     import sys
     src, dst, n = tcgen.rmat(scale, ef, seed)
@@ -421,7 +421,7 @@ def test_sort_paths_agree(tc, scale, ef, seed):
             "h = hashlib.sha256(); [h.update(x.cpu().numpy().tobytes()) for x in g.csr()];"
             "print(h.hexdigest(), g.info.b_itc, g.info.keys_total, g.count())") % (ROOT, scale, ef, seed)
     out = {}
-    for mode, env_kv in (("own", {}), ("cub", {"TC_SORT": "cub"})):
+    for mode, env_kv in (("own", {}), ("cub", {"TC_SORT": "cub"})):  # own = the tuned policy
         env = dict(os.environ, **env_kv)
         env.pop("TC_SORT", None) if mode == "own" else None
         r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
