@@ -387,12 +387,14 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
   }
 }
 
-__global__ void k_group_mark(const uint32_t* __restrict__ key, int64_t S,
-                             int32_t* __restrict__ mark) {
-  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S;
-       s += (int64_t)gridDim.x * blockDim.x)
-    mark[s] = (s == 0 || key[s] != key[s - 1]) ? 1 : 0;
-}
+// 1 at the first segment of each group (its sort key differs from the
+// previous one): read on the fly by the group-index scan (no mark array).
+struct GroupStart {
+  const uint32_t* key;
+  __host__ __device__ int32_t operator()(int64_t s) const {
+    return (s == 0 || key[s] != key[s - 1]) ? 1 : 0;
+  }
+};
 
 // Per segment (sorted live edge): start, length, group, work units; per
 // group (at its first segment): row start, d+(v) and its table.
@@ -1222,11 +1224,10 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
 
   DevBuf<int32_t> gincl(S, s);
   {
-    DevBuf<int32_t> mark(S, s);
-    k_group_mark<<<grid_for(S), TPB, 0, s>>>(key_sorted, S, mark.get());
-    TC_LAUNCH();
+    cub::TransformInputIterator<int32_t, GroupStart, cub::CountingInputIterator<int64_t>> marks(
+        cub::CountingInputIterator<int64_t>(0), GroupStart{key_sorted});
     cub_run(s, [&](void* t, size_t& b) {
-      return cub::DeviceScan::InclusiveSum(t, b, mark.get(), gincl.get(), S, s);
+      return cub::DeviceScan::InclusiveSum(t, b, marks, gincl.get(), S, s);
     });
   }
   const int64_t G = (int64_t)d2h(gincl.get() + (S - 1), s);

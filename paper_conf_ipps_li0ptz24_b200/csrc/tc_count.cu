@@ -60,9 +60,6 @@ constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flig
 #ifndef TC_PF_SHORT
 #define TC_PF_SHORT 1  // produce: L2 prefetch of every short-class edge's keys at staging (r2y: C2 -1.6%)
 #endif
-#ifndef TC_XSHFL
-#define TC_XSHFL 0  // walk_long: next batch's descriptors read one word per lane + shuffles (1: x, 2: x, z, zw)
-#endif
 #ifndef TC_L2PF
 #define TC_L2PF 1  // walk_long: L2 prefetch of the key lines TC_L2PF batches ahead (0: off;
 #endif             // r2v C3 k_count 42.2 -> 38.9 ms, C4 564 -> 545 ms with 1)
@@ -412,73 +409,25 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
   const int lane = threadIdx.x & 31;
   const int32_t* colL = lane_base(pv.col, lane);
   int t = t0;
-  // TC_XSHFL (A/B knob, 8-tile batches): the next batch's descriptors are read
-  // one word per lane while this batch's loads are in flight (lanes 0-7: x,
-  // 8-15: x again for the last-line prefetch, 16-23: z, 24-31: zw) and handed
-  // out by shuffles instead of broadcast LDS.128s
-  constexpr bool kShfl = TC_XSHFL > 0 && kB == 8;
-  int nd = 0;
-  bool have = false;
   for (; t + kB <= t1; t += kB) {
-    int32_t key[kB];
-    int z[kB], zw[kB];
-    if constexpr (kShfl) {
-      int x[kB];
-      if (have) {
-#pragma unroll
-        for (int u = 0; u < kB; ++u) {
-          x[u] = __shfl_sync(0xffffffffu, nd, u);
-          if (TC_XSHFL >= 2) {
-            z[u] = __shfl_sync(0xffffffffu, nd, 16 + u);
-            zw[u] = __shfl_sync(0xffffffffu, nd, 24 + u);
-          }
-        }
-      } else {
-#pragma unroll
-        for (int q = 0; q < kB; q += 4) {
-          *reinterpret_cast<int4*>(x + q) = *reinterpret_cast<const int4*>(c.sT0 + t + q);
-          if (TC_XSHFL >= 2) {
-            *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
-            *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
-          }
-        }
-      }
-      have = t + 2 * kB <= t1;  // warp-uniform
-      if (have) {
-        const int q = lane & 7, f = lane >> 3;
-        nd = (f < 2 ? c.sT0 : (f == 2 ? c.sT1 : c.sT2))[t + kB + q];
-        if (f < 2) asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + ((uint32_t)nd + (f ? 31u : 0u))));
-      } else if (lane < 2 * kB && t + kB + (lane % kB) < t1) {
-        const uint32_t xx = (uint32_t)c.sT0[t + kB + (lane % kB)] + (lane >= kB ? 31u : 0u);
-        asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + xx));
-      }
-#pragma unroll
-      for (int u = 0; u < kB; ++u) key[u] = __ldg(colL + (uint32_t)x[u]);
-      if (TC_XSHFL < 2) {
-#pragma unroll
-        for (int q = 0; q < kB; q += 4) {
-          *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
-          *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
-        }
-      }
-    } else {
 #if TC_L2PF
-      // pull the key lines of the batch TC_L2PF batches ahead into L2 while this
-      // batch's loads are outstanding: the loads in flight per lane are bounded
-      // by registers, a prefetch holds none (lane u < kB takes tile u's first
-      // line, lane kB + u its last)
-      if (lane < 2 * kB && t + TC_L2PF * kB + (lane % kB) < t1) {
-        const int q = lane % kB;
-        const uint32_t x = (uint32_t)c.sT0[t + TC_L2PF * kB + q] + (lane >= kB ? 31u : 0u);
-        asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + x));
-      }
+    // pull the key lines of the batch TC_L2PF batches ahead into L2 while this
+    // batch's loads are outstanding: the loads in flight per lane are bounded
+    // by registers, a prefetch holds none (lane u < kB takes tile u's first
+    // line, lane kB + u its last)
+    if (lane < 2 * kB && t + TC_L2PF * kB + (lane % kB) < t1) {
+      const int q = lane % kB;
+      const uint32_t x = (uint32_t)c.sT0[t + TC_L2PF * kB + q] + (lane >= kB ? 31u : 0u);
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(pv.col + x));
+    }
 #endif
-      load_batch<kB>(c, colL, t, key);
+    int32_t key[kB];
+    load_batch<kB>(c, colL, t, key);
+    int z[kB], zw[kB];
 #pragma unroll
-      for (int q = 0; q < kB; q += 4) {
-        *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
-        *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
-      }
+    for (int q = 0; q < kB; q += 4) {
+      *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
+      *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
     }
     int zw_or = 0;  // first-lane fields are < 64, so the OR's code bits are the OR of the codes
 #pragma unroll

@@ -217,6 +217,17 @@ r4e)
     env $kv timeout 900 python bench.py --steps 10 --warmup 3 --no-balance --out $O/r4e_bench_c3_$tag.json > $O/r4e_bench_c3_$tag.log 2>&1
   done
   ;;
+r4f)
+  # next batch's descriptors by shuffles (TC_XSHFL 1: x, 2: x, z, zw) vs broadcast LDS.128
+  for c in C3; do
+    bash scripts/gpu_abbuild.sh r4f_$c $c 10 "" "-DTC_XSHFL=1" "-DTC_XSHFL=2" "" "-DTC_XSHFL=2"
+  done
+  rm -f build/tc_count.o paper_conf_ipps_li0ptz24_b200/libtc.so; make -s NVEXTRA=-DTC_XSHFL=2 paper_conf_ipps_li0ptz24_b200/libtc.so > /dev/null 2>&1
+  timeout 900 python -m pytest -q -x tests/test_gpu_parity.py -k "closed_forms or c1_rmat10 or rmat_medium or options or karate or golden or full_size" > $O/r4f_pytest_xshfl2.txt 2>&1; echo "rc=$?" >> $O/r4f_pytest_xshfl2.txt
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_count -s 2 -c 1 \
+    -o $O/r4f_c3_xshfl2 python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e --no-sharded --no-balance > $O/r4f_ncu.log 2>&1
+  rm -f build/tc_count.o paper_conf_ipps_li0ptz24_b200/libtc.so; make -s paper_conf_ipps_li0ptz24_b200/libtc.so > /dev/null 2>&1
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
