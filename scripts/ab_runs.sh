@@ -228,6 +228,19 @@ r4f)
     -o $O/r4f_c3_xshfl2 python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e --no-sharded --no-balance > $O/r4f_ncu.log 2>&1
   rm -f build/tc_count.o paper_conf_ipps_li0ptz24_b200/libtc.so; make -s paper_conf_ipps_li0ptz24_b200/libtc.so > /dev/null 2>&1
   ;;
+r4g)
+  # short class: L2 prefetch of each group's N+(v) at staging; 4 staging loads in flight per thread
+  for c in C2 C5 C3; do
+    bash scripts/gpu_abbuild.sh r4g_$c $c 10 "" "-DTC_PF_ROWS_SHORT=1" "-DTC_FLAT_PB=4" "-DTC_PF_ROWS_SHORT=1 -DTC_FLAT_PB=4" ""
+  done
+  ;;
+r4h)
+  # long class: one packed {first lane, bitmap flag, word base} descriptor word per tile (TC_PACKED)
+  rm -f build/tc_count.o paper_conf_ipps_li0ptz24_b200/libtc.so; make -s NVEXTRA=-DTC_PACKED=1 paper_conf_ipps_li0ptz24_b200/libtc.so > /dev/null 2>&1
+  timeout 900 python -m pytest -q -x tests/test_gpu_parity.py -k "closed_forms or c1_rmat10 or rmat_medium or options or karate or golden or full_size or huge or cap or skewed" > $O/r4h_pytest_packed.txt 2>&1; echo "rc=$?" >> $O/r4h_pytest_packed.txt
+  bash scripts/gpu_abbuild.sh r4h_C3 C3 10 "" "-DTC_PACKED=1" "" "-DTC_PACKED=1"
+  bash scripts/gpu_abbuild.sh r4h_C4 C4 3 "" "-DTC_PACKED=1"
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
