@@ -57,9 +57,6 @@ constexpr int kUnrollLong = 8;   // tail batch of the long class
 #define TC_BATCH_LONG 8
 #endif
 constexpr int kBatchLong = TC_BATCH_LONG;  // tiles per batch: key loads in flight per lane
-#ifndef TC_PACKED
-#define TC_PACKED 0  // walk_long: one packed {first lane, bitmap flag, word base} word per tile (A/B knob)
-#endif
 #ifndef TC_PF_SHORT
 #define TC_PF_SHORT 1  // produce: L2 prefetch of every short-class edge's keys at staging (r2y: C2 -1.6%)
 #endif
@@ -426,32 +423,10 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
 #endif
     int32_t key[kB];
     load_batch<kB>(c, colL, t, key);
-#if TC_PACKED
-    {
-      // one packed word per tile: all-bitmap batches need no other field
-      uint32_t zf[kB];
-#pragma unroll
-      for (int q = 0; q < kB; q += 4)
-        *reinterpret_cast<uint4*>(zf + q) = *reinterpret_cast<const uint4*>(c.sT1 + t + q);
-      uint32_t zf_or = 0;
-#pragma unroll
-      for (int u = 0; u < kB; ++u) zf_or |= zf[u];
-      if (!(zf_or & (1u << 26))) {
-        const uint32_t lim = (uint32_t)(lane + 1) << 27;  // lane >= first valid lane
-#pragma unroll
-        for (int u = 0; u < kB; ++u) {
-          const unsigned word = (unsigned)c.sT0[((uint32_t)(key[u] >> 5) + zf[u]) & 0x3FFFFFFu];
-          const unsigned hit = (__funnelshift_r(word, 0u, (unsigned)key[u]) & 1u) ^ 1u;
-          if (zf[u] < lim) cnt += hit;
-        }
-        continue;
-      }
-    }
-#endif
     int z[kB], zw[kB];
 #pragma unroll
     for (int q = 0; q < kB; q += 4) {
-      *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>((TC_PACKED ? c.sT3 : c.sT1) + t + q);
+      *reinterpret_cast<int4*>(z + q) = *reinterpret_cast<const int4*>(c.sT1 + t + q);
       *reinterpret_cast<int4*>(zw + q) = *reinterpret_cast<const int4*>(c.sT2 + t + q);
     }
     int zw_or = 0;  // first-lane fields are < 64, so the OR's code bits are the OR of the codes
@@ -483,7 +458,7 @@ __device__ __forceinline__ unsigned walk_long(const ChunkSmem& c, int t0, int t1
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const int tt = min(t + u, t1 - 1);
-      z[u] = (TC_PACKED ? c.sT3 : c.sT1)[tt];
+      z[u] = c.sT1[tt];
       zw[u] = c.sT2[tt] | (t + u < t1 ? 0 : 32);  // first valid lane 32: none
     }
 #pragma unroll
@@ -887,18 +862,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
           c.sT0[t] = (int)(uint32_t)(p - (32 - lanes));
           const int zt = d.x < 0 ? toff : (int)(c.sHash - c.sT0) + (d.y <= 0 ? d.x + d.y : d.x);
           const int zwt = ((d.x < 0 ? -1 : (d.y <= 0 ? 0 : d.y)) * 64) | (32 - lanes);
-#if TC_PACKED
-          // packed fast-path word: first valid lane << 27 | not-a-bitmap << 26 |
-          // the bitmap's word base z mod 2^26 (z > -2^26: the window's first word
-          // is < 2^25, k_seg_fill; the probed word (key >> 5) + z is < 2^15, so
-          // ((key >> 5) + packed) mod 2^26 is that word); hash and huge tiles keep
-          // z / zw in sT3 / sT2
-          const bool bm = d.x >= 0 && d.y <= 0;
-          c.sT1[t] = (int)(((uint32_t)(32 - lanes) << 27) | (bm ? ((uint32_t)zt & 0x3FFFFFFu) : (1u << 26)));
-          c.sT3[t] = zt;
-#else
           c.sT1[t] = zt;
-#endif
           c.sT2[t] = zwt;
         }
       }
