@@ -474,7 +474,12 @@ TC_API tc_status tc_mc_buffer_create(size_t bytes, void** handle, uint64_t** d_u
                                      uint64_t** d_mc);
 TC_API void tc_mc_buffer_destroy(void* handle);
 
-/* Release a graph (NULL is a no-op).  Stream-ordered frees on the build stream. */
+/* Release a graph (NULL is a no-op).  Waits on the host for the work the
+ * stream-ordered entry points (tc_count_async, tc_count_range[_fused],
+ * tc_count_variant, tc_support, tc_edge_list) enqueued on the graph, on
+ * whatever stream, up to this call -- not for the whole device, so a build
+ * running on another stream is not waited for -- then frees the graph's
+ * buffers stream-ordered. */
 TC_API void tc_free(tc_graph* g);
 
 /*

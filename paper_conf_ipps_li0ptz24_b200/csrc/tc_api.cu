@@ -10,6 +10,8 @@
 #include <new>
 #include <vector>
 
+#include <mutex>
+
 #include "tc_internal.cuh"
 
 namespace {
@@ -61,10 +63,18 @@ namespace {
 constexpr int kMaxDevices = 64;
 
 // Release threshold "never": freed blocks stay mapped across syncs (without
-// this every build re-maps its scratch, tens of ms at config C2).
+// this every build re-maps its scratch, tens of ms at config C2).  No
+// internal reuse dependencies: a block freed on one stream is not handed to
+// an allocation on another stream by making that stream wait for the first
+// one's work, which serialised a count on one stream with a build on another
+// (C3 pipelined e2e 124 -> 100 ms per step, profiles/r4o_pipe3.txt); blocks
+// are still reused when their free is known complete (event dependencies,
+// opportunistic reuse).
 void keep_mapped(cudaMemPool_t pool) {
   uint64_t thr = UINT64_MAX;
   cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  int no = 0;
+  cudaMemPoolSetAttribute(pool, cudaMemPoolReuseAllowInternalDependencies, &no);
 }
 
 // The device's default pool (persistent buffers) or the library's own scratch
@@ -72,6 +82,8 @@ void keep_mapped(cudaMemPool_t pool) {
 cudaMemPool_t pool_of(bool persistent) {
   static cudaMemPool_t scratch[kMaxDevices] = {};
   static bool default_ready[kMaxDevices] = {};
+  static std::mutex mu;  // first use may come from several host threads
+  std::lock_guard<std::mutex> lk(mu);
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) {
     cudaGetLastError();
@@ -208,6 +220,21 @@ namespace {
 
 // Rebinds every stream-ordered buffer of the graph to `s` so frees are
 // ordered after the work that used them.
+// Record that work reading g was enqueued on s (tc_free waits for it).
+void note_use(const tc_graph* g, void* stream) {
+  const cudaStream_t s = (cudaStream_t)stream;
+  std::lock_guard<std::mutex> lk(g->use_mu);
+  for (auto& u : g->uses)
+    if (u.s == s) {
+      TC_CUDA(cudaEventRecord(u.ev, s));
+      return;
+    }
+  tc_graph::Use u{s, nullptr};
+  TC_CUDA(cudaEventCreateWithFlags(&u.ev, cudaEventDisableTiming));
+  g->uses.push_back(u);
+  TC_CUDA(cudaEventRecord(u.ev, s));
+}
+
 void rebind(tc_graph* g, cudaStream_t s) {
   g->row_ptr.s = g->col.s = g->perm.s = s;
   tc::Plan& P = g->plan;
@@ -351,6 +378,7 @@ tc_status tc_count_async(const tc_graph* g, void* stream, uint64_t* d_count) {
     require(g && d_count, "NULL argument");
     tc::count_chunks(g, 0, g->plan.n_chunks, 0, g->plan.S, (cudaStream_t)stream,
                      reinterpret_cast<unsigned long long*>(d_count));
+    note_use(g, stream);
   });
 }
 
@@ -360,10 +388,20 @@ tc_status tc_count(const tc_graph* g, void* stream, uint64_t* h_count) {
     cudaStream_t s = (cudaStream_t)stream;
     tc::DevBuf<unsigned long long> d(1, s);
     tc::count_chunks(g, 0, g->plan.n_chunks, 0, g->plan.S, s, d.get());
-    unsigned long long h = 0;
-    TC_CUDA(cudaMemcpyAsync(&h, d.get(), sizeof(h), cudaMemcpyDeviceToHost, s));
+    // the 8-B result lands in pinned memory: a copy into pageable (stack)
+    // memory held a build's H2D copies on another stream back until this
+    // count finished (C3 pipelined e2e: 124 vs 100 ms per step,
+    // profiles/r4o_pipeline_variants.txt)
+    thread_local struct Pinned {
+      unsigned long long* p = nullptr;
+      ~Pinned() {
+        if (p) cudaFreeHost(p);
+      }
+    } pin;
+    if (!pin.p) TC_CUDA(cudaMallocHost(&pin.p, sizeof(unsigned long long)));
+    TC_CUDA(cudaMemcpyAsync(pin.p, d.get(), sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
     TC_CUDA(cudaStreamSynchronize(s));
-    *h_count = h;
+    *h_count = *pin.p;
   });
 }
 
@@ -378,6 +416,7 @@ tc_status tc_count_range(const tc_graph* g, int64_t e_begin, int64_t e_end, void
     chunk_range(g, e_begin, e_end, &c_begin, &c_end);
     tc::count_chunks(g, c_begin, c_end, e_begin, e_end, (cudaStream_t)stream,
                      reinterpret_cast<unsigned long long*>(d_partial));
+    note_use(g, stream);
   });
 }
 
@@ -401,6 +440,7 @@ tc_status tc_count_range_fused(const tc_graph* g, int64_t e_begin, int64_t e_end
     unsigned long long* tot = reinterpret_cast<unsigned long long*>(d_total);
     if (tc::count_chunks(g, c_begin, c_end, e_begin, e_end, (cudaStream_t)stream, tot, &f) == 0)
       tc::fused_finish(tot, f, (cudaStream_t)stream);
+    note_use(g, stream);
   });
 }
 
@@ -421,6 +461,7 @@ tc_status tc_count_variant(const tc_graph* g, int32_t variant, void* stream, uin
     require(variant == TC_VARIANT_POLAK || variant == TC_VARIANT_TRUST, "unknown variant");
     tc::count_variant(g, variant, (cudaStream_t)stream,
                       reinterpret_cast<unsigned long long*>(d_count));
+    note_use(g, stream);
   });
 }
 
@@ -429,6 +470,7 @@ tc_status tc_support(const tc_graph* g, void* stream, uint32_t* d_support) {
     require(g != nullptr, "graph is NULL");
     require(g->m == 0 || d_support != nullptr, "d_support is NULL");
     tc::support_all(g, (cudaStream_t)stream, reinterpret_cast<unsigned*>(d_support));
+    note_use(g, stream);
   });
 }
 
@@ -437,6 +479,7 @@ tc_status tc_edge_list(const tc_graph* g, void* stream, int32_t* d_u, int32_t* d
     require(g != nullptr, "graph is NULL");
     require(g->m == 0 || (d_u && d_v), "d_u/d_v is NULL");
     tc::edge_ends(g, (cudaStream_t)stream, d_u, d_v);
+    note_use(g, stream);
   });
 }
 
@@ -850,7 +893,16 @@ tc_status tc_build_from_oriented(const uint64_t* d_okeys, int64_t m, const int32
 
 void tc_free(tc_graph* g) {
   if (!g) return;
-  cudaDeviceSynchronize();
+  // the graph's own build and replans completed before they returned; wait
+  // for the work other streams enqueued on it, then free stream-ordered
+  {
+    std::lock_guard<std::mutex> lk(g->use_mu);
+    for (auto& u : g->uses) {
+      cudaEventSynchronize(u.ev);
+      cudaEventDestroy(u.ev);
+    }
+    g->uses.clear();
+  }
   rebind(g, nullptr);
   delete g;
 }

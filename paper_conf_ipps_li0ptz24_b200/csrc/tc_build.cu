@@ -948,8 +948,6 @@ void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen,
   DevBuf<int> err(1, s);
   DevBuf<int64_t> nsel(1, s);
   DevBuf<UniqTail> tail(1, s);
-  TC_CUDA(cudaMemsetAsync(err.get(), 0, sizeof(int), s));
-  TC_CUDA(cudaMemsetAsync(nsel.get(), 0, sizeof(int64_t), s));
   struct Res {
     cudaStream_t cs = nullptr;
     cudaEvent_t ready = nullptr, ev[8] = {};
@@ -966,8 +964,13 @@ void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen,
   TC_CUDA(cudaStreamCreateWithFlags(&r.cs, cudaStreamNonBlocking));
   TC_CUDA(cudaEventCreateWithFlags(&r.ready, cudaEventDisableTiming));
   for (int i = 0; i < pieces; ++i) TC_CUDA(cudaEventCreateWithFlags(&r.ev[i], cudaEventDisableTiming));
+  // the copies wait only for the stream-ordered allocations: nothing that
+  // needs an SM may sit between them and the event (a memset there waited
+  // behind a count kernel running on another stream and held the H2D back)
   TC_CUDA(cudaEventRecord(r.ready, s));  // the device buffers exist (stream-ordered allocs)
   TC_CUDA(cudaStreamWaitEvent(r.cs, r.ready, 0));
+  TC_CUDA(cudaMemsetAsync(err.get(), 0, sizeof(int), s));
+  TC_CUDA(cudaMemsetAsync(nsel.get(), 0, sizeof(int64_t), s));
   int64_t lo[9];
   for (int i = 0; i <= pieces; ++i) lo[i] = m_gen * i / pieces;
   for (int i = 0; i < pieces; ++i) {

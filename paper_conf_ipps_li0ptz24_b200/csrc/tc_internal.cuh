@@ -200,6 +200,15 @@ struct tc_graph {
   tc::Plan plan;
   uint64_t b_itc = 0;
   float ms[6] = {0, 0, 0, 0, 0, 0};
+  // Streams that ran work reading this graph (the stream-ordered entry points
+  // record an event after their launches): tc_free waits for these events
+  // only, not for the whole device (a build on another stream runs on).
+  struct Use {
+    cudaStream_t s;
+    cudaEvent_t ev;
+  };
+  mutable std::mutex use_mu;
+  mutable std::vector<Use> uses;
 };
 
 namespace tc {

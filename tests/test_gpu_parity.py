@@ -485,3 +485,48 @@ def test_more_than_2_31_edges(tc):
         assert g.count() == c * comb(k, 3)
         b = g.partition(3)
         assert sum(int(g.count_range(b[r], b[r + 1]).item()) for r in range(3)) == c * comb(k, 3)
+
+
+def test_close_waits_only_for_its_own_work(tc):
+    """tc_free waits for the work other streams enqueued on the graph (the
+    stream-ordered entry points record an event), not for the device: a graph
+    closed right after an async count on another stream still yields T."""
+    src, dst, n = tcgen.rmat(16, 16, 21)
+    want = oracle.triangles(src, dst)
+    s = torch.cuda.Stream()
+    out = torch.zeros(1, dtype=torch.int64, device="cuda")
+    g = tc.build_csr(dev(src), dev(dst), n)
+    g.count_async(out=out, stream=s)
+    g.close()
+    junk = [torch.full((1 << 22,), -1, dtype=torch.int32, device="cuda") for _ in range(4)]
+    s.synchronize()
+    assert int(out.item()) == want
+    del junk
+
+
+def test_build_and_count_on_two_streams_concurrently(tc):
+    """The pipelined use (bench.py e2e_pipelined): graph i+1 is built from
+    host pairs on one stream in a second host thread while graph i is counted
+    on another stream; every count equals the oracle's."""
+    import threading
+    src, dst, n = tcgen.rmat(17, 16, 22)
+    want = oracle.triangles(src, dst)
+    ps = torch.from_numpy(src).pin_memory()
+    pd = torch.from_numpy(dst).pin_memory()
+    sb, sc = torch.cuda.Stream(), torch.cuda.Stream()
+    g = tc.build_csr_host(ps, pd, n, stream=sb)
+    for _ in range(3):
+        res = {}
+
+        def build():
+            with torch.cuda.stream(sb):
+                res["g"] = tc.build_csr_host(ps, pd, n, stream=sb)
+
+        th = threading.Thread(target=build)
+        th.start()
+        assert g.count(stream=sc) == want
+        th.join()
+        g.close()
+        g = res["g"]
+    assert g.count(stream=sc) == want
+    g.close()
