@@ -874,7 +874,7 @@ __device__ __forceinline__ void produce(const PlanView& pv, int64_t cix, int64_t
 #ifndef TC_INS_UNROLL
 #define TC_INS_UNROLL 4
 #endif
-  constexpr int kInsU = TC_INS_UNROLL;  // N+(v) row loads in flight per producer lane
+  constexpr int kInsU = kB >= 4 ? TC_INS_UNROLL : 4;  // N+(v) row loads in flight per producer lane (long-class producers; the flat kernel keeps 4)
   const int pw = pt >> 5, npw = PT >> 5;
   const int NI = c.sGP[G];
   const int i0 = (int)((unsigned)NI * (unsigned)pw / (unsigned)npw),

@@ -241,6 +241,17 @@ r4h)
   bash scripts/gpu_abbuild.sh r4h_C3 C3 10 "" "-DTC_PACKED=1" "" "-DTC_PACKED=1"
   bash scripts/gpu_abbuild.sh r4h_C4 C4 3 "" "-DTC_PACKED=1"
   ;;
+r4u)
+  # mbarrier try_wait suspend-time hint (TC_WAIT_HINT ns; 0 = a bare try_wait spin loop)
+  bash scripts/gpu_ab.sh r4u_C3 C3 10 "" "TC_WAIT_HINT=100" "TC_WAIT_HINT=500" "TC_WAIT_HINT=2000" "TC_WAIT_HINT=10000" ""
+  bash scripts/gpu_ab.sh r4u_C2 C2 10 "" "TC_WAIT_HINT=500" "TC_WAIT_HINT=2000"
+  bash scripts/gpu_ab.sh r4u_C4 C4 3 "" "TC_WAIT_HINT=500" "TC_WAIT_HINT=2000"
+  ;;
+r4v)
+  # producers' row loads in flight per lane in the insert walk (TC_INS_UNROLL, compile time)
+  bash scripts/gpu_abbuild.sh r4v_C3 C3 10 "" "-DTC_INS_UNROLL=8" "-DTC_INS_UNROLL=16" ""
+  bash scripts/gpu_abbuild.sh r4v_C2 C2 10 "" "-DTC_INS_UNROLL=8" "-DTC_INS_UNROLL=16"
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
