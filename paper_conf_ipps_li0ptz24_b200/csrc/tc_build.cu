@@ -346,7 +346,7 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
                             const int32_t* __restrict__ rowid, const int4* __restrict__ vmm,
                             int64_t m, int long_min, int bits,
                             uint32_t dead, uint32_t* __restrict__ skey, uint64_t* __restrict__ sval,
-                            unsigned long long* stats) {
+                            unsigned long long* stats, int long_bitmap_factor) {
   typedef cub::BlockReduce<unsigned long long, TPB> BR;
   __shared__ typename BR::TempStorage tmp;
   unsigned long long b = 0, keys = 0, nl = 0, nlong = 0, klong = 0;
@@ -361,13 +361,19 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
       lo = lower_bound_i32(col, p + 1, rend, w.x);
       len = upper_bound_i32(col, lo, rend, w.y) - lo;
     }
-    const uint32_t cls = len < long_min ? 1u : 0u;
+    // long class: len >= long_min (and, with TC_LONG_BITMAP, only edges whose
+    // head gets a bitmap table; the others are flattened with the short class)
+    bool lng = len >= long_min;
+    if (long_bitmap_factor > 0 && lng)
+      lng = (w.x >> 5) < (1 << 25) &&
+            (int64_t)((w.y >> 5) - (w.x >> 5) + 1) <= (int64_t)long_bitmap_factor * w.z;
+    const uint32_t cls = lng ? 0u : 1u;
     skey[p] = len > 0 ? ((cls << bits) | (uint32_t)v) : dead;
     sval[p] = ((uint64_t)lo << 24) | (uint64_t)len;  // len <= d+(u) < 2^24
     keys += (unsigned long long)len;
     nl += len > 0;
-    nlong += len >= long_min;
-    klong += len >= long_min ? (unsigned long long)len : 0ull;
+    nlong += lng;
+    klong += lng ? (unsigned long long)len : 0ull;
   }
   unsigned long long r0 = BR(tmp).Sum(b);
   __syncthreads();
@@ -1143,6 +1149,7 @@ Tuning tuning_from_env() {
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
   t.batch = get("TC_BATCH", t.batch, 0, 64);
   t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 3);
+  t.long_bitmap = get("TC_LONG_BITMAP", t.long_bitmap, 0, 1);
   return t;
 }
 
@@ -1152,6 +1159,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   P = Plan();
   P.opt = opt;
   P.block = opt.block_threads;
+  P.tune = tuning_from_env();
   const int64_t m = g->m, n = g->n;
   // the count kernel's tile descriptors address keys by a 32-bit col index
   if (m > (int64_t)0xFFFFFFFFll) fail(TC_ERR_UNSUPPORTED, "more than 2^32 - 1 unique edges");
@@ -1189,7 +1197,8 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     constexpr int64_t kSmallGraph = int64_t(1) << 20;
     const int long_min = (opt.long_min_auto && m < kSmallGraph) ? (1 << 30) : std::max(opt.long_min, 32);
     k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), vmm.get(), m, long_min,
-                                            g->bits, dead, skey.get(), sval.get(), stats.get());
+                                            g->bits, dead, skey.get(), sval.get(), stats.get(),
+                                            P.tune.long_bitmap ? opt.bitmap_factor : 0);
     TC_LAUNCH();
   }
   rowid.reset();
@@ -1235,7 +1244,6 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   }
   const int64_t G = (int64_t)d2h(gincl.get() + (S - 1), s);
   P.G = G;
-  P.tune = tuning_from_env();
   // SMEM of one chunk slot of the count kernel; a table may use at most half
   // of it (bigger tables are "huge": probed in global memory)
   const int64_t slot_limit = max_chunk_smem(P.tune);

@@ -252,6 +252,14 @@ r4v)
   bash scripts/gpu_abbuild.sh r4v_C3 C3 10 "" "-DTC_INS_UNROLL=8" "-DTC_INS_UNROLL=16" ""
   bash scripts/gpu_abbuild.sh r4v_C2 C2 10 "" "-DTC_INS_UNROLL=8" "-DTC_INS_UNROLL=16"
   ;;
+r4w)
+  # long class only for edges whose head gets a bitmap table (TC_LONG_BITMAP): the hash-table heads of
+  # the producer-bound head of the long class go to the flattened kernel
+  TC_LONG_BITMAP=1 timeout 900 python -m pytest -q -x tests/test_gpu_parity.py -k "closed_forms or c1_rmat10 or rmat_medium or options or karate or golden or full_size or huge or cap or skewed or c2_chung or c5_lattice" > $O/r4w_pytest_long_bitmap.txt 2>&1; echo "rc=$?" >> $O/r4w_pytest_long_bitmap.txt
+  bash scripts/gpu_ab.sh r4w_C3 C3 10 "" "TC_LONG_BITMAP=1" "" "TC_LONG_BITMAP=1"
+  bash scripts/gpu_ab.sh r4w_C2 C2 10 "" "TC_LONG_BITMAP=1"
+  bash scripts/gpu_ab.sh r4w_C4 C4 3 "" "TC_LONG_BITMAP=1"
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
