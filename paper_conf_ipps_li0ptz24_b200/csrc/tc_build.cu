@@ -346,7 +346,7 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
                             const int32_t* __restrict__ rowid, const int4* __restrict__ vmm,
                             int64_t m, int long_min, int bits,
                             uint32_t dead, uint32_t* __restrict__ skey, uint64_t* __restrict__ sval,
-                            unsigned long long* stats, int long_bitmap_factor) {
+                            unsigned long long* stats, int hash_dmax, int bitmap_factor) {
   typedef cub::BlockReduce<unsigned long long, TPB> BR;
   __shared__ typename BR::TempStorage tmp;
   unsigned long long b = 0, keys = 0, nl = 0, nlong = 0, klong = 0;
@@ -361,12 +361,14 @@ __global__ void k_edge_trim(const int64_t* __restrict__ row_ptr, const int32_t* 
       lo = lower_bound_i32(col, p + 1, rend, w.x);
       len = upper_bound_i32(col, lo, rend, w.y) - lo;
     }
-    // long class: len >= long_min (and, with TC_LONG_BITMAP, only edges whose
-    // head gets a bitmap table; the others are flattened with the short class)
+    // long class: len >= long_min; with TC_LONG_HASH_DMAX = D > 0, an edge
+    // whose head gets a hash table (no bitmap) with d+(v) <= D is flattened
+    // with the short class instead (tiny tables, few edges per group: the
+    // producer-bound head of the long class)
     bool lng = len >= long_min;
-    if (long_bitmap_factor > 0 && lng)
+    if (hash_dmax > 0 && lng && w.z <= hash_dmax)
       lng = (w.x >> 5) < (1 << 25) &&
-            (int64_t)((w.y >> 5) - (w.x >> 5) + 1) <= (int64_t)long_bitmap_factor * w.z;
+            (int64_t)((w.y >> 5) - (w.x >> 5) + 1) <= (int64_t)bitmap_factor * w.z;
     const uint32_t cls = lng ? 0u : 1u;
     skey[p] = len > 0 ? ((cls << bits) | (uint32_t)v) : dead;
     sval[p] = ((uint64_t)lo << 24) | (uint64_t)len;  // len <= d+(u) < 2^24
@@ -1149,7 +1151,8 @@ Tuning tuning_from_env() {
   t.max_kicks = get("TC_CUCKOO_KICKS", t.max_kicks, 0, 4096);
   t.batch = get("TC_BATCH", t.batch, 0, 64);
   t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 3);
-  t.long_bitmap = get("TC_LONG_BITMAP", t.long_bitmap, 0, 1);
+  t.long_hash_dmax = get("TC_LONG_HASH_DMAX", t.long_hash_dmax, 0, 1 << 30);
+  t.chunk_order = get("TC_CHUNK_ORDER", t.chunk_order, 0, 1);
   return t;
 }
 
@@ -1198,7 +1201,7 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
     const int long_min = (opt.long_min_auto && m < kSmallGraph) ? (1 << 30) : std::max(opt.long_min, 32);
     k_edge_trim<<<grid_for(m), TPB, 0, s>>>(row_ptr, col, rowid.get(), vmm.get(), m, long_min,
                                             g->bits, dead, skey.get(), sval.get(), stats.get(),
-                                            P.tune.long_bitmap ? opt.bitmap_factor : 0);
+                                            P.tune.long_hash_dmax, opt.bitmap_factor);
     TC_LAUNCH();
   }
   rowid.reset();

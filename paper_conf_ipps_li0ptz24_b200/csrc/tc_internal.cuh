@@ -153,7 +153,8 @@ struct Tuning {
   int batch = 0;          // long-class tiles per batch for block_threads <= 768 (TC_BATCH; see count_kernel)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
-  int long_bitmap = 0;    // long class only for edges whose head gets a bitmap (TC_LONG_BITMAP)
+  int long_hash_dmax = 0; // hash-table heads with d+(v) <= this go to the short class (TC_LONG_HASH_DMAX)
+  int chunk_order = 0;    // long class: 1 = each CTA alternates chunks from both ends (TC_CHUNK_ORDER)
 };
 Tuning tuning_from_env();
 

@@ -260,6 +260,25 @@ r4w)
   bash scripts/gpu_ab.sh r4w_C2 C2 10 "" "TC_LONG_BITMAP=1"
   bash scripts/gpu_ab.sh r4w_C4 C4 3 "" "TC_LONG_BITMAP=1"
   ;;
+r4x)
+  # hash-table heads with d+(v) <= D flattened with the short class (TC_LONG_HASH_DMAX)
+  bash scripts/gpu_ab.sh r4x_C3 C3 10 "" "TC_LONG_HASH_DMAX=16" "TC_LONG_HASH_DMAX=32" "TC_LONG_HASH_DMAX=64" "TC_LONG_HASH_DMAX=128" ""
+  bash scripts/gpu_ab.sh r4x_C4 C4 3 "" "TC_LONG_HASH_DMAX=32" "TC_LONG_HASH_DMAX=64"
+  ;;
+r4y)
+  # hash table size (table_factor slots per N+(v) entry; default 6)
+  bash scripts/gpu_ab.sh r4y_C3 C3 10 "" "BENCH_OPT=table_factor=3" "BENCH_OPT=table_factor=4" "BENCH_OPT=table_factor=8" ""
+  bash scripts/gpu_ab.sh r4y_C2 C2 10 "" "BENCH_OPT=table_factor=3" "BENCH_OPT=table_factor=4"
+  bash scripts/gpu_ab.sh r4y_C3d C3 10 "" "TC_LONG_HASH_DMAX=128" "TC_LONG_HASH_DMAX=256" "TC_LONG_HASH_DMAX=512" "TC_LONG_HASH_DMAX=1024" ""
+  ;;
+r5a)
+  # long-class chunks taken alternately from both ends of the range by every CTA (TC_CHUNK_ORDER=1)
+  TC_CHUNK_ORDER=1 timeout 900 python -m pytest -q -x tests/test_gpu_parity.py -k "closed_forms or c1_rmat10 or rmat_medium or options or karate or golden or full_size or huge or cap or skewed or partition or ranges or async" > $O/r5a_pytest_chunk_order.txt 2>&1; echo "rc=$?" >> $O/r5a_pytest_chunk_order.txt
+  bash scripts/gpu_ab.sh r5a_C3 C3 10 "" "TC_CHUNK_ORDER=1" "" "TC_CHUNK_ORDER=1"
+  bash scripts/gpu_ab.sh r5a_C4 C4 3 "" "TC_CHUNK_ORDER=1" "TC_LONG_HASH_DMAX=128"
+  bash scripts/gpu_ab.sh r5a_C2 C2 10 "" "TC_LONG_HASH_DMAX=128" "TC_CHUNK_ORDER=1"
+  bash scripts/gpu_ab.sh r5a_C3b C3 10 "TC_LONG_HASH_DMAX=128" "TC_LONG_HASH_DMAX=128 TC_CHUNK_ORDER=1" ""
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
