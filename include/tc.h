@@ -89,7 +89,10 @@ typedef struct {
   int32_t long_min;     /* trimmed suffixes with >= long_min keys go to the
                            warp-per-edge tile class, shorter ones to the flattened
                            class (default 32; values below 32 act as 32, since a
-                           tile holds 32 keys of its own edge; 2^30 = all short) */
+                           tile holds 32 keys of its own edge; 2^30 = all short).
+                           Edges whose head gets a hash table with d+(v) <= 128
+                           are flattened whatever their length (env
+                           TC_LONG_HASH_DMAX; 0 = pure length split)         */
   int32_t probe_mode;   /* 0 = two-choice (cuckoo) tables with linear-probing
                            fallback per chunk, 1 = linear probing only (default 0) */
   int32_t bitmap_factor; /* a head v whose window [min N+(v), max N+(v)] needs at most

@@ -1152,7 +1152,6 @@ Tuning tuning_from_env() {
   t.batch = get("TC_BATCH", t.batch, 0, 64);
   t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 3);
   t.long_hash_dmax = get("TC_LONG_HASH_DMAX", t.long_hash_dmax, 0, 1 << 30);
-  t.chunk_order = get("TC_CHUNK_ORDER", t.chunk_order, 0, 1);
   return t;
 }
 
