@@ -74,7 +74,8 @@ void keep_mapped(cudaMemPool_t pool) {
   uint64_t thr = UINT64_MAX;
   cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
   int no = 0;
-  cudaMemPoolSetAttribute(pool, cudaMemPoolReuseAllowInternalDependencies, &no);
+  static const bool allow = std::getenv("TC_POOL_INTERNAL_DEPS") != nullptr;  // A/B knob
+  if (!allow) cudaMemPoolSetAttribute(pool, cudaMemPoolReuseAllowInternalDependencies, &no);
 }
 
 // The device's default pool (persistent buffers) or the library's own scratch
@@ -893,6 +894,8 @@ tc_status tc_build_from_oriented(const uint64_t* d_okeys, int64_t m, const int32
 
 void tc_free(tc_graph* g) {
   if (!g) return;
+  static const bool devsync = std::getenv("TC_FREE_DEVSYNC") != nullptr;  // A/B knob
+  if (devsync) cudaDeviceSynchronize();
   // the graph's own build and replans completed before they returned; wait
   // for the work other streams enqueued on it, then free stream-ordered
   {

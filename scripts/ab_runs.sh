@@ -279,6 +279,16 @@ r5a)
   bash scripts/gpu_ab.sh r5a_C2 C2 10 "" "TC_LONG_HASH_DMAX=128" "TC_CHUNK_ORDER=1"
   bash scripts/gpu_ab.sh r5a_C3b C3 10 "TC_LONG_HASH_DMAX=128" "TC_LONG_HASH_DMAX=128 TC_CHUNK_ORDER=1" ""
   ;;
+r5c)
+  # e2e step spread: pool internal reuse dependencies and tc_free's device sync (A/B knobs)
+  for c in C5 C3; do
+    for kv in "" "TC_POOL_INTERNAL_DEPS=1" "TC_FREE_DEVSYNC=1" "TC_POOL_INTERNAL_DEPS=1 TC_FREE_DEVSYNC=1" ""; do
+      tag=$(echo "${kv:-default}" | tr ' =' '__')
+      env $kv timeout 900 python bench.py --config $c --steps 3 --warmup 3 --e2e-steps 20 --no-balance --no-sharded --no-cpu-baseline --no-e2e-pipelined --out $O/r5c_${c}_$tag.json > $O/r5c_${c}_$tag.log 2>&1
+      python -c "import json,sys; d=json.load(open('$O/r5c_${c}_$tag.json')); e=d['e2e']['step_ms']; print('$c', '$tag', round(sum(e)/len(e),1), [round(x) for x in e])" >> $O/r5c_e2e.txt 2>&1
+    done
+  done
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt

@@ -22,9 +22,8 @@ for v in polak trust; do for c in C1 C2 C5 C3; do
     --no-balance --out $O/${T}_bench_${v}_$(echo $c | tr C c).json > $O/${T}_bench_${v}_$c.log 2>&1
 done; done
 timeout 1800 python scripts/oracle_times.py > $O/${T}_oracle_times.jsonl 2> $O/${T}_oracle_times.err
-for tool in racecheck synccheck memcheck; do
-  timeout 900 compute-sanitizer --tool $tool --print-limit 50 python scripts/sanitize_case.py > $O/${T}_sanitize_${tool}.txt 2>&1; echo "rc=$?" >> $O/${T}_sanitize_${tool}.txt
-done
+# (compute-sanitizer is closed on the gpurun pool since r4a; the r2b / r2j logs are the last runs:
+#  for tool in racecheck synccheck memcheck: compute-sanitizer --tool $tool python scripts/sanitize_case.py)
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/${T}_launches_c3.csv \
   python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu-baseline --no-sharded --no-balance > $O/${T}_launches.log 2>&1
 for c in C3 C2; do
