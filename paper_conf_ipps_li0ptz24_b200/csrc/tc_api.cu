@@ -63,19 +63,12 @@ namespace {
 constexpr int kMaxDevices = 64;
 
 // Release threshold "never": freed blocks stay mapped across syncs (without
-// this every build re-maps its scratch, tens of ms at config C2).  No
-// internal reuse dependencies: a block freed on one stream is not handed to
-// an allocation on another stream by making that stream wait for the first
-// one's work, which serialised a count on one stream with a build on another
-// (C3 pipelined e2e 124 -> 100 ms per step, profiles/r4o_pipe3.txt); blocks
-// are still reused when their free is known complete (event dependencies,
-// opportunistic reuse).
+// this every build re-maps its scratch, tens of ms at config C2).  (Turning
+// off the pools' internal cross-stream reuse dependencies made the host
+// entry's steps vary, C5 13 -> 13-119 ms, profiles/r5c_e2e.txt; kept on.)
 void keep_mapped(cudaMemPool_t pool) {
   uint64_t thr = UINT64_MAX;
   cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-  int no = 0;
-  static const bool allow = std::getenv("TC_POOL_INTERNAL_DEPS") != nullptr;  // A/B knob
-  if (!allow) cudaMemPoolSetAttribute(pool, cudaMemPoolReuseAllowInternalDependencies, &no);
 }
 
 // The device's default pool (persistent buffers) or the library's own scratch
@@ -387,22 +380,34 @@ tc_status tc_count(const tc_graph* g, void* stream, uint64_t* h_count) {
   return guarded([&] {
     require(g && h_count, "NULL argument");
     cudaStream_t s = (cudaStream_t)stream;
-    tc::DevBuf<unsigned long long> d(1, s);
-    tc::count_chunks(g, 0, g->plan.n_chunks, 0, g->plan.S, s, d.get());
-    // the 8-B result lands in pinned memory: a copy into pageable (stack)
-    // memory held a build's H2D copies on another stream back until this
-    // count finished (C3 pipelined e2e: 124 vs 100 ms per step,
-    // profiles/r4o_pipeline_variants.txt)
-    thread_local struct Pinned {
-      unsigned long long* p = nullptr;
-      ~Pinned() {
-        if (p) cudaFreeHost(p);
+    // The 8-B result: a per-thread device word (no pool allocation, so no
+    // reuse dependency on another stream's frees) copied into per-thread
+    // pinned memory (a copy into pageable stack memory held a build's H2D
+    // copies on another stream back until this count finished: C3 pipelined
+    // e2e 124 vs 100 ms per step, profiles/r4o_pipeline_variants.txt).  The
+    // call is synchronous, so one word per thread and device suffices.
+    thread_local struct Result {
+      int dev = -1;
+      unsigned long long* d = nullptr;
+      unsigned long long* h = nullptr;
+      ~Result() {
+        if (d) cudaFree(d);
+        if (h) cudaFreeHost(h);
       }
-    } pin;
-    if (!pin.p) TC_CUDA(cudaMallocHost(&pin.p, sizeof(unsigned long long)));
-    TC_CUDA(cudaMemcpyAsync(pin.p, d.get(), sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
+    } res;
+    int dev = 0;
+    TC_CUDA(cudaGetDevice(&dev));
+    if (res.dev != dev) {
+      if (res.d) cudaFree(res.d);
+      res.d = nullptr;
+      TC_CUDA(cudaMalloc(&res.d, sizeof(unsigned long long)));
+      res.dev = dev;
+    }
+    if (!res.h) TC_CUDA(cudaMallocHost(&res.h, sizeof(unsigned long long)));
+    tc::count_chunks(g, 0, g->plan.n_chunks, 0, g->plan.S, s, res.d);
+    TC_CUDA(cudaMemcpyAsync(res.h, res.d, sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
     TC_CUDA(cudaStreamSynchronize(s));
-    *h_count = *pin.p;
+    *h_count = *res.h;
   });
 }
 
@@ -894,8 +899,6 @@ tc_status tc_build_from_oriented(const uint64_t* d_okeys, int64_t m, const int32
 
 void tc_free(tc_graph* g) {
   if (!g) return;
-  static const bool devsync = std::getenv("TC_FREE_DEVSYNC") != nullptr;  // A/B knob
-  if (devsync) cudaDeviceSynchronize();
   // the graph's own build and replans completed before they returned; wait
   // for the work other streams enqueued on it, then free stream-ordered
   {

@@ -289,6 +289,16 @@ r5c)
     done
   done
   ;;
+r5d)
+  # e2e steps and the pipelined leg with pool reuse dependencies on + per-thread count result
+  timeout 600 python scripts/diag_pipeline3.py > $O/r5d_pipe3.txt 2>&1
+  for c in C5 C3 C2; do
+    for rep in 1 2; do
+      timeout 900 python bench.py --config $c --steps 3 --warmup 3 --e2e-steps 20 --no-balance --no-sharded --no-cpu-baseline --out $O/r5d_${c}_$rep.json > $O/r5d_${c}_$rep.log 2>&1
+      python -c "import json; d=json.load(open('$O/r5d_${c}_$rep.json')); e=d['e2e']['step_ms']; print('$c', $rep, round(sum(e)/len(e),1), [round(x) for x in e], 'pipelined', round(d['e2e_pipelined']['ms_per_step'],1))" >> $O/r5d_e2e.txt 2>&1
+    done
+  done
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
