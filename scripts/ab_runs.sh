@@ -299,6 +299,13 @@ r5d)
     done
   done
   ;;
+r5i)
+  # consumers insert N+(v) of insert-heavy long-class chunks (TC_CONS_INSERT = R: when inserts x R > key lanes)
+  TC_CONS_INSERT=1 timeout 900 python -m pytest -q -x tests/test_gpu_parity.py -k "closed_forms or c1_rmat10 or rmat_medium or options or karate or golden or full_size or huge or cap or skewed or partition or ranges" > $O/r5i_pytest_cons_insert.txt 2>&1; echo "rc=$?" >> $O/r5i_pytest_cons_insert.txt
+  TC_CONS_INSERT=1000 TC_CUCKOO_KICKS=0 timeout 900 python -m pytest -q -x tests/test_gpu_parity.py tests/test_gpu_robust.py -k "closed_forms or c1_rmat10 or rmat_medium or options or cuckoo" > $O/r5i_pytest_cons_insert_cuckoo.txt 2>&1; echo "rc=$?" >> $O/r5i_pytest_cons_insert_cuckoo.txt
+  bash scripts/gpu_ab.sh r5i_C3 C3 10 "" "TC_CONS_INSERT=1" "TC_CONS_INSERT=2" "TC_CONS_INSERT=4" "TC_CONS_INSERT=16" ""
+  bash scripts/gpu_ab.sh r5i_C4 C4 3 "" "TC_CONS_INSERT=2" "TC_CONS_INSERT=4"
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
