@@ -531,6 +531,7 @@ def main():
         ps = torch.from_numpy(src).pin_memory()
         pd = torch.from_numpy(dst).pin_memory()
         ts = []
+        detail = []  # per step: host ms of the build call, the partition, the count + D2H; build phase ms (events)
         n_chunks = 0
         for i in range(1 + k2):  # first one warms the pinned path
             if world > 1:
@@ -539,30 +540,40 @@ def main():
             x0 = torch.cuda.Event(enable_timing=True)
             x1 = torch.cuda.Event(enable_timing=True)
             x0.record(stream)
+            h0 = time.perf_counter()
             if world > 1:  # each rank copies and sorts only its slice (f2)
                 g2 = tc.build_csr_sharded(ps[lo:hi].to(dev, non_blocking=True),
                                           pd[lo:hi].to(dev, non_blocking=True), n,
                                           options=opts or None)
             else:
                 g2 = tc.build_csr_host(ps, pd, n, options=opts or None)
+            h1 = time.perf_counter()
             b = g2.partition(world, profile) if profile is not None else g2.partition(world)
+            h2 = time.perf_counter()
             o2 = g2.count_range(b[rank], b[rank + 1])
             if world > 1:
                 dist.all_reduce(o2)
             t_e2e = int(o2.item()) & (2**64 - 1)
+            h3 = time.perf_counter()
             x1.record(stream)
             torch.cuda.synchronize()
-            n_chunks = g2.info.n_chunks
+            inf2 = g2.info
+            n_chunks = inf2.n_chunks
+            phases = [round(x, 1) for x in (inf2.ms_canon, inf2.ms_sort_unique, inf2.ms_degree_rank,
+                                             inf2.ms_orient_csr, inf2.ms_plan, inf2.ms_total)]
             g2.close()
             assert t_e2e == T, (t_e2e, T)
             if i:
                 ts.append(x0.elapsed_time(x1))
+                detail.append([round(1e3 * (h1 - h0), 1), round(1e3 * (h2 - h1), 1), round(1e3 * (h3 - h2), 1),
+                               phases])
         et = torch.tensor([sum(ts)], dtype=torch.float64, device=dev)
         if world > 1:
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
         e2e_ms = float(et[0]) / max(1, len(ts))
         e2e = {"value": m / (e2e_ms / 1e3), "unit": UNIT, "ms_per_step": e2e_ms,
                "step_ms": [round(x, 3) for x in ts],
+               "step_host_ms_build_partition_count": detail,
                "h2d_bytes_per_step": int(src.nbytes + dst.nbytes) * (hi - lo) // max(1, len(src)),
                "d2h_bytes_per_step": 8 + 8 * (n_chunks + 1) + 96,
                "what": ("tc_build_csr_host (H2D of the raw pinned edge list + a1..a6)" if world == 1

@@ -2,6 +2,7 @@
 // translation (no exception crosses the ABI), the allocator hook, and the
 // host-side range/partition logic.  SURVEY.md §8(b).
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cmath>
 #include <cstdlib>
@@ -57,6 +58,29 @@ void check_cuda(cudaError_t e, const char* what, const char* file, int line) {
   char buf[512];
   snprintf(buf, sizeof(buf), "%s: %s (%s:%d)", what, cudaGetErrorString(e), file, line);
   fail(TC_ERR_CUDA, buf);
+}
+
+bool host_trace_on() {
+  static const bool on = std::getenv("TC_HOST_TRACE") != nullptr;
+  return on;
+}
+namespace {
+thread_local std::vector<std::pair<const char*, std::chrono::steady_clock::time_point>> g_marks;
+}
+void host_mark(const char* what) {
+  if (host_trace_on()) g_marks.emplace_back(what, std::chrono::steady_clock::now());
+}
+void host_trace_flush() {
+  if (!host_trace_on() || g_marks.empty()) return;
+  std::string line = "[tc host]";
+  for (size_t i = 1; i < g_marks.size(); ++i) {
+    char b[96];
+    snprintf(b, sizeof(b), " %s %.2f", g_marks[i].first,
+             std::chrono::duration<double, std::milli>(g_marks[i].second - g_marks[i - 1].second).count());
+    line += b;
+  }
+  fprintf(stderr, "%s\n", line.c_str());
+  g_marks.clear();
 }
 
 namespace {
@@ -131,14 +155,30 @@ void* dev_alloc(size_t bytes, cudaStream_t s, bool persistent) {
 // Grow the scratch pool in one step so that a build's scratch allocations
 // reuse already-mapped memory: mapping physical memory inside the build
 // (pool growth on demand) made identical builds vary by 3-10x in time.
+// The scratch pool only ever grows (release threshold "never"; trim_pools
+// resets it), and nothing holds scratch between builds, so once it has been
+// grown to `bytes` a later build of at most that size skips the driver
+// queries: they cost 0.1-9 ms per build of the host entry at C2 and made its
+// steps vary (TC_HOST_TRACE, profiles/r5m_*).
+std::atomic<uint64_t> g_reserved_hint[64];
+
 void reserve_pool(size_t bytes, cudaStream_t s) {
   if (g_alloc || bytes == 0) return;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) {
+    cudaGetLastError();
+    return;
+  }
+  if ((uint64_t)bytes <= g_reserved_hint[dev].load(std::memory_order_relaxed)) return;
   cudaMemPool_t pool = pool_of(false);
   if (!pool) return;
   uint64_t reserved = 0, used = 0;
   cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved);
   cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used);
-  if (reserved - used >= bytes) return;
+  if (reserved - used >= bytes) {
+    if (used == 0) g_reserved_hint[dev].store(reserved, std::memory_order_relaxed);
+    return;
+  }
   size_t free_b = 0, total_b = 0;
   cudaMemGetInfo(&free_b, &total_b);
   const size_t want = bytes - (size_t)(reserved - used);
@@ -146,7 +186,10 @@ void reserve_pool(size_t bytes, cudaStream_t s) {
   const size_t grow = want < cap ? want : cap;
   if (grow == 0) return;
   void* p = nullptr;
-  if (cudaMallocFromPoolAsync(&p, grow, pool, s) == cudaSuccess && p) cudaFreeAsync(p, s);
+  if (cudaMallocFromPoolAsync(&p, grow, pool, s) == cudaSuccess && p) {
+    cudaFreeAsync(p, s);
+    if (used == 0) g_reserved_hint[dev].store(reserved + grow, std::memory_order_relaxed);
+  }
   cudaGetLastError();
 }
 
@@ -154,6 +197,7 @@ void reserve_pool(size_t bytes, cudaStream_t s) {
 // device back to the driver: tc_release_memory.
 void trim_pools() {
   TC_CUDA(cudaDeviceSynchronize());
+  for (auto& h : g_reserved_hint) h.store(0, std::memory_order_relaxed);
   for (bool persistent : {false, true}) {
     cudaMemPool_t pool = pool_of(persistent);
     if (pool) TC_CUDA(cudaMemPoolTrimTo(pool, 0));
@@ -273,13 +317,17 @@ tc_status build_impl(const int32_t* src, const int32_t* dst, int64_t num_edges,
     // + the a2 hash set (u64, capacity the power of two >= 2 num_edges)
     size_t cap = 1024;
     while ((int64_t)cap < 2 * num_edges && num_edges <= (int64_t(1) << 25)) cap <<= 1;
+    tc::host_mark("start");
     tc::reserve_pool((size_t)num_edges * (host ? 80 : 72) + (size_t)nv * 48 + cap * 8, s);
+    tc::host_mark("reserve_pool");
     g = new tc_graph();
     if (host) {
       tc::build_graph_host(src, dst, num_edges, num_vertices, flags, opt, s, g);
     } else {
       tc::build_graph(src, dst, num_edges, num_vertices, flags, opt, s, g);
     }
+    tc::host_mark("return");
+    tc::host_trace_flush();
   });
   if (st != TC_OK) {
     if (g) {

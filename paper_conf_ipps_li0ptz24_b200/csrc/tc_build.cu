@@ -825,6 +825,7 @@ static void build_tail(uint64_t* ukey, int64_t m, DevBuf<uint64_t>& ka, DevBuf<u
   const int bits = bits_for(std::max<int64_t>(n, 2));
   g->m = m;
   tm.mark();
+  host_mark("a2_done");
 
   // a3 + a4
   DevBuf<int32_t> deg(std::max<int64_t>(n, 1), s);
@@ -859,9 +860,12 @@ static void build_tail(uint64_t* ukey, int64_t m, DevBuf<uint64_t>& ka, DevBuf<u
   kb.reset();
   rank.reset();
   tm.mark();
+  host_mark("a3_a5");
   build_plan(g, opt, s);
+  host_mark("plan_issued");
   tm.mark();
   TC_CUDA(cudaStreamSynchronize(s));
+  host_mark("plan_sync");
   g->ms[0] = tm.ms(0, 1);
   g->ms[1] = tm.ms(1, 2);
   g->ms[2] = tm.ms(2, 3);
@@ -933,6 +937,7 @@ void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen,
     return k == 1 || k == 2 || k == 4 || k == 8 ? k : 8;
   }();
   DevBuf<int32_t> ds(std::max<int64_t>(m_gen, 1), s), dd(std::max<int64_t>(m_gen, 1), s);
+  host_mark("alloc_pairs");
   if (n < 0 || pieces == 1 || m_gen <= (int64_t(1) << 25) ||
       m_gen / pieces > (int64_t)0x7fffffff) {  // (cub merge counts are int)
     if (m_gen) {
@@ -949,6 +954,7 @@ void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen,
   // time at C3 varied between 86 and 161 ms over identical builds (the phase
   // events inside stayed at 85 ms), with it it is 85-88 ms (profiles/r2t_e2e_c3.txt).
   TC_CUDA(cudaStreamSynchronize(s));
+  host_mark("sync_alloc");
   g->n_input = n;
   const int bits = bits_for(std::max<int64_t>(n, 2));
   const uint64_t sent = (uint64_t(1) << (2 * bits)) - 1;
@@ -977,6 +983,7 @@ void build_graph_host(const int32_t* h_src, const int32_t* h_dst, int64_t m_gen,
   // behind a count kernel running on another stream and held the H2D back)
   TC_CUDA(cudaEventRecord(r.ready, s));  // the device buffers exist (stream-ordered allocs)
   TC_CUDA(cudaStreamWaitEvent(r.cs, r.ready, 0));
+  host_mark("streams_events");
   TC_CUDA(cudaMemsetAsync(err.get(), 0, sizeof(int), s));
   TC_CUDA(cudaMemsetAsync(nsel.get(), 0, sizeof(int64_t), s));
   int64_t lo[9];

@@ -71,6 +71,13 @@ struct DevBuf {
   T* get() const { return p; }
 };
 
+// ---------------------------------------------------------------- host trace
+// TC_HOST_TRACE=1: host timestamps of a build's steps, one stderr line per
+// build (diagnosing host-side delays of the host entry point).
+bool host_trace_on();
+void host_mark(const char* what);  // no-op unless TC_HOST_TRACE
+void host_trace_flush();
+
 // ---------------------------------------------------------------- options
 struct Options {
   int chunk_cost = 16384;
