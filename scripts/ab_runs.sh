@@ -306,6 +306,24 @@ r5i)
   bash scripts/gpu_ab.sh r5i_C3 C3 10 "" "TC_CONS_INSERT=1" "TC_CONS_INSERT=2" "TC_CONS_INSERT=4" "TC_CONS_INSERT=16" ""
   bash scripts/gpu_ab.sh r5i_C4 C4 3 "" "TC_CONS_INSERT=2" "TC_CONS_INSERT=4"
   ;;
+r6b)
+  # chunk sizes (plan option chunk_cost: long chunks 4x, short 1x) and the short-class divisor
+  bash scripts/gpu_ab.sh r6b_C3 C3 10 "" "BENCH_OPT=chunk_cost=12288" "BENCH_OPT=chunk_cost=24576" "BENCH_OPT=chunk_cost=32768" "TC_CS_DIV=2" ""
+  bash scripts/gpu_ab.sh r6b_C2 C2 10 "" "BENCH_OPT=chunk_cost=12288" "BENCH_OPT=chunk_cost=24576" "BENCH_OPT=chunk_cost=32768" "TC_CS_DIV=2"
+  bash scripts/gpu_ab.sh r6b_C5 C5 10 "" "BENCH_OPT=chunk_cost=8192" "BENCH_OPT=chunk_cost=24576"
+  ;;
+r6c)
+  # flat kernel: 3 CTAs x 384 threads (54 registers) with 3 / 4 tiles of keys in flight per warp
+  for c in C2 C5 C3; do
+    bash scripts/gpu_abbuild.sh r6c_$c $c 10 "" "-DTC_FLAT_CTAS=3 -DTC_UNROLL_SHORT=3" "-DTC_FLAT_CTAS=3 -DTC_UNROLL_SHORT=4" ""
+  done
+  ;;
+r6d)
+  # long-class chunk cost multiplier (TC_LONG_CHUNK; long chunks = x * chunk_cost, default 4)
+  bash scripts/gpu_ab.sh r6d_C3 C3 10 "" "TC_LONG_CHUNK=5" "TC_LONG_CHUNK=6" "TC_LONG_CHUNK=8" "TC_LONG_CHUNK=12" ""
+  bash scripts/gpu_ab.sh r6d_C2 C2 10 "" "TC_LONG_CHUNK=6" "TC_LONG_CHUNK=8"
+  bash scripts/gpu_ab.sh r6d_C4 C4 3 "" "TC_LONG_CHUNK=6" "TC_LONG_CHUNK=8"
+  ;;
 *) echo "unknown tag $T"; exit 1;;
 esac
 echo done > $O/${T}_done.txt
