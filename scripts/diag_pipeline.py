@@ -1,3 +1,5 @@
+"""Pipelined e2e timeline (C3): per step, how long the main thread waits for graph i+1's
+build (second host thread, own stream) and how long graph i's count and close take."""
 import sys, time, os, concurrent.futures
 sys.path.insert(0, os.getcwd())
 import numpy as np, torch, tcgen
