@@ -77,8 +77,7 @@ TC_API tc_status tc_set_allocator(tc_alloc_fn alloc, tc_free_fn free_fn, void* c
  * change the count; the property tests vary them).  0 in a field = default.
  */
 typedef struct {
-  int32_t chunk_cost;   /* cost units per short-class work chunk (default 16384;
-                           long-class chunks are 6x: env TC_LONG_CHUNK)          */
+  int32_t chunk_cost;   /* cost units per work chunk (default 16384)               */
   int32_t seg_cost;     /* fixed cost per live oriented edge (default 4)          */
   int32_t huge_degree;  /* d+(v) above which N+(v) is probed in global memory by
                            binary search instead of an SMEM hash (default 8192)    */

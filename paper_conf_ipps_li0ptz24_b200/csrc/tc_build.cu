@@ -1159,7 +1159,6 @@ Tuning tuning_from_env() {
   t.batch = get("TC_BATCH", t.batch, 0, 64);
   t.prod_groups = get("TC_PROD_GROUPS", t.prod_groups, 1, 3);
   t.long_hash_dmax = get("TC_LONG_HASH_DMAX", t.long_hash_dmax, 0, 1 << 30);
-  t.long_chunk = get("TC_LONG_CHUNK", t.long_chunk, 1, 64);
   return t;
 }
 
@@ -1312,13 +1311,13 @@ void build_plan(tc_graph* g, const Options& opt, cudaStream_t s) {
   tr("groups + prefixes + costs");
   P.units_total = (int64_t)units_total;
 
-  // Chunking, per class: cost chunks (long class Tuning::long_chunk = 6x
-  // larger: its edges carry ~150 keys each), then every chunk is split where its SMEM layout would
+  // Chunking, per class: cost chunks (long class 4x larger: its edges carry
+  // ~150 keys each), then every chunk is split where its SMEM layout would
   // exceed one of the count kernel's chunk slots (only outliers split).
   // short chunks of half the cost when edges carry ~1 key (C5 road lattice:
   // 1.05 keys per live edge, 0.114 -> 0.073 ms; C2 at 5.4 keys: neutral)
   const int cs_div = P.tune.cs_div ? P.tune.cs_div : (P.keys_total < 2 * S ? 2 : 1);
-  const int64_t CL = std::max<int64_t>((int64_t)P.tune.long_chunk * opt.chunk_cost, 64),
+  const int64_t CL = std::max<int64_t>(4ll * opt.chunk_cost, 64),
                 CS = std::max<int64_t>(opt.chunk_cost / cs_div, 64);
   {
     const int64_t nL0 = (cost_long + CL - 1) / CL, nS0 = (cost_short + CS - 1) / CS, nc0 = nL0 + nS0;

@@ -160,8 +160,6 @@ struct Tuning {
   int batch = 0;          // long-class tiles per batch for block_threads <= 768 (TC_BATCH; see count_kernel)
   int max_kicks = 96;     // cuckoo displacements before a chunk rebuilds with linear probing (TC_CUCKOO_KICKS;
                           // 0 forces the rebuild of every chunk with a hash table: tests)
-  int long_chunk = 6;     // long-class chunk cost = long_chunk x chunk_cost (TC_LONG_CHUNK; r6d: 4 -> 6
-                          // C3 step 44.6 -> 43.4 ms, C4 563 -> 538, C2 equal; 8: 44.7, 12: 49.7)
   int long_hash_dmax = 128;  // long-class candidates whose head gets a hash table with d+(v) <= this
                             // go to the short class (TC_LONG_HASH_DMAX; 0 = off; r4x/r4y/r5a: C3 step
                             // 44.4 -> 43.9 ms, C2 1.313 -> 1.283, C4 558 -> 555)
